@@ -1,0 +1,305 @@
+#!/usr/bin/env python
+"""Benchmark of the Central Graph keyword-search hot path (BASELINE.json metric: p50 query latency,
+queries/s and GTEPS on the Wikidata-scale synthetic graph).
+
+A step = one query through the whole hot path (activation gate, search, central detection,
+extraction + level-cover + Eq. 6 score of every central graph, radix-select top-k, answer emit).
+
+  python bench.py [--gpus N --steps K --warmup W]          CUDA path (libkgs), one rank per GPU
+  python bench.py --impl reference [...]                   the CPU oracle on this box's host cores
+
+N = 1: workload C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keywords, top-20), the
+queries cycled from its 350-query latency set.  N > 1 (torchrun): workload C4 (configs[3]: the same
+graph, 4096 queries with q ~ U{2..8}) sharded round-robin over ranks, each rank holding a replicated
+graph; after the timed steps the ranks all-gather their top-k headers over NCCL (inside the timed
+region).  Scaling is weak (K queries per rank).
+
+Timing: W warm-up steps; then K steps, each bracketed by CUDA events on the launching stream; between
+steps L2 is flushed (a 512 MiB write, outside the events); barrier + synchronize on both sides; the
+max over ranks.  `value` = queries / second of device time (graph and keyword ids resident in HBM);
+`e2e` = the same through kgs_query with host keyword ids and the answers copied back (wall clock).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "p50 query latency (ms) & queries/s, Wikidata-scale graph; GTEPS"
+
+
+def _env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+        self.th = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.index), "-lms", "100"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+            return
+        self.th = threading.Thread(target=self._read, daemon=True)
+        self.th.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        if self.th:
+            self.th.join(timeout=2)
+        sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        smax = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            if len(r) >= 9:
+                for nm, v in zip(names, r[5:9]):
+                    if v.lower() == "active":
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def bfs_algorithmic_bytes(st: dict) -> float:
+    """SURVEY.md §8(d) / DESIGN.md "Roofline": bytes the search must move for this query.
+    per expanded frontier entry: 16 B row_ptr + 2 B own status + 1 B activation + 4 B queue slot;
+    per inspected arc: 4 B col_idx + 2 B neighbour status;
+    per new (node, keyword) hit: 1 B M write + 1 B new-hit mask + 4 B next-queue slot (amortised);
+    per touched node: 2 B status reset."""
+    return (st["frontier_total"] * 23.0 + st["arcs_scanned"] * 6.0 + st.get("hits", 0) * 6.0)
+
+
+# ------------------------------------------------------------------------------------------ workloads
+def build_workload(name: str, rank: int, world: int):
+    import synth
+    t0 = time.time()
+    w = synth.make_workload(name)
+    return w, time.time() - t0
+
+
+def run_reference(args):
+    """The oracle, as it stands, on host cores (bench.py --impl reference)."""
+    rank, world = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1)
+    if rank != 0:
+        return 0
+    import oracle
+    name = "C3" if world == 1 else "C4"
+    w, gen_s = build_workload(name, 0, 1)
+    qs = w.queries
+    for i in range(args.warmup):
+        oracle.query(w.graph, qs[i % len(qs)], w.k)
+    lat = []
+    t_all = time.perf_counter()
+    for i in range(args.steps):
+        kw = qs[(args.warmup + i) % len(qs)]
+        t0 = time.perf_counter()
+        oracle.query(w.graph, kw, w.k)
+        lat.append((time.perf_counter() - t0) * 1e3)
+    tot = time.perf_counter() - t_all
+    qps = args.steps / tot
+    line = {"impl": "reference", "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot * 1e3 / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "config": {"workload": name, "graph": f"R-MAT scale 25 edge factor 8 ({w.graph.n} nodes, "
+                                                   f"{w.graph.n_arcs} arcs)", "k": w.k, "queries": len(qs)},
+            "p50_ms": statistics.median(lat),
+            "cpu_baseline": {"value": qps, "unit": "queries/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} consecutive {name} queries after {args.warmup} warm-up"},
+            "e2e": {"value": qps, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="kgs", choices=["kgs", "reference"])
+    ap.add_argument("--cpu-sample-s", type=float, default=15.0)
+    ap.add_argument("--e2e-steps", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    rank, world, local = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1), _env_int("LOCAL_RANK", 0)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = local
+    torch.cuda.set_device(dev)
+    import paper_conf_icde_yangajtw19_b200 as kgs
+
+    name = "C3" if world == 1 else "C4"
+    w, gen_s = build_workload(name, rank, world)
+    g = w.graph
+    t0 = time.time()
+    G = kgs.kgs_load_graph(g, device=dev)
+    load_s = time.time() - t0
+    queries = w.queries[rank::world] if world > 1 else w.queries
+    qdev = [torch.tensor(list(kw), dtype=torch.int32, device=f"cuda:{dev}") for kw in queries]
+    stream = torch.cuda.current_stream(dev)
+    sh = stream.cuda_stream
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=f"cuda:{dev}")
+    p = kgs.kgs_params_default()
+
+    def step(i):
+        j = i % len(queries)
+        kgs.kgs_query_device(G, qdev[j].data_ptr(), len(queries[j]), w.k, p, sh)
+
+    # warm-up (also builds the activation cache for alpha)
+    for i in range(args.warmup):
+        step(i)
+        kgs.kgs_query_fetch(G, len(queries[i % len(queries)]), 0, sh)
+    torch.cuda.synchronize(dev)
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    stats = []
+    clk = ClockSampler(dev)
+    clk.start()
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
+    t_wall = time.perf_counter()
+    for i in range(args.steps):
+        flush.fill_(i & 0xFF)                       # L2 flush between timed steps (outside the events)
+        ev[i][0].record(stream)
+        step(args.warmup + i)
+        ev[i][1].record(stream)
+        r = kgs.kgs_query_fetch(G, len(queries[(args.warmup + i) % len(queries)]), 0, sh)  # after ev: not timed
+        stats.append(r.stats)
+    gather_ms = 0.0
+    if dist:
+        # NCCL gather of every rank's top-k headers (central, depth, key) to all ranks (config C4)
+        hdr = torch.zeros((args.steps, w.k, 3), dtype=torch.float64, device=f"cuda:{dev}")
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        out = [torch.empty_like(hdr) for _ in range(world)]
+        dist.all_gather(out, hdr)
+        e1.record(stream)
+    torch.cuda.synchronize(dev)
+    if dist:
+        dist.barrier()
+        gather_ms = e0.elapsed_time(e1)
+    wall = time.perf_counter() - t_wall
+    clocks = clk.stop()
+    lat = [a.elapsed_time(b) for a, b in ev]
+    dev_ms = sum(lat) + gather_ms
+    if dist:
+        t = torch.tensor([dev_ms], dtype=torch.float64, device=f"cuda:{dev}")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev_ms = float(t.item())
+    total_queries = args.steps * world
+    value = total_queries / (dev_ms / 1e3)
+    arcs = sum(s["arcs_scanned"] for s in stats)
+    search_ms = sum(s["ms_search"] for s in stats)
+    td_ms = sum(s["ms_topdown"] for s in stats)
+
+    # e2e: host keyword ids -> kgs_query -> answers on the host (wall clock, includes H2D / D2H)
+    e2e_steps = args.e2e_steps or args.steps
+    e2e_lat = []
+    d2h = 0
+    for i in range(e2e_steps):
+        kw = list(queries[(args.warmup + i) % len(queries)])
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        r = kgs.kgs_query(G, kw, w.k, p, sh)
+        e2e_lat.append((time.perf_counter() - t0) * 1e3)
+        d2h += sum(16 + 8 + a.nodes.nbytes + a.arcs.nbytes for a in r.answers)
+    e2e_qps = e2e_steps / (sum(e2e_lat) / 1e3)
+    h2d = sum(4 * len(queries[(args.warmup + i) % len(queries)]) for i in range(e2e_steps)) / e2e_steps
+
+    if rank != 0:
+        if dist:
+            dist.destroy_process_group()
+        return 0
+    peak, peak_kind = load_peaks()
+    bfs_bytes = sum(bfs_algorithmic_bytes(s) for s in stats)
+    achieved = bfs_bytes / (search_ms / 1e3) / 1e9 if search_ms > 0 else 0.0
+    line = {
+        "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {g.n} nodes, {g.n_arcs} arcs",
+                   "k": w.k, "queries": len(w.queries), "alpha": 0.1, "lambda": 0.2,
+                   "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
+                   "load_s": round(load_s, 1), "parallelism": f"query-sharded x{world}" if world > 1 else "single"},
+        "p50_ms": statistics.median(lat), "p95_ms": float(np.percentile(lat, 95)),
+        "gteps": arcs / (dev_ms / 1e3) / 1e9 * (world if world > 1 else 1) if dev_ms else 0.0,
+        "phase_ms": {"search": search_ms / args.steps, "topdown": td_ms / args.steps},
+        "roofline": {"kernel": "k_search", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": None, "peak_kind": peak_kind,
+                     "algorithmic_bytes_per_query": bfs_bytes / args.steps},
+        "e2e": {"value": e2e_qps, "unit": "queries/s", "p50_ms": statistics.median(e2e_lat),
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h / e2e_steps},
+        "gpu_launches": 7 * args.steps,
+        "clocks": clocks,
+        "stats_mean": {k: float(np.mean([s[k] for s in stats])) for k in
+                       ("levels", "n_centrals", "frontier_total", "arcs_scanned", "overflow")},
+    }
+    if not args.no_cpu_baseline:
+        import oracle
+        t0 = time.perf_counter()
+        done = 0
+        while time.perf_counter() - t0 < args.cpu_sample_s and done < len(queries):
+            oracle.query(g, queries[done], w.k)
+            done += 1
+        el = time.perf_counter() - t0
+        line["cpu_baseline"] = {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
+                                "sample": f"first {done} {name} queries ({el:.1f} s, single-threaded oracle)"}
+    print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,177 @@
+/* kgs.h — C-ABI of the B200-native Central Graph keyword-search hot path (libkgs.so).
+ *
+ * The method is Yang, Agrawal, Jagadish, Tung, Wu, "An Efficient Parallel Keyword Search Engine on
+ * Knowledge Graphs", ICDE 2019.  "P:Lnnn" cites a line of that paper's text; "R<n>" names a
+ * reading of an ambiguous passage listed in DESIGN.md "Readings".
+ *
+ * Problem (Def. 4): given a knowledge graph G (CSR, node weights, keyword -> nodes
+ * inverted index), a query Q of q keyword ids and k, run one BFS instance B_i per keyword from
+ * T_i = nodes containing t_i, level-synchronously and gated by minimum activation levels
+ * (Eqs. 3-5), until at least k Central Nodes (nodes hit by every B_i) are identified;
+ * extract each Central Graph top-down (Thm. V.4, Alg. 3), prune it with level-cover
+ * (P:L454), score it by Eq. 6 and return the k best.
+ *
+ * Conventions for every call:
+ *   - Every entry point returns kgs_status (0 = KGS_OK, < 0 = error) except the void/free/count
+ *     helpers.  Nothing aborts or throws across the ABI; on error, kgs_last_error() returns a
+ *     thread-local message and every output pointer is left NULL/unchanged.
+ *   - Host pointers are only read during the call; the caller keeps ownership.  Device pointers are
+ *     only accepted where a name or flag says so.
+ *   - A kgs_graph is immutable after load and may serve several threads; queries on one graph are
+ *     serialised internally (one workspace per graph in this version).
+ *   - All work is enqueued on the caller's CUDA stream (NULL = legacy default stream); kgs_query
+ *     returns after the results have been copied to host memory (it synchronises that stream).
+ */
+#ifndef KGS_H
+#define KGS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    KGS_OK = 0,
+    KGS_EINVAL = -1,    /* malformed argument (see each call) */
+    KGS_ENOMEM = -2,    /* device or host allocation failed */
+    KGS_ECUDA = -3,     /* a CUDA runtime/launch error (message from kgs_last_error) */
+    KGS_ENCCL = -4,     /* reserved for the multi-GPU layer */
+    KGS_EINTERNAL = -5  /* an internal invariant failed */
+} kgs_status;
+
+#define KGS_MAX_Q 8        /* q <= 8: one 8-byte M row and a uint8 hit mask per node */
+#define KGS_MAX_K 4096     /* top-k selection sorts the winners inside one CTA */
+#define KGS_INF_LEVEL 255  /* "infinity" in the uint8 node-keyword matrix M */
+
+#define KGS_INPUT_DEVICE_PTRS 1  /* kgs_graph_desc arrays are device pointers (copied, not borrowed) */
+
+#define KGS_EXTRACT_EXACT 0    /* Thm. V.4 + "predecessor not yet central" (reading R12, default) */
+#define KGS_EXTRACT_LITERAL 1  /* Thm. V.4 exactly as printed */
+
+#define KGS_STOP_K 0              /* |C| >= k after identification at level d (Thm. V.3) */
+#define KGS_STOP_EXHAUSTED 1      /* the joint frontier became empty (no pending work) */
+#define KGS_STOP_MAX_DEPTH 2      /* level reached params.max_depth (truncated) */
+#define KGS_STOP_EMPTY_KEYWORD 3  /* some T_i is empty: nothing can be central (reading R17) */
+
+/* Graph description for kgs_load_graph (node-weighted graph stored as CSR).
+ *   n_nodes     number of nodes, 0 <= n < 2^31.
+ *   n_arcs      number of CSR entries (a bi-directed KG stores every edge as two arcs, reading R21).
+ *   row_ptr     [n_nodes + 1], row_ptr[0] = 0, non-decreasing, row_ptr[n] = n_arcs.
+ *   col_idx     [n_arcs], 0 <= id < n_nodes.  Out-arcs: B_i expands u -> col_idx (reading R1).
+ *   weight      [n_nodes], normalised node weight w' in [0, 1] (Eq. 2 + min-max).
+ *               Snapped to the 2^-24 grid on load (reading R15) so Eq. 6 sums are exact.
+ *   n_keywords  vocabulary size V >= 1.
+ *   kw_ptr      [V + 1] int64 offsets, kw_nodes[kw_ptr[t] .. kw_ptr[t+1]) = T_t, strictly increasing.
+ *   avg_dist_A  A, the sampled average shortest distance (Table II), > 0.
+ *   symmetric   1: in-arcs == out-arcs (bi-directed KG).  0: the library builds the reverse CSR used
+ *               by extraction (reading R1).
+ *   device      CUDA device ordinal the graph lives on.
+ *   flags       KGS_INPUT_DEVICE_PTRS or 0. */
+typedef struct {
+    int64_t n_nodes, n_arcs;
+    const int64_t *row_ptr;
+    const int32_t *col_idx;
+    const float *weight;
+    int64_t n_keywords;
+    const int64_t *kw_ptr;
+    const int32_t *kw_nodes;
+    double avg_dist_A;
+    int32_t symmetric;
+    int32_t device;
+    int32_t flags;
+} kgs_graph_desc;
+
+typedef struct kgs_graph kgs_graph;   /* opaque: device CSR (+ reverse), weights, index, workspace */
+typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ optional M / centrals) */
+
+/* Per-query parameters (Table III, Eq. 6).
+ *   alpha          in (0, 1), default 0.1 (Eqs. 3-5).
+ *   lambda         >= 0, default 0.2 (Eq. 6).
+ *   max_depth      1..254, default 254 (255 encodes infinity in M).
+ *   block_central  1 (default): a node identified as central no longer expands (Alg. 2 ln 2).
+ *   extract_mode   KGS_EXTRACT_EXACT (default) or KGS_EXTRACT_LITERAL.
+ *   level_cover    1 (default): apply level-cover pruning; 0 returns unpruned Central Graphs.
+ *   want_levels    1: also copy M and the central list back (for parity checks); default 0. */
+typedef struct {
+    double alpha, lambda;
+    int32_t max_depth, block_central, extract_mode, level_cover, want_levels, reserved;
+} kgs_params;
+
+/* One answer (a pruned Central Graph).  Pointers live until kgs_result_free. */
+typedef struct {
+    int32_t central;     /* the Central Node id */
+    int32_t depth;       /* d(C) = max_i h^i_c (Eq. 1, Lemma V.1), before pruning */
+    float score;         /* (float)score_key */
+    double score_key;    /* Eq. 6 in fp64: pow(d, lambda) * sum of w over the pruned graph; smaller is better (R14) */
+    int64_t n_nodes;
+    const int32_t *nodes;  /* ascending node ids */
+    int64_t n_arcs;
+    const int32_t *arcs;   /* [2 * n_arcs] (pred, succ) pairs, lexicographic, unique, union over keywords */
+} kgs_answer;
+
+/* Statistics of one query.  Times are CUDA-event milliseconds of the phases (P:L532 profile). */
+typedef struct {
+    int32_t levels;        /* BFS level at which the search stopped (d when stop_reason == KGS_STOP_K) */
+    int32_t stop_reason;   /* KGS_STOP_* */
+    int64_t n_centrals;    /* |C|: all Central Nodes identified (candidates for top-down) */
+    int64_t count;         /* answers returned = min(k, |C|) */
+    int64_t frontier_total;/* sum over levels of the joint frontier size */
+    int64_t arcs_scanned;  /* out-arcs inspected by expansion (GTEPS numerator) */
+    int64_t overflow;      /* Central Graphs extracted by the large-graph path */
+    int64_t hits;          /* (node, keyword) pairs newly hit by expansion (M entries written) */
+    float ms_search, ms_topdown, ms_total;
+} kgs_stats;
+
+/* Load a graph onto params-independent device state.  Validates the CSR and the index
+ * (KGS_EINVAL: n out of range, row_ptr not monotone / wrong ends, col_idx out of range,
+ * weight not finite or outside [0, 1], kw_ptr malformed, kw_nodes out of range or not strictly
+ * increasing per keyword, A <= 0).  On success *out owns all device memory of the graph. */
+kgs_status kgs_load_graph(const kgs_graph_desc *desc, kgs_graph **out);
+void kgs_free_graph(kgs_graph *g);
+
+void kgs_params_default(kgs_params *p);
+
+/* Answer one query (Alg. 1).
+ *   kw_ids       host array of q distinct keyword ids in [0, n_keywords).
+ *   q            1..KGS_MAX_Q.   k  1..KGS_MAX_K.
+ *   p            NULL = defaults.
+ *   cuda_stream  cudaStream_t to enqueue on (NULL = default stream).
+ * Returns KGS_EINVAL for q/k/params out of range or duplicate / out-of-range keyword ids.  An empty
+ * T_i is not an error: the result has count 0 and stop_reason KGS_STOP_EMPTY_KEYWORD.
+ * On success *out is a new result the caller frees with kgs_result_free. */
+kgs_status kgs_query(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, const kgs_params *p,
+                     void *cuda_stream, kgs_result **out);
+
+/* Device-resident variant for pipelines and benchmarks: kw_ids_dev is a DEVICE array of q keyword ids
+ * (validated on the device: invalid ids give count 0 and stop_reason -1 in the device header).
+ * Enqueues the whole query on the stream and returns without synchronising; the answers stay in the
+ * graph's device workspace until the next query on this graph.  kgs_query_fetch (same stream)
+ * copies them to a host result, synchronising the stream. */
+kgs_status kgs_query_device(kgs_graph *g, const int32_t *kw_ids_dev, int32_t q, int32_t k, const kgs_params *p,
+                            void *cuda_stream);
+kgs_status kgs_query_fetch(kgs_graph *g, void *cuda_stream, kgs_result **out);
+
+/* Result accessors.  kgs_result_count = min(k, |C|); answers are ranked by (score_key asc, central asc). */
+int32_t kgs_result_count(const kgs_result *r);
+kgs_status kgs_result_answer(const kgs_result *r, int32_t i, kgs_answer *a);
+/* M (n * q bytes, node-major, 255 = infinity) — only if params.want_levels was 1, else KGS_EINVAL. */
+kgs_status kgs_result_levels(const kgs_result *r, uint8_t *M, int64_t cap);
+/* Central list ascending with depths (all of C) — only if want_levels was 1.  *n = |C|. */
+kgs_status kgs_result_centrals(const kgs_result *r, int32_t *ids, uint8_t *depth, double *score_key, int64_t cap,
+                               int64_t *n);
+/* Activation levels a (n bytes, Eqs. 3-5 at the query's alpha) — only if want_levels was 1. */
+kgs_status kgs_result_activation(const kgs_result *r, uint8_t *a, int64_t cap);
+kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s);
+void kgs_result_free(kgs_result *r);
+
+/* Thread-local message describing the last non-OK status of this thread. */
+const char *kgs_last_error(void);
+
+/* Library build/version string. */
+const char *kgs_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* KGS_H */

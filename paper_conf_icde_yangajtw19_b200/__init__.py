@@ -1,0 +1,249 @@
+"""B200-native Central Graph keyword search (Yang et al., ICDE 2019) — Python binding of libkgs.so.
+
+Argument marshalling only: every step of the query path runs in the CUDA kernels behind the C-ABI
+declared in ``include/kgs.h``.  There is no CPU fallback: if ``libkgs.so`` is missing or no CUDA
+device is present, the calls raise.
+
+The names mirror the C-ABI (``kgs_load_graph``, ``kgs_query``, ``kgs_query_device``, ...); the
+``Graph`` / ``Result`` classes are thin owners of the opaque handles.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libkgs.so")
+
+KGS_OK, KGS_EINVAL, KGS_ENOMEM, KGS_ECUDA, KGS_ENCCL, KGS_EINTERNAL = 0, -1, -2, -3, -4, -5
+KGS_MAX_Q, KGS_MAX_K = 8, 4096
+KGS_INPUT_DEVICE_PTRS = 1
+KGS_EXTRACT_EXACT, KGS_EXTRACT_LITERAL = 0, 1
+KGS_STOP_K, KGS_STOP_EXHAUSTED, KGS_STOP_MAX_DEPTH, KGS_STOP_EMPTY_KEYWORD = 0, 1, 2, 3
+
+
+class KgsError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"kgs status {status}: {msg}")
+        self.status = status
+
+
+class kgs_graph_desc(ctypes.Structure):
+    _fields_ = [("n_nodes", ctypes.c_int64), ("n_arcs", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("weight", ctypes.c_void_p),
+                ("n_keywords", ctypes.c_int64), ("kw_ptr", ctypes.c_void_p), ("kw_nodes", ctypes.c_void_p),
+                ("avg_dist_A", ctypes.c_double), ("symmetric", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("flags", ctypes.c_int32)]
+
+
+class kgs_params(ctypes.Structure):
+    _fields_ = [("alpha", ctypes.c_double), ("lambda_", ctypes.c_double), ("max_depth", ctypes.c_int32),
+                ("block_central", ctypes.c_int32), ("extract_mode", ctypes.c_int32),
+                ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+
+
+class kgs_answer(ctypes.Structure):
+    _fields_ = [("central", ctypes.c_int32), ("depth", ctypes.c_int32), ("score", ctypes.c_float),
+                ("score_key", ctypes.c_double), ("n_nodes", ctypes.c_int64),
+                ("nodes", ctypes.POINTER(ctypes.c_int32)), ("n_arcs", ctypes.c_int64),
+                ("arcs", ctypes.POINTER(ctypes.c_int32))]
+
+
+class kgs_stats(ctypes.Structure):
+    _fields_ = [("levels", ctypes.c_int32), ("stop_reason", ctypes.c_int32), ("n_centrals", ctypes.c_int64),
+                ("count", ctypes.c_int64), ("frontier_total", ctypes.c_int64), ("arcs_scanned", ctypes.c_int64),
+                ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
+                ("ms_total", ctypes.c_float)]
+
+
+EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
+            "kgs_query_fetch", "kgs_result_count", "kgs_result_answer", "kgs_result_levels",
+            "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_free",
+            "kgs_last_error", "kgs_version"]
+
+_lib = None
+
+
+def lib():
+    """Load libkgs.so (raises if it was not built: the product has no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built; run `make` (or __graft_entry__.build())")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        L.kgs_load_graph.argtypes = [ctypes.POINTER(kgs_graph_desc), ctypes.POINTER(vp)]
+        L.kgs_load_graph.restype = i32
+        L.kgs_free_graph.argtypes = [vp]
+        L.kgs_free_graph.restype = None
+        L.kgs_params_default.argtypes = [ctypes.POINTER(kgs_params)]
+        L.kgs_params_default.restype = None
+        L.kgs_query.argtypes = [vp, vp, i32, i32, ctypes.POINTER(kgs_params), vp, ctypes.POINTER(vp)]
+        L.kgs_query.restype = i32
+        L.kgs_query_device.argtypes = [vp, vp, i32, i32, ctypes.POINTER(kgs_params), vp]
+        L.kgs_query_device.restype = i32
+        L.kgs_query_fetch.argtypes = [vp, vp, ctypes.POINTER(vp)]
+        L.kgs_query_fetch.restype = i32
+        L.kgs_result_count.argtypes = [vp]
+        L.kgs_result_count.restype = i32
+        L.kgs_result_answer.argtypes = [vp, i32, ctypes.POINTER(kgs_answer)]
+        L.kgs_result_answer.restype = i32
+        L.kgs_result_levels.argtypes = [vp, vp, i64]
+        L.kgs_result_levels.restype = i32
+        L.kgs_result_activation.argtypes = [vp, vp, i64]
+        L.kgs_result_activation.restype = i32
+        L.kgs_result_centrals.argtypes = [vp, vp, vp, vp, i64, ctypes.POINTER(i64)]
+        L.kgs_result_centrals.restype = i32
+        L.kgs_result_stats.argtypes = [vp, ctypes.POINTER(kgs_stats)]
+        L.kgs_result_stats.restype = i32
+        L.kgs_result_free.argtypes = [vp]
+        L.kgs_result_free.restype = None
+        L.kgs_last_error.argtypes = []
+        L.kgs_last_error.restype = ctypes.c_char_p
+        L.kgs_version.argtypes = []
+        L.kgs_version.restype = ctypes.c_char_p
+        _lib = L
+    return _lib
+
+
+def _check(st: int):
+    if st != KGS_OK:
+        raise KgsError(st, lib().kgs_last_error().decode())
+
+
+def kgs_params_default() -> kgs_params:
+    p = kgs_params()
+    lib().kgs_params_default(ctypes.byref(p))
+    return p
+
+
+def make_params(alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=KGS_EXTRACT_EXACT,
+                level_cover=1, want_levels=0) -> kgs_params:
+    p = kgs_params_default()
+    p.alpha, p.lambda_, p.max_depth = float(alpha), float(lam), int(max_depth)
+    p.block_central, p.extract_mode = int(block_central), int(extract_mode)
+    p.level_cover, p.want_levels = int(level_cover), int(want_levels)
+    return p
+
+
+class Graph:
+    """Owner of a kgs_graph handle (device CSR, weights, keyword index, query workspace)."""
+
+    def __init__(self, handle, n, n_keywords):
+        self.handle = handle
+        self.n = n
+        self.n_keywords = n_keywords
+
+    def close(self):
+        if self.handle:
+            lib().kgs_free_graph(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def kgs_load_graph(g, device: int = 0) -> Graph:
+    """Load a graph given as host numpy arrays (attributes row_ptr, col_idx, weight, kw_ptr, kw_nodes,
+    A, symmetric — e.g. a synth.Graph)."""
+    rp = np.ascontiguousarray(g.row_ptr, np.int64)
+    ci = np.ascontiguousarray(g.col_idx, np.int32)
+    w = np.ascontiguousarray(g.weight, np.float32)
+    kp = np.ascontiguousarray(g.kw_ptr, np.int64)
+    kn = np.ascontiguousarray(g.kw_nodes, np.int32)
+    d = kgs_graph_desc(rp.shape[0] - 1, ci.shape[0], rp.ctypes.data, ci.ctypes.data, w.ctypes.data,
+                       kp.shape[0] - 1, kp.ctypes.data, kn.ctypes.data if kn.size else None, float(g.A),
+                       1 if getattr(g, "symmetric", True) else 0, int(device), 0)
+    h = ctypes.c_void_p()
+    _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
+    return Graph(h, rp.shape[0] - 1, kp.shape[0] - 1)
+
+
+@dataclass
+class Answer:
+    central: int
+    depth: int
+    score: float
+    score_key: float
+    nodes: np.ndarray
+    arcs: np.ndarray   # [n_arcs, 2]
+
+
+@dataclass
+class Result:
+    answers: list
+    stats: dict
+    M: np.ndarray | None = None
+    a: np.ndarray | None = None
+    centrals: np.ndarray | None = None
+    central_depth: np.ndarray | None = None
+    central_key: np.ndarray | None = None
+
+
+def _read_result(h, n, q, want_levels) -> Result:
+    L = lib()
+    try:
+        cnt = L.kgs_result_count(h)
+        answers = []
+        a = kgs_answer()
+        for i in range(cnt):
+            _check(L.kgs_result_answer(h, i, ctypes.byref(a)))
+            nodes = np.ctypeslib.as_array(a.nodes, shape=(a.n_nodes,)).copy() if a.n_nodes else np.zeros(0, np.int32)
+            arcs = (np.ctypeslib.as_array(a.arcs, shape=(2 * a.n_arcs,)).copy().reshape(-1, 2) if a.n_arcs
+                    else np.zeros((0, 2), np.int32))
+            answers.append(Answer(a.central, a.depth, a.score, a.score_key, nodes, arcs))
+        st = kgs_stats()
+        _check(L.kgs_result_stats(h, ctypes.byref(st)))
+        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
+        res = Result(answers, stats)
+        if want_levels:
+            M = np.empty(n * q, np.uint8)
+            _check(L.kgs_result_levels(h, M.ctypes.data, M.size))
+            act = np.empty(n, np.uint8)
+            _check(L.kgs_result_activation(h, act.ctypes.data, act.size))
+            nc = ctypes.c_int64()
+            cap = n
+            ids = np.empty(cap, np.int32)
+            dep = np.empty(cap, np.uint8)
+            key = np.empty(cap, np.float64)
+            _check(L.kgs_result_centrals(h, ids.ctypes.data, dep.ctypes.data, key.ctypes.data, cap, ctypes.byref(nc)))
+            k = nc.value
+            res.M, res.a = M.reshape(n, q), act
+            res.centrals, res.central_depth, res.central_key = ids[:k].copy(), dep[:k].copy(), key[:k].copy()
+        return res
+    finally:
+        L.kgs_result_free(h)
+
+
+def kgs_query(graph: Graph, kw_ids, k: int, params: kgs_params | None = None, stream: int = 0) -> Result:
+    """One query with host keyword ids; answers copied back to the host (kgs_query)."""
+    kw = np.ascontiguousarray(np.asarray(kw_ids, dtype=np.int32))
+    p = params if params is not None else kgs_params_default()
+    h = ctypes.c_void_p()
+    _check(lib().kgs_query(graph.handle, kw.ctypes.data, int(kw.shape[0]), int(k), ctypes.byref(p),
+                           ctypes.c_void_p(stream), ctypes.byref(h)))
+    return _read_result(h, graph.n, int(kw.shape[0]), p.want_levels)
+
+
+def kgs_query_device(graph: Graph, kw_ids_dev_ptr: int, q: int, k: int, params: kgs_params | None = None,
+                     stream: int = 0) -> None:
+    """Enqueue a query whose keyword ids are already in device memory; no synchronisation."""
+    p = params if params is not None else kgs_params_default()
+    _check(lib().kgs_query_device(graph.handle, ctypes.c_void_p(kw_ids_dev_ptr), int(q), int(k), ctypes.byref(p),
+                                  ctypes.c_void_p(stream)))
+
+
+def kgs_query_fetch(graph: Graph, q: int, want_levels: int = 0, stream: int = 0) -> Result:
+    h = ctypes.c_void_p()
+    _check(lib().kgs_query_fetch(graph.handle, ctypes.c_void_p(stream), ctypes.byref(h)))
+    return _read_result(h, graph.n, q, want_levels)
+
+
+def kgs_version() -> str:
+    return lib().kgs_version().decode()

@@ -1,0 +1,132 @@
+// kgs_internal.h — device data layout and kernel entry points shared by the libkgs translation units.
+// Product code (CUDA path).  Shares nothing with oracle/.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/kgs.h"
+
+namespace kgs {
+
+constexpr int kMaxQ = KGS_MAX_Q;
+constexpr int kWarp = 32;
+
+// Degree classes for the expansion's load balance: light nodes are expanded by
+// warp batches, heavy ones by a CTA each, huge ones by the whole grid.
+constexpr int64_t kHeavyDeg = 2048;
+constexpr int64_t kHugeDeg = 65536;
+enum : uint8_t { CLS_LIGHT = 0, CLS_HEAVY = 1, CLS_HUGE = 2 };
+
+// Per-warp shared-memory capacity of the Central Graph extractor.
+constexpr int kExtNodes = 256;
+constexpr int kExtArcs = 512;
+constexpr int kExtHash = 512;
+constexpr int kExtWarps = 4;  // warps per CTA in the extractor
+// Per-CTA global-memory arena of the large-graph extractor.
+constexpr int kBigNodes = 1 << 16;
+constexpr int kBigArcs = 1 << 18;
+constexpr int kBigHash = 1 << 17;
+constexpr int kBigCtas = 64;
+
+// Device control block, zeroed at the start of every query.
+struct Ctl {
+    uint32_t qcount[3][256];       // ring slot counts per degree class
+    uint32_t work[256];            // dynamic work counters per level (light batches)
+    uint32_t n_central;
+    uint32_t n_touched;
+    uint32_t n_overflow;
+    uint32_t work_ext;
+    int32_t fatal;                 // non-zero: an arena overflowed beyond the large path
+    uint32_t pad0;
+    int32_t levels;
+    int32_t stop_reason;
+    int32_t empty_keyword;
+    int32_t pad;
+    unsigned long long frontier_total;
+    unsigned long long arcs_scanned;
+    unsigned long long hits;       // new (node, keyword) hits (M entries written)
+    uint32_t hist[12][256];        // radix-select histograms (one per digit)
+    unsigned long long thr_hi;     // selected threshold (composite key)
+    unsigned long long thr_lo;
+    uint32_t sel_count;
+    uint32_t pad2;
+    unsigned long long arena_used[2];  // emitted nodes / arcs
+};
+
+struct DevGraph {
+    int64_t n, m;
+    const int64_t *row_ptr;
+    const int32_t *col_idx;
+    const int64_t *in_ptr;
+    const int32_t *in_idx;
+    const float *weight;
+    const uint8_t *cls;       // degree class per node
+    int64_t n_kw;
+    const int64_t *kw_ptr;
+    const int32_t *kw_nodes;
+};
+
+// Per-query device state (all sized for n at load time).
+struct DevWork {
+    uint8_t *act;       // [n] activation levels at act_alpha (Eqs. 3-5)
+    uint16_t *st;       // [n] low byte: hit mask hm (bit i <=> M[v][i] finite); high byte: gate (0 for K, else a)
+    uint32_t *nm;       // [ceil(n/4)] new hits of the current level, one byte per node
+    uint8_t *M;         // [n*8] hitting levels, node-major, valid where the hm bit is set
+    int32_t *ring[3];   // per class: [R][cap_c] frontier queues, slot = level % R
+    int64_t cap[3];     // per class capacity (light = n, heavy/huge = number of such nodes)
+    uint32_t *fbits;    // [R][W] frontier membership bitmaps (dedup of pushes)
+    int64_t W;          // words per bitmap
+    int R;              // ring size = amax + 2
+    int32_t *touched;   // [n] nodes whose hm became non-zero (sparse reset of the next query)
+    int32_t *centrals;  // [n] central ids in identification order
+    uint8_t *cdepth;    // [n] depth per central
+    double *ckey;       // [n] Eq. 6 key per central
+    int32_t *overflow;  // [n] centrals whose graph exceeds the shared-memory extractor
+    uint8_t *cflag;     // [n] 1 = overflowed the shared-memory extractor
+    int32_t *sel;       // [KGS_MAX_K] ranked winners (index into centrals)
+    int32_t *kw_dev;    // [KGS_MAX_Q] query keyword ids
+    double *dpow;       // [256] pow(d, lambda) per depth (host libm)
+    Ctl *ctl;
+    const Ctl *prev;    // previous query's control block (sparse reset), nullptr -> full reset
+    // emitted answers
+    int32_t *ans_hdr;   // [KGS_MAX_K][4]: central, depth, n_nodes, n_arcs
+    double *ans_key;    // [KGS_MAX_K]
+    long long *ans_off; // [KGS_MAX_K][2]: offsets into the node / arc arenas
+    int32_t *arena_nodes;
+    int32_t *arena_arcs;  // pairs
+    long long arena_nodes_cap, arena_arcs_cap;
+    // large-graph extractor arenas
+    void *big_ws;
+    size_t big_bytes, big_bytes_emit;
+    int big_hcap, big_ncap, big_acap, big_ctas;
+};
+
+struct QueryArgs {
+    DevGraph g;
+    DevWork w;
+    int q;
+    int k;
+    int max_depth;
+    int block_central;
+    int extract_mode;
+    int level_cover;
+    int full_reset;     // 1: reset st for all nodes; 0: only the previous query's touched nodes (w.prev)
+    int prev_R;
+};
+
+// ---- launchers (return cudaError_t) ----
+cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha, uint8_t *act, uint32_t *amax,
+                              cudaStream_t s);
+cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s);
+cudaError_t launch_snap_weights(float *w, int64_t n, cudaStream_t s);
+cudaError_t launch_search(const QueryArgs &a, int grid, int block, cudaStream_t s);
+int search_max_grid(int device, int block);
+cudaError_t launch_extract(const QueryArgs &a, int grid, cudaStream_t s);
+cudaError_t launch_select(const QueryArgs &a, int grid, cudaStream_t s);
+int select_max_grid(int device);
+cudaError_t launch_emit(const QueryArgs &a, int grid, cudaStream_t s);
+size_t big_arena_bytes(int hcap, int ncap, int acap, bool with_sort);
+cudaError_t launch_levels_out(const QueryArgs &a, uint8_t *out, cudaStream_t s);
+cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s);
+
+}  // namespace kgs

@@ -1,0 +1,368 @@
+// search.cu — bottom-up search of the Central Graph method on sm_100a (product CUDA path).
+//
+//   k_activation   Eqs. 3-5: w, alpha, A -> uint8 activation level a, cached per alpha.
+//   k_search       Alg. 1 ln 1-7 + Alg. 2 (L244-284) as ONE persistent cooperative kernel:
+//                  reset -> initialise M / sources (L254) -> per level { merge new hits + identify
+//                  central nodes (L262-266, Lemma V.1) -> termination (Def. 4, Thm. V.3) -> expansion
+//                  (Alg. 2, gated by a, L210) } with two grid barriers per level and no host round trip.
+//
+// Data layout:
+//   st[v]   uint16: low byte = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of the level),
+//           high byte = gate (0 if v contains a query keyword, else a_v).  One 2-byte load per inspected arc.
+//   nm[v]   uint8 (packed in 32-bit words for atomicOr): bits newly hit during the current level.
+//   M[v*8+i] uint8 hitting level, written once per (v, i) by the thread that set the bit; never reset.
+//   Frontier: three degree-class rings (light / heavy / huge) of R = amax+2 level slots, deduplicated by
+//   a bitmap per slot.  A node is re-queued exactly at the level where it can make progress again:
+//   a_v if it is not yet active (Alg. 2 ln 5-7), gate(n)-1 if a neighbour n is still gated (ln 18-19).
+//
+// Snapshot semantics (reading R10): expansion at level l reads hm as of the start of the level; new hits
+// accumulate in nm and are merged in the next merge phase, so the result equals the sequential Alg. 2
+// (Thm. V.2).  All writes are idempotent (bits OR-ed, level l+1 written once).
+#include <cooperative_groups.h>
+
+#include "kgs_internal.h"
+
+namespace cg = cooperative_groups;
+
+namespace kgs {
+
+// ------------------------------------------------------------------------------------------ activation
+__global__ void k_activation(const float *__restrict__ w, int64_t n, double A, double alpha,
+                             uint8_t *__restrict__ act, uint32_t *amax) {
+    uint32_t local = 0;
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const double wv = (double)w[v];
+        double x;
+        if (wv < alpha) {            // Eq. 4 reward, Eq. 5 first case
+            const double reward = __ddiv_rn(__dmul_rn(A, __dsub_rn(alpha, wv)), alpha);
+            x = __dsub_rn(A, reward);
+        } else if (wv == alpha) {    // Eq. 5 second case
+            x = A;
+        } else {                     // Eq. 3 penalty, Eq. 5 third case
+            const double penalty = __ddiv_rn(__dmul_rn(A, __dsub_rn(wv, alpha)), __dsub_rn(1.0, alpha));
+            x = __dadd_rn(A, penalty);
+        }
+        double r = floor(__dadd_rn(x, 0.5));   // nearest integer, halves up (R4)
+        r = r < 0.0 ? 0.0 : (r > 254.0 ? 254.0 : r);
+        const uint8_t a = (uint8_t)r;
+        act[v] = a;
+        local = local > a ? local : a;
+    }
+    local = __reduce_max_sync(0xffffffffu, local);
+    if ((threadIdx.x & 31) == 0) atomicMax(amax, local);
+}
+
+cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha, uint8_t *act, uint32_t *amax,
+                              cudaStream_t s) {
+    cudaMemsetAsync(amax, 0, sizeof(uint32_t), s);
+    if (n > 0) {
+        int grid = (int)((n + 255) / 256);
+        if (grid > 148 * 16) grid = 148 * 16;
+        k_activation<<<grid, 256, 0, s>>>(w, n, A, alpha, act, amax);
+    }
+    return cudaGetLastError();
+}
+
+__global__ void k_degree_class(const int64_t *__restrict__ rp, int64_t n, uint8_t *__restrict__ cls) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t d = rp[v + 1] - rp[v];
+        cls[v] = d > kHugeDeg ? CLS_HUGE : (d > kHeavyDeg ? CLS_HEAVY : CLS_LIGHT);
+    }
+}
+cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s) {
+    if (n > 0) {
+        int grid = (int)((n + 255) / 256);
+        if (grid > 148 * 16) grid = 148 * 16;
+        k_degree_class<<<grid, 256, 0, s>>>(row_ptr, n, cls);
+    }
+    return cudaGetLastError();
+}
+
+// Reading R15: weights on the 2^-24 grid make every fp64 sum of Eq. 6 exact and order-independent.
+__global__ void k_snap(float *w, int64_t n) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const double x = (double)w[v] * 16777216.0;
+        w[v] = (float)(floor(x + 0.5) * (1.0 / 16777216.0));
+    }
+}
+cudaError_t launch_snap_weights(float *w, int64_t n, cudaStream_t s) {
+    if (n > 0) {
+        int grid = (int)((n + 255) / 256);
+        if (grid > 148 * 16) grid = 148 * 16;
+        k_snap<<<grid, 256, 0, s>>>(w, n);
+    }
+    return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------ helpers
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned r;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+    return r;
+}
+
+// Append to a list with one atomic per group of converged lanes sharing the same counter.
+__device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
+    const unsigned mask = __activemask();
+    const unsigned peers = __match_any_sync(mask, key);
+    const int leader = __ffs(peers) - 1;
+    const int rank = __popc(peers & lanemask_lt());
+    uint32_t base = 0;
+    if ((int)lane_id() == leader) base = atomicAdd(counter, (uint32_t)__popc(peers));
+    base = __shfl_sync(peers, base, leader);
+    return base + rank;
+}
+
+struct SearchCtx {
+    const QueryArgs &a;
+    int R;
+    uint32_t full;
+};
+
+// Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1 for level L).
+__device__ __forceinline__ void push(const QueryArgs &a, int R, int32_t v, int L) {
+    const int s = L % R;
+    uint32_t *word = a.w.fbits + (int64_t)s * a.w.W + (v >> 5);
+    const uint32_t bit = 1u << (v & 31);
+    if (__ldcg(word) & bit) return;
+    if (atomicOr(word, bit) & bit) return;
+    const int c = a.g.cls[v];
+    const uint32_t pos = agg_slot(&a.w.ctl->qcount[c][s], (unsigned)((c << 8) | s));
+    a.w.ring[c][(int64_t)s * a.w.cap[c] + pos] = v;
+}
+
+// One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask).
+__device__ __forceinline__ void visit_arc(const QueryArgs &a, int R, int l, int32_t v, uint32_t hmv, int32_t x,
+                                          unsigned long long &hits) {
+    const uint32_t sx = __ldcg(a.w.st + x);
+    const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
+    if (!bits) return;
+    const uint32_t gate = sx >> 8;
+    if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
+        const uint32_t sh = (uint32_t)(x & 3) << 3;
+        uint32_t *nw = a.w.nm + (x >> 2);
+        const uint32_t cur = (__ldcg(nw) >> sh) & 0xFFu;
+        if (!(bits & ~cur)) return;
+        const uint32_t old = (atomicOr(nw, bits << sh) >> sh) & 0xFFu;
+        const uint32_t nb = bits & ~old;
+        if (nb) {
+            hits += __popc(nb);
+            uint8_t *row = a.w.M + (int64_t)x * 8;
+            const uint8_t lv = (uint8_t)(l + 1);
+#pragma unroll
+            for (int i = 0; i < kMaxQ; ++i)
+                if (nb & (1u << i)) row[i] = lv;          // ln 21: m_xi <- l+1
+            if (old == 0) push(a, R, x, l + 1);           // ln 22: FIdentifier[x] <- 1 (first new bit)
+        }
+    } else {
+        push(a, R, v, (int)gate - 1);                     // ln 19: v must retry when x opens
+    }
+}
+
+// Alg. 2 ln 2-7 for node v at level l: returns its expansion mask (0 = does not expand now).
+__device__ __forceinline__ uint32_t prepare(const QueryArgs &a, int R, int l, uint32_t full, int32_t v, bool leader) {
+    const uint32_t hm = __ldcg(a.w.st + v) & 0xFFu;
+    if (a.block_central && hm == full) return 0;          // ln 2-3: central nodes do not expand
+    const int av = a.w.act[v];
+    if (av > l) {                                          // ln 5-7: not yet active
+        if (leader) push(a, R, v, av);
+        return 0;
+    }
+    return hm;                                             // ln 8-11: every hit instance has m <= l
+}
+
+// ------------------------------------------------------------------------------------------ search
+__global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
+    const int64_t n = a.g.n;
+    const int R = a.w.R;
+    const int amax = R - 2;
+    const uint32_t full = (1u << a.q) - 1u;
+    Ctl *ctl = a.w.ctl;
+    uint8_t *st8 = reinterpret_cast<uint8_t *>(a.w.st);
+    uint8_t *nm8 = reinterpret_cast<uint8_t *>(a.w.nm);
+
+    // ---- reset the state the previous query left behind
+    if (a.full_reset) {
+        for (int64_t v = gtid; v < n; v += gsz) a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
+        for (int64_t v = gtid; v < (n + 3) / 4; v += gsz) a.w.nm[v] = 0u;
+        for (int64_t j = gtid; j < (int64_t)R * a.w.W; j += gsz) a.w.fbits[j] = 0u;
+    } else {
+        const Ctl *pv = a.w.prev;
+        const int64_t pt = (int64_t)pv->n_touched;
+        for (int64_t j = gtid; j < pt; j += gsz) {
+            const int32_t v = a.w.touched[j];
+            a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
+        }
+        for (int c = 0; c < 3; ++c)
+            for (int s = 0; s < a.prev_R; ++s) {
+                const uint32_t cnt = pv->qcount[c][s];
+                for (int64_t j = gtid; j < (int64_t)cnt; j += gsz) {
+                    const int32_t v = a.w.ring[c][(int64_t)s * a.w.cap[c] + j];
+                    a.w.fbits[(int64_t)s * a.w.W + (v >> 5)] = 0u;
+                }
+            }
+    }
+    // ---- initialisation: M = 0 on T_i, keyword nodes ungated, F_0 = K
+    bool empty = false;
+    for (int i = 0; i < a.q; ++i) {
+        const int32_t t = a.w.kw_dev[i];
+        if (a.g.kw_ptr[t + 1] == a.g.kw_ptr[t]) empty = true;
+    }
+    grid.sync();
+    for (int i = 0; i < a.q; ++i) {
+        const int32_t t = a.w.kw_dev[i];
+        const int64_t b = a.g.kw_ptr[t], e = a.g.kw_ptr[t + 1];
+        for (int64_t j = b + gtid; j < e; j += gsz) {
+            const int32_t v = a.g.kw_nodes[j];
+            a.w.M[(int64_t)v * 8 + i] = 0;
+            st8[2 * (int64_t)v + 1] = 0;                                  // keyword node: no gate (L210)
+            atomicOr(a.w.nm + (v >> 2), (1u << i) << ((v & 3) * 8));      // hit in B_i at level 0
+            push(a, R, v, 0);
+        }
+    }
+    grid.sync();
+
+    unsigned long long my_arcs = 0, my_hits = 0;
+    for (int l = 0;; ++l) {
+        // ---- enqueue frontiers: anything pending at this or a later level?
+        uint32_t pend = 0;
+        const int top = l > amax ? l : amax;
+        for (int L = l; L <= top; ++L) {
+            const int s = L % R;
+            pend += __ldcg(&ctl->qcount[0][s]) + __ldcg(&ctl->qcount[1][s]) + __ldcg(&ctl->qcount[2][s]);
+        }
+        if (pend == 0) {
+            if (gtid == 0) { ctl->stop_reason = empty ? KGS_STOP_EMPTY_KEYWORD : KGS_STOP_EXHAUSTED; ctl->levels = l; }
+            break;
+        }
+        const int s = l % R;
+        const uint32_t c0 = __ldcg(&ctl->qcount[0][s]), c1 = __ldcg(&ctl->qcount[1][s]),
+                       c2 = __ldcg(&ctl->qcount[2][s]);
+        const int64_t total = (int64_t)c0 + c1 + c2;
+        // ---- merge new hits into hm and identify central nodes (only frontiers can change, L262)
+        for (int64_t j = gtid; j < total; j += gsz) {
+            int32_t v;
+            if (j < c0) v = a.w.ring[0][(int64_t)s * a.w.cap[0] + j];
+            else if (j < (int64_t)c0 + c1) v = a.w.ring[1][(int64_t)s * a.w.cap[1] + (j - c0)];
+            else v = a.w.ring[2][(int64_t)s * a.w.cap[2] + (j - c0 - c1)];
+            a.w.fbits[(int64_t)s * a.w.W + (v >> 5)] = 0u;
+            const uint32_t b = nm8[v];
+            if (b) {
+                nm8[v] = 0;
+                const uint32_t old = st8[2 * (int64_t)v];
+                const uint32_t nw = old | b;
+                st8[2 * (int64_t)v] = (uint8_t)nw;
+                if (old == 0) a.w.touched[agg_slot(&ctl->n_touched, 0u)] = v;
+                if (nw == full && old != full) {                            // Lemma V.1: depth = l
+                    const uint32_t ci = agg_slot(&ctl->n_central, 1u);
+                    a.w.centrals[ci] = v;
+                    a.w.cdepth[ci] = (uint8_t)l;
+                }
+            }
+        }
+        if (gtid == 0) ctl->frontier_total += (unsigned long long)total;
+        grid.sync();
+        if (gtid == 0 && l > 0) {
+            const int sp = (l - 1) % R;
+            ctl->qcount[0][sp] = 0; ctl->qcount[1][sp] = 0; ctl->qcount[2][sp] = 0;
+        }
+        // ---- termination (Def. 4 / Thm. V.3; reading R9: no expansion at d)
+        if (empty) {   // some T_i is empty: M holds the initialisation, nothing can be central (R17)
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_EMPTY_KEYWORD; ctl->levels = 0; ctl->empty_keyword = 1; }
+            break;
+        }
+        const uint32_t nc = __ldcg(&ctl->n_central);
+        if (nc >= (uint32_t)a.k) {
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_K; ctl->levels = l; }
+            break;
+        }
+        if (l == a.max_depth) {
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_MAX_DEPTH; ctl->levels = l; }
+            break;
+        }
+        // ---- expansion (Alg. 2)
+        // huge nodes: the whole grid strides over one node's arcs
+        for (uint32_t j = 0; j < c2; ++j) {
+            const int32_t v = a.w.ring[2][(int64_t)s * a.w.cap[2] + j];
+            const uint32_t hm = prepare(a, R, l, full, v, gtid == 0);
+            if (!hm) continue;
+            const int64_t b = a.g.row_ptr[v], e = a.g.row_ptr[v + 1];
+            if (gtid == 0) my_arcs += (unsigned long long)(e - b);
+            for (int64_t p = b + gtid; p < e; p += gsz) visit_arc(a, R, l, v, hm, __ldcs(a.g.col_idx + p), my_hits);
+        }
+        // heavy nodes: one CTA per node
+        for (uint32_t j = blockIdx.x; j < c1; j += gridDim.x) {
+            const int32_t v = a.w.ring[1][(int64_t)s * a.w.cap[1] + j];
+            const uint32_t hm = prepare(a, R, l, full, v, threadIdx.x == 0);
+            if (!hm) continue;
+            const int64_t b = a.g.row_ptr[v], e = a.g.row_ptr[v + 1];
+            if (threadIdx.x == 0) my_arcs += (unsigned long long)(e - b);
+            for (int64_t p = b + threadIdx.x; p < e; p += blockDim.x) visit_arc(a, R, l, v, hm, __ldcs(a.g.col_idx + p), my_hits);
+        }
+        // light nodes: dynamic batches of 32 frontier nodes per warp, arcs balanced across the lanes
+        const unsigned lane = lane_id();
+        for (;;) {
+            uint32_t base = 0;
+            if (lane == 0) base = atomicAdd(&ctl->work[l], 32u);
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (base >= c0) break;
+            const uint32_t idx = base + lane;
+            int32_t v = -1;
+            uint32_t hm = 0;
+            int64_t start = 0;
+            int deg = 0;
+            if (idx < c0) {
+                v = a.w.ring[0][(int64_t)s * a.w.cap[0] + idx];
+                hm = prepare(a, R, l, full, v, true);
+                if (hm) {
+                    start = a.g.row_ptr[v];
+                    deg = (int)(a.g.row_ptr[v + 1] - start);
+                }
+            }
+            int incl = deg;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(0xffffffffu, incl, o);
+                if ((int)lane >= o) incl += t;
+            }
+            const int tot = __shfl_sync(0xffffffffu, incl, 31);
+            if (lane == 0) my_arcs += (unsigned long long)tot;
+            const int excl = incl - deg;
+            for (int e0 = 0; e0 < tot; e0 += 32) {
+                const int e = e0 + (int)lane;
+                int pos = 0;
+#pragma unroll
+                for (int b = 16; b > 0; b >>= 1) {
+                    const int val = __shfl_sync(0xffffffffu, incl, pos + b - 1);
+                    if (val <= e) pos += b;
+                }
+                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
+                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
+                const uint32_t hm_o = __shfl_sync(0xffffffffu, hm, pos);
+                const int32_t v_o = __shfl_sync(0xffffffffu, v, pos);
+                if (e < tot) visit_arc(a, R, l, v_o, hm_o, __ldcs(a.g.col_idx + st_o + (e - ex_o)), my_hits);
+            }
+        }
+        grid.sync();
+    }
+    if (my_arcs) atomicAdd(&ctl->arcs_scanned, my_arcs);
+    if (my_hits) atomicAdd(&ctl->hits, my_hits);
+}
+
+int search_max_grid(int device, int block) {
+    int per_sm = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_search, block, 0);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    return per_sm * sms;
+}
+
+cudaError_t launch_search(const QueryArgs &a, int grid, int block, cudaStream_t s) {
+    void *args[] = {(void *)&a};
+    return cudaLaunchCooperativeKernel((const void *)k_search, dim3(grid), dim3(block), args, 0, s);
+}
+
+}  // namespace kgs

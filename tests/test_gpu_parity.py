@@ -1,0 +1,154 @@
+"""CUDA path (through the C-ABI) vs the oracle, element by element on the same seeded inputs.
+
+Bit-exact: activation levels a, the hitting-level matrix M, the central set with depths, every
+central's Eq. 6 key, the ranked top-k ids, the answer subgraphs, stop level / reason.  fp32 scores
+must agree within 1e-5 relative (BASELINE.json north_star); they are in fact identical because the
+fp64 keys are exact (reading R15), and the test checks both.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import refimpl as R
+import synth
+
+pytestmark = pytest.mark.gpu
+
+kgs = pytest.importorskip("paper_conf_icde_yangajtw19_b200")
+
+
+def _gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def compare(G, g, kw, k, *, alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=0,
+            level_cover=1, full=True):
+    o = oracle.query(g, kw, k, alpha=alpha, lam=lam, max_depth=max_depth, block_central=block_central,
+                     extract_mode=extract_mode, level_cover=level_cover)
+    p = kgs.make_params(alpha=alpha, lam=lam, max_depth=max_depth, block_central=block_central,
+                        extract_mode=extract_mode, level_cover=level_cover, want_levels=1 if full else 0)
+    r = kgs.kgs_query(G, kw, k, p)
+    assert o.status == 0
+    ctx = f"kw={list(kw)} k={k} alpha={alpha} lam={lam} md={max_depth} blk={block_central} ext={extract_mode} lc={level_cover}"
+    if full:
+        assert (r.a == o.a).all(), ctx
+        bad = np.argwhere(r.M != o.M)
+        assert bad.size == 0, f"{ctx}: M differs at {bad[:5].tolist()} gpu={r.M[tuple(bad[0])]} ora={o.M[tuple(bad[0])]}"
+        assert r.centrals.tolist() == o.centrals.tolist(), ctx
+        assert r.central_depth.tolist() == o.central_depth.tolist(), ctx
+        assert r.central_key.tolist() == o.central_key.tolist(), ctx
+    assert r.stats["stop_reason"] == o.stop_reason, ctx
+    if o.stop_reason != oracle.STOP_EMPTY_KEYWORD:
+        assert r.stats["levels"] == o.levels, ctx
+    assert r.stats["n_centrals"] == len(o.centrals), ctx
+    assert len(r.answers) == len(o.answers), ctx
+    for ra, oa in zip(r.answers, o.answers):
+        assert ra.central == oa.central and ra.depth == oa.depth, ctx
+        assert ra.score_key == oa.key, ctx
+        assert ra.score == oa.score and abs(ra.score - oa.score) <= 1e-5 * max(abs(oa.score), 1e-30), ctx
+        assert ra.nodes.tolist() == oa.nodes.tolist(), ctx
+        assert ra.arcs.tolist() == oa.arcs.tolist(), ctx
+    return r, o
+
+
+def test_golden_examples():
+    _gpu()
+    d = R.load_golden("fig2_examples_1_3.json")
+    g = R.golden_graph(d)
+    G = kgs.kgs_load_graph(g)
+    for c in d["cases"]:
+        for lc in (0, 1):
+            r, _ = compare(G, g, d["query"], c["k"], alpha=d["alpha"], block_central=c["block_central"], level_cover=lc)
+            assert r.M.tolist() == c["M"]
+    for name in ("fig4_example_4.json", "fig5_example_5.json"):
+        d = R.load_golden(name)
+        g = R.golden_graph(d)
+        G = kgs.kgs_load_graph(g)
+        r, _ = compare(G, g, d["query"], d["k"], alpha=d["alpha"], lam=d["lambda"])
+        assert r.M.tolist() == d["M"]
+        assert r.answers[0].nodes.tolist() == d["answer"]["nodes"]
+    d = R.load_golden("fig4_example_4.json")
+    assert r is not None
+
+
+def test_random_small_graphs_all_modes():
+    _gpu()
+    rng = np.random.default_rng(2024)
+    for case in range(160):
+        n = int(rng.integers(4, 70))
+        directed = bool(rng.random() < 0.4)
+        q = int(rng.integers(1, 9))
+        g = R.random_graph(rng, n, float(rng.uniform(0.03, 0.3)), directed, q, kw_size=(1, 5),
+                           wmax=float(rng.choice([0.0, 0.2, 1.0])))
+        G = kgs.kgs_load_graph(g)
+        kw = list(range(q))
+        for _ in range(3):
+            compare(G, g, kw, int(rng.choice([1, 2, 5, 40])), alpha=float(rng.choice([0.05, 0.1, 0.4])),
+                    lam=float(rng.choice([0.0, 0.2, 1.0])), max_depth=int(rng.choice([1, 3, 254])),
+                    block_central=int(rng.integers(0, 2)), extract_mode=int(rng.integers(0, 2)),
+                    level_cover=int(rng.integers(0, 2)))
+        G.close()
+
+
+def test_c1_all_queries():
+    """Config C1 (BASELINE.json configs[0]): 100 three-keyword queries, top-5."""
+    _gpu()
+    w = synth.make_workload("C1")
+    G = kgs.kgs_load_graph(w.graph)
+    for kw in w.queries:
+        compare(G, w.graph, kw, w.k)
+
+
+def test_c2_queries_and_state_reuse():
+    """Config C2 (1M nodes / 8M edges, 2-4 keywords, top-20): sampled queries; the workspace is reused
+    across queries (sparse reset) and alpha changes in between, so stale state would show."""
+    _gpu()
+    w = synth.make_workload("C2")
+    G = kgs.kgs_load_graph(w.graph)
+    qs = w.queries[::10]
+    for j, kw in enumerate(qs):
+        compare(G, w.graph, kw, w.k, alpha=0.4 if j % 7 == 3 else 0.1, full=(j % 3 == 0))
+    # determinism (Thm. V.2): same query twice, interleaved with another one
+    r1 = kgs.kgs_query(G, qs[0], w.k)
+    kgs.kgs_query(G, qs[1], w.k)
+    r2 = kgs.kgs_query(G, qs[0], w.k)
+    assert [(a.central, a.score_key) for a in r1.answers] == [(a.central, a.score_key) for a in r2.answers]
+
+
+def test_ragged_and_degenerate():
+    """Empty keyword set, q = 1, k > |C|, a node containing all keywords, max_depth truncation,
+    isolated nodes and a graph whose size is not a multiple of any tile."""
+    _gpu()
+    g = synth.from_edges(7, [(0, 1), (1, 2), (2, 3), (4, 5)], [0.5, 0, 0, 0, 0, 0, 0.25],
+                         [[0, 2], [2], [], [6], [3, 5]], 2.0)
+    G = kgs.kgs_load_graph(g)
+    compare(G, g, [0], 5)
+    compare(G, g, [0, 1], 1)
+    compare(G, g, [0, 2], 3)
+    compare(G, g, [0, 3], 3)
+    compare(G, g, [1, 4], 100)
+    compare(G, g, [0, 4], 100, max_depth=1)
+    with pytest.raises(kgs.KgsError):
+        kgs.kgs_query(G, [0, 0], 1)
+    with pytest.raises(kgs.KgsError):
+        kgs.kgs_query(G, [0], 0)
+    with pytest.raises(kgs.KgsError):
+        kgs.kgs_query(G, [99], 1)
+
+
+def test_device_resident_path():
+    """kgs_query_device (keyword ids already in HBM) + kgs_query_fetch give the same answers."""
+    _gpu()
+    import torch
+    w = synth.make_workload("C1")
+    G = kgs.kgs_load_graph(w.graph)
+    for kw in w.queries[:10]:
+        t = torch.tensor(kw, dtype=torch.int32, device="cuda")
+        s = torch.cuda.current_stream().cuda_stream
+        kgs.kgs_query_device(G, t.data_ptr(), len(kw), w.k, None, s)
+        r = kgs.kgs_query_fetch(G, len(kw), 0, s)
+        o = oracle.query(w.graph, kw, w.k)
+        assert [a.central for a in r.answers] == [a.central for a in o.answers]
+        assert [a.score_key for a in r.answers] == [a.key for a in o.answers]
