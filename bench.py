@@ -128,7 +128,8 @@ def run_reference(args):
     import oracle
     name = "C3" if world == 1 else "C4"
     w, gen_s = build_workload(name, 0, 1)
-    qs = w.queries
+    order = np.random.default_rng(12345).permutation(len(w.queries))
+    qs = [w.queries[i] for i in order]
     for i in range(args.warmup):
         oracle.query(w.graph, qs[i % len(qs)], w.k)
     lat = []
@@ -184,7 +185,10 @@ def main():
     t0 = time.time()
     G = kgs.kgs_load_graph(g, device=dev)
     load_s = time.time() - t0
-    queries = w.queries[rank::world] if world > 1 else w.queries
+    # a fixed permutation so every window of steps mixes all query sizes (the config lists them by q)
+    order = np.random.default_rng(12345).permutation(len(w.queries))
+    allq = [w.queries[i] for i in order]
+    queries = allq[rank::world] if world > 1 else allq
     qdev = [torch.tensor(list(kw), dtype=torch.int32, device=f"cuda:{dev}") for kw in queries]
     stream = torch.cuda.current_stream(dev)
     sh = stream.cuda_stream
@@ -290,11 +294,11 @@ def main():
         t0 = time.perf_counter()
         done = 0
         while time.perf_counter() - t0 < args.cpu_sample_s and done < len(queries):
-            oracle.query(g, queries[done], w.k)
+            oracle.query(g, queries[(args.warmup + done) % len(queries)], w.k)
             done += 1
         el = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
-                                "sample": f"first {done} {name} queries ({el:.1f} s, single-threaded oracle)"}
+                                "sample": f"the first {done} timed {name} queries ({el:.1f} s, single-threaded oracle)"}
     print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

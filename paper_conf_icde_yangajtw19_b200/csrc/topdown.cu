@@ -500,6 +500,14 @@ __global__ void __launch_bounds__(256) k_select(QueryArgs a) {
     const uint32_t nc = ctl->n_central;
     const uint32_t kk = (uint32_t)a.k < nc ? (uint32_t)a.k : nc;
     if (kk == 0) { if (blockIdx.x == 0 && threadIdx.x == 0) ctl->sel_count = 0; return; }
+    if (nc <= (uint32_t)KGS_MAX_K) {
+        // small candidate set: k_rank sorts all of it in one CTA, no grid-wide passes needed
+        if (blockIdx.x == 0) {
+            for (uint32_t i = threadIdx.x; i < nc; i += blockDim.x) a.w.sel[i] = (int32_t)i;
+            if (threadIdx.x == 0) ctl->sel_count = nc;
+        }
+        return;
+    }
     const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gsz = (int64_t)gridDim.x * blockDim.x;
     uint64_t phi = 0;
     uint32_t plo = 0;
@@ -580,7 +588,9 @@ __global__ void __launch_bounds__(1024) k_rank(QueryArgs a) {
             }
             __syncthreads();
         }
-    for (int i = threadIdx.x; i < (int)cnt; i += blockDim.x) a.w.sel[i] = kid[i];
+    const int keep = (int)cnt < a.k ? (int)cnt : a.k;
+    for (int i = threadIdx.x; i < keep; i += blockDim.x) a.w.sel[i] = kid[i];
+    if (threadIdx.x == 0) a.w.ctl->sel_count = (uint32_t)keep;
 }
 
 // ------------------------------------------------------------------------------------------ emit
