@@ -163,6 +163,10 @@ kgs_status kgs_result_centrals(const kgs_result *r, int32_t *ids, uint8_t *depth
 /* Activation levels a (n bytes, Eqs. 3-5 at the query's alpha) — only if want_levels was 1. */
 kgs_status kgs_result_activation(const kgs_result *r, uint8_t *a, int64_t cap);
 kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s);
+/* Phase trace of the search kernel (the paper's per-phase profile): *n stamps, each a
+ * tag (0 start, 1 reset, 2 sources, 3 merge+identify, 4 expansion, 5..8 top-down pre-pass: seeds,
+ * merge, expansion, CSR, 9 end of search) and a %globaltimer time in ns, in execution order. */
+kgs_status kgs_result_phases(const kgs_result *r, int32_t *tags, uint64_t *t_ns, int32_t cap, int32_t *n);
 void kgs_result_free(kgs_result *r);
 
 /* Thread-local message describing the last non-OK status of this thread. */

@@ -61,8 +61,10 @@ class kgs_stats(ctypes.Structure):
 
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
             "kgs_query_fetch", "kgs_result_count", "kgs_result_answer", "kgs_result_levels",
-            "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_free",
-            "kgs_last_error", "kgs_version"]
+            "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_phases",
+            "kgs_result_free", "kgs_last_error", "kgs_version"]
+
+PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr", "search_end"]
 
 _lib = None
 
@@ -99,6 +101,8 @@ def lib():
         L.kgs_result_centrals.restype = i32
         L.kgs_result_stats.argtypes = [vp, ctypes.POINTER(kgs_stats)]
         L.kgs_result_stats.restype = i32
+        L.kgs_result_phases.argtypes = [vp, vp, vp, i32, ctypes.POINTER(i32)]
+        L.kgs_result_phases.restype = i32
         L.kgs_result_free.argtypes = [vp]
         L.kgs_result_free.restype = None
         L.kgs_last_error.argtypes = []
@@ -201,6 +205,17 @@ def _read_result(h, n, q, want_levels) -> Result:
         st = kgs_stats()
         _check(L.kgs_result_stats(h, ctypes.byref(st)))
         stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
+        tags = np.zeros(64, np.int32)
+        tns = np.zeros(64, np.uint64)
+        nph = ctypes.c_int32()
+        _check(L.kgs_result_phases(h, tags.ctypes.data, tns.ctypes.data, 64, ctypes.byref(nph)))
+        m = min(nph.value, 64)
+        # per-phase durations (us): time from the previous stamp to this one, summed by phase name
+        ph = {}
+        for i in range(1, m):
+            nm = PHASE_NAMES[tags[i]] if 0 <= tags[i] < len(PHASE_NAMES) else str(tags[i])
+            ph[nm] = ph.get(nm, 0.0) + (int(tns[i]) - int(tns[i - 1])) / 1e3
+        stats["phases_us"] = ph
         res = Result(answers, stats)
         if want_levels:
             M = np.empty(n * q, np.uint8)

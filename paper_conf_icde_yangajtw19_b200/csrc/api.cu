@@ -92,8 +92,8 @@ struct kgs_graph {
     int64_t *row_ptr = nullptr, *in_ptr = nullptr, *kw_ptr = nullptr;
     int32_t *col_idx = nullptr, *in_idx = nullptr, *kw_nodes = nullptr;
     float *weight = nullptr;
-    uint8_t *cls = nullptr;
-    int64_t n_heavy = 0, n_huge = 0;
+    uint8_t *cls = nullptr, *cls_in = nullptr;
+    int64_t n_heavy = 0, n_huge = 0, n_heavy_in = 0, n_huge_in = 0;
     // workspace
     DevWork w{};
     uint32_t *amax_dev = nullptr;
@@ -131,6 +131,8 @@ struct kgs_result {
     int64_t n = 0;
     int q = 0;
     kgs_stats stats{};
+    std::vector<int32_t> ph_tag;
+    std::vector<uint64_t> ph_ns;
 };
 
 extern "C" {
@@ -158,9 +160,11 @@ void kgs_free_graph(kgs_graph *g) {
                     g->w.nm, g->w.M, g->w.ring[0], g->w.ring[1], g->w.ring[2], g->w.fbits, g->w.touched,
                     g->w.centrals, g->w.cdepth, g->w.ckey, g->w.overflow, g->w.cflag, g->w.sel, g->w.kw_dev,
                     g->w.dpow, g->ctl_pair[0], g->ctl_pair[1], g->w.ans_hdr, g->w.ans_key, g->w.ans_off,
-                    g->w.arena_nodes, g->w.arena_arcs, g->w.big_ws, g->amax_dev};
+                    g->w.arena_nodes, g->w.arena_arcs, g->w.big_ws, g->amax_dev, g->w.pd_state, g->w.pd_cid,
+                    g->w.pd_touched, g->w.pd_ring[0], g->w.pd_ring[1], g->w.pd_ring[2], g->w.pcnt, g->w.pred_ptr,
+                    g->w.pred_u, g->w.pred_b, g->w.pa_u, g->w.pa_x, g->w.pa_b, g->w.pa_slot, g->w.scan_tmp};
     for (void *p : ptrs) if (p) cudaFree(p);
-    if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); }
+    if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
     void *hp[] = {g->h_ctl, g->h_kw, g->h_dpow, g->h_hdr, g->h_key, g->h_off};
     for (void *p : hp) if (p) cudaFreeHost(p);
     for (auto &e : g->ev) cudaEventDestroy(e);
@@ -250,7 +254,8 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     }
     // reverse CSR for extraction along in-arcs (reading R1)
     if (g->symmetric) {
-        g->in_ptr = g->row_ptr; g->in_idx = g->col_idx;
+        g->in_ptr = g->row_ptr; g->in_idx = g->col_idx; g->cls_in = g->cls;
+        g->n_heavy_in = g->n_heavy; g->n_huge_in = g->n_huge;
     } else {
         std::vector<int32_t> ci(m);
         if (on_dev) G_TRY(cudaMemcpy(ci.data(), d->col_idx, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
@@ -266,6 +271,12 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         G_TRY(dmalloc(&g->in_idx, m));
         G_TRY(cudaMemcpy(g->in_ptr, ip.data(), sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice));
         if (m) G_TRY(cudaMemcpy(g->in_idx, ii.data(), sizeof(int32_t) * m, cudaMemcpyHostToDevice));
+        G_TRY(dmalloc(&g->cls_in, n));
+        G_TRY(launch_degree_class(g->in_ptr, n, g->cls_in, 0));
+        for (int64_t v = 0; v < n; ++v) {
+            const int64_t dg_ = ip[v + 1] - ip[v];
+            if (dg_ > kHugeDeg) ++g->n_huge_in; else if (dg_ > kHeavyDeg) ++g->n_heavy_in;
+        }
     }
     // per-query workspace sized for n (rings are sized at the first query: they depend on alpha)
     DevWork &w = g->w;
@@ -305,6 +316,22 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     G_TRY(cudaMallocHost(&g->h_key, sizeof(double) * KGS_MAX_K));
     G_TRY(cudaMallocHost(&g->h_off, sizeof(long long) * 2 * KGS_MAX_K));
     w.cap[0] = n; w.cap[1] = g->n_heavy; w.cap[2] = g->n_huge;
+    // shared predecessor DAG of the top-down pre-pass
+    w.pd_cap[0] = n; w.pd_cap[1] = g->n_heavy_in; w.pd_cap[2] = g->n_huge_in;
+    w.pcap = std::max<int64_t>(std::min<int64_t>(m, int64_t(64) << 20), 1 << 20);
+    G_TRY(dmalloc(&w.pd_state, n));
+    G_TRY(dmalloc(&w.pd_cid, n));
+    G_TRY(dmalloc(&w.pd_touched, n));
+    for (int c = 0; c < 3; ++c) G_TRY(dmalloc(&w.pd_ring[c], 2 * (size_t)std::max<int64_t>(w.pd_cap[c], 1)));
+    G_TRY(dmalloc(&w.pcnt, n));
+    G_TRY(dmalloc(&w.pred_ptr, n + 1));
+    G_TRY(dmalloc(&w.pred_u, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.pred_b, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.pa_u, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.pa_x, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.pa_b, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.pa_slot, (size_t)w.pcap));
+    G_TRY(dmalloc(&w.scan_tmp, 4096));
     w.W = (n + 31) / 32;
     g->search_grid = search_max_grid(g->device, g->search_block);
     g->select_grid = select_max_grid(g->device);
@@ -381,6 +408,7 @@ kgs_status enqueue(kgs_graph *g, int32_t q, int32_t k, const kgs_params &p, cuda
     QueryArgs a{};
     a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx;
     a.g.in_ptr = g->in_ptr; a.g.in_idx = g->in_idx; a.g.weight = g->weight; a.g.cls = g->cls;
+    a.g.cls_in = g->cls_in;
     a.g.n_kw = g->n_kw; a.g.kw_ptr = g->kw_ptr; a.g.kw_nodes = g->kw_nodes;
     a.w = w;
     a.q = q; a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0;
@@ -482,6 +510,10 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
     st.arcs_scanned = (int64_t)c.arcs_scanned;
     st.overflow = c.n_overflow;
     st.hits = (int64_t)c.hits;
+    for (int i = 0; i < std::min(c.n_stamp, 64); ++i) {
+        r->ph_tag.push_back(c.stamp_tag[i]);
+        r->ph_ns.push_back(c.stamp[i]);
+    }
     cudaEventElapsedTime(&st.ms_search, g->ev[0], g->ev[1]);
     cudaEventElapsedTime(&st.ms_topdown, g->ev[1], g->ev[2]);
     cudaEventElapsedTime(&st.ms_total, g->ev[0], g->ev[2]);
@@ -576,6 +608,17 @@ kgs_status kgs_result_centrals(const kgs_result *r, int32_t *ids, uint8_t *depth
 kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s) {
     if (!r || !s) return fail(KGS_EINVAL, "null argument");
     *s = r->stats;
+    return KGS_OK;
+}
+
+kgs_status kgs_result_phases(const kgs_result *r, int32_t *tags, uint64_t *t_ns, int32_t cap, int32_t *n) {
+    if (!r || !n) return fail(KGS_EINVAL, "null argument");
+    *n = (int32_t)r->ph_tag.size();
+    const int32_t m = std::min<int32_t>(cap, *n);
+    for (int32_t i = 0; i < m; ++i) {
+        if (tags) tags[i] = r->ph_tag[i];
+        if (t_ns) t_ns[i] = r->ph_ns[i];
+    }
     return KGS_OK;
 }
 

@@ -51,7 +51,28 @@ struct Ctl {
     uint32_t sel_count;
     uint32_t pad2;
     unsigned long long arena_used[2];  // emitted nodes / arcs
+    // shared predecessor DAG (top-down pre-pass)
+    uint32_t pd_qcount[3][2];
+    uint32_t n_cid;                // nodes of the union of closures that have predecessor lists
+    uint32_t n_parcs;              // predecessor arcs found
+    unsigned long long td_arcs;    // in-arcs inspected by the pre-pass
+    int32_t pd_rounds;
+    int32_t pad3;
+    uint32_t pd_work[256];         // dynamic work counters per pre-pass round
+    // phase timestamps (%globaltimer, ns) written by thread 0 of the search kernel
+    int32_t n_stamp;
+    int32_t pad4;
+    unsigned long long stamp[64];
+    int32_t stamp_tag[64];
 };
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+// tags of the phase stamps
+enum { TS_START = 0, TS_RESET, TS_SCATTER, TS_MERGE, TS_EXPAND, TS_PD_SEED, TS_PD_MERGE, TS_PD_EXPAND, TS_PD_CSR, TS_END };
 
 struct DevGraph {
     int64_t n, m;
@@ -60,7 +81,8 @@ struct DevGraph {
     const int64_t *in_ptr;
     const int32_t *in_idx;
     const float *weight;
-    const uint8_t *cls;       // degree class per node
+    const uint8_t *cls;       // degree class per node (out-arcs)
+    const uint8_t *cls_in;    // degree class per node (in-arcs; == cls for a symmetric graph)
     int64_t n_kw;
     const int64_t *kw_ptr;
     const int32_t *kw_nodes;
@@ -95,6 +117,22 @@ struct DevWork {
     int32_t *arena_nodes;
     int32_t *arena_arcs;  // pairs
     long long arena_nodes_cap, arena_arcs_cap;
+    // shared predecessor DAG over the union of all Central Graphs
+    uint32_t *pd_state;   // [n] byte0 = bits to expand this round, byte1 = bits for the next round, byte2 = done
+    int32_t *pd_cid;      // [n] compact id of a node with a predecessor list, -1 otherwise
+    int32_t *pd_touched;  // [n] node of each compact id (reset list)
+    int32_t *pd_ring[3];  // per in-degree class: [2][pd_cap_c] round queues
+    int64_t pd_cap[3];
+    int32_t *pcnt;        // [n] predecessors per compact id
+    int32_t *pred_ptr;    // [n+1] CSR offsets per compact id
+    int32_t *pred_u;      // [pcap] predecessor node
+    uint16_t *pred_b;     // [pcap] low byte: keyword bits of the arc; high byte: zb(pred) (source bits)
+    int32_t *pa_u;        // [pcap] arcs in discovery order
+    int32_t *pa_x;        // [pcap] compact id of the successor
+    uint16_t *pa_b;       // [pcap]
+    int32_t *pa_slot;     // [pcap] position inside the successor's list
+    int32_t *scan_tmp;    // [4096] block sums of the CSR scan
+    int64_t pcap;
     // large-graph extractor arenas
     void *big_ws;
     size_t big_bytes, big_bytes_emit;

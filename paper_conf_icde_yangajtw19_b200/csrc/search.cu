@@ -114,11 +114,14 @@ __device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
     return base + rank;
 }
 
-struct SearchCtx {
-    const QueryArgs &a;
-    int R;
-    uint32_t full;
-};
+// phase timestamp by the grid's first thread (read back into kgs_stats-like debug output)
+#define KGS_STAMP(tag)                                                                            \
+    do {                                                                                          \
+        if (gtid == 0) {                                                                          \
+            const int _i = ctl->n_stamp;                                                          \
+            if (_i < 64) { ctl->stamp[_i] = globaltimer_ns(); ctl->stamp_tag[_i] = (tag); ctl->n_stamp = _i + 1; } \
+        }                                                                                         \
+    } while (0)
 
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1 for level L).
 __device__ __forceinline__ void push(const QueryArgs &a, int R, int32_t v, int L) {
@@ -172,6 +175,251 @@ __device__ __forceinline__ uint32_t prepare(const QueryArgs &a, int R, int l, ui
     return hm;                                             // ln 8-11: every hit instance has m <= l
 }
 
+// ------------------------------------------------------------------------------------------ pre-pass
+// Shared predecessor DAG (top-down): whether u -> x is a B_i-predecessor arc
+// (Thm. V.4 + reading R12) depends only on M, a and K, never on the central node whose graph is being
+// extracted.  So the backward closure of ALL central nodes is computed once, level by level, with the
+// same degree-balanced scheme as the expansion, and every arc that passes the test is stored in a CSR
+// keyed by its successor.  Each Central Graph is then a walk over these short lists (topdown.cu).
+__device__ __forceinline__ void pd_push(const QueryArgs &a, int slot, int32_t u) {
+    const int c = a.g.cls_in[u];
+    const uint32_t pos = agg_slot(&a.w.ctl->pd_qcount[c][slot], (unsigned)((c << 8) | slot));
+    a.w.pd_ring[c][(int64_t)slot * a.w.pd_cap[c] + pos] = u;
+}
+
+// Thm. V.4 test of in-arc u -> x for the keyword bits P of x (hx = M row of x, gx = gate(x) - 1).
+__device__ __forceinline__ uint32_t pred_test(const QueryArgs &a, uint32_t full, bool exact_block, uint32_t P,
+                                              uint64_t hx, int gx, int32_t u, uint32_t &zbu) {
+    const uint32_t hmu = __ldcg(a.w.st + u) & 0xFFu;
+    const uint32_t cand = P & hmu;
+    if (!cand) return 0;
+    const int au = a.w.act[u];
+    const uint64_t Mu = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + u);
+    uint32_t pb = 0, zb = 0;
+    int maxrow = 0;
+#pragma unroll
+    for (int i = 0; i < kMaxQ; ++i) {
+        if (!((hmu >> i) & 1u)) continue;
+        const int mu = (int)((Mu >> (8 * i)) & 0xFF);
+        maxrow = maxrow > mu ? maxrow : mu;
+        if (mu == 0) zb |= 1u << i;
+        if (!((cand >> i) & 1u)) continue;
+        int need = au > mu ? au : mu;
+        need = need > gx ? need : gx;
+        if ((int)((hx >> (8 * i)) & 0xFF) == need + 1) pb |= 1u << i;   // m_xi = 1 + max{a_u, m_ui, g_x}
+    }
+    if (pb && exact_block && hmu == full) {
+#pragma unroll
+        for (int i = 0; i < kMaxQ; ++i)   // u central at depth maxrow: it only expanded at levels < maxrow
+            if (((pb >> i) & 1u) && maxrow <= (int)((hx >> (8 * i)) & 0xFF) - 1) pb &= ~(1u << i);
+    }
+    zbu = zb;
+    return pb;
+}
+
+__device__ __forceinline__ void pd_visit(const QueryArgs &a, uint32_t full, bool exact_block, uint32_t P, uint64_t hx,
+                                         int gx, int32_t cidx, int32_t u, int nslot) {
+    uint32_t zbu = 0;
+    const uint32_t pb = pred_test(a, full, exact_block, P, hx, gx, u, zbu);
+    if (!pb) return;
+    const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(a.w.pcnt + cidx), (unsigned)cidx);
+    const uint32_t ai = agg_slot(&a.w.ctl->n_parcs, 0xFFFFFFFFu);
+    if ((int64_t)ai < a.w.pcap) {
+        a.w.pa_u[ai] = u;
+        a.w.pa_x[ai] = cidx;
+        a.w.pa_b[ai] = (uint16_t)(pb | (zbu << 8));
+        a.w.pa_slot[ai] = (int32_t)pos;
+    } else {
+        atomicExch(&a.w.ctl->fatal, 5);
+    }
+    const uint32_t nb = pb & ~zbu;        // sources (m = 0) have no predecessors
+    if (nb) {
+        const uint32_t old = atomicOr(a.w.pd_state + u, nb << 8);
+        if (((old >> 8) & 0xFFu) == 0) pd_push(a, nslot, u);
+    }
+}
+
+struct PdNode {
+    uint32_t P;
+    uint64_t hx;
+    int gx;
+    int32_t cidx;
+};
+
+__device__ __forceinline__ PdNode pd_prepare(const QueryArgs &a, int32_t x) {
+    PdNode nd;
+    nd.P = __ldcg(a.w.pd_state + x) & 0xFFu;
+    nd.hx = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + x);
+    nd.gx = (int)(__ldcg(a.w.st + x) >> 8) - 1;
+    nd.cidx = __ldcg(a.w.pd_cid + x);
+    return nd;
+}
+
+__device__ __forceinline__ int block_excl_scan(int x, int *total, int *sh) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    int incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    __syncthreads();
+    if (lane == 31) sh[wid] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int acc = 0;
+        for (int w = 0; w < nw; ++w) { const int t = sh[w]; sh[w] = acc; acc += t; }
+        sh[32] = acc;
+    }
+    __syncthreads();
+    const int r = sh[wid] + incl - x;
+    *total = sh[32];
+    __syncthreads();
+    return r;
+}
+
+__device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid, int64_t gsz, uint32_t full) {
+    Ctl *ctl = a.w.ctl;
+    const bool exact_block = a.extract_mode == KGS_EXTRACT_EXACT && a.block_central;
+    const uint32_t nc = __ldcg(&ctl->n_central);
+    // seeds: every central node, for every keyword it did not contain itself
+    for (int64_t j = gtid; j < nc; j += gsz) {
+        const int32_t c = a.w.centrals[j];
+        const uint64_t Mc = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + c);
+        uint32_t zbc = 0;
+        for (int i = 0; i < a.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
+        const uint32_t bits = full & ~zbc;
+        if (bits) { atomicOr(a.w.pd_state + c, bits << 8); pd_push(a, 0, c); }
+    }
+    grid.sync();
+    KGS_STAMP(TS_PD_SEED);
+    unsigned long long my_arcs = 0;
+    int r = 0;
+    for (;; ++r) {
+        const int slot = r & 1;
+        const uint32_t c0 = __ldcg(&ctl->pd_qcount[0][slot]), c1 = __ldcg(&ctl->pd_qcount[1][slot]),
+                       c2 = __ldcg(&ctl->pd_qcount[2][slot]);
+        const int64_t total = (int64_t)c0 + c1 + c2;
+        if (total == 0) break;
+        if (gtid == 0) { ctl->pd_qcount[0][slot ^ 1] = 0; ctl->pd_qcount[1][slot ^ 1] = 0; ctl->pd_qcount[2][slot ^ 1] = 0; }
+        // merge: bits to expand this round = newly requested bits not expanded before
+        for (int64_t j = gtid; j < total; j += gsz) {
+            int32_t u;
+            if (j < c0) u = a.w.pd_ring[0][(int64_t)slot * a.w.pd_cap[0] + j];
+            else if (j < (int64_t)c0 + c1) u = a.w.pd_ring[1][(int64_t)slot * a.w.pd_cap[1] + (j - c0)];
+            else u = a.w.pd_ring[2][(int64_t)slot * a.w.pd_cap[2] + (j - c0 - c1)];
+            const uint32_t s = __ldcg(a.w.pd_state + u);
+            const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
+            const uint32_t bits = nx & ~dn;
+            a.w.pd_state[u] = bits | ((dn | bits) << 16);
+            if (bits && __ldcg(a.w.pd_cid + u) < 0) {
+                const uint32_t cid = agg_slot(&ctl->n_cid, 1u);
+                a.w.pd_cid[u] = (int32_t)cid;
+                a.w.pd_touched[cid] = u;
+            }
+        }
+        grid.sync();
+        KGS_STAMP(TS_PD_MERGE);
+        const int ns = slot ^ 1;
+        for (uint32_t j = 0; j < c2; ++j) {                       // huge: whole grid per node
+            const int32_t x = a.w.pd_ring[2][(int64_t)slot * a.w.pd_cap[2] + j];
+            const PdNode nd = pd_prepare(a, x);
+            if (!nd.P) continue;
+            const int64_t b = a.g.in_ptr[x], e = a.g.in_ptr[x + 1];
+            if (gtid == 0) my_arcs += (unsigned long long)(e - b);
+            for (int64_t p = b + gtid; p < e; p += gsz)
+                pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, __ldcs(a.g.in_idx + p), ns);
+        }
+        for (uint32_t j = blockIdx.x; j < c1; j += gridDim.x) {  // heavy: one CTA per node
+            const int32_t x = a.w.pd_ring[1][(int64_t)slot * a.w.pd_cap[1] + j];
+            const PdNode nd = pd_prepare(a, x);
+            if (!nd.P) continue;
+            const int64_t b = a.g.in_ptr[x], e = a.g.in_ptr[x + 1];
+            if (threadIdx.x == 0) my_arcs += (unsigned long long)(e - b);
+            for (int64_t p = b + threadIdx.x; p < e; p += blockDim.x)
+                pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, __ldcs(a.g.in_idx + p), ns);
+        }
+        const unsigned lane = lane_id();
+        for (;;) {                                                 // light: warp batches of 32 nodes
+            uint32_t base = 0;
+            if (lane == 0) base = atomicAdd(&ctl->pd_work[r & 255], 32u);
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (base >= c0) break;
+            const uint32_t idx = base + lane;
+            PdNode nd{0, 0, 0, -1};
+            int64_t start = 0;
+            int deg = 0;
+            if (idx < c0) {
+                const int32_t x = a.w.pd_ring[0][(int64_t)slot * a.w.pd_cap[0] + idx];
+                nd = pd_prepare(a, x);
+                if (nd.P) { start = a.g.in_ptr[x]; deg = (int)(a.g.in_ptr[x + 1] - start); }
+            }
+            int incl = deg;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(0xffffffffu, incl, o);
+                if ((int)lane >= o) incl += t;
+            }
+            const int tot = __shfl_sync(0xffffffffu, incl, 31);
+            if (lane == 0) my_arcs += (unsigned long long)tot;
+            const int excl = incl - deg;
+            for (int e0 = 0; e0 < tot; e0 += 32) {
+                const int e = e0 + (int)lane;
+                int pos = 0;
+#pragma unroll
+                for (int bb = 16; bb > 0; bb >>= 1) {
+                    const int val = __shfl_sync(0xffffffffu, incl, pos + bb - 1);
+                    if (val <= e) pos += bb;
+                }
+                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
+                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
+                const uint32_t P_o = __shfl_sync(0xffffffffu, nd.P, pos);
+                const uint64_t hx_o = __shfl_sync(0xffffffffu, (unsigned long long)nd.hx, pos);
+                const int gx_o = __shfl_sync(0xffffffffu, nd.gx, pos);
+                const int32_t cid_o = __shfl_sync(0xffffffffu, nd.cidx, pos);
+                if (e < tot)
+                    pd_visit(a, full, exact_block, P_o, hx_o, gx_o, cid_o, __ldcs(a.g.in_idx + st_o + (e - ex_o)), ns);
+            }
+        }
+        grid.sync();
+        KGS_STAMP(TS_PD_EXPAND);
+    }
+    if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
+    if (gtid == 0) ctl->pd_rounds = r;
+    // CSR of the predecessor lists: exclusive scan of pcnt over compact ids, then scatter
+    __shared__ int sh[40];
+    const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
+    const int64_t chunk = (ncid + gridDim.x - 1) / gridDim.x;
+    const int64_t lo = (int64_t)blockIdx.x * chunk, hi = lo + chunk < ncid ? lo + chunk : ncid;
+    int run = 0;
+    for (int64_t t0 = lo; t0 < hi; t0 += blockDim.x) {
+        const int64_t j = t0 + threadIdx.x;
+        const int v = j < hi ? __ldcg(a.w.pcnt + j) : 0;
+        int tot;
+        const int ex = block_excl_scan(v, &tot, sh);
+        if (j < hi) a.w.pred_ptr[j] = run + ex;
+        run += tot;
+    }
+    if (threadIdx.x == 0) a.w.scan_tmp[blockIdx.x] = run;
+    grid.sync();
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        int acc = 0;
+        for (unsigned b = 0; b < gridDim.x; ++b) { const int t = __ldcg(a.w.scan_tmp + b); a.w.scan_tmp[b] = acc; acc += t; }
+        a.w.pred_ptr[ncid] = acc;
+    }
+    grid.sync();
+    const int off = __ldcg(a.w.scan_tmp + blockIdx.x);
+    for (int64_t j = lo + threadIdx.x; j < hi; j += blockDim.x) a.w.pred_ptr[j] += off;
+    grid.sync();
+    KGS_STAMP(TS_PD_CSR);
+    const int64_t np = (int64_t)__ldcg(&ctl->n_parcs) < a.w.pcap ? (int64_t)__ldcg(&ctl->n_parcs) : a.w.pcap;
+    for (int64_t ai = gtid; ai < np; ai += gsz) {
+        const int64_t pos = (int64_t)__ldcg(a.w.pred_ptr + a.w.pa_x[ai]) + a.w.pa_slot[ai];
+        a.w.pred_u[pos] = a.w.pa_u[ai];
+        a.w.pred_b[pos] = a.w.pa_b[ai];
+    }
+}
+
 // ------------------------------------------------------------------------------------------ search
 __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     cg::grid_group grid = cg::this_grid();
@@ -184,13 +432,19 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     Ctl *ctl = a.w.ctl;
     uint8_t *st8 = reinterpret_cast<uint8_t *>(a.w.st);
     uint8_t *nm8 = reinterpret_cast<uint8_t *>(a.w.nm);
+    KGS_STAMP(TS_START);
 
     // ---- reset the state the previous query left behind
     if (a.full_reset) {
         for (int64_t v = gtid; v < n; v += gsz) a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
         for (int64_t v = gtid; v < (n + 3) / 4; v += gsz) a.w.nm[v] = 0u;
         for (int64_t j = gtid; j < (int64_t)R * a.w.W; j += gsz) a.w.fbits[j] = 0u;
+        for (int64_t v = gtid; v < n; v += gsz) { a.w.pd_state[v] = 0u; a.w.pd_cid[v] = -1; a.w.pcnt[v] = 0; }
     } else {
+        for (int64_t j = gtid; j < (int64_t)a.w.prev->n_cid; j += gsz) {
+            const int32_t v = a.w.pd_touched[j];
+            a.w.pd_state[v] = 0u; a.w.pd_cid[v] = -1; a.w.pcnt[j] = 0;
+        }
         const Ctl *pv = a.w.prev;
         const int64_t pt = (int64_t)pv->n_touched;
         for (int64_t j = gtid; j < pt; j += gsz) {
@@ -213,6 +467,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
         if (a.g.kw_ptr[t + 1] == a.g.kw_ptr[t]) empty = true;
     }
     grid.sync();
+    KGS_STAMP(TS_RESET);
     for (int i = 0; i < a.q; ++i) {
         const int32_t t = a.w.kw_dev[i];
         const int64_t b = a.g.kw_ptr[t], e = a.g.kw_ptr[t + 1];
@@ -225,6 +480,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
         }
     }
     grid.sync();
+    KGS_STAMP(TS_SCATTER);
 
     unsigned long long my_arcs = 0, my_hits = 0;
     for (int l = 0;; ++l) {
@@ -266,6 +522,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
         }
         if (gtid == 0) ctl->frontier_total += (unsigned long long)total;
         grid.sync();
+        KGS_STAMP(TS_MERGE);
         if (gtid == 0 && l > 0) {
             const int sp = (l - 1) % R;
             ctl->qcount[0][sp] = 0; ctl->qcount[1][sp] = 0; ctl->qcount[2][sp] = 0;
@@ -348,9 +605,13 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
             }
         }
         grid.sync();
+        KGS_STAMP(TS_EXPAND);
     }
     if (my_arcs) atomicAdd(&ctl->arcs_scanned, my_arcs);
     if (my_hits) atomicAdd(&ctl->hits, my_hits);
+    grid.sync();
+    KGS_STAMP(TS_END);
+    pred_dag(a, grid, gtid, gsz, full);
 }
 
 int search_max_grid(int device, int block) {

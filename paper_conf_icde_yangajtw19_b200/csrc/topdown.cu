@@ -136,7 +136,6 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
 template <class Team>
 __device__ bool central_graph(const Team &T, Arena &S, const QueryArgs &a, int32_t c, int depth, double *key) {
     const uint32_t full = (1u << a.q) - 1u;
-    const bool exact_block = a.extract_mode == KGS_EXTRACT_EXACT && a.block_central;
     const int r = T.rank(), ts = T.size();
     for (int i = r; i < S.hcap; i += ts) { S.hkey[i] = -1; S.hval[i] = -1; }
     for (int i = r; i < S.ncap; i += ts) { S.inmask[i] = 0; S.pending[i] = 0; S.keep[i] = 0; }
@@ -166,11 +165,10 @@ __device__ bool central_graph(const Team &T, Arena &S, const QueryArgs &a, int32
                 const int32_t x = S.id[j];
                 S.b_j[r] = j;
                 S.b_P[r] = P;
-                S.b_hx[r] = *reinterpret_cast<const uint64_t *>(a.w.M + (int64_t)x * 8);
-                S.b_gx[r] = (int)(a.w.st[x] >> 8) - 1;
-                const int64_t s0 = a.g.in_ptr[x];
+                const int32_t cid = a.w.pd_cid[x];   // predecessor list from the shared DAG
+                int64_t s0 = 0;
+                if (P && cid >= 0) { s0 = a.w.pred_ptr[cid]; deg = (int)(a.w.pred_ptr[cid + 1] - s0); }
                 S.b_start[r] = s0;
-                if (P) deg = (int)(a.g.in_ptr[x + 1] - s0);
             }
             int tot;
             const int ex = T.scan_excl(deg, &tot);
@@ -185,34 +183,12 @@ __device__ bool central_graph(const Team &T, Arena &S, const QueryArgs &a, int32
                 }
                 const int o = lo;
                 const int exo = o ? S.b_incl[o - 1] : 0;
-                const int32_t u = a.g.in_idx[S.b_start[o] + (e - exo)];
-                const uint32_t P = S.b_P[o];
-                const uint32_t su = a.w.st[u];
-                const uint32_t hmu = su & 0xFFu;
-                const uint32_t cand = P & hmu;
-                if (!cand) continue;
-                const uint64_t hx = S.b_hx[o];
-                const int gx = S.b_gx[o];
-                const int au = a.w.act[u];
-                const uint64_t Mu = *reinterpret_cast<const uint64_t *>(a.w.M + (int64_t)u * 8);
-                uint32_t pb = 0;
-                int maxrow = 0;
-                for (int i = 0; i < a.q; ++i) {
-                    const int mu = (int)((Mu >> (8 * i)) & 0xFF);
-                    if ((hmu >> i) & 1u) maxrow = maxrow > mu ? maxrow : mu;
-                    if (!((cand >> i) & 1u)) continue;
-                    int need = au > mu ? au : mu;
-                    need = need > gx ? need : gx;
-                    if ((int)((hx >> (8 * i)) & 0xFF) == need + 1) pb |= 1u << i;  // Thm. V.4
-                }
-                if (pb && exact_block && hmu == full) {
-                    for (int i = 0; i < a.q; ++i)   // u central at depth maxrow: expanded only before it
-                        if (((pb >> i) & 1u) && maxrow <= (int)((hx >> (8 * i)) & 0xFF) - 1) pb &= ~(1u << i);
-                }
+                const int64_t pi = S.b_start[o] + (e - exo);
+                const int32_t u = a.w.pred_u[pi];
+                const uint32_t bz = a.w.pred_b[pi];
+                const uint32_t pb = bz & S.b_P[o] & 0xFFu;   // Thm. V.4 arc for the keywords x needs here
                 if (!pb) continue;
-                uint32_t zbu = 0;
-                for (int i = 0; i < a.q; ++i)
-                    if (((hmu >> i) & 1u) && ((Mu >> (8 * i)) & 0xFF) == 0) zbu |= 1u << i;
+                const uint32_t zbu = bz >> 8;
                 const int j = arena_insert(S, u, zbu);
                 if (j < 0) continue;
                 const uint32_t old = atomicOr(S.inmask + j, pb);
