@@ -175,6 +175,92 @@ __device__ __forceinline__ uint32_t prepare(const QueryArgs &a, int R, int l, ui
     return hm;                                             // ln 8-11: every hit instance has m <= l
 }
 
+// ------------------------------------------------------------------------------------------ load balance
+// Frontier nodes above kHeavyDeg (heavy and huge classes) are expanded in tiles of blockDim entries:
+// every CTA computes the same tile prefix of degrees in shared memory, then the tile's arcs form one
+// index space that all threads of the grid stride over (owner found by binary search).  A hub's arcs
+// are thus spread over the whole GPU instead of one warp or one CTA.
+__device__ __forceinline__ long long block_excl_scan64(long long x, long long *total, long long *sh) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    long long incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    __syncthreads();
+    if (lane == 31) sh[wid] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long acc = 0;
+        for (int w = 0; w < nw; ++w) { const long long t = sh[w]; sh[w] = acc; acc += t; }
+        sh[32] = acc;
+    }
+    __syncthreads();
+    const long long r = sh[wid] + incl - x;
+    *total = sh[32];
+    __syncthreads();
+    return r;
+}
+
+constexpr int kTileMax = 512;   // == blockDim of the persistent kernel
+
+struct FwdNode {
+    int32_t v;
+    uint32_t hm;
+};
+
+template <class NodeT>
+struct BigTile {
+    long long incl[kTileMax];
+    long long start[kTileMax];
+    NodeT node[kTileMax];
+    long long scan[40];
+};
+
+template <class NodeT, class Prep, class Visit>
+__device__ __forceinline__ void expand_big(const int32_t *ring1, uint32_t c1, const int32_t *ring2, uint32_t c2,
+                                           const int64_t *ptr, const int32_t *idx, BigTile<NodeT> &S, int64_t gtid,
+                                           int64_t gsz, Prep prep, Visit visit, unsigned long long &arcs) {
+    const uint32_t cb = c1 + c2;
+    for (uint32_t t0 = 0; t0 < cb; t0 += blockDim.x) {
+        const int nt = (int)min((uint32_t)blockDim.x, cb - t0);
+        const int j = threadIdx.x;
+        long long deg = 0, st = 0;
+        if (j < nt) {
+            const uint32_t e = t0 + j;
+            const int32_t v = e < c1 ? ring1[e] : ring2[e - c1];
+            NodeT nd;
+            if (prep(v, blockIdx.x == 0, nd)) { st = ptr[v]; deg = ptr[v + 1] - st; }
+            S.node[j] = nd;
+            S.start[j] = st;
+        }
+        long long T;
+        const long long ex = block_excl_scan64(deg, &T, S.scan);
+        S.incl[j] = ex + deg;
+        __syncthreads();
+        if (gtid == 0) arcs += (unsigned long long)T;
+        for (long long e = gtid; e < T; e += gsz) {
+            int lo = 0, hi = nt - 1;
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (S.incl[mid] > e) hi = mid; else lo = mid + 1;
+            }
+            const long long exo = lo ? S.incl[lo - 1] : 0;
+            visit(S.node[lo], __ldcs(idx + S.start[lo] + (e - exo)));
+        }
+        __syncthreads();
+    }
+}
+
+// light-batch size: 32 frontier nodes per warp when the frontier is large, fewer (down to 1) when it
+// is small, so that every warp of the grid gets work
+__device__ __forceinline__ uint32_t light_batch(uint32_t c0, int64_t gsz) {
+    const uint32_t warps = (uint32_t)(gsz >> 5);
+    uint32_t b = (c0 + 2 * warps - 1) / (2 * warps);
+    return b < 1 ? 1u : (b > 32 ? 32u : b);
+}
+
 // ------------------------------------------------------------------------------------------ pre-pass
 // Shared predecessor DAG (top-down): whether u -> x is a B_i-predecessor arc
 // (Thm. V.4 + reading R12) depends only on M, a and K, never on the central node whose graph is being
@@ -282,6 +368,7 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
     Ctl *ctl = a.w.ctl;
     const bool exact_block = a.extract_mode == KGS_EXTRACT_EXACT && a.block_central;
     const uint32_t nc = __ldcg(&ctl->n_central);
+    __shared__ BigTile<PdNode> s_bigb;
     // seeds: every central node, for every keyword it did not contain itself
     for (int64_t j = gtid; j < nc; j += gsz) {
         const int32_t c = a.w.centrals[j];
@@ -321,35 +408,27 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
         grid.sync();
         KGS_STAMP(TS_PD_MERGE);
         const int ns = slot ^ 1;
-        for (uint32_t j = 0; j < c2; ++j) {                       // huge: whole grid per node
-            const int32_t x = a.w.pd_ring[2][(int64_t)slot * a.w.pd_cap[2] + j];
-            const PdNode nd = pd_prepare(a, x);
-            if (!nd.P) continue;
-            const int64_t b = a.g.in_ptr[x], e = a.g.in_ptr[x + 1];
-            if (gtid == 0) my_arcs += (unsigned long long)(e - b);
-            for (int64_t p = b + gtid; p < e; p += gsz)
-                pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, __ldcs(a.g.in_idx + p), ns);
-        }
-        for (uint32_t j = blockIdx.x; j < c1; j += gridDim.x) {  // heavy: one CTA per node
-            const int32_t x = a.w.pd_ring[1][(int64_t)slot * a.w.pd_cap[1] + j];
-            const PdNode nd = pd_prepare(a, x);
-            if (!nd.P) continue;
-            const int64_t b = a.g.in_ptr[x], e = a.g.in_ptr[x + 1];
-            if (threadIdx.x == 0) my_arcs += (unsigned long long)(e - b);
-            for (int64_t p = b + threadIdx.x; p < e; p += blockDim.x)
-                pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, __ldcs(a.g.in_idx + p), ns);
-        }
+        // heavy and huge nodes: tiles spread over the whole grid
+        expand_big(a.w.pd_ring[1] + (int64_t)slot * a.w.pd_cap[1], c1, a.w.pd_ring[2] + (int64_t)slot * a.w.pd_cap[2],
+                   c2, a.g.in_ptr, a.g.in_idx, s_bigb, gtid, gsz,
+                   [&](int32_t x, bool, PdNode &nd) {
+                       nd = pd_prepare(a, x);
+                       return nd.P != 0;
+                   },
+                   [&](const PdNode &nd, int32_t u) { pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, u, ns); },
+                   my_arcs);
         const unsigned lane = lane_id();
-        for (;;) {                                                 // light: warp batches of 32 nodes
+        const uint32_t B = light_batch(c0, gsz);
+        for (;;) {                                                 // light: warp batches
             uint32_t base = 0;
-            if (lane == 0) base = atomicAdd(&ctl->pd_work[r & 255], 32u);
+            if (lane == 0) base = atomicAdd(&ctl->pd_work[r & 255], B);
             base = __shfl_sync(0xffffffffu, base, 0);
             if (base >= c0) break;
             const uint32_t idx = base + lane;
             PdNode nd{0, 0, 0, -1};
             int64_t start = 0;
             int deg = 0;
-            if (idx < c0) {
+            if (lane < B && idx < c0) {
                 const int32_t x = a.w.pd_ring[0][(int64_t)slot * a.w.pd_cap[0] + idx];
                 nd = pd_prepare(a, x);
                 if (nd.P) { start = a.g.in_ptr[x]; deg = (int)(a.g.in_ptr[x + 1] - start); }
@@ -402,10 +481,17 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
     }
     if (threadIdx.x == 0) a.w.scan_tmp[blockIdx.x] = run;
     grid.sync();
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        int acc = 0;
-        for (unsigned b = 0; b < gridDim.x; ++b) { const int t = __ldcg(a.w.scan_tmp + b); a.w.scan_tmp[b] = acc; acc += t; }
-        a.w.pred_ptr[ncid] = acc;
+    if (blockIdx.x == 0) {   // exclusive scan of the per-CTA sums (gridDim <= a few blockDim)
+        int carry = 0;
+        for (unsigned b0 = 0; b0 < gridDim.x; b0 += blockDim.x) {
+            const unsigned b = b0 + threadIdx.x;
+            const int v = b < gridDim.x ? __ldcg(a.w.scan_tmp + b) : 0;
+            int tot;
+            const int ex = block_excl_scan(v, &tot, sh);
+            if (b < gridDim.x) a.w.scan_tmp[b] = carry + ex;
+            carry += tot;
+        }
+        if (threadIdx.x == 0) a.w.pred_ptr[ncid] = carry;
     }
     grid.sync();
     const int off = __ldcg(a.w.scan_tmp + blockIdx.x);
@@ -432,6 +518,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     Ctl *ctl = a.w.ctl;
     uint8_t *st8 = reinterpret_cast<uint8_t *>(a.w.st);
     uint8_t *nm8 = reinterpret_cast<uint8_t *>(a.w.nm);
+    __shared__ BigTile<FwdNode> s_big;
     KGS_STAMP(TS_START);
 
     // ---- reset the state the previous query left behind
@@ -447,6 +534,9 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
         }
         const Ctl *pv = a.w.prev;
         const int64_t pt = (int64_t)pv->n_touched;
+        if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
+            for (int64_t v = gtid; v < n; v += gsz) a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
+        } else
         for (int64_t j = gtid; j < pt; j += gsz) {
             const int32_t v = a.w.touched[j];
             a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
@@ -542,29 +632,21 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
             break;
         }
         // ---- expansion (Alg. 2)
-        // huge nodes: the whole grid strides over one node's arcs
-        for (uint32_t j = 0; j < c2; ++j) {
-            const int32_t v = a.w.ring[2][(int64_t)s * a.w.cap[2] + j];
-            const uint32_t hm = prepare(a, R, l, full, v, gtid == 0);
-            if (!hm) continue;
-            const int64_t b = a.g.row_ptr[v], e = a.g.row_ptr[v + 1];
-            if (gtid == 0) my_arcs += (unsigned long long)(e - b);
-            for (int64_t p = b + gtid; p < e; p += gsz) visit_arc(a, R, l, v, hm, __ldcs(a.g.col_idx + p), my_hits);
-        }
-        // heavy nodes: one CTA per node
-        for (uint32_t j = blockIdx.x; j < c1; j += gridDim.x) {
-            const int32_t v = a.w.ring[1][(int64_t)s * a.w.cap[1] + j];
-            const uint32_t hm = prepare(a, R, l, full, v, threadIdx.x == 0);
-            if (!hm) continue;
-            const int64_t b = a.g.row_ptr[v], e = a.g.row_ptr[v + 1];
-            if (threadIdx.x == 0) my_arcs += (unsigned long long)(e - b);
-            for (int64_t p = b + threadIdx.x; p < e; p += blockDim.x) visit_arc(a, R, l, v, hm, __ldcs(a.g.col_idx + p), my_hits);
-        }
-        // light nodes: dynamic batches of 32 frontier nodes per warp, arcs balanced across the lanes
+        // heavy and huge nodes: tiles whose arcs are spread over the whole grid
+        expand_big(a.w.ring[1] + (int64_t)s * a.w.cap[1], c1, a.w.ring[2] + (int64_t)s * a.w.cap[2], c2,
+                   a.g.row_ptr, a.g.col_idx, s_big, gtid, gsz,
+                   [&](int32_t v, bool leader, FwdNode &nd) {
+                       nd.v = v;
+                       nd.hm = prepare(a, R, l, full, v, leader);
+                       return nd.hm != 0;
+                   },
+                   [&](const FwdNode &nd, int32_t x) { visit_arc(a, R, l, nd.v, nd.hm, x, my_hits); }, my_arcs);
+        // light nodes: dynamic batches of frontier nodes per warp, arcs balanced across the lanes
         const unsigned lane = lane_id();
+        const uint32_t B = light_batch(c0, gsz);
         for (;;) {
             uint32_t base = 0;
-            if (lane == 0) base = atomicAdd(&ctl->work[l], 32u);
+            if (lane == 0) base = atomicAdd(&ctl->work[l], B);
             base = __shfl_sync(0xffffffffu, base, 0);
             if (base >= c0) break;
             const uint32_t idx = base + lane;
@@ -572,7 +654,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
             uint32_t hm = 0;
             int64_t start = 0;
             int deg = 0;
-            if (idx < c0) {
+            if (lane < B && idx < c0) {
                 v = a.w.ring[0][(int64_t)s * a.w.cap[0] + idx];
                 hm = prepare(a, R, l, full, v, true);
                 if (hm) {
@@ -607,8 +689,12 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
         grid.sync();
         KGS_STAMP(TS_EXPAND);
     }
-    if (my_arcs) atomicAdd(&ctl->arcs_scanned, my_arcs);
-    if (my_hits) atomicAdd(&ctl->hits, my_hits);
+    my_arcs = __reduce_add_sync(0xffffffffu, (unsigned)my_arcs) + 0ull;   // per-warp totals fit 32 bits
+    my_hits = __reduce_add_sync(0xffffffffu, (unsigned)my_hits) + 0ull;
+    if ((threadIdx.x & 31) == 0) {
+        if (my_arcs) atomicAdd(&ctl->arcs_scanned, my_arcs);
+        if (my_hits) atomicAdd(&ctl->hits, my_hits);
+    }
     grid.sync();
     KGS_STAMP(TS_END);
     pred_dag(a, grid, gtid, gsz, full);
