@@ -93,7 +93,7 @@ struct kgs_graph {
     int32_t *col_idx = nullptr, *in_idx = nullptr, *kw_nodes = nullptr;
     float *weight = nullptr;
     uint8_t *cls = nullptr, *cls_in = nullptr;
-    int64_t n_heavy = 0, n_huge = 0, n_heavy_in = 0, n_huge_in = 0;
+    int64_t n_big = 0, n_big_in = 0;   // nodes with more than kBigDeg out- / in-arcs
     // workspace
     DevWork w{};
     uint32_t *amax_dev = nullptr;
@@ -157,11 +157,11 @@ void kgs_free_graph(kgs_graph *g) {
     cudaSetDevice(g->device);
     cudaDeviceSynchronize();
     void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->w.act, g->w.st,
-                    g->w.nm, g->w.M, g->w.ring[0], g->w.ring[1], g->w.ring[2], g->w.fbits, g->w.touched,
+                    g->w.nm, g->w.M, g->w.qlight, g->w.qbig, g->w.pd_bits, g->w.fbits, g->w.touched,
                     g->w.centrals, g->w.cdepth, g->w.ckey, g->w.overflow, g->w.cflag, g->w.sel, g->w.kw_dev,
                     g->w.dpow, g->ctl_pair[0], g->ctl_pair[1], g->w.ans_hdr, g->w.ans_key, g->w.ans_off,
                     g->w.arena_nodes, g->w.arena_arcs, g->w.big_ws, g->amax_dev, g->w.pd_state, g->w.pd_cid,
-                    g->w.pd_touched, g->w.pd_ring[0], g->w.pd_ring[1], g->w.pd_ring[2], g->w.pcnt, g->w.pred_ptr,
+                    g->w.pd_touched, g->w.pd_qlight, g->w.pd_qbig, g->w.pcnt, g->w.pred_ptr,
                     g->w.pred_u, g->w.pred_b, g->w.pa_u, g->w.pa_x, g->w.pa_b, g->w.pa_slot, g->w.scan_tmp};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
@@ -250,12 +250,12 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     G_TRY(launch_degree_class(g->row_ptr, n, g->cls, 0));
     for (int64_t v = 0; v < n; ++v) {
         const int64_t dg_ = rp[v + 1] - rp[v];
-        if (dg_ > kHugeDeg) ++g->n_huge; else if (dg_ > kHeavyDeg) ++g->n_heavy;
+        if (dg_ > kBigDeg) ++g->n_big;
     }
     // reverse CSR for extraction along in-arcs (reading R1)
     if (g->symmetric) {
         g->in_ptr = g->row_ptr; g->in_idx = g->col_idx; g->cls_in = g->cls;
-        g->n_heavy_in = g->n_heavy; g->n_huge_in = g->n_huge;
+        g->n_big_in = g->n_big;
     } else {
         std::vector<int32_t> ci(m);
         if (on_dev) G_TRY(cudaMemcpy(ci.data(), d->col_idx, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
@@ -275,7 +275,7 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         G_TRY(launch_degree_class(g->in_ptr, n, g->cls_in, 0));
         for (int64_t v = 0; v < n; ++v) {
             const int64_t dg_ = ip[v + 1] - ip[v];
-            if (dg_ > kHugeDeg) ++g->n_huge_in; else if (dg_ > kHeavyDeg) ++g->n_heavy_in;
+            if (dg_ > kBigDeg) ++g->n_big_in;
         }
     }
     // per-query workspace sized for n (rings are sized at the first query: they depend on alpha)
@@ -315,14 +315,17 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     G_TRY(cudaMallocHost(&g->h_hdr, sizeof(int32_t) * 4 * KGS_MAX_K));
     G_TRY(cudaMallocHost(&g->h_key, sizeof(double) * KGS_MAX_K));
     G_TRY(cudaMallocHost(&g->h_off, sizeof(long long) * 2 * KGS_MAX_K));
-    w.cap[0] = n; w.cap[1] = g->n_heavy; w.cap[2] = g->n_huge;
+    w.W = ((n + 31) / 32 + 7) / 8 * 8;   // words per bitmap, a multiple of 8 (16-byte vector access)
+    G_TRY(dmalloc(&w.qlight, n));
+    G_TRY(dmalloc(&w.qbig, g->n_big));
     // shared predecessor DAG of the top-down pre-pass
-    w.pd_cap[0] = n; w.pd_cap[1] = g->n_heavy_in; w.pd_cap[2] = g->n_huge_in;
     w.pcap = std::max<int64_t>(std::min<int64_t>(m, int64_t(64) << 20), 1 << 20);
     G_TRY(dmalloc(&w.pd_state, n));
     G_TRY(dmalloc(&w.pd_cid, n));
     G_TRY(dmalloc(&w.pd_touched, n));
-    for (int c = 0; c < 3; ++c) G_TRY(dmalloc(&w.pd_ring[c], 2 * (size_t)std::max<int64_t>(w.pd_cap[c], 1)));
+    G_TRY(dmalloc(&w.pd_bits, 2 * w.W));
+    G_TRY(dmalloc(&w.pd_qlight, n));
+    G_TRY(dmalloc(&w.pd_qbig, g->n_big_in));
     G_TRY(dmalloc(&w.pcnt, n));
     G_TRY(dmalloc(&w.pred_ptr, n + 1));
     G_TRY(dmalloc(&w.pred_u, (size_t)w.pcap));
@@ -332,7 +335,6 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     G_TRY(dmalloc(&w.pa_b, (size_t)w.pcap));
     G_TRY(dmalloc(&w.pa_slot, (size_t)w.pcap));
     G_TRY(dmalloc(&w.scan_tmp, 4096));
-    w.W = (n + 31) / 32;
     g->search_grid = search_max_grid(g->device, g->search_block);
     g->select_grid = select_max_grid(g->device);
     int sms = 148;
@@ -380,11 +382,6 @@ kgs_status enqueue(kgs_graph *g, int32_t q, int32_t k, const kgs_params &p, cuda
     const int R = g->amax + 2;
     if (R > g->R_alloc) {
         CUDA_TRY(cudaStreamSynchronize(s));
-        for (int c = 0; c < 3; ++c) {
-            if (w.ring[c]) cudaFree(w.ring[c]);
-            w.ring[c] = nullptr;
-            CUDA_TRY(dmalloc(&w.ring[c], (size_t)R * (size_t)std::max<int64_t>(w.cap[c], 1)));
-        }
         if (w.fbits) cudaFree(w.fbits);
         CUDA_TRY(dmalloc(&w.fbits, (size_t)R * (size_t)w.W));
         g->R_alloc = R;

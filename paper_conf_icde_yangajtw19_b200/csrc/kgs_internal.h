@@ -11,11 +11,10 @@ namespace kgs {
 constexpr int kMaxQ = KGS_MAX_Q;
 constexpr int kWarp = 32;
 
-// Degree classes for the expansion's load balance: light nodes are expanded by
-// warp batches, heavy ones by a CTA each, huge ones by the whole grid.
-constexpr int64_t kHeavyDeg = 2048;
-constexpr int64_t kHugeDeg = 65536;
-enum : uint8_t { CLS_LIGHT = 0, CLS_HEAVY = 1, CLS_HUGE = 2 };
+// Degree classes for the expansion's load balance: light frontier nodes are
+// expanded by warp batches, big ones (more than kBigDeg arcs) in tiles spread over the whole grid.
+constexpr int64_t kBigDeg = 2048;
+enum : uint8_t { CLS_LIGHT = 0, CLS_BIG = 1 };
 
 // Per-warp shared-memory capacity of the Central Graph extractor.
 constexpr int kExtNodes = 256;
@@ -30,8 +29,8 @@ constexpr int kBigCtas = 64;
 
 // Device control block, zeroed at the start of every query.
 struct Ctl {
-    uint32_t qcount[3][256];       // ring slot counts per degree class
-    uint32_t work[256];            // dynamic work counters per level (light batches)
+    uint32_t slot_flag[256];       // level slot s has pending frontier bits
+    uint32_t qn[2][2];             // [level parity][light, big] compacted frontier sizes
     uint32_t n_central;
     uint32_t n_touched;
     uint32_t n_overflow;
@@ -46,19 +45,17 @@ struct Ctl {
     unsigned long long arcs_scanned;
     unsigned long long hits;       // new (node, keyword) hits (M entries written)
     uint32_t hist[12][256];        // radix-select histograms (one per digit)
-    unsigned long long thr_hi;     // selected threshold (composite key)
-    unsigned long long thr_lo;
     uint32_t sel_count;
     uint32_t pad2;
     unsigned long long arena_used[2];  // emitted nodes / arcs
     // shared predecessor DAG (top-down pre-pass)
-    uint32_t pd_qcount[3][2];
+    uint32_t pd_flag[2];
+    uint32_t pd_qn[2][2];
     uint32_t n_cid;                // nodes of the union of closures that have predecessor lists
     uint32_t n_parcs;              // predecessor arcs found
     unsigned long long td_arcs;    // in-arcs inspected by the pre-pass
     int32_t pd_rounds;
     int32_t pad3;
-    uint32_t pd_work[256];         // dynamic work counters per pre-pass round
     // phase timestamps (%globaltimer, ns) written by thread 0 of the search kernel
     int32_t n_stamp;
     int32_t pad4;
@@ -94,11 +91,11 @@ struct DevWork {
     uint16_t *st;       // [n] low byte: hit mask hm (bit i <=> M[v][i] finite); high byte: gate (0 for K, else a)
     uint32_t *nm;       // [ceil(n/4)] new hits of the current level, one byte per node
     uint8_t *M;         // [n*8] hitting levels, node-major, valid where the hm bit is set
-    int32_t *ring[3];   // per class: [R][cap_c] frontier queues, slot = level % R
-    int64_t cap[3];     // per class capacity (light = n, heavy/huge = number of such nodes)
-    uint32_t *fbits;    // [R][W] frontier membership bitmaps (dedup of pushes)
-    int64_t W;          // words per bitmap
-    int R;              // ring size = amax + 2
+    uint32_t *fbits;    // [R][W] frontier bitmaps, slot = level % R (FIdentifier)
+    int64_t W;          // 32-bit words per bitmap
+    int R;              // ring of level slots = amax + 2
+    int32_t *qlight;    // [n] compacted frontier of the current level, light nodes (ascending ids per CTA)
+    int32_t *qbig;      // [n_big] compacted frontier, big nodes
     int32_t *touched;   // [n] nodes whose hm became non-zero (sparse reset of the next query)
     int32_t *centrals;  // [n] central ids in identification order
     uint8_t *cdepth;    // [n] depth per central
@@ -121,8 +118,9 @@ struct DevWork {
     uint32_t *pd_state;   // [n] byte0 = bits to expand this round, byte1 = bits for the next round, byte2 = done
     int32_t *pd_cid;      // [n] compact id of a node with a predecessor list, -1 otherwise
     int32_t *pd_touched;  // [n] node of each compact id (reset list)
-    int32_t *pd_ring[3];  // per in-degree class: [2][pd_cap_c] round queues
-    int64_t pd_cap[3];
+    uint32_t *pd_bits;    // [2][W] round bitmaps
+    int32_t *pd_qlight;   // [n]
+    int32_t *pd_qbig;     // [n_big_in]
     int32_t *pcnt;        // [n] predecessors per compact id
     int32_t *pred_ptr;    // [n+1] CSR offsets per compact id
     int32_t *pred_u;      // [pcap] predecessor node
@@ -148,7 +146,7 @@ struct QueryArgs {
     int block_central;
     int extract_mode;
     int level_cover;
-    int full_reset;     // 1: reset st for all nodes; 0: only the previous query's touched nodes (w.prev)
+    int full_reset;     // 1: reset all per-node state; 0: only what the previous query (w.prev) touched
     int prev_R;
 };
 

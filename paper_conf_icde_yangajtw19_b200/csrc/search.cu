@@ -2,22 +2,28 @@
 //
 //   k_activation   Eqs. 3-5: w, alpha, A -> uint8 activation level a, cached per alpha.
 //   k_search       Alg. 1 ln 1-7 + Alg. 2 (L244-284) as ONE persistent cooperative kernel:
-//                  reset -> initialise M / sources (L254) -> per level { merge new hits + identify
-//                  central nodes (L262-266, Lemma V.1) -> termination (Def. 4, Thm. V.3) -> expansion
-//                  (Alg. 2, gated by a, L210) } with two grid barriers per level and no host round trip.
+//                  reset -> initialise M / sources (L254) -> per level { enqueue frontiers = compact the
+//                  level's bitmap, merge new hits, identify central nodes (L256-266, Lemma V.1) ->
+//                  termination (Def. 4, Thm. V.3) -> expansion (Alg. 2, gated by a, L210) }, then the
+//                  top-down pre-pass (shared predecessor DAG, see pred_dag), with two grid barriers per
+//                  level and no host round trip.
 //
 // Data layout:
 //   st[v]   uint16: low byte = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of the level),
 //           high byte = gate (0 if v contains a query keyword, else a_v).  One 2-byte load per inspected arc.
 //   nm[v]   uint8 (packed in 32-bit words for atomicOr): bits newly hit during the current level.
 //   M[v*8+i] uint8 hitting level, written once per (v, i) by the thread that set the bit; never reset.
-//   Frontier: three degree-class rings (light / heavy / huge) of R = amax+2 level slots, deduplicated by
-//   a bitmap per slot.  A node is re-queued exactly at the level where it can make progress again:
-//   a_v if it is not yet active (Alg. 2 ln 5-7), gate(n)-1 if a neighbour n is still gated (ln 18-19).
+//   fbits   one frontier bitmap per level slot (R = amax+2 slots): "FIdentifier[v] <- 1 for level L" is one
+//           atomicOr on a bitmap word, so pushes never contend on a queue counter.  A node is re-queued
+//           exactly at the level where it can make progress again: a_v if it is not yet active (Alg. 2
+//           ln 5-7), gate(n)-1 if a neighbour n is still gated (ln 18-19).
+//   Each level starts by compacting its bitmap into light / big queues (block-aggregated appends, node
+//   ids ascending within a CTA's word range); big nodes (> kBigDeg arcs) are expanded in tiles whose arcs
+//   are spread over the whole grid, light ones by warp batches.
 //
 // Snapshot semantics (reading R10): expansion at level l reads hm as of the start of the level; new hits
-// accumulate in nm and are merged in the next merge phase, so the result equals the sequential Alg. 2
-// (Thm. V.2).  All writes are idempotent (bits OR-ed, level l+1 written once).
+// accumulate in nm and are merged when the next level is compacted, so the result equals the sequential
+// Alg. 2 (Thm. V.2).  All writes are idempotent (bits OR-ed, level l+1 written once).
 #include <cooperative_groups.h>
 
 #include "kgs_internal.h"
@@ -64,10 +70,8 @@ cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha,
 }
 
 __global__ void k_degree_class(const int64_t *__restrict__ rp, int64_t n, uint8_t *__restrict__ cls) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t d = rp[v + 1] - rp[v];
-        cls[v] = d > kHugeDeg ? CLS_HUGE : (d > kHeavyDeg ? CLS_HEAVY : CLS_LIGHT);
-    }
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        cls[v] = (rp[v + 1] - rp[v]) > kBigDeg ? CLS_BIG : CLS_LIGHT;
 }
 cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s) {
     if (n > 0) {
@@ -114,7 +118,7 @@ __device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
     return base + rank;
 }
 
-// phase timestamp by the grid's first thread (read back into kgs_stats-like debug output)
+// phase timestamp by the grid's first thread (kgs_result_phases)
 #define KGS_STAMP(tag)                                                                            \
     do {                                                                                          \
         if (gtid == 0) {                                                                          \
@@ -123,22 +127,129 @@ __device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
         }                                                                                         \
     } while (0)
 
-// Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1 for level L).
-__device__ __forceinline__ void push(const QueryArgs &a, int R, int32_t v, int L) {
-    const int s = L % R;
-    uint32_t *word = a.w.fbits + (int64_t)s * a.w.W + (v >> 5);
+__device__ __forceinline__ long long block_excl_scan64(long long x, long long *total, long long *sh) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    long long incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    __syncthreads();
+    if (lane == 31) sh[wid] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long acc = 0;
+        for (int w = 0; w < nw; ++w) { const long long t = sh[w]; sh[w] = acc; acc += t; }
+        sh[32] = acc;
+    }
+    __syncthreads();
+    const long long r = sh[wid] + incl - x;
+    *total = sh[32];
+    __syncthreads();
+    return r;
+}
+
+// ------------------------------------------------------------------------------------------ frontier
+// Set v's bit in bitmap `bits` (one level slot); `flag` records that the slot is non-empty.
+__device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t v) {
+    uint32_t *word = bits + (v >> 5);
     const uint32_t bit = 1u << (v & 31);
     if (__ldcg(word) & bit) return;
-    if (atomicOr(word, bit) & bit) return;
-    const int c = a.g.cls[v];
-    const uint32_t pos = agg_slot(&a.w.ctl->qcount[c][s], (unsigned)((c << 8) | s));
-    a.w.ring[c][(int64_t)s * a.w.cap[c] + pos] = v;
+    if (!(atomicOr(word, bit) & bit) && !__ldcg(flag)) *flag = 1u;
+}
+
+// Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
+__device__ __forceinline__ void push(const QueryArgs &a, int R, int32_t v, int L) {
+    const int s = L % R;
+    set_bit(a.w.fbits + (int64_t)s * a.w.W, &a.w.ctl->slot_flag[s], v);
+}
+
+// Enqueue frontiers: compact a bitmap (which is cleared) into the light / big queues.
+// on_node(v) runs once per set bit and returns whether v goes to the aux list; on_aux(v, pos) runs
+// when v is written there.  Light and aux appends cost one atomic per CTA per tile of blockDim words.
+constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16-byte loads)
+
+template <class OnNode, class OnAux>
+__device__ __forceinline__ void compact(uint32_t *bits, int64_t W, const uint8_t *cls, int32_t *ql, uint32_t *nl,
+                                        int32_t *qb, uint32_t *nb, int32_t *aux, uint32_t *naux, long long *sh,
+                                        OnNode on_node, OnAux on_aux) {
+    const int64_t step = (int64_t)blockDim.x * kWpt;                  // words per CTA iteration
+    const int64_t cw = ((W + gridDim.x - 1) / gridDim.x + kWpt - 1) / kWpt * kWpt;
+    const int64_t w0 = (int64_t)blockIdx.x * cw, w1 = w0 + cw < W ? w0 + cw : W;
+    for (int64_t base = w0; base < w1; base += step) {
+        const int64_t wi = base + (int64_t)threadIdx.x * kWpt;         // multiple of kWpt: 16-byte aligned
+        uint32_t word[kWpt];
+        if (wi + kWpt <= w1) {
+            const uint4 x0 = __ldcg(reinterpret_cast<const uint4 *>(bits + wi));
+            const uint4 x1 = __ldcg(reinterpret_cast<const uint4 *>(bits + wi + 4));
+            word[0] = x0.x; word[1] = x0.y; word[2] = x0.z; word[3] = x0.w;
+            word[4] = x1.x; word[5] = x1.y; word[6] = x1.z; word[7] = x1.w;
+            if ((x0.x | x0.y | x0.z | x0.w) != 0u) *reinterpret_cast<uint4 *>(bits + wi) = make_uint4(0, 0, 0, 0);
+            if ((x1.x | x1.y | x1.z | x1.w) != 0u) *reinterpret_cast<uint4 *>(bits + wi + 4) = make_uint4(0, 0, 0, 0);
+        } else {
+#pragma unroll
+            for (int k = 0; k < kWpt; ++k) {
+                word[k] = (wi + k < w1) ? __ldcg(bits + wi + k) : 0u;
+                if (word[k]) bits[wi + k] = 0u;
+            }
+        }
+        // (A) node ids of the set bits -> the CTA's segment of the frontier queue (stores only)
+        int cnt = 0;
+#pragma unroll
+        for (int k = 0; k < kWpt; ++k) cnt += __popc(word[k]);
+        long long tot;
+        const long long ex = block_excl_scan64(cnt, &tot, sh);
+        if (threadIdx.x == 0) sh[34] = tot ? (long long)atomicAdd(nl, (uint32_t)tot) : 0;
+        __syncthreads();
+        const uint32_t seg0 = (uint32_t)sh[34];
+        uint32_t p = seg0 + (uint32_t)ex;
+#pragma unroll
+        for (int k = 0; k < kWpt; ++k)
+            for (uint32_t m = word[k]; m; m &= m - 1) ql[p++] = (int32_t)((wi + k) * 32 + __ffs(m) - 1);
+        __syncthreads();   // the segment is visible to the whole CTA
+        // (B) one node per thread: on_node (merge / identify), big nodes moved to qb, aux appends
+        for (long long c0 = 0; c0 < tot; c0 += blockDim.x) {
+            const long long j = c0 + threadIdx.x;
+            int32_t v = -1;
+            int flag = 0;
+            if (j < tot) {
+                v = ql[seg0 + j];
+                flag = on_node(v) ? 1 : 0;
+                if (cls[v] != CLS_LIGHT) { qb[atomicAdd(nb, 1u)] = v; ql[seg0 + j] = -1; }
+            }
+            long long atot;
+            const long long aex = block_excl_scan64(flag, &atot, sh);
+            if (threadIdx.x == 0) sh[35] = atot ? (long long)atomicAdd(naux, (uint32_t)atot) : 0;
+            __syncthreads();
+            if (flag) {
+                const uint32_t pos = (uint32_t)sh[35] + (uint32_t)aex;
+                aux[pos] = v;
+                on_aux(v, pos);
+            }
+        }
+    }
+}
+
+// st[v] = a_v << 8 (hit mask 0, gate = a) for v in [0, n), 8 nodes per thread-step
+__device__ __forceinline__ void reset_st_dense(uint16_t *st, const uint8_t *act, int64_t n, int64_t gtid, int64_t gsz) {
+    const int64_t n8 = n / 8;
+    for (int64_t j = gtid; j < n8; j += gsz) {
+        const uint2 av = *reinterpret_cast<const uint2 *>(act + j * 8);
+        uint4 o;
+        o.x = ((av.x & 0xFFu) << 8) | ((av.x & 0xFF00u) << 16);
+        o.y = ((av.x >> 8) & 0xFF00u) | ((av.x >> 24) << 24);
+        o.z = ((av.y & 0xFFu) << 8) | ((av.y & 0xFF00u) << 16);
+        o.w = ((av.y >> 8) & 0xFF00u) | ((av.y >> 24) << 24);
+        *reinterpret_cast<uint4 *>(st + j * 8) = o;
+    }
+    for (int64_t v = n8 * 8 + gtid; v < n; v += gsz) st[v] = (uint16_t)((uint16_t)act[v] << 8);
 }
 
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask).
+// sx = st[x], gathered by the caller.
 __device__ __forceinline__ void visit_arc(const QueryArgs &a, int R, int l, int32_t v, uint32_t hmv, int32_t x,
-                                          unsigned long long &hits) {
-    const uint32_t sx = __ldcg(a.w.st + x);
+                                          uint32_t sx, unsigned &hits) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = sx >> 8;
@@ -176,33 +287,9 @@ __device__ __forceinline__ uint32_t prepare(const QueryArgs &a, int R, int l, ui
 }
 
 // ------------------------------------------------------------------------------------------ load balance
-// Frontier nodes above kHeavyDeg (heavy and huge classes) are expanded in tiles of blockDim entries:
-// every CTA computes the same tile prefix of degrees in shared memory, then the tile's arcs form one
-// index space that all threads of the grid stride over (owner found by binary search).  A hub's arcs
-// are thus spread over the whole GPU instead of one warp or one CTA.
-__device__ __forceinline__ long long block_excl_scan64(long long x, long long *total, long long *sh) {
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
-    long long incl = x;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const long long t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
-    }
-    __syncthreads();
-    if (lane == 31) sh[wid] = incl;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        long long acc = 0;
-        for (int w = 0; w < nw; ++w) { const long long t = sh[w]; sh[w] = acc; acc += t; }
-        sh[32] = acc;
-    }
-    __syncthreads();
-    const long long r = sh[wid] + incl - x;
-    *total = sh[32];
-    __syncthreads();
-    return r;
-}
-
+// Big frontier nodes are expanded in tiles of blockDim entries: every CTA computes the same tile prefix of
+// degrees in shared memory, then the tile's arcs form one index space that all threads of the grid stride
+// over (owner found by binary search).  A hub's arcs are spread over the whole GPU.
 constexpr int kTileMax = 512;   // == blockDim of the persistent kernel
 
 struct FwdNode {
@@ -210,73 +297,146 @@ struct FwdNode {
     uint32_t hm;
 };
 
+struct PdNode {
+    uint32_t P;      // keyword bits to expand backwards
+    uint64_t hx;     // M row of the node
+    int gx;          // gate - 1
+    int32_t cidx;    // compact id
+};
+
 template <class NodeT>
 struct BigTile {
     long long incl[kTileMax];
     long long start[kTileMax];
     NodeT node[kTileMax];
-    long long scan[40];
 };
 
+constexpr int kBigUnroll = 4;
+constexpr int kLightUnroll = 2;
+
 template <class NodeT, class Prep, class Visit>
-__device__ __forceinline__ void expand_big(const int32_t *ring1, uint32_t c1, const int32_t *ring2, uint32_t c2,
-                                           const int64_t *ptr, const int32_t *idx, BigTile<NodeT> &S, int64_t gtid,
+__device__ __forceinline__ void expand_big(const int32_t *qb, uint32_t cb, const int64_t *ptr, const int32_t *idx,
+                                           const uint16_t *st, BigTile<NodeT> &S, long long *sh, int64_t gtid,
                                            int64_t gsz, Prep prep, Visit visit, unsigned long long &arcs) {
-    const uint32_t cb = c1 + c2;
     for (uint32_t t0 = 0; t0 < cb; t0 += blockDim.x) {
         const int nt = (int)min((uint32_t)blockDim.x, cb - t0);
         const int j = threadIdx.x;
-        long long deg = 0, st = 0;
+        long long deg = 0, s0 = 0;
         if (j < nt) {
-            const uint32_t e = t0 + j;
-            const int32_t v = e < c1 ? ring1[e] : ring2[e - c1];
+            const int32_t v = __ldcg(qb + t0 + j);
             NodeT nd;
-            if (prep(v, blockIdx.x == 0, nd)) { st = ptr[v]; deg = ptr[v + 1] - st; }
+            if (prep(v, blockIdx.x == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
             S.node[j] = nd;
-            S.start[j] = st;
+            S.start[j] = s0;
         }
         long long T;
-        const long long ex = block_excl_scan64(deg, &T, S.scan);
+        const long long ex = block_excl_scan64(deg, &T, sh);
         S.incl[j] = ex + deg;
         __syncthreads();
         if (gtid == 0) arcs += (unsigned long long)T;
-        for (long long e = gtid; e < T; e += gsz) {
-            int lo = 0, hi = nt - 1;
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (S.incl[mid] > e) hi = mid; else lo = mid + 1;
+        // kBigUnroll arcs per thread per step: the index and status gathers of all of them are issued
+        // before any of them is processed (memory-level parallelism for a latency-bound loop)
+        for (long long e = gtid; e < T; e += kBigUnroll * gsz) {
+            int own[kBigUnroll];
+            int32_t x[kBigUnroll];
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k) {
+                const long long ek = e + k * gsz;
+                own[k] = -1;
+                x[k] = 0;
+                if (ek < T) {
+                    int lo = 0, hi = nt - 1;
+                    while (lo < hi) {
+                        const int mid = (lo + hi) >> 1;
+                        if (S.incl[mid] > ek) hi = mid; else lo = mid + 1;
+                    }
+                    const long long exo = lo ? S.incl[lo - 1] : 0;
+                    own[k] = lo;
+                    x[k] = __ldcs(idx + S.start[lo] + (ek - exo));
+                }
             }
-            const long long exo = lo ? S.incl[lo - 1] : 0;
-            visit(S.node[lo], __ldcs(idx + S.start[lo] + (e - exo)));
+            uint32_t sx[kBigUnroll];
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k) sx[k] = own[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k)
+                if (own[k] >= 0) visit(S.node[own[k]], x[k], sx[k]);
         }
         __syncthreads();
     }
 }
 
-// light-batch size: 32 frontier nodes per warp when the frontier is large, fewer (down to 1) when it
-// is small, so that every warp of the grid gets work
-__device__ __forceinline__ uint32_t light_batch(uint32_t c0, int64_t gsz) {
+// Light frontier nodes: warp w takes batches w, w + #warps, ... of B nodes each (no shared counter);
+// the batch's arcs are balanced over the 32 lanes by a warp scan and a shuffle binary search.
+// B = 32 when the frontier is large, fewer (down to 1) when it is small so that every warp gets work.
+template <class NodeT, class Prep, class Visit>
+__device__ __forceinline__ void expand_light(const int32_t *ql, uint32_t c0, const int64_t *ptr, const int32_t *idx,
+                                             const uint16_t *st, int64_t gtid, int64_t gsz, Prep prep, Visit visit,
+                                             unsigned long long &arcs) {
     const uint32_t warps = (uint32_t)(gsz >> 5);
-    uint32_t b = (c0 + 2 * warps - 1) / (2 * warps);
-    return b < 1 ? 1u : (b > 32 ? 32u : b);
+    uint32_t B = (c0 + 2 * warps - 1) / (2 * warps);
+    B = B < 1 ? 1u : (B > 32 ? 32u : B);
+    const uint32_t nbatch = (c0 + B - 1) / B;
+    const unsigned lane = lane_id();
+    for (uint32_t bi = (uint32_t)(gtid >> 5); bi < nbatch; bi += warps) {
+        const uint32_t i = bi * B + lane;
+        NodeT nd{};
+        int64_t start = 0;
+        int deg = 0;
+        if (lane < B && i < c0) {
+            const int32_t v = __ldcg(ql + i);   // -1: a big node, expanded by expand_big
+            if (v >= 0 && prep(v, true, nd)) { start = ptr[v]; deg = (int)(ptr[v + 1] - start); }
+        }
+        int incl = deg;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if ((int)lane >= o) incl += t;
+        }
+        const int tot = __shfl_sync(0xffffffffu, incl, 31);
+        if (lane == 0) arcs += (unsigned long long)tot;
+        const int excl = incl - deg;
+        for (int e0 = 0; e0 < tot; e0 += 32 * kLightUnroll) {
+            NodeT no[kLightUnroll];
+            int32_t x[kLightUnroll];
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k) {
+                const int e = e0 + 32 * k + (int)lane;
+                int pos = 0;
+#pragma unroll
+                for (int bb = 16; bb > 0; bb >>= 1) {
+                    const int val = __shfl_sync(0xffffffffu, incl, pos + bb - 1);
+                    if (val <= e) pos += bb;
+                }
+                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
+                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
+                const uint32_t *src = reinterpret_cast<const uint32_t *>(&nd);
+                uint32_t *dst = reinterpret_cast<uint32_t *>(&no[k]);
+#pragma unroll
+                for (int w = 0; w < (int)(sizeof(NodeT) / 4); ++w) dst[w] = __shfl_sync(0xffffffffu, src[w], pos);
+                x[k] = e < tot ? __ldcs(idx + st_o + (e - ex_o)) : -1;
+            }
+            uint32_t sx[kLightUnroll];
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k) sx[k] = x[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k)
+                if (x[k] >= 0) visit(no[k], x[k], sx[k]);
+        }
+    }
 }
 
 // ------------------------------------------------------------------------------------------ pre-pass
 // Shared predecessor DAG (top-down): whether u -> x is a B_i-predecessor arc
 // (Thm. V.4 + reading R12) depends only on M, a and K, never on the central node whose graph is being
-// extracted.  So the backward closure of ALL central nodes is computed once, level by level, with the
-// same degree-balanced scheme as the expansion, and every arc that passes the test is stored in a CSR
-// keyed by its successor.  Each Central Graph is then a walk over these short lists (topdown.cu).
-__device__ __forceinline__ void pd_push(const QueryArgs &a, int slot, int32_t u) {
-    const int c = a.g.cls_in[u];
-    const uint32_t pos = agg_slot(&a.w.ctl->pd_qcount[c][slot], (unsigned)((c << 8) | slot));
-    a.w.pd_ring[c][(int64_t)slot * a.w.pd_cap[c] + pos] = u;
-}
+// extracted.  So the backward closure of ALL central nodes is computed once, round by round, with the
+// same load balancing as the expansion, and every arc that passes the test is stored in a CSR keyed by
+// its successor.  Each Central Graph is then a walk over these short lists (topdown.cu).
 
 // Thm. V.4 test of in-arc u -> x for the keyword bits P of x (hx = M row of x, gx = gate(x) - 1).
 __device__ __forceinline__ uint32_t pred_test(const QueryArgs &a, uint32_t full, bool exact_block, uint32_t P,
-                                              uint64_t hx, int gx, int32_t u, uint32_t &zbu) {
-    const uint32_t hmu = __ldcg(a.w.st + u) & 0xFFu;
+                                              uint64_t hx, int gx, int32_t u, uint32_t su, uint32_t &zbu) {
+    const uint32_t hmu = su & 0xFFu;   // su = st[u], gathered by the caller
     const uint32_t cand = P & hmu;
     if (!cand) return 0;
     const int au = a.w.act[u];
@@ -303,16 +463,16 @@ __device__ __forceinline__ uint32_t pred_test(const QueryArgs &a, uint32_t full,
     return pb;
 }
 
-__device__ __forceinline__ void pd_visit(const QueryArgs &a, uint32_t full, bool exact_block, uint32_t P, uint64_t hx,
-                                         int gx, int32_t cidx, int32_t u, int nslot) {
+__device__ __forceinline__ void pd_visit(const QueryArgs &a, uint32_t full, bool exact_block, const PdNode &nd,
+                                         int32_t u, uint32_t su, uint32_t *nbits, uint32_t *nflag) {
     uint32_t zbu = 0;
-    const uint32_t pb = pred_test(a, full, exact_block, P, hx, gx, u, zbu);
+    const uint32_t pb = pred_test(a, full, exact_block, nd.P, nd.hx, nd.gx, u, su, zbu);
     if (!pb) return;
-    const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(a.w.pcnt + cidx), (unsigned)cidx);
+    const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(a.w.pcnt + nd.cidx), (unsigned)nd.cidx);
     const uint32_t ai = agg_slot(&a.w.ctl->n_parcs, 0xFFFFFFFFu);
     if ((int64_t)ai < a.w.pcap) {
         a.w.pa_u[ai] = u;
-        a.w.pa_x[ai] = cidx;
+        a.w.pa_x[ai] = nd.cidx;
         a.w.pa_b[ai] = (uint16_t)(pb | (zbu << 8));
         a.w.pa_slot[ai] = (int32_t)pos;
     } else {
@@ -321,53 +481,31 @@ __device__ __forceinline__ void pd_visit(const QueryArgs &a, uint32_t full, bool
     const uint32_t nb = pb & ~zbu;        // sources (m = 0) have no predecessors
     if (nb) {
         const uint32_t old = atomicOr(a.w.pd_state + u, nb << 8);
-        if (((old >> 8) & 0xFFu) == 0) pd_push(a, nslot, u);
+        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u);
     }
 }
 
-struct PdNode {
-    uint32_t P;
-    uint64_t hx;
-    int gx;
-    int32_t cidx;
-};
-
-__device__ __forceinline__ PdNode pd_prepare(const QueryArgs &a, int32_t x) {
-    PdNode nd;
+__device__ __forceinline__ bool pd_prepare(const QueryArgs &a, int32_t x, PdNode &nd) {
     nd.P = __ldcg(a.w.pd_state + x) & 0xFFu;
     nd.hx = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + x);
     nd.gx = (int)(__ldcg(a.w.st + x) >> 8) - 1;
     nd.cidx = __ldcg(a.w.pd_cid + x);
-    return nd;
+    return nd.P != 0;
 }
 
-__device__ __forceinline__ int block_excl_scan(int x, int *total, int *sh) {
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
-    int incl = x;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
-    }
-    __syncthreads();
-    if (lane == 31) sh[wid] = incl;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int acc = 0;
-        for (int w = 0; w < nw; ++w) { const int t = sh[w]; sh[w] = acc; acc += t; }
-        sh[32] = acc;
-    }
-    __syncthreads();
-    const int r = sh[wid] + incl - x;
-    *total = sh[32];
-    __syncthreads();
-    return r;
+__device__ __forceinline__ int block_excl_scan(int x, int *total, long long *sh) {
+    long long t;
+    const long long r = block_excl_scan64((long long)x, &t, sh);
+    *total = (int)t;
+    return (int)r;
 }
 
-__device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid, int64_t gsz, uint32_t full) {
+__device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid, int64_t gsz, uint32_t full,
+                         long long *sh) {
     Ctl *ctl = a.w.ctl;
     const bool exact_block = a.extract_mode == KGS_EXTRACT_EXACT && a.block_central;
     const uint32_t nc = __ldcg(&ctl->n_central);
+    const int64_t W = a.w.W;
     __shared__ BigTile<PdNode> s_bigb;
     // seeds: every central node, for every keyword it did not contain itself
     for (int64_t j = gtid; j < nc; j += gsz) {
@@ -376,7 +514,7 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
         uint32_t zbc = 0;
         for (int i = 0; i < a.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
         const uint32_t bits = full & ~zbc;
-        if (bits) { atomicOr(a.w.pd_state + c, bits << 8); pd_push(a, 0, c); }
+        if (bits) { atomicOr(a.w.pd_state + c, bits << 8); set_bit(a.w.pd_bits, &ctl->pd_flag[0], c); }
     }
     grid.sync();
     KGS_STAMP(TS_PD_SEED);
@@ -384,89 +522,38 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
     int r = 0;
     for (;; ++r) {
         const int slot = r & 1;
-        const uint32_t c0 = __ldcg(&ctl->pd_qcount[0][slot]), c1 = __ldcg(&ctl->pd_qcount[1][slot]),
-                       c2 = __ldcg(&ctl->pd_qcount[2][slot]);
-        const int64_t total = (int64_t)c0 + c1 + c2;
-        if (total == 0) break;
-        if (gtid == 0) { ctl->pd_qcount[0][slot ^ 1] = 0; ctl->pd_qcount[1][slot ^ 1] = 0; ctl->pd_qcount[2][slot ^ 1] = 0; }
+        if (!__ldcg(&ctl->pd_flag[slot])) break;
+        uint32_t *qn = ctl->pd_qn[slot];
+        if (gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; }
         // merge: bits to expand this round = newly requested bits not expanded before
-        for (int64_t j = gtid; j < total; j += gsz) {
-            int32_t u;
-            if (j < c0) u = a.w.pd_ring[0][(int64_t)slot * a.w.pd_cap[0] + j];
-            else if (j < (int64_t)c0 + c1) u = a.w.pd_ring[1][(int64_t)slot * a.w.pd_cap[1] + (j - c0)];
-            else u = a.w.pd_ring[2][(int64_t)slot * a.w.pd_cap[2] + (j - c0 - c1)];
-            const uint32_t s = __ldcg(a.w.pd_state + u);
-            const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
-            const uint32_t bits = nx & ~dn;
-            a.w.pd_state[u] = bits | ((dn | bits) << 16);
-            if (bits && __ldcg(a.w.pd_cid + u) < 0) {
-                const uint32_t cid = agg_slot(&ctl->n_cid, 1u);
-                a.w.pd_cid[u] = (int32_t)cid;
-                a.w.pd_touched[cid] = u;
-            }
-        }
+        compact(a.w.pd_bits + (int64_t)slot * W, W, a.g.cls_in, a.w.pd_qlight, &qn[0], a.w.pd_qbig, &qn[1],
+                a.w.pd_touched, &ctl->n_cid, sh,
+                [&](int32_t u) {
+                    const uint32_t s = __ldcg(a.w.pd_state + u);
+                    const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
+                    const uint32_t bits = nx & ~dn;
+                    a.w.pd_state[u] = bits | ((dn | bits) << 16);
+                    return bits != 0 && __ldcg(a.w.pd_cid + u) < 0;
+                },
+                [&](int32_t u, uint32_t pos) { a.w.pd_cid[u] = (int32_t)pos; });
         grid.sync();
         KGS_STAMP(TS_PD_MERGE);
-        const int ns = slot ^ 1;
-        // heavy and huge nodes: tiles spread over the whole grid
-        expand_big(a.w.pd_ring[1] + (int64_t)slot * a.w.pd_cap[1], c1, a.w.pd_ring[2] + (int64_t)slot * a.w.pd_cap[2],
-                   c2, a.g.in_ptr, a.g.in_idx, s_bigb, gtid, gsz,
-                   [&](int32_t x, bool, PdNode &nd) {
-                       nd = pd_prepare(a, x);
-                       return nd.P != 0;
-                   },
-                   [&](const PdNode &nd, int32_t u) { pd_visit(a, full, exact_block, nd.P, nd.hx, nd.gx, nd.cidx, u, ns); },
-                   my_arcs);
-        const unsigned lane = lane_id();
-        const uint32_t B = light_batch(c0, gsz);
-        for (;;) {                                                 // light: warp batches
-            uint32_t base = 0;
-            if (lane == 0) base = atomicAdd(&ctl->pd_work[r & 255], B);
-            base = __shfl_sync(0xffffffffu, base, 0);
-            if (base >= c0) break;
-            const uint32_t idx = base + lane;
-            PdNode nd{0, 0, 0, -1};
-            int64_t start = 0;
-            int deg = 0;
-            if (lane < B && idx < c0) {
-                const int32_t x = a.w.pd_ring[0][(int64_t)slot * a.w.pd_cap[0] + idx];
-                nd = pd_prepare(a, x);
-                if (nd.P) { start = a.g.in_ptr[x]; deg = (int)(a.g.in_ptr[x + 1] - start); }
-            }
-            int incl = deg;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int t = __shfl_up_sync(0xffffffffu, incl, o);
-                if ((int)lane >= o) incl += t;
-            }
-            const int tot = __shfl_sync(0xffffffffu, incl, 31);
-            if (lane == 0) my_arcs += (unsigned long long)tot;
-            const int excl = incl - deg;
-            for (int e0 = 0; e0 < tot; e0 += 32) {
-                const int e = e0 + (int)lane;
-                int pos = 0;
-#pragma unroll
-                for (int bb = 16; bb > 0; bb >>= 1) {
-                    const int val = __shfl_sync(0xffffffffu, incl, pos + bb - 1);
-                    if (val <= e) pos += bb;
-                }
-                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
-                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
-                const uint32_t P_o = __shfl_sync(0xffffffffu, nd.P, pos);
-                const uint64_t hx_o = __shfl_sync(0xffffffffu, (unsigned long long)nd.hx, pos);
-                const int gx_o = __shfl_sync(0xffffffffu, nd.gx, pos);
-                const int32_t cid_o = __shfl_sync(0xffffffffu, nd.cidx, pos);
-                if (e < tot)
-                    pd_visit(a, full, exact_block, P_o, hx_o, gx_o, cid_o, __ldcs(a.g.in_idx + st_o + (e - ex_o)), ns);
-            }
-        }
+        const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
+        if (gtid == 0) ctl->pd_flag[slot] = 0u;   // read by every thread before the barrier above
+        uint32_t *nbits = a.w.pd_bits + (int64_t)(slot ^ 1) * W;
+        uint32_t *nflag = &ctl->pd_flag[slot ^ 1];
+        auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(a, x, nd); };
+        auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) {
+            pd_visit(a, full, exact_block, nd, u, su, nbits, nflag);
+        };
+        expand_big(a.w.pd_qbig, c1, a.g.in_ptr, a.g.in_idx, a.w.st, s_bigb, sh, gtid, gsz, prep, visit, my_arcs);
+        expand_light<PdNode>(a.w.pd_qlight, c0, a.g.in_ptr, a.g.in_idx, a.w.st, gtid, gsz, prep, visit, my_arcs);
         grid.sync();
         KGS_STAMP(TS_PD_EXPAND);
     }
     if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
     if (gtid == 0) ctl->pd_rounds = r;
     // CSR of the predecessor lists: exclusive scan of pcnt over compact ids, then scatter
-    __shared__ int sh[40];
     const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
     const int64_t chunk = (ncid + gridDim.x - 1) / gridDim.x;
     const int64_t lo = (int64_t)blockIdx.x * chunk, hi = lo + chunk < ncid ? lo + chunk : ncid;
@@ -481,7 +568,7 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
     }
     if (threadIdx.x == 0) a.w.scan_tmp[blockIdx.x] = run;
     grid.sync();
-    if (blockIdx.x == 0) {   // exclusive scan of the per-CTA sums (gridDim <= a few blockDim)
+    if (blockIdx.x == 0) {   // exclusive scan of the per-CTA sums
         int carry = 0;
         for (unsigned b0 = 0; b0 < gridDim.x; b0 += blockDim.x) {
             const unsigned b = b0 + threadIdx.x;
@@ -512,6 +599,7 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     const int64_t gtid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t gsz = (int64_t)gridDim.x * blockDim.x;
     const int64_t n = a.g.n;
+    const int64_t W = a.w.W;
     const int R = a.w.R;
     const int amax = R - 2;
     const uint32_t full = (1u << a.q) - 1u;
@@ -519,38 +607,35 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     uint8_t *st8 = reinterpret_cast<uint8_t *>(a.w.st);
     uint8_t *nm8 = reinterpret_cast<uint8_t *>(a.w.nm);
     __shared__ BigTile<FwdNode> s_big;
+    __shared__ long long sh[40];
     KGS_STAMP(TS_START);
 
     // ---- reset the state the previous query left behind
     if (a.full_reset) {
-        for (int64_t v = gtid; v < n; v += gsz) a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
+        reset_st_dense(a.w.st, a.w.act, n, gtid, gsz);
         for (int64_t v = gtid; v < (n + 3) / 4; v += gsz) a.w.nm[v] = 0u;
-        for (int64_t j = gtid; j < (int64_t)R * a.w.W; j += gsz) a.w.fbits[j] = 0u;
+        for (int64_t j = gtid; j < (int64_t)R * W; j += gsz) a.w.fbits[j] = 0u;
+        for (int64_t j = gtid; j < 2 * W; j += gsz) a.w.pd_bits[j] = 0u;
         for (int64_t v = gtid; v < n; v += gsz) { a.w.pd_state[v] = 0u; a.w.pd_cid[v] = -1; a.w.pcnt[v] = 0; }
     } else {
-        for (int64_t j = gtid; j < (int64_t)a.w.prev->n_cid; j += gsz) {
+        const Ctl *pv = a.w.prev;
+        for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
             const int32_t v = a.w.pd_touched[j];
             a.w.pd_state[v] = 0u; a.w.pd_cid[v] = -1; a.w.pcnt[j] = 0;
         }
-        const Ctl *pv = a.w.prev;
         const int64_t pt = (int64_t)pv->n_touched;
         if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
-            for (int64_t v = gtid; v < n; v += gsz) a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
-        } else
-        for (int64_t j = gtid; j < pt; j += gsz) {
-            const int32_t v = a.w.touched[j];
-            a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
-        }
-        for (int c = 0; c < 3; ++c)
-            for (int s = 0; s < a.prev_R; ++s) {
-                const uint32_t cnt = pv->qcount[c][s];
-                for (int64_t j = gtid; j < (int64_t)cnt; j += gsz) {
-                    const int32_t v = a.w.ring[c][(int64_t)s * a.w.cap[c] + j];
-                    a.w.fbits[(int64_t)s * a.w.W + (v >> 5)] = 0u;
-                }
+            reset_st_dense(a.w.st, a.w.act, n, gtid, gsz);
+        } else {
+            for (int64_t j = gtid; j < pt; j += gsz) {
+                const int32_t v = a.w.touched[j];
+                a.w.st[v] = (uint16_t)((uint16_t)a.w.act[v] << 8);
             }
+        }
+        for (int s = 0; s < a.prev_R; ++s)   // level slots still pending when the previous query stopped
+            if (pv->slot_flag[s])
+                for (int64_t j = gtid; j < W; j += gsz) a.w.fbits[(int64_t)s * W + j] = 0u;
     }
-    // ---- initialisation (P:L254): M = 0 on T_i, keyword nodes ungated, F_0 = K
     bool empty = false;
     for (int i = 0; i < a.q; ++i) {
         const int32_t t = a.w.kw_dev[i];
@@ -558,11 +643,19 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     }
     grid.sync();
     KGS_STAMP(TS_RESET);
-    for (int i = 0; i < a.q; ++i) {
-        const int32_t t = a.w.kw_dev[i];
-        const int64_t b = a.g.kw_ptr[t], e = a.g.kw_ptr[t + 1];
-        for (int64_t j = b + gtid; j < e; j += gsz) {
-            const int32_t v = a.g.kw_nodes[j];
+    // ---- initialisation (P:L254): M = 0 on T_i, keyword nodes ungated, F_0 = K
+    {   // one flat grid-stride loop over the concatenation T_0 | T_1 | ... | T_{q-1}
+        int64_t kb[kMaxQ], ko[kMaxQ + 1];
+        ko[0] = 0;
+        for (int i = 0; i < a.q; ++i) {
+            const int32_t t = a.w.kw_dev[i];
+            kb[i] = a.g.kw_ptr[t];
+            ko[i + 1] = ko[i] + (a.g.kw_ptr[t + 1] - kb[i]);
+        }
+        for (int64_t j = gtid; j < ko[a.q]; j += gsz) {
+            int i = 0;
+            while (j >= ko[i + 1]) ++i;
+            const int32_t v = a.g.kw_nodes[kb[i] + (j - ko[i])];
             a.w.M[(int64_t)v * 8 + i] = 0;
             st8[2 * (int64_t)v + 1] = 0;                                  // keyword node: no gate (L210)
             atomicOr(a.w.nm + (v >> 2), (1u << i) << ((v & 3) * 8));      // hit in B_i at level 0
@@ -572,51 +665,42 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
     grid.sync();
     KGS_STAMP(TS_SCATTER);
 
-    unsigned long long my_arcs = 0, my_hits = 0;
+    unsigned long long my_arcs = 0;
+    unsigned my_hits = 0;
     for (int l = 0;; ++l) {
         // ---- enqueue frontiers: anything pending at this or a later level?
-        uint32_t pend = 0;
+        bool pend = false;
         const int top = l > amax ? l : amax;
-        for (int L = l; L <= top; ++L) {
-            const int s = L % R;
-            pend += __ldcg(&ctl->qcount[0][s]) + __ldcg(&ctl->qcount[1][s]) + __ldcg(&ctl->qcount[2][s]);
-        }
-        if (pend == 0) {
+        for (int L = l; L <= top; ++L) pend |= __ldcg(&ctl->slot_flag[L % R]) != 0u;
+        if (!pend) {
             if (gtid == 0) { ctl->stop_reason = empty ? KGS_STOP_EMPTY_KEYWORD : KGS_STOP_EXHAUSTED; ctl->levels = l; }
             break;
         }
         const int s = l % R;
-        const uint32_t c0 = __ldcg(&ctl->qcount[0][s]), c1 = __ldcg(&ctl->qcount[1][s]),
-                       c2 = __ldcg(&ctl->qcount[2][s]);
-        const int64_t total = (int64_t)c0 + c1 + c2;
-        // ---- merge new hits into hm and identify central nodes (only frontiers can change, L262)
-        for (int64_t j = gtid; j < total; j += gsz) {
-            int32_t v;
-            if (j < c0) v = a.w.ring[0][(int64_t)s * a.w.cap[0] + j];
-            else if (j < (int64_t)c0 + c1) v = a.w.ring[1][(int64_t)s * a.w.cap[1] + (j - c0)];
-            else v = a.w.ring[2][(int64_t)s * a.w.cap[2] + (j - c0 - c1)];
-            a.w.fbits[(int64_t)s * a.w.W + (v >> 5)] = 0u;
-            const uint32_t b = nm8[v];
-            if (b) {
-                nm8[v] = 0;
-                const uint32_t old = st8[2 * (int64_t)v];
-                const uint32_t nw = old | b;
-                st8[2 * (int64_t)v] = (uint8_t)nw;
-                if (old == 0) a.w.touched[agg_slot(&ctl->n_touched, 0u)] = v;
-                if (nw == full && old != full) {                            // Lemma V.1: depth = l
-                    const uint32_t ci = agg_slot(&ctl->n_central, 1u);
-                    a.w.centrals[ci] = v;
-                    a.w.cdepth[ci] = (uint8_t)l;
-                }
-            }
-        }
-        if (gtid == 0) ctl->frontier_total += (unsigned long long)total;
+        uint32_t *qn = ctl->qn[l & 1];
+        if (gtid == 0) { ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; }
+        // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
+        compact(a.w.fbits + (int64_t)s * W, W, a.g.cls, a.w.qlight, &qn[0], a.w.qbig, &qn[1], a.w.touched,
+                &ctl->n_touched, sh,
+                [&](int32_t v) {
+                    const uint32_t b = nm8[v];
+                    if (!b) return false;
+                    nm8[v] = 0;
+                    const uint32_t old = st8[2 * (int64_t)v];
+                    const uint32_t nw = old | b;
+                    st8[2 * (int64_t)v] = (uint8_t)nw;
+                    if (nw == full && old != full) {                        // Lemma V.1: depth = l
+                        const uint32_t ci = agg_slot(&ctl->n_central, 1u);
+                        a.w.centrals[ci] = v;
+                        a.w.cdepth[ci] = (uint8_t)l;
+                    }
+                    return old == 0;
+                },
+                [&](int32_t, uint32_t) {});
         grid.sync();
         KGS_STAMP(TS_MERGE);
-        if (gtid == 0 && l > 0) {
-            const int sp = (l - 1) % R;
-            ctl->qcount[0][sp] = 0; ctl->qcount[1][sp] = 0; ctl->qcount[2][sp] = 0;
-        }
+        const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
+        if (gtid == 0) ctl->frontier_total += (unsigned long long)c0 + c1;
         // ---- termination (Def. 4 / Thm. V.3; reading R9: no expansion at d)
         if (empty) {   // some T_i is empty: M holds the initialisation, nothing can be central (R17)
             if (gtid == 0) { ctl->stop_reason = KGS_STOP_EMPTY_KEYWORD; ctl->levels = 0; ctl->empty_keyword = 1; }
@@ -632,72 +716,36 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
             break;
         }
         // ---- expansion (Alg. 2)
-        // heavy and huge nodes: tiles whose arcs are spread over the whole grid
-        expand_big(a.w.ring[1] + (int64_t)s * a.w.cap[1], c1, a.w.ring[2] + (int64_t)s * a.w.cap[2], c2,
-                   a.g.row_ptr, a.g.col_idx, s_big, gtid, gsz,
-                   [&](int32_t v, bool leader, FwdNode &nd) {
-                       nd.v = v;
-                       nd.hm = prepare(a, R, l, full, v, leader);
-                       return nd.hm != 0;
-                   },
-                   [&](const FwdNode &nd, int32_t x) { visit_arc(a, R, l, nd.v, nd.hm, x, my_hits); }, my_arcs);
-        // light nodes: dynamic batches of frontier nodes per warp, arcs balanced across the lanes
-        const unsigned lane = lane_id();
-        const uint32_t B = light_batch(c0, gsz);
-        for (;;) {
-            uint32_t base = 0;
-            if (lane == 0) base = atomicAdd(&ctl->work[l], B);
-            base = __shfl_sync(0xffffffffu, base, 0);
-            if (base >= c0) break;
-            const uint32_t idx = base + lane;
-            int32_t v = -1;
-            uint32_t hm = 0;
-            int64_t start = 0;
-            int deg = 0;
-            if (lane < B && idx < c0) {
-                v = a.w.ring[0][(int64_t)s * a.w.cap[0] + idx];
-                hm = prepare(a, R, l, full, v, true);
-                if (hm) {
-                    start = a.g.row_ptr[v];
-                    deg = (int)(a.g.row_ptr[v + 1] - start);
-                }
-            }
-            int incl = deg;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int t = __shfl_up_sync(0xffffffffu, incl, o);
-                if ((int)lane >= o) incl += t;
-            }
-            const int tot = __shfl_sync(0xffffffffu, incl, 31);
-            if (lane == 0) my_arcs += (unsigned long long)tot;
-            const int excl = incl - deg;
-            for (int e0 = 0; e0 < tot; e0 += 32) {
-                const int e = e0 + (int)lane;
-                int pos = 0;
-#pragma unroll
-                for (int b = 16; b > 0; b >>= 1) {
-                    const int val = __shfl_sync(0xffffffffu, incl, pos + b - 1);
-                    if (val <= e) pos += b;
-                }
-                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
-                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
-                const uint32_t hm_o = __shfl_sync(0xffffffffu, hm, pos);
-                const int32_t v_o = __shfl_sync(0xffffffffu, v, pos);
-                if (e < tot) visit_arc(a, R, l, v_o, hm_o, __ldcs(a.g.col_idx + st_o + (e - ex_o)), my_hits);
-            }
-        }
+        // slot s is consumed; nothing pushes to level l + R during this level (pushes reach <= max(l+1, amax))
+        if (gtid == 0) ctl->slot_flag[s] = 0u;
+        auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
+            nd.v = v;
+            nd.hm = prepare(a, R, l, full, v, leader);
+            return nd.hm != 0;
+        };
+        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(a, R, l, nd.v, nd.hm, x, sx, my_hits); };
+        expand_big(a.w.qbig, c1, a.g.row_ptr, a.g.col_idx, a.w.st, s_big, sh, gtid, gsz, prep, visit, my_arcs);
+        expand_light<FwdNode>(a.w.qlight, c0, a.g.row_ptr, a.g.col_idx, a.w.st, gtid, gsz, prep, visit, my_arcs);
         grid.sync();
         KGS_STAMP(TS_EXPAND);
     }
-    my_arcs = __reduce_add_sync(0xffffffffu, (unsigned)my_arcs) + 0ull;   // per-warp totals fit 32 bits
-    my_hits = __reduce_add_sync(0xffffffffu, (unsigned)my_hits) + 0ull;
+    const unsigned wa = __reduce_add_sync(0xffffffffu, (unsigned)my_arcs);   // per-warp totals fit 32 bits
+    const unsigned wh = __reduce_add_sync(0xffffffffu, my_hits);
+    __shared__ unsigned long long s_sum[2];
+    if (threadIdx.x < 2) s_sum[threadIdx.x] = 0ull;
+    __syncthreads();
     if ((threadIdx.x & 31) == 0) {
-        if (my_arcs) atomicAdd(&ctl->arcs_scanned, my_arcs);
-        if (my_hits) atomicAdd(&ctl->hits, my_hits);
+        if (wa) atomicAdd(&s_sum[0], (unsigned long long)wa);
+        if (wh) atomicAdd(&s_sum[1], (unsigned long long)wh);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {      // one global atomic per CTA
+        if (s_sum[0]) atomicAdd(&ctl->arcs_scanned, s_sum[0]);
+        if (s_sum[1]) atomicAdd(&ctl->hits, s_sum[1]);
     }
     grid.sync();
     KGS_STAMP(TS_END);
-    pred_dag(a, grid, gtid, gsz, full);
+    pred_dag(a, grid, gtid, gsz, full, sh);
 }
 
 int search_max_grid(int device, int block) {
