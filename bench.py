@@ -120,6 +120,62 @@ def build_workload(name: str, rank: int, world: int):
     return w, time.time() - t0
 
 
+class _RemoteGraph:
+    """Sizes of a graph received from rank 0 (host arrays stay on rank 0)."""
+
+    def __init__(self, n, n_arcs):
+        self.n, self.n_arcs = n, n_arcs
+
+
+def load_replicated(name, rank, world, dev, kgs):
+    """Rank 0 generates the workload once; every rank receives the arrays over NCCL (device to device)
+    and loads its replica from device pointers (KGS_INPUT_DEVICE_PTRS)."""
+    import torch
+    import torch.distributed as dist
+    from types import SimpleNamespace
+    t0 = time.time()
+    cuda = f"cuda:{dev}"
+    if rank == 0:
+        w, _ = build_workload(name, 0, 1)
+        g = w.graph
+        qmax = max(len(q) for q in w.queries)
+        meta = torch.tensor([g.n, g.n_arcs, g.n_keywords, g.kw_nodes.shape[0], len(w.queries), qmax, w.k],
+                            dtype=torch.int64, device=cuda)
+        A = torch.tensor([g.A], dtype=torch.float64, device=cuda)
+    else:
+        meta = torch.zeros(7, dtype=torch.int64, device=cuda)
+        A = torch.zeros(1, dtype=torch.float64, device=cuda)
+    dist.broadcast(meta, 0)
+    dist.broadcast(A, 0)
+    n, m, V, P, nq, qmax, k = (int(x) for x in meta.tolist())
+    if rank == 0:
+        t = [torch.from_numpy(g.row_ptr).to(cuda), torch.from_numpy(g.col_idx).to(cuda),
+             torch.from_numpy(g.weight).to(cuda), torch.from_numpy(g.kw_ptr).to(cuda),
+             torch.from_numpy(g.kw_nodes).to(cuda)]
+        qt = torch.full((nq, qmax), -1, dtype=torch.int32)
+        for i, q in enumerate(w.queries):
+            qt[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
+        qt = qt.to(cuda)
+    else:
+        t = [torch.empty(n + 1, dtype=torch.int64, device=cuda), torch.empty(m, dtype=torch.int32, device=cuda),
+             torch.empty(n, dtype=torch.float32, device=cuda), torch.empty(V + 1, dtype=torch.int64, device=cuda),
+             torch.empty(P, dtype=torch.int32, device=cuda)]
+        qt = torch.empty((nq, qmax), dtype=torch.int32, device=cuda)
+    for x in t:
+        dist.broadcast(x, 0)
+    dist.broadcast(qt, 0)
+    gen_s = time.time() - t0
+    t1 = time.time()
+    G = kgs.kgs_load_graph_device(n, m, t[0].data_ptr(), t[1].data_ptr(), t[2].data_ptr(), V, t[3].data_ptr(),
+                                  t[4].data_ptr(), float(A.item()), True, dev)
+    torch.cuda.synchronize(dev)
+    load_s = time.time() - t1
+    del t
+    qh = qt.cpu().numpy()
+    queries = [tuple(int(x) for x in row if x >= 0) for row in qh]
+    return SimpleNamespace(queries=queries, k=k), _RemoteGraph(n, m), G, gen_s, load_s
+
+
 def run_reference(args):
     """The oracle, as it stands, on host cores (bench.py --impl reference)."""
     rank, world = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1)
@@ -180,11 +236,14 @@ def main():
     import paper_conf_icde_yangajtw19_b200 as kgs
 
     name = "C3" if world == 1 else "C4"
-    w, gen_s = build_workload(name, rank, world)
-    g = w.graph
-    t0 = time.time()
-    G = kgs.kgs_load_graph(g, device=dev)
-    load_s = time.time() - t0
+    if world == 1:
+        w, gen_s = build_workload(name, rank, world)
+        g = w.graph
+        t0 = time.time()
+        G = kgs.kgs_load_graph(g, device=dev)
+        load_s = time.time() - t0
+    else:
+        w, g, G, gen_s, load_s = load_replicated(name, rank, world, dev, kgs)
     # a fixed permutation so every window of steps mixes all query sizes (the config lists them by q)
     order = np.random.default_rng(12345).permutation(len(w.queries))
     allq = [w.queries[i] for i in order]
@@ -207,6 +266,7 @@ def main():
 
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     stats = []
+    answers = []
     clk = ClockSampler(dev)
     clk.start()
     if dist:
@@ -220,14 +280,16 @@ def main():
         ev[i][1].record(stream)
         r = kgs.kgs_query_fetch(G, len(queries[(args.warmup + i) % len(queries)]), 0, sh)  # after ev: not timed
         stats.append(r.stats)
+        answers.append([(a.central, a.depth, a.score_key) for a in r.answers])
     gather_ms = 0.0
     if dist:
-        # NCCL gather of every rank's top-k headers (central, depth, key) to all ranks (config C4)
-        hdr = torch.zeros((args.steps, w.k, 3), dtype=torch.float64, device=f"cuda:{dev}")
+        # NCCL all-gather of every rank's top-k headers (central, depth, key) (config C4)
+        from paper_conf_icde_yangajtw19_b200 import dist as kd
+        qids = [int(order[(rank + world * ((args.warmup + i) % len(queries))) % len(order)]) for i in range(args.steps)]
+        hdr = kd.pack_headers(qids, answers, w.k).to(f"cuda:{dev}")
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        out = [torch.empty_like(hdr) for _ in range(world)]
-        dist.all_gather(out, hdr)
+        merged = kd.gather_headers(hdr, args.steps * world, world)
         e1.record(stream)
     torch.cuda.synchronize(dev)
     if dist:
@@ -289,7 +351,7 @@ def main():
         "stats_mean": {k: float(np.mean([s[k] for s in stats])) for k in
                        ("levels", "n_centrals", "frontier_total", "arcs_scanned", "overflow")},
     }
-    if not args.no_cpu_baseline:
+    if not args.no_cpu_baseline and world == 1:
         import oracle
         t0 = time.perf_counter()
         done = 0

@@ -120,6 +120,8 @@ typedef struct {
     int64_t arcs_scanned;  /* out-arcs inspected by expansion (GTEPS numerator) */
     int64_t overflow;      /* Central Graphs extracted by the large-graph path */
     int64_t hits;          /* (node, keyword) pairs newly hit by expansion (M entries written) */
+    int64_t td_arcs;       /* in-arcs inspected by the top-down predecessor pre-pass */
+    int64_t td_pred_arcs;  /* predecessor arcs (Thm. V.4) in the union of all Central Graphs */
     float ms_search, ms_topdown, ms_total;
 } kgs_stats;
 

@@ -55,7 +55,8 @@ class kgs_answer(ctypes.Structure):
 class kgs_stats(ctypes.Structure):
     _fields_ = [("levels", ctypes.c_int32), ("stop_reason", ctypes.c_int32), ("n_centrals", ctypes.c_int64),
                 ("count", ctypes.c_int64), ("frontier_total", ctypes.c_int64), ("arcs_scanned", ctypes.c_int64),
-                ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
+                ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("td_arcs", ctypes.c_int64),
+                ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float)]
 
 
@@ -167,6 +168,18 @@ def kgs_load_graph(g, device: int = 0) -> Graph:
     h = ctypes.c_void_p()
     _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
     return Graph(h, rp.shape[0] - 1, kp.shape[0] - 1)
+
+
+def kgs_load_graph_device(n, n_arcs, row_ptr_ptr, col_idx_ptr, weight_ptr, n_keywords, kw_ptr_ptr, kw_nodes_ptr,
+                          A: float, symmetric: bool = True, device: int = 0) -> Graph:
+    """Load a graph whose arrays already live in device memory (KGS_INPUT_DEVICE_PTRS): raw device
+    pointers (e.g. torch CUDA tensors' data_ptr()), int64 row_ptr / kw_ptr, int32 col_idx / kw_nodes,
+    float32 weight.  The library copies them; the caller keeps ownership."""
+    d = kgs_graph_desc(int(n), int(n_arcs), row_ptr_ptr, col_idx_ptr, weight_ptr, int(n_keywords), kw_ptr_ptr,
+                       kw_nodes_ptr, float(A), 1 if symmetric else 0, int(device), KGS_INPUT_DEVICE_PTRS)
+    h = ctypes.c_void_p()
+    _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
+    return Graph(h, int(n), int(n_keywords))
 
 
 @dataclass

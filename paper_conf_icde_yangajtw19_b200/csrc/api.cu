@@ -113,6 +113,8 @@ struct kgs_graph {
     int32_t *h_hdr = nullptr;
     double *h_key = nullptr;
     long long *h_off = nullptr;
+    int32_t *h_nodes = nullptr, *h_arcs = nullptr;   // pinned staging of the emitted answer lists
+    size_t h_nodes_cap = 0, h_arcs_cap = 0;
     cudaEvent_t ev[4];
     std::mutex mu;
     // last enqueued query (for kgs_query_fetch)
@@ -165,7 +167,7 @@ void kgs_free_graph(kgs_graph *g) {
                     g->w.pred_u, g->w.pred_b, g->w.pa_u, g->w.pa_x, g->w.pa_b, g->w.pa_slot, g->w.scan_tmp};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
-    void *hp[] = {g->h_ctl, g->h_kw, g->h_dpow, g->h_hdr, g->h_key, g->h_off};
+    void *hp[] = {g->h_ctl, g->h_kw, g->h_dpow, g->h_hdr, g->h_key, g->h_off, g->h_nodes, g->h_arcs};
     for (void *p : hp) if (p) cudaFreeHost(p);
     for (auto &e : g->ev) cudaEventDestroy(e);
     delete g;
@@ -446,14 +448,27 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
     r->ans.resize(cnt);
     r->nodes.resize(cnt);
     r->arcs.resize(cnt);
+    // the emitted node / arc lists: one pinned copy of each used arena prefix, then split on the host
+    const size_t used_n = (size_t)c.arena_used[0], used_a = (size_t)c.arena_used[1];
+    if (used_n > g->h_nodes_cap) {
+        if (g->h_nodes) cudaFreeHost(g->h_nodes);
+        g->h_nodes_cap = std::max<size_t>(used_n, 2 * g->h_nodes_cap);
+        CUDA_TRY(cudaMallocHost(&g->h_nodes, sizeof(int32_t) * g->h_nodes_cap));
+    }
+    if (2 * used_a > g->h_arcs_cap) {
+        if (g->h_arcs) cudaFreeHost(g->h_arcs);
+        g->h_arcs_cap = std::max<size_t>(2 * used_a, 2 * g->h_arcs_cap);
+        CUDA_TRY(cudaMallocHost(&g->h_arcs, sizeof(int32_t) * g->h_arcs_cap));
+    }
+    if (used_n) CUDA_TRY(cudaMemcpyAsync(g->h_nodes, w.arena_nodes, sizeof(int32_t) * used_n, cudaMemcpyDeviceToHost, s));
+    if (used_a) CUDA_TRY(cudaMemcpyAsync(g->h_arcs, w.arena_arcs, sizeof(int32_t) * 2 * used_a, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
     for (int i = 0; i < cnt; ++i) {
         const int32_t *h = g->h_hdr + 4 * i;
-        r->nodes[i].resize(h[2]);
-        r->arcs[i].resize(2 * (size_t)h[3]);
-        if (h[2]) CUDA_TRY(cudaMemcpyAsync(r->nodes[i].data(), w.arena_nodes + g->h_off[2 * i], sizeof(int32_t) * h[2],
-                                           cudaMemcpyDeviceToHost, s));
-        if (h[3]) CUDA_TRY(cudaMemcpyAsync(r->arcs[i].data(), w.arena_arcs + 2 * g->h_off[2 * i + 1],
-                                           sizeof(int32_t) * 2 * h[3], cudaMemcpyDeviceToHost, s));
+        const int32_t *pn = g->h_nodes + g->h_off[2 * i];
+        const int32_t *pa = g->h_arcs + 2 * g->h_off[2 * i + 1];
+        r->nodes[i].assign(pn, pn + h[2]);
+        r->arcs[i].assign(pa, pa + 2 * (size_t)h[3]);
     }
     if (g->last_p.want_levels) {
         const int64_t n = g->n, q = g->last_q;
@@ -507,6 +522,8 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
     st.arcs_scanned = (int64_t)c.arcs_scanned;
     st.overflow = c.n_overflow;
     st.hits = (int64_t)c.hits;
+    st.td_arcs = (int64_t)c.td_arcs;
+    st.td_pred_arcs = (int64_t)c.n_parcs;
     for (int i = 0; i < std::min(c.n_stamp, 64); ++i) {
         r->ph_tag.push_back(c.stamp_tag[i]);
         r->ph_ns.push_back(c.stamp[i]);
