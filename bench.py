@@ -103,6 +103,17 @@ def load_peaks():
         return 6650.0, "fallback"
 
 
+def load_traffic():
+    """Mean DRAM bytes per k_search launch from the newest committed ncu capture (profiles/)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_k_search_traffic.json")))
+    if not files:
+        return None, None
+    with open(files[-1]) as f:
+        d = json.load(f)
+    return d.get("mean_dram_bytes_per_launch"), os.path.basename(files[-1])
+
+
 def bfs_algorithmic_bytes(st: dict) -> float:
     """SURVEY.md §8(d) / DESIGN.md "Roofline": bytes the search must move for this query.
     per expanded frontier entry: 16 B row_ptr + 2 B own status + 1 B activation + 4 B queue slot;
@@ -328,6 +339,7 @@ def main():
             dist.destroy_process_group()
         return 0
     peak, peak_kind = load_peaks()
+    traffic, traffic_src = load_traffic()
     bfs_bytes = sum(bfs_algorithmic_bytes(s) for s in stats)
     achieved = bfs_bytes / (search_ms / 1e3) / 1e9 if search_ms > 0 else 0.0
     line = {
@@ -342,11 +354,13 @@ def main():
         "gteps": arcs / (dev_ms / 1e3) / 1e9 * (world if world > 1 else 1) if dev_ms else 0.0,
         "phase_ms": {"search": search_ms / args.steps, "topdown": td_ms / args.steps},
         "roofline": {"kernel": "k_search", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": None, "peak_kind": peak_kind,
+                     "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                     "peak_kind": peak_kind,
                      "algorithmic_bytes_per_query": bfs_bytes / args.steps},
         "e2e": {"value": e2e_qps, "unit": "queries/s", "p50_ms": statistics.median(e2e_lat),
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h / e2e_steps},
-        "gpu_launches": 7 * args.steps,
+        # ours per query: k_search, k_extract, k_extract_big, k_select, k_rank, k_emit
+        "gpu_launches": 6 * args.steps,
         "clocks": clocks,
         "stats_mean": {k: float(np.mean([s[k] for s in stats])) for k in
                        ("levels", "n_centrals", "frontier_total", "arcs_scanned", "overflow")},
