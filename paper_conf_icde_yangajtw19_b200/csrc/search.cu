@@ -151,12 +151,16 @@ __device__ __forceinline__ long long block_excl_scan64(long long x, long long *t
 }
 
 // ------------------------------------------------------------------------------------------ frontier
-// Set v's bit in bitmap `bits` (one level slot); `flag` records that the slot is non-empty.
+// Set v's bit in bitmap `bits` (one level slot); `flag` records that the slot is non-empty.  The bit is
+// set with a reduction (no return value: one round trip less); the flag is stored once per group of
+// converged lanes.
 __device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t v) {
     uint32_t *word = bits + (v >> 5);
     const uint32_t bit = 1u << (v & 31);
     if (__ldcg(word) & bit) return;
-    if (!(atomicOr(word, bit) & bit) && !__ldcg(flag)) *flag = 1u;
+    asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
+    const unsigned mask = __activemask();
+    if ((int)lane_id() == __ffs(mask) - 1 && !__ldcg(flag)) *flag = 1u;   // stores to one line contend
 }
 
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
@@ -504,20 +508,10 @@ __device__ void pred_dag(const QueryArgs &a, cg::grid_group &grid, int64_t gtid,
                          long long *sh) {
     Ctl *ctl = a.w.ctl;
     const bool exact_block = a.extract_mode == KGS_EXTRACT_EXACT && a.block_central;
-    const uint32_t nc = __ldcg(&ctl->n_central);
     const int64_t W = a.w.W;
     __shared__ BigTile<PdNode> s_bigb;
-    // seeds: every central node, for every keyword it did not contain itself
-    for (int64_t j = gtid; j < nc; j += gsz) {
-        const int32_t c = a.w.centrals[j];
-        const uint64_t Mc = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + c);
-        uint32_t zbc = 0;
-        for (int i = 0; i < a.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
-        const uint32_t bits = full & ~zbc;
-        if (bits) { atomicOr(a.w.pd_state + c, bits << 8); set_bit(a.w.pd_bits, &ctl->pd_flag[0], c); }
-    }
-    grid.sync();
-    KGS_STAMP(TS_PD_SEED);
+    // seeds (every central node, for every keyword it did not contain itself) were set when each
+    // central was identified (k_search merge step): round 0 starts from them.
     unsigned long long my_arcs = 0;
     int r = 0;
     for (;; ++r) {
@@ -693,6 +687,14 @@ __global__ void __launch_bounds__(512, 2) k_search(QueryArgs a) {
                         const uint32_t ci = agg_slot(&ctl->n_central, 1u);
                         a.w.centrals[ci] = v;
                         a.w.cdepth[ci] = (uint8_t)l;
+                        // seed of the top-down pre-pass: expand backwards every keyword v does not contain
+                        const uint64_t Mv = __ldcg(reinterpret_cast<const unsigned long long *>(a.w.M) + v);
+                        uint32_t zb = 0;
+                        for (int i = 0; i < a.q; ++i) if (((Mv >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
+                        if (full & ~zb) {
+                            a.w.pd_state[v] = (full & ~zb) << 8;
+                            set_bit(a.w.pd_bits, &ctl->pd_flag[0], v);
+                        }
                     }
                     return old == 0;
                 },
