@@ -53,6 +53,7 @@ typedef enum {
 #define KGS_STOP_EXHAUSTED 1      /* the joint frontier became empty (no pending work) */
 #define KGS_STOP_MAX_DEPTH 2      /* level reached params.max_depth (truncated) */
 #define KGS_STOP_EMPTY_KEYWORD 3  /* some T_i is empty: nothing can be central (reading R17) */
+#define KGS_STOP_INVALID_QUERY (-1) /* device batch only: q out of range, keyword id out of range or repeated */
 
 /* Graph description for kgs_load_graph (node-weighted graph stored as CSR).
  *   n_nodes     number of nodes, 0 <= n < 2^31.
@@ -122,7 +123,9 @@ typedef struct {
     int64_t hits;          /* (node, keyword) pairs newly hit by expansion (M entries written) */
     int64_t td_arcs;       /* in-arcs inspected by the top-down predecessor pre-pass */
     int64_t td_pred_arcs;  /* predecessor arcs (Thm. V.4) in the union of all Central Graphs */
-    float ms_search, ms_topdown, ms_total;
+    float ms_search, ms_topdown, ms_total;   /* this query: bottom-up search, top-down, total (device clock) */
+    float ms_launch;       /* the whole engine launch that answered it (all queries of the batch) */
+    int32_t group;         /* engine group (set of CTAs) that answered the query */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index
@@ -153,6 +156,23 @@ kgs_status kgs_query(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, 
 kgs_status kgs_query_device(kgs_graph *g, const int32_t *kw_ids_dev, int32_t q, int32_t k, const kgs_params *p,
                             void *cuda_stream);
 kgs_status kgs_query_fetch(kgs_graph *g, void *cuda_stream, kgs_result **out);
+
+/* Answer a batch of independent queries in ONE launch (BASELINE.json configs[3]).
+ *   Query j has the keywords kw_ids[q_ptr[j] .. q_ptr[j+1]) (host arrays, q_ptr[0] = 0).
+ *   n_groups  how many queries run at the same time: the engine's CTAs are split into that many groups,
+ *             each answering whole queries and taking the next one from a device counter (0 = default 8;
+ *             clamped to [1, n_queries]).  Results do not depend on it.
+ *   results   [n_queries] receives one kgs_result per query (free each with kgs_result_free).
+ * Validation as kgs_query for every query (KGS_EINVAL, nothing enqueued). */
+kgs_status kgs_query_batch(kgs_graph *g, int32_t n_queries, const int32_t *q_ptr, const int32_t *kw_ids, int32_t k,
+                           const kgs_params *p, int32_t n_groups, void *cuda_stream, kgs_result **results);
+/* Device-resident batch: kw_dev [n_queries][KGS_MAX_Q] (unused slots ignored) and qlen_dev [n_queries] in
+ * device memory.  Invalid queries are detected on the device and reported with stop_reason
+ * KGS_STOP_INVALID_QUERY.  Enqueues without synchronising; kgs_query_batch_fetch (same stream) copies
+ * the n_queries results back, synchronising the stream. */
+kgs_status kgs_query_batch_device(kgs_graph *g, int32_t n_queries, const int32_t *kw_dev, const int32_t *qlen_dev,
+                                  int32_t k, const kgs_params *p, int32_t n_groups, void *cuda_stream);
+kgs_status kgs_query_batch_fetch(kgs_graph *g, void *cuda_stream, kgs_result **results);
 
 /* Result accessors.  kgs_result_count = min(k, |C|); answers are ranked by (score_key asc, central asc). */
 int32_t kgs_result_count(const kgs_result *r);

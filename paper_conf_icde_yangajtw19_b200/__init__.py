@@ -57,15 +57,18 @@ class kgs_stats(ctypes.Structure):
                 ("count", ctypes.c_int64), ("frontier_total", ctypes.c_int64), ("arcs_scanned", ctypes.c_int64),
                 ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("td_arcs", ctypes.c_int64),
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
-                ("ms_total", ctypes.c_float)]
+                ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32)]
 
 
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
             "kgs_query_fetch", "kgs_result_count", "kgs_result_answer", "kgs_result_levels",
             "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_phases",
-            "kgs_result_free", "kgs_last_error", "kgs_version"]
+            "kgs_result_free", "kgs_last_error", "kgs_version", "kgs_query_batch", "kgs_query_batch_device",
+            "kgs_query_batch_fetch"]
 
-PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr", "search_end"]
+PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
+               "search_end", "extract", "extract_big", "select", "emit"]
+KGS_STOP_INVALID_QUERY = -1
 
 _lib = None
 
@@ -102,6 +105,12 @@ def lib():
         L.kgs_result_centrals.restype = i32
         L.kgs_result_stats.argtypes = [vp, ctypes.POINTER(kgs_stats)]
         L.kgs_result_stats.restype = i32
+        L.kgs_query_batch.argtypes = [vp, i32, vp, vp, i32, ctypes.POINTER(kgs_params), i32, vp, vp]
+        L.kgs_query_batch.restype = i32
+        L.kgs_query_batch_device.argtypes = [vp, i32, vp, vp, i32, ctypes.POINTER(kgs_params), i32, vp]
+        L.kgs_query_batch_device.restype = i32
+        L.kgs_query_batch_fetch.argtypes = [vp, vp, vp]
+        L.kgs_query_batch_fetch.restype = i32
         L.kgs_result_phases.argtypes = [vp, vp, vp, i32, ctypes.POINTER(i32)]
         L.kgs_result_phases.restype = i32
         L.kgs_result_free.argtypes = [vp]
@@ -271,6 +280,35 @@ def kgs_query_fetch(graph: Graph, q: int, want_levels: int = 0, stream: int = 0)
     h = ctypes.c_void_p()
     _check(lib().kgs_query_fetch(graph.handle, ctypes.c_void_p(stream), ctypes.byref(h)))
     return _read_result(h, graph.n, q, want_levels)
+
+
+def kgs_query_batch(graph: Graph, queries, k: int, params: kgs_params | None = None, n_groups: int = 0,
+                    stream: int = 0) -> list:
+    """A batch of queries in one engine launch (host keyword ids in, host results out)."""
+    p = params if params is not None else kgs_params_default()
+    qp = np.zeros(len(queries) + 1, np.int32)
+    for j, kw in enumerate(queries):
+        qp[j + 1] = qp[j] + len(kw)
+    kw = np.ascontiguousarray(np.concatenate([np.asarray(q, np.int32) for q in queries]), np.int32)
+    hs = (ctypes.c_void_p * len(queries))()
+    _check(lib().kgs_query_batch(graph.handle, len(queries), qp.ctypes.data, kw.ctypes.data, int(k), ctypes.byref(p),
+                                 int(n_groups), ctypes.c_void_p(stream), hs))
+    return [_read_result(ctypes.c_void_p(hs[j]), graph.n, len(queries[j]), 0) for j in range(len(queries))]
+
+
+def kgs_query_batch_device(graph: Graph, n_queries: int, kw_dev_ptr: int, qlen_dev_ptr: int, k: int,
+                           params: kgs_params | None = None, n_groups: int = 0, stream: int = 0) -> None:
+    """Enqueue a batch whose padded keyword rows [n][8] and lengths [n] are in device memory."""
+    p = params if params is not None else kgs_params_default()
+    _check(lib().kgs_query_batch_device(graph.handle, int(n_queries), ctypes.c_void_p(kw_dev_ptr),
+                                        ctypes.c_void_p(qlen_dev_ptr), int(k), ctypes.byref(p), int(n_groups),
+                                        ctypes.c_void_p(stream)))
+
+
+def kgs_query_batch_fetch(graph: Graph, qlens, stream: int = 0) -> list:
+    hs = (ctypes.c_void_p * len(qlens))()
+    _check(lib().kgs_query_batch_fetch(graph.handle, ctypes.c_void_p(stream), hs))
+    return [_read_result(ctypes.c_void_p(hs[j]), graph.n, int(qlens[j]), 0) for j in range(len(qlens))]
 
 
 def kgs_version() -> str:

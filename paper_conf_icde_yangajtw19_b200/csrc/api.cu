@@ -1,6 +1,6 @@
-// api.cu — the C-ABI of libkgs (include/kgs.h): graph loading, query orchestration, result handles.
-// Host code only orchestrates: every step of the query path runs in the kernels of search.cu and
-// topdown.cu.  There is no CPU fallback; without a CUDA device every call fails with KGS_ECUDA.
+// api.cu — the C-ABI of libkgs (include/kgs.h): graph loading, the query engine's buffers, result handles.
+// Host code only validates and orchestrates: every step of the query path runs in engine.cu's kernel.
+// There is no CPU fallback; without a CUDA device every call fails with KGS_ECUDA.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -38,49 +38,29 @@ cudaError_t dmalloc(T **p, size_t count) {
     return cudaMalloc((void **)p, sizeof(T) * (count > 0 ? count : 1));
 }
 
+template <class T>
+cudaError_t grow_pinned(T **p, size_t *cap, size_t need) {
+    if (need <= *cap) return cudaSuccess;
+    if (*p) cudaFreeHost(*p);
+    *p = nullptr;
+    const size_t c = std::max(need, 2 * *cap);
+    cudaError_t e = cudaMallocHost((void **)p, sizeof(T) * c);
+    *cap = e == cudaSuccess ? c : 0;
+    return e;
+}
+
+template <class T>
+cudaError_t grow_dev(T **p, size_t *cap, size_t need) {
+    if (need <= *cap) return cudaSuccess;
+    if (*p) cudaFree(*p);
+    *p = nullptr;
+    const size_t c = std::max(need, 2 * *cap);
+    cudaError_t e = cudaMalloc((void **)p, sizeof(T) * c);
+    *cap = e == cudaSuccess ? c : 0;
+    return e;
+}
+
 }  // namespace
-
-// ------------------------------------------------------------------------------------------ kernels
-namespace kgs {
-__global__ void k_validate(DevGraph g, int32_t *err) {
-    const int64_t gt = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gs = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = gt; v < g.n; v += gs) {
-        if (g.row_ptr[v + 1] < g.row_ptr[v]) atomicOr(err, 1);
-        const float w = g.weight[v];
-        if (!(w >= 0.0f && w <= 1.0f)) atomicOr(err, 4);
-    }
-    for (int64_t j = gt; j < g.m; j += gs) {
-        const int32_t x = g.col_idx[j];
-        if (x < 0 || x >= g.n) atomicOr(err, 2);
-    }
-    for (int64_t t = gt; t < g.n_kw; t += gs) {
-        const int64_t b = g.kw_ptr[t], e = g.kw_ptr[t + 1];
-        if (e < b) { atomicOr(err, 8); continue; }
-        for (int64_t j = b; j < e; ++j) {
-            const int32_t v = g.kw_nodes[j];
-            if (v < 0 || v >= g.n || (j > b && v <= g.kw_nodes[j - 1])) { atomicOr(err, 16); break; }
-        }
-    }
-}
-cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s) {
-    k_validate<<<148 * 8, 256, 0, s>>>(g, err);
-    return cudaGetLastError();
-}
-
-// M for parity output: n*q bytes, 255 where the hit bit is clear
-__global__ void k_levels_out(QueryArgs a, uint8_t *out) {
-    const int64_t gt = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gs = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = gt; v < a.g.n; v += gs) {
-        const uint32_t hm = a.w.st[v] & 0xFFu;
-        for (int i = 0; i < a.q; ++i)
-            out[v * a.q + i] = ((hm >> i) & 1u) ? a.w.M[v * 8 + i] : (uint8_t)KGS_INF_LEVEL;
-    }
-}
-cudaError_t launch_levels_out(const QueryArgs &a, uint8_t *out, cudaStream_t s) {
-    k_levels_out<<<148 * 8, 256, 0, s>>>(a, out);
-    return cudaGetLastError();
-}
-}  // namespace kgs
 
 // ------------------------------------------------------------------------------------------ objects
 struct kgs_graph {
@@ -94,31 +74,58 @@ struct kgs_graph {
     float *weight = nullptr;
     uint8_t *cls = nullptr, *cls_in = nullptr;
     int64_t n_big = 0, n_big_in = 0;   // nodes with more than kBigDeg out- / in-arcs
-    // workspace
-    DevWork w{};
+    // per-alpha / per-lambda caches
+    uint8_t *act = nullptr;
     uint32_t *amax_dev = nullptr;
     double act_alpha = -1.0;
-    int amax = 0;
-    int R_alloc = 0;
+    int amax = 0, R = 0, R_alloc = 0;
+    int64_t W = 0;
+    double *dpow = nullptr;
     double dpow_lambda = -1.0;
-    Ctl *ctl_pair[2] = {nullptr, nullptr};
-    int query_no = 0;
-    bool state_valid = false;  // st/nm/fbits consistent with act and R of the last query
-    int last_R = 0;
-    int search_grid = 0, search_block = 512, select_grid = 0, extract_grid = 0;
+    // engine groups
+    std::vector<DevWork> works;         // host copies of the per-group workspaces
+    std::vector<int64_t> pcaps;
+    DevWork *works_dev = nullptr;
+    int works_dev_n = 0;
+    GroupBar *bars = nullptr;
+    int grid = 0;
+    char *warp_arenas = nullptr, *cta_arenas = nullptr;
+    size_t warp_arena_bytes = 0, cta_arena_bytes = 0;
+    // batch buffers
+    int32_t *d_kw = nullptr, *d_qlen = nullptr;
+    size_t d_kw_cap = 0, d_qlen_cap = 0;
+    QOut *d_qout = nullptr;
+    size_t d_qout_cap = 0;
+    int32_t *d_hdr = nullptr;
+    size_t d_hdr_cap = 0;
+    double *d_key = nullptr;
+    size_t d_key_cap = 0;
+    long long *d_off = nullptr;
+    size_t d_off_cap = 0;
+    int32_t *d_nodes = nullptr, *d_arcs = nullptr;
+    size_t d_nodes_cap = 0, d_arcs_cap = 0;
+    unsigned long long *d_ctr = nullptr;   // [0] next query, [1..2] arena counters
     // pinned host staging
-    Ctl *h_ctl = nullptr;
-    int32_t *h_kw = nullptr;
-    double *h_dpow = nullptr;
+    int32_t *h_kw = nullptr, *h_qlen = nullptr;
+    size_t h_kw_cap = 0, h_qlen_cap = 0;
+    QOut *h_qout = nullptr;
+    size_t h_qout_cap = 0;
     int32_t *h_hdr = nullptr;
+    size_t h_hdr_cap = 0;
     double *h_key = nullptr;
+    size_t h_key_cap = 0;
     long long *h_off = nullptr;
-    int32_t *h_nodes = nullptr, *h_arcs = nullptr;   // pinned staging of the emitted answer lists
+    size_t h_off_cap = 0;
+    int32_t *h_nodes = nullptr, *h_arcs = nullptr;
     size_t h_nodes_cap = 0, h_arcs_cap = 0;
-    cudaEvent_t ev[4];
+    unsigned long long *h_ctr = nullptr;
+    double *h_dpow = nullptr;
+    uint32_t *h_amax = nullptr;
+    cudaEvent_t ev[2];
     std::mutex mu;
-    // last enqueued query (for kgs_query_fetch)
-    int last_q = 0, last_k = 0;
+    // the last enqueued batch (for the fetch calls)
+    int last_nq = 0, last_k = 0, last_G = 1;
+    std::vector<int> last_q;
     kgs_params last_p{};
     bool pending = false;
 };
@@ -137,10 +144,65 @@ struct kgs_result {
     std::vector<uint64_t> ph_ns;
 };
 
+namespace {
+
+void free_work(DevWork &w) {
+    void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.centrals, w.cdepth, w.ckey, w.overflow,
+                 w.cflag, w.sel, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
+                 w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
+                 w.gstate};
+    for (void *x : p) if (x) cudaFree(x);
+    w = DevWork{};
+}
+
+// one group's workspace, sized for the graph (fbits for the current R)
+kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
+    const int64_t n = g->n;
+    w = DevWork{};
+    CUDA_TRY(dmalloc(&w.st, n));
+    CUDA_TRY(dmalloc(&w.nm, (n + 3) / 4));
+    CUDA_TRY(dmalloc(&w.M, n * 8));
+    CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max(g->R, 2) * (size_t)g->W));
+    CUDA_TRY(dmalloc(&w.qlight, n));
+    CUDA_TRY(dmalloc(&w.qbig, g->n_big));
+    CUDA_TRY(dmalloc(&w.touched, n));
+    CUDA_TRY(dmalloc(&w.centrals, n));
+    CUDA_TRY(dmalloc(&w.cdepth, n));
+    CUDA_TRY(dmalloc(&w.ckey, n));
+    CUDA_TRY(dmalloc(&w.overflow, n));
+    CUDA_TRY(dmalloc(&w.cflag, n));
+    CUDA_TRY(dmalloc(&w.sel, KGS_MAX_K));
+    CUDA_TRY(dmalloc(&w.ctl[0], 1));
+    CUDA_TRY(dmalloc(&w.ctl[1], 1));
+    CUDA_TRY(cudaMemset(w.ctl[0], 0, sizeof(Ctl)));
+    CUDA_TRY(cudaMemset(w.ctl[1], 0, sizeof(Ctl)));
+    CUDA_TRY(dmalloc(&w.pd_state, n));
+    CUDA_TRY(dmalloc(&w.pd_cid, n));
+    CUDA_TRY(dmalloc(&w.pd_touched, n));
+    CUDA_TRY(dmalloc(&w.pd_bits, 2 * g->W));
+    CUDA_TRY(dmalloc(&w.pd_qlight, n));
+    CUDA_TRY(dmalloc(&w.pd_qbig, g->n_big_in));
+    CUDA_TRY(dmalloc(&w.pcnt, n));
+    CUDA_TRY(dmalloc(&w.pred_ptr, n + 1));
+    w.pcap = pcap;
+    CUDA_TRY(dmalloc(&w.pred_u, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.pred_b, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.pa_u, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.pa_x, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.pa_b, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.pa_slot, (size_t)pcap));
+    CUDA_TRY(dmalloc(&w.scan_tmp, 4096));
+    CUDA_TRY(dmalloc(&w.gstate, 4));
+    CUDA_TRY(cudaMemset(w.gstate, 0, 4 * sizeof(uint32_t)));   // not valid: the first query resets densely
+    return KGS_OK;
+}
+
+}  // namespace
+
 extern "C" {
 
 const char *kgs_last_error(void) { return g_err.c_str(); }
-const char *kgs_version(void) { return "kgs 0.1 sm_100a (" __DATE__ ")"; }
+const char *kgs_version(void) { return "kgs 0.2 sm_100a engine (" __DATE__ ")"; }
 
 void kgs_params_default(kgs_params *p) {
     if (!p) return;
@@ -158,16 +220,14 @@ void kgs_free_graph(kgs_graph *g) {
     if (!g) return;
     cudaSetDevice(g->device);
     cudaDeviceSynchronize();
-    void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->w.act, g->w.st,
-                    g->w.nm, g->w.M, g->w.qlight, g->w.qbig, g->w.pd_bits, g->w.fbits, g->w.touched,
-                    g->w.centrals, g->w.cdepth, g->w.ckey, g->w.overflow, g->w.cflag, g->w.sel, g->w.kw_dev,
-                    g->w.dpow, g->ctl_pair[0], g->ctl_pair[1], g->w.ans_hdr, g->w.ans_key, g->w.ans_off,
-                    g->w.arena_nodes, g->w.arena_arcs, g->w.big_ws, g->amax_dev, g->w.pd_state, g->w.pd_cid,
-                    g->w.pd_touched, g->w.pd_qlight, g->w.pd_qbig, g->w.pcnt, g->w.pred_ptr,
-                    g->w.pred_u, g->w.pred_b, g->w.pa_u, g->w.pa_x, g->w.pa_b, g->w.pa_slot, g->w.scan_tmp};
+    for (auto &w : g->works) free_work(w);
+    void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->act, g->amax_dev, g->dpow,
+                    g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
+                    g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
-    void *hp[] = {g->h_ctl, g->h_kw, g->h_dpow, g->h_hdr, g->h_key, g->h_off, g->h_nodes, g->h_arcs};
+    void *hp[] = {g->h_kw, g->h_qlen, g->h_qout, g->h_hdr, g->h_key, g->h_off, g->h_nodes, g->h_arcs, g->h_ctr,
+                  g->h_dpow, g->h_amax};
     for (void *p : hp) if (p) cudaFreeHost(p);
     for (auto &e : g->ev) cudaEventDestroy(e);
     delete g;
@@ -176,12 +236,12 @@ void kgs_free_graph(kgs_graph *g) {
 kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     if (!d || !out) return fail(KGS_EINVAL, "null argument");
     *out = nullptr;
-    if (d->n_nodes < 0 || d->n_nodes >= (int64_t(1) << 31) || d->n_arcs < 0 || d->n_keywords < 1 ||
-        !(d->avg_dist_A > 0.0) || !std::isfinite(d->avg_dist_A))
+    if (d->n_nodes < 0 || d->n_nodes >= (int64_t(1) << 31) || d->n_arcs < 0 || d->n_arcs >= (int64_t(1) << 40) ||
+        d->n_keywords < 1 || !(d->avg_dist_A > 0.0) || !std::isfinite(d->avg_dist_A))
         return fail(KGS_EINVAL, "n_nodes / n_arcs / n_keywords / avg_dist_A out of range");
     if (d->n_nodes > 0 && (!d->row_ptr || !d->weight)) return fail(KGS_EINVAL, "missing row_ptr / weight");
     if (d->n_arcs > 0 && !d->col_idx) return fail(KGS_EINVAL, "missing col_idx");
-    if (!d->kw_ptr) return fail(KGS_EINVAL, "missing kw_ptr");
+    if (!d->kw_ptr || !d->row_ptr) return fail(KGS_EINVAL, "missing kw_ptr / row_ptr");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
         return fail(KGS_ECUDA, "no CUDA device available (libkgs has no CPU path)");
@@ -191,16 +251,16 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     const cudaMemcpyKind kind = on_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
     const int64_t n = d->n_nodes, m = d->n_arcs, V = d->n_keywords;
 
-    // host-side structural checks on the offsets (cheap; also needed for class counts / reverse CSR)
+    // host-side structural checks on the offsets (also needed for class counts / the reverse CSR)
     std::vector<int64_t> rp(n + 1), kp(V + 1);
-    if (n >= 0) {
-        if (on_dev) CUDA_TRY(cudaMemcpy(rp.data(), d->row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost));
-        else std::memcpy(rp.data(), d->row_ptr, sizeof(int64_t) * (n + 1));
-    }
+    if (on_dev) CUDA_TRY(cudaMemcpy(rp.data(), d->row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost));
+    else std::memcpy(rp.data(), d->row_ptr, sizeof(int64_t) * (n + 1));
     if (on_dev) CUDA_TRY(cudaMemcpy(kp.data(), d->kw_ptr, sizeof(int64_t) * (V + 1), cudaMemcpyDeviceToHost));
     else std::memcpy(kp.data(), d->kw_ptr, sizeof(int64_t) * (V + 1));
     if (rp[0] != 0 || rp[n] != m) return fail(KGS_EINVAL, "row_ptr[0] must be 0 and row_ptr[n] == n_arcs");
-    if (kp[0] != 0 || kp[V] < 0) return fail(KGS_EINVAL, "kw_ptr[0] must be 0");
+    for (int64_t v = 0; v < n; ++v)
+        if (rp[v + 1] < rp[v]) return fail(KGS_EINVAL, "row_ptr not non-decreasing");
+    if (kp[0] != 0) return fail(KGS_EINVAL, "kw_ptr[0] must be 0");
     for (int64_t t = 0; t < V; ++t)
         if (kp[t + 1] < kp[t]) return fail(KGS_EINVAL, "kw_ptr not non-decreasing");
     const int64_t P = kp[V];
@@ -250,14 +310,11 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     }
     G_TRY(launch_snap_weights(g->weight, n, 0));
     G_TRY(launch_degree_class(g->row_ptr, n, g->cls, 0));
-    for (int64_t v = 0; v < n; ++v) {
-        const int64_t dg_ = rp[v + 1] - rp[v];
-        if (dg_ > kBigDeg) ++g->n_big;
-    }
+    for (int64_t v = 0; v < n; ++v)
+        if (rp[v + 1] - rp[v] > kBigDeg) ++g->n_big;
     // reverse CSR for extraction along in-arcs (reading R1)
     if (g->symmetric) {
-        g->in_ptr = g->row_ptr; g->in_idx = g->col_idx; g->cls_in = g->cls;
-        g->n_big_in = g->n_big;
+        g->in_ptr = g->row_ptr; g->in_idx = g->col_idx; g->cls_in = g->cls; g->n_big_in = g->n_big;
     } else {
         std::vector<int32_t> ci(m);
         if (on_dev) G_TRY(cudaMemcpy(ci.data(), d->col_idx, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
@@ -275,74 +332,24 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         if (m) G_TRY(cudaMemcpy(g->in_idx, ii.data(), sizeof(int32_t) * m, cudaMemcpyHostToDevice));
         G_TRY(dmalloc(&g->cls_in, n));
         G_TRY(launch_degree_class(g->in_ptr, n, g->cls_in, 0));
-        for (int64_t v = 0; v < n; ++v) {
-            const int64_t dg_ = ip[v + 1] - ip[v];
-            if (dg_ > kBigDeg) ++g->n_big_in;
-        }
+        for (int64_t v = 0; v < n; ++v)
+            if (ip[v + 1] - ip[v] > kBigDeg) ++g->n_big_in;
     }
-    // per-query workspace sized for n (rings are sized at the first query: they depend on alpha)
-    DevWork &w = g->w;
-    G_TRY(dmalloc(&w.act, n));
-    G_TRY(dmalloc(&w.st, n));
-    G_TRY(dmalloc(&w.nm, (n + 3) / 4));
-    G_TRY(dmalloc(&w.M, n * 8));
-    G_TRY(dmalloc(&w.touched, n));
-    G_TRY(dmalloc(&w.centrals, n));
-    G_TRY(dmalloc(&w.cdepth, n));
-    G_TRY(dmalloc(&w.ckey, n));
-    G_TRY(dmalloc(&w.overflow, n));
-    G_TRY(dmalloc(&w.cflag, n));
-    G_TRY(dmalloc(&w.sel, KGS_MAX_K));
-    G_TRY(dmalloc(&w.kw_dev, KGS_MAX_Q));
-    G_TRY(dmalloc(&w.dpow, 256));
-    G_TRY(dmalloc(&g->ctl_pair[0], 1));
-    G_TRY(dmalloc(&g->ctl_pair[1], 1));
-    G_TRY(cudaMemset(g->ctl_pair[0], 0, sizeof(Ctl)));
-    G_TRY(cudaMemset(g->ctl_pair[1], 0, sizeof(Ctl)));
-    G_TRY(dmalloc(&w.ans_hdr, 4 * KGS_MAX_K));
-    G_TRY(dmalloc(&w.ans_key, KGS_MAX_K));
-    G_TRY(dmalloc(&w.ans_off, 2 * KGS_MAX_K));
-    w.arena_nodes_cap = (long long)KGS_MAX_K * kExtNodes + 4 * (long long)kBigNodes;
-    w.arena_arcs_cap = (long long)KGS_MAX_K * kExtArcs + 4 * (long long)kBigArcs;
-    G_TRY(dmalloc(&w.arena_nodes, (size_t)w.arena_nodes_cap));
-    G_TRY(dmalloc(&w.arena_arcs, 2 * (size_t)w.arena_arcs_cap));
-    w.big_hcap = kBigHash; w.big_ncap = kBigNodes; w.big_acap = kBigArcs; w.big_ctas = kBigCtas;
-    w.big_bytes = big_arena_bytes(kBigHash, kBigNodes, kBigArcs, false);
-    w.big_bytes_emit = big_arena_bytes(kBigHash, kBigNodes, kBigArcs, true);
-    G_TRY(cudaMalloc(&w.big_ws, w.big_bytes_emit * kBigCtas));
+    g->W = ((n + 31) / 32 + 7) / 8 * 8;   // words per bitmap, a multiple of 8 (16-byte vector access)
+    G_TRY(dmalloc(&g->act, n));
     G_TRY(dmalloc(&g->amax_dev, 1));
-    G_TRY(cudaMallocHost(&g->h_ctl, sizeof(Ctl)));
-    G_TRY(cudaMallocHost(&g->h_kw, sizeof(int32_t) * KGS_MAX_Q));
-    G_TRY(cudaMallocHost(&g->h_dpow, sizeof(double) * 256));
-    G_TRY(cudaMallocHost(&g->h_hdr, sizeof(int32_t) * 4 * KGS_MAX_K));
-    G_TRY(cudaMallocHost(&g->h_key, sizeof(double) * KGS_MAX_K));
-    G_TRY(cudaMallocHost(&g->h_off, sizeof(long long) * 2 * KGS_MAX_K));
-    w.W = ((n + 31) / 32 + 7) / 8 * 8;   // words per bitmap, a multiple of 8 (16-byte vector access)
-    G_TRY(dmalloc(&w.qlight, n));
-    G_TRY(dmalloc(&w.qbig, g->n_big));
-    // shared predecessor DAG of the top-down pre-pass
-    w.pcap = std::max<int64_t>(std::min<int64_t>(m, int64_t(64) << 20), 1 << 20);
-    G_TRY(dmalloc(&w.pd_state, n));
-    G_TRY(dmalloc(&w.pd_cid, n));
-    G_TRY(dmalloc(&w.pd_touched, n));
-    G_TRY(dmalloc(&w.pd_bits, 2 * w.W));
-    G_TRY(dmalloc(&w.pd_qlight, n));
-    G_TRY(dmalloc(&w.pd_qbig, g->n_big_in));
-    G_TRY(dmalloc(&w.pcnt, n));
-    G_TRY(dmalloc(&w.pred_ptr, n + 1));
-    G_TRY(dmalloc(&w.pred_u, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.pred_b, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.pa_u, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.pa_x, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.pa_b, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.pa_slot, (size_t)w.pcap));
-    G_TRY(dmalloc(&w.scan_tmp, 4096));
-    g->search_grid = search_max_grid(g->device, g->search_block);
-    g->select_grid = select_max_grid(g->device);
-    int sms = 148;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device);
-    g->extract_grid = sms * 4;
-    if (g->search_grid <= 0 || g->select_grid <= 0) return bail(fail(KGS_ECUDA, "occupancy query failed"));
+    G_TRY(dmalloc(&g->dpow, 256));
+    G_TRY(dmalloc(&g->d_ctr, 4));
+    G_TRY(cudaMallocHost(&g->h_ctr, 4 * sizeof(unsigned long long)));
+    G_TRY(cudaMallocHost(&g->h_dpow, 256 * sizeof(double)));
+    G_TRY(cudaMallocHost(&g->h_amax, sizeof(uint32_t)));
+    // the engine: one persistent cooperative grid; extraction arenas per warp and per CTA
+    g->grid = engine_max_grid(g->device);
+    if (g->grid <= 0) return bail(fail(KGS_ECUDA, "engine occupancy query failed"));
+    g->warp_arena_bytes = arena_bytes_host(kExtHash, kExtNodes, kExtArcs, 32, true);
+    g->cta_arena_bytes = arena_bytes_host(kBigHash, kBigNodes, kBigArcs, kBlock, true);
+    G_TRY(cudaMalloc(&g->warp_arenas, g->warp_arena_bytes * (size_t)g->grid * (kBlock / 32)));
+    G_TRY(cudaMalloc(&g->cta_arenas, g->cta_arena_bytes * (size_t)g->grid));
     G_TRY(cudaDeviceSynchronize());
 #undef G_TRY
     *out = g;
@@ -351,137 +358,215 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
 
 }  // extern "C"
 
-// ------------------------------------------------------------------------------------------ query
+// ------------------------------------------------------------------------------------------ query engine
 namespace {
 
-kgs_status check_params(const kgs_graph *g, const kgs_params &p, int32_t q, int32_t k) {
-    if (q < 1 || q > KGS_MAX_Q) return fail(KGS_EINVAL, "q must be in [1, 8]");
+kgs_status check_params(const kgs_params &p, int32_t k) {
     if (k < 1 || k > KGS_MAX_K) return fail(KGS_EINVAL, "k must be in [1, 4096]");
     if (!(p.alpha > 0.0 && p.alpha < 1.0)) return fail(KGS_EINVAL, "alpha must be in (0, 1)");
     if (!(p.lambda >= 0.0) || !std::isfinite(p.lambda)) return fail(KGS_EINVAL, "lambda must be >= 0");
     if (p.max_depth < 1 || p.max_depth > 254) return fail(KGS_EINVAL, "max_depth must be in [1, 254]");
     if (p.extract_mode != KGS_EXTRACT_EXACT && p.extract_mode != KGS_EXTRACT_LITERAL)
         return fail(KGS_EINVAL, "extract_mode");
-    (void)g;
     return KGS_OK;
 }
 
-// Enqueue the whole query on stream s; keyword ids already in g->w.kw_dev.
-kgs_status enqueue(kgs_graph *g, int32_t q, int32_t k, const kgs_params &p, cudaStream_t s) {
-    DevWork &w = g->w;
-    bool full_reset = !g->state_valid;
+kgs_status check_query(const kgs_graph *g, const int32_t *kw, int32_t q) {
+    if (q < 1 || q > KGS_MAX_Q) return fail(KGS_EINVAL, "q must be in [1, 8]");
+    for (int i = 0; i < q; ++i) {
+        if (kw[i] < 0 || kw[i] >= g->n_kw) return fail(KGS_EINVAL, "keyword id out of range");
+        for (int j = 0; j < i; ++j)
+            if (kw[j] == kw[i]) return fail(KGS_EINVAL, "duplicate keyword id");
+    }
+    return KGS_OK;
+}
+
+// per-alpha activation cache, level-slot ring, per-lambda depth factors, G group workspaces
+kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
+    bool invalidate = false;
     if (p.alpha != g->act_alpha) {
-        // activation cache (Eqs. 3-5) — recomputed only when alpha changes; amax sizes the rings
-        CUDA_TRY(launch_activation(g->weight, g->n, g->A, p.alpha, w.act, g->amax_dev, s));
-        uint32_t amax = 0;
-        CUDA_TRY(cudaMemcpyAsync(&g->h_ctl->levels, g->amax_dev, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        // activation cache (Eqs. 3-5) — recomputed only when alpha changes; amax sizes the level ring
+        CUDA_TRY(launch_activation(g->weight, g->n, g->A, p.alpha, g->act, g->amax_dev, s));
+        CUDA_TRY(cudaMemcpyAsync(g->h_amax, g->amax_dev, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         CUDA_TRY(cudaStreamSynchronize(s));
-        std::memcpy(&amax, &g->h_ctl->levels, sizeof(uint32_t));
-        g->amax = (int)amax;
+        g->amax = (int)*g->h_amax;
         g->act_alpha = p.alpha;
-        full_reset = true;
+        g->R = g->amax + 2;
+        invalidate = true;
     }
-    const int R = g->amax + 2;
-    if (R > g->R_alloc) {
+    if (g->R > g->R_alloc) {   // bigger ring: reallocate every group's bitmaps
         CUDA_TRY(cudaStreamSynchronize(s));
-        if (w.fbits) cudaFree(w.fbits);
-        CUDA_TRY(dmalloc(&w.fbits, (size_t)R * (size_t)w.W));
-        g->R_alloc = R;
-        full_reset = true;
+        for (auto &w : g->works) {
+            cudaFree(w.fbits);
+            w.fbits = nullptr;
+            CUDA_TRY(dmalloc(&w.fbits, (size_t)g->R * (size_t)g->W));
+        }
+        g->R_alloc = g->R;
+        invalidate = true;
     }
-    if (R != g->last_R) full_reset = true;
-    w.R = R;
+    if ((int)g->works.size() < G) {
+        CUDA_TRY(cudaStreamSynchronize(s));
+        // predecessor-arc capacity per group: 64 M for the single-query group, 16 M for the others
+        while ((int)g->works.size() < G) {
+            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, g->works.empty() ? (64ll << 20) : (16ll << 20)), 1 << 20);
+            DevWork w;
+            kgs_status st = alloc_work(g, w, pcap);
+            if (st != KGS_OK) { free_work(w); return st; }
+            g->works.push_back(w);
+        }
+        g->R_alloc = std::max(g->R_alloc, std::max(g->R, 2));
+        if (g->works_dev) cudaFree(g->works_dev);
+        if (g->bars) cudaFree(g->bars);
+        CUDA_TRY(dmalloc(&g->works_dev, g->works.size()));
+        CUDA_TRY(dmalloc(&g->bars, g->works.size()));
+        CUDA_TRY(cudaMemset(g->bars, 0, sizeof(GroupBar) * g->works.size()));
+        g->works_dev_n = 0;
+    }
+    if (g->works_dev_n != (int)g->works.size() || invalidate) {
+        CUDA_TRY(cudaMemcpyAsync(g->works_dev, g->works.data(), sizeof(DevWork) * g->works.size(), cudaMemcpyHostToDevice, s));
+        g->works_dev_n = (int)g->works.size();
+    }
+    if (invalidate)
+        for (auto &w : g->works) CUDA_TRY(cudaMemsetAsync(w.gstate, 0, 4 * sizeof(uint32_t), s));
     if (p.lambda != g->dpow_lambda) {
         // Eq. 6 depth factor d^lambda from the host libm (reading R15), one value per depth
         CUDA_TRY(cudaStreamSynchronize(s));
         for (int dd = 0; dd < 256; ++dd) g->h_dpow[dd] = std::pow((double)dd, p.lambda);
-        CUDA_TRY(cudaMemcpyAsync(w.dpow, g->h_dpow, sizeof(double) * 256, cudaMemcpyHostToDevice, s));
+        CUDA_TRY(cudaMemcpyAsync(g->dpow, g->h_dpow, sizeof(double) * 256, cudaMemcpyHostToDevice, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
         g->dpow_lambda = p.lambda;
     }
-    Ctl *cur = g->ctl_pair[g->query_no & 1];
-    Ctl *prev = g->ctl_pair[(g->query_no + 1) & 1];
-    CUDA_TRY(cudaMemsetAsync(cur, 0, sizeof(Ctl), s));
-    w.ctl = cur;
-    w.prev = full_reset ? nullptr : prev;
+    return KGS_OK;
+}
 
-    QueryArgs a{};
-    a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx;
-    a.g.in_ptr = g->in_ptr; a.g.in_idx = g->in_idx; a.g.weight = g->weight; a.g.cls = g->cls;
-    a.g.cls_in = g->cls_in;
-    a.g.n_kw = g->n_kw; a.g.kw_ptr = g->kw_ptr; a.g.kw_nodes = g->kw_nodes;
-    a.w = w;
-    a.q = q; a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0;
-    a.extract_mode = p.extract_mode; a.level_cover = p.level_cover ? 1 : 0;
-    a.full_reset = full_reset ? 1 : 0;
-    a.prev_R = g->last_R;
-
+// Enqueue one engine launch for nq queries whose padded keyword rows / lengths are in g->d_kw / d_qlen.
+kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaStream_t s, int qconst = 0) {
+    G = std::max(1, std::min(G, nq));
+    kgs_status st = prepare(g, p, G, s);
+    if (st != KGS_OK) return st;
+    CUDA_TRY(grow_dev(&g->d_qout, &g->d_qout_cap, (size_t)nq));
+    CUDA_TRY(grow_dev(&g->d_hdr, &g->d_hdr_cap, (size_t)nq * k * 4));
+    CUDA_TRY(grow_dev(&g->d_key, &g->d_key_cap, (size_t)nq * k));
+    CUDA_TRY(grow_dev(&g->d_off, &g->d_off_cap, (size_t)nq * k * 2));
+    CUDA_TRY(grow_dev(&g->d_nodes, &g->d_nodes_cap, (size_t)nq * k * 64 + (4u << 20)));
+    CUDA_TRY(grow_dev(&g->d_arcs, &g->d_arcs_cap, 2 * ((size_t)nq * k * 64 + (4u << 20))));
+    CUDA_TRY(cudaMemsetAsync(g->d_ctr, 0, 4 * sizeof(unsigned long long), s));
+    EngineArgs a{};
+    a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx; a.g.in_ptr = g->in_ptr;
+    a.g.in_idx = g->in_idx; a.g.weight = g->weight; a.g.cls = g->cls; a.g.cls_in = g->cls_in; a.g.n_kw = g->n_kw;
+    a.g.kw_ptr = g->kw_ptr; a.g.kw_nodes = g->kw_nodes;
+    a.act = g->act; a.R = g->R; a.W = g->W; a.dpow = g->dpow;
+    a.works = g->works_dev; a.bars = g->bars; a.G = G;
+    a.nq = nq; a.kw = g->d_kw; a.qlen = g->d_qlen; a.qconst = qconst;
+    a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
+    a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
+    a.level_cover = p.level_cover ? 1 : 0;
+    a.qout = g->d_qout; a.out_hdr = g->d_hdr; a.out_key = g->d_key; a.out_off = g->d_off;
+    a.out_nodes = g->d_nodes; a.out_arcs = g->d_arcs;
+    a.out_nodes_cap = (long long)g->d_nodes_cap; a.out_arcs_cap = (long long)(g->d_arcs_cap / 2);
+    a.out_used = g->d_ctr + 1;
+    a.warp_arenas = g->warp_arenas; a.warp_arena_bytes = g->warp_arena_bytes;
+    a.cta_arenas = g->cta_arenas; a.cta_arena_bytes = g->cta_arena_bytes;
     CUDA_TRY(cudaEventRecord(g->ev[0], s));
-    CUDA_TRY(launch_search(a, g->search_grid, g->search_block, s));
+    CUDA_TRY(launch_engine(a, g->grid, s));
     CUDA_TRY(cudaEventRecord(g->ev[1], s));
-    CUDA_TRY(launch_extract(a, g->extract_grid, s));
-    CUDA_TRY(launch_select(a, g->select_grid, s));
-    CUDA_TRY(launch_emit(a, std::min<int>(k, w.big_ctas), s));
-    CUDA_TRY(cudaEventRecord(g->ev[2], s));
-    g->query_no++;
-    g->state_valid = true;
-    g->last_R = R;
-    g->last_q = q; g->last_k = k; g->last_p = p;
+    g->last_nq = nq; g->last_k = k; g->last_G = G; g->last_p = p;
     g->pending = true;
     return KGS_OK;
 }
 
-kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
+// Copy the last batch's results back (synchronises s) into results[0..nq).
+kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
     if (!g->pending) return fail(KGS_EINVAL, "no query enqueued on this graph");
-    DevWork &w = g->w;
-    Ctl *cur = g->ctl_pair[(g->query_no + 1) & 1];  // the last enqueued query's block
-    CUDA_TRY(cudaMemcpyAsync(g->h_ctl, cur, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaMemcpyAsync(g->h_hdr, w.ans_hdr, sizeof(int32_t) * 4 * g->last_k, cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaMemcpyAsync(g->h_key, w.ans_key, sizeof(double) * g->last_k, cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaMemcpyAsync(g->h_off, w.ans_off, sizeof(long long) * 2 * g->last_k, cudaMemcpyDeviceToHost, s));
+    const int nq = g->last_nq, k = g->last_k;
+    CUDA_TRY(grow_pinned(&g->h_qout, &g->h_qout_cap, (size_t)nq));
+    CUDA_TRY(grow_pinned(&g->h_hdr, &g->h_hdr_cap, (size_t)nq * k * 4));
+    CUDA_TRY(grow_pinned(&g->h_key, &g->h_key_cap, (size_t)nq * k));
+    CUDA_TRY(grow_pinned(&g->h_off, &g->h_off_cap, (size_t)nq * k * 2));
+    CUDA_TRY(cudaMemcpyAsync(g->h_qout, g->d_qout, sizeof(QOut) * nq, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaMemcpyAsync(g->h_hdr, g->d_hdr, sizeof(int32_t) * nq * k * 4, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaMemcpyAsync(g->h_key, g->d_key, sizeof(double) * nq * k, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaMemcpyAsync(g->h_off, g->d_off, sizeof(long long) * nq * k * 2, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaMemcpyAsync(g->h_ctr, g->d_ctr, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     g->pending = false;
-    const Ctl &c = *g->h_ctl;
-    if (c.fatal) return fail(KGS_EINTERNAL, "a Central Graph exceeded the large-graph extractor capacity");
-    kgs_result *r = new kgs_result();
-    r->n = g->n; r->q = g->last_q;
-    const int cnt = (int)std::min<uint32_t>(c.sel_count, (uint32_t)g->last_k);
-    r->ans.resize(cnt);
-    r->nodes.resize(cnt);
-    r->arcs.resize(cnt);
-    // the emitted node / arc lists: one pinned copy of each used arena prefix, then split on the host
-    const size_t used_n = (size_t)c.arena_used[0], used_a = (size_t)c.arena_used[1];
-    if (used_n > g->h_nodes_cap) {
-        if (g->h_nodes) cudaFreeHost(g->h_nodes);
-        g->h_nodes_cap = std::max<size_t>(used_n, 2 * g->h_nodes_cap);
-        CUDA_TRY(cudaMallocHost(&g->h_nodes, sizeof(int32_t) * g->h_nodes_cap));
-    }
-    if (2 * used_a > g->h_arcs_cap) {
-        if (g->h_arcs) cudaFreeHost(g->h_arcs);
-        g->h_arcs_cap = std::max<size_t>(2 * used_a, 2 * g->h_arcs_cap);
-        CUDA_TRY(cudaMallocHost(&g->h_arcs, sizeof(int32_t) * g->h_arcs_cap));
-    }
-    if (used_n) CUDA_TRY(cudaMemcpyAsync(g->h_nodes, w.arena_nodes, sizeof(int32_t) * used_n, cudaMemcpyDeviceToHost, s));
-    if (used_a) CUDA_TRY(cudaMemcpyAsync(g->h_arcs, w.arena_arcs, sizeof(int32_t) * 2 * used_a, cudaMemcpyDeviceToHost, s));
+    const size_t used_n = (size_t)g->h_ctr[1], used_a = (size_t)g->h_ctr[2];
+    CUDA_TRY(grow_pinned(&g->h_nodes, &g->h_nodes_cap, std::max<size_t>(used_n, 1)));
+    CUDA_TRY(grow_pinned(&g->h_arcs, &g->h_arcs_cap, std::max<size_t>(2 * used_a, 1)));
+    if (used_n) CUDA_TRY(cudaMemcpyAsync(g->h_nodes, g->d_nodes, sizeof(int32_t) * used_n, cudaMemcpyDeviceToHost, s));
+    if (used_a) CUDA_TRY(cudaMemcpyAsync(g->h_arcs, g->d_arcs, sizeof(int32_t) * 2 * used_a, cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
-    for (int i = 0; i < cnt; ++i) {
-        const int32_t *h = g->h_hdr + 4 * i;
-        const int32_t *pn = g->h_nodes + g->h_off[2 * i];
-        const int32_t *pa = g->h_arcs + 2 * g->h_off[2 * i + 1];
-        r->nodes[i].assign(pn, pn + h[2]);
-        r->arcs[i].assign(pa, pa + 2 * (size_t)h[3]);
+    float ms_all = 0.f;
+    cudaEventElapsedTime(&ms_all, g->ev[0], g->ev[1]);
+    for (int j = 0; j < nq; ++j) {
+        const QOut &o = g->h_qout[j];
+        if (o.fatal) {
+            for (int t = 0; t < j; ++t) { delete results[t]; results[t] = nullptr; }
+            return fail(KGS_EINTERNAL, "a Central Graph exceeded the large-graph extractor capacity (query " +
+                                           std::to_string(j) + ", code " + std::to_string(o.fatal) + ")");
+        }
     }
-    if (g->last_p.want_levels) {
-        const int64_t n = g->n, q = g->last_q;
+    for (int j = 0; j < nq; ++j) {
+        const QOut &o = g->h_qout[j];
+        kgs_result *r = new kgs_result();
+        r->n = g->n;
+        r->q = g->last_q.empty() ? 0 : g->last_q[j];
+        const int cnt = std::max(0, std::min(o.count, k));
+        r->ans.resize(cnt); r->nodes.resize(cnt); r->arcs.resize(cnt);
+        for (int i = 0; i < cnt; ++i) {
+            const int64_t ai = (int64_t)j * k + i;
+            const int32_t *h = g->h_hdr + 4 * ai;
+            const int32_t *pn = g->h_nodes + g->h_off[2 * ai];
+            const int32_t *pa = g->h_arcs + 2 * g->h_off[2 * ai + 1];
+            r->nodes[i].assign(pn, pn + h[2]);
+            r->arcs[i].assign(pa, pa + 2 * (size_t)h[3]);
+            kgs_answer &an = r->ans[i];
+            an.central = h[0];
+            an.depth = h[1];
+            an.score_key = g->h_key[ai];
+            an.score = (float)an.score_key;
+            an.n_nodes = h[2];
+            an.nodes = r->nodes[i].data();
+            an.n_arcs = h[3];
+            an.arcs = r->arcs[i].data();
+        }
+        kgs_stats &st = r->stats;
+        st.levels = o.levels;
+        st.stop_reason = o.stop_reason;
+        st.n_centrals = o.n_central;
+        st.count = cnt;
+        st.frontier_total = (int64_t)o.frontier_total;
+        st.arcs_scanned = (int64_t)o.arcs_scanned;
+        st.overflow = o.n_overflow;
+        st.hits = (int64_t)o.hits;
+        st.td_arcs = (int64_t)o.td_arcs;
+        st.td_pred_arcs = o.n_parcs;
+        st.group = o.group;
+        if (o.stop_reason != KGS_STOP_INVALID_QUERY && o.t_end >= o.t_start) {
+            st.ms_search = (float)((double)(o.t_search_end - o.t_start) * 1e-6);
+            st.ms_topdown = (float)((double)(o.t_end - o.t_search_end) * 1e-6);
+            st.ms_total = (float)((double)(o.t_end - o.t_start) * 1e-6);
+        }
+        st.ms_launch = ms_all;
+        for (int i = 0; i < std::min(o.n_stamp, kMaxStamps); ++i) {
+            r->ph_tag.push_back(o.stamp_tag[i]);
+            r->ph_ns.push_back(o.stamp[i]);
+        }
+        results[j] = r;
+    }
+    // parity view of a single query (want_levels): M, activation levels and every central of group 0
+    if (g->last_p.want_levels && nq == 1 && results[0]) {
+        kgs_result *r = results[0];
+        const int64_t n = g->n, q = r->q;
+        const DevWork &w = g->works[0];
         uint8_t *dM = nullptr;
         CUDA_TRY(dmalloc(&dM, n * q));
-        QueryArgs a{};
-        a.g.n = n; a.w = w; a.q = (int)q;
-        CUDA_TRY(launch_levels_out(a, dM, s));
+        CUDA_TRY(launch_levels_out(w.st, w.M, n, (int)q, dM, s));
         r->M.resize(n * q);
         r->act.resize(n);
         CUDA_TRY(cudaMemcpyAsync(r->M.data(), dM, n * q, cudaMemcpyDeviceToHost, s));
-        CUDA_TRY(cudaMemcpyAsync(r->act.data(), w.act, n, cudaMemcpyDeviceToHost, s));
-        const uint32_t nc = c.n_central;
+        CUDA_TRY(cudaMemcpyAsync(r->act.data(), g->act, n, cudaMemcpyDeviceToHost, s));
+        const uint32_t nc = g->h_qout[0].n_central;
         std::vector<int32_t> ids(nc);
         std::vector<uint8_t> dep(nc);
         std::vector<double> key(nc);
@@ -500,38 +585,25 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
         for (uint32_t i = 0; i < nc; ++i) { r->centrals[i] = ids[ord[i]]; r->cdepth[i] = dep[ord[i]]; r->ckey[i] = key[ord[i]]; }
         r->has_levels = true;
     }
-    CUDA_TRY(cudaStreamSynchronize(s));
-    for (int i = 0; i < cnt; ++i) {
-        const int32_t *h = g->h_hdr + 4 * i;
-        kgs_answer &an = r->ans[i];
-        an.central = h[0];
-        an.depth = h[1];
-        an.score_key = g->h_key[i];
-        an.score = (float)an.score_key;
-        an.n_nodes = h[2];
-        an.nodes = r->nodes[i].data();
-        an.n_arcs = h[3];
-        an.arcs = r->arcs[i].data();
+    return KGS_OK;
+}
+
+// stage host keyword rows into the padded device layout [nq][KGS_MAX_Q]
+kgs_status stage_host(kgs_graph *g, int nq, const int32_t *q_ptr, const int32_t *kw_ids, cudaStream_t s) {
+    CUDA_TRY(cudaStreamSynchronize(s));   // pinned staging may still be in use by a previous copy
+    CUDA_TRY(grow_pinned(&g->h_kw, &g->h_kw_cap, (size_t)nq * KGS_MAX_Q));
+    CUDA_TRY(grow_pinned(&g->h_qlen, &g->h_qlen_cap, (size_t)nq));
+    CUDA_TRY(grow_dev(&g->d_kw, &g->d_kw_cap, (size_t)nq * KGS_MAX_Q));
+    CUDA_TRY(grow_dev(&g->d_qlen, &g->d_qlen_cap, (size_t)nq));
+    g->last_q.assign(nq, 0);
+    for (int j = 0; j < nq; ++j) {
+        const int q = q_ptr[j + 1] - q_ptr[j];
+        g->h_qlen[j] = q;
+        g->last_q[j] = q;
+        for (int i = 0; i < KGS_MAX_Q; ++i) g->h_kw[(int64_t)j * KGS_MAX_Q + i] = i < q ? kw_ids[q_ptr[j] + i] : -1;
     }
-    kgs_stats &st = r->stats;
-    st.levels = c.levels;
-    st.stop_reason = c.stop_reason;
-    st.n_centrals = c.n_central;
-    st.count = cnt;
-    st.frontier_total = (int64_t)c.frontier_total;
-    st.arcs_scanned = (int64_t)c.arcs_scanned;
-    st.overflow = c.n_overflow;
-    st.hits = (int64_t)c.hits;
-    st.td_arcs = (int64_t)c.td_arcs;
-    st.td_pred_arcs = (int64_t)c.n_parcs;
-    for (int i = 0; i < std::min(c.n_stamp, 64); ++i) {
-        r->ph_tag.push_back(c.stamp_tag[i]);
-        r->ph_ns.push_back(c.stamp[i]);
-    }
-    cudaEventElapsedTime(&st.ms_search, g->ev[0], g->ev[1]);
-    cudaEventElapsedTime(&st.ms_topdown, g->ev[1], g->ev[2]);
-    cudaEventElapsedTime(&st.ms_total, g->ev[0], g->ev[2]);
-    *out = r;
+    CUDA_TRY(cudaMemcpyAsync(g->d_kw, g->h_kw, sizeof(int32_t) * nq * KGS_MAX_Q, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(g->d_qlen, g->h_qlen, sizeof(int32_t) * nq, cudaMemcpyHostToDevice, s));
     return KGS_OK;
 }
 
@@ -539,48 +611,106 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **out) {
 
 extern "C" {
 
-kgs_status kgs_query_device(kgs_graph *g, const int32_t *kw_ids_dev, int32_t q, int32_t k, const kgs_params *pp,
-                            void *cuda_stream) {
-    if (!g || !kw_ids_dev) return fail(KGS_EINVAL, "null argument");
-    kgs_params p;
-    if (pp) p = *pp; else kgs_params_default(&p);
-    kgs_status st = check_params(g, p, q, k);
-    if (st != KGS_OK) return st;
-    std::lock_guard<std::mutex> lk(g->mu);
-    cudaStream_t s = (cudaStream_t)cuda_stream;
-    CUDA_TRY(cudaSetDevice(g->device));
-    CUDA_TRY(cudaMemcpyAsync(g->w.kw_dev, kw_ids_dev, sizeof(int32_t) * q, cudaMemcpyDeviceToDevice, s));
-    return enqueue(g, q, k, p, s);
-}
-
-kgs_status kgs_query_fetch(kgs_graph *g, void *cuda_stream, kgs_result **out) {
-    if (!g || !out) return fail(KGS_EINVAL, "null argument");
-    std::lock_guard<std::mutex> lk(g->mu);
-    CUDA_TRY(cudaSetDevice(g->device));
-    return fetch(g, (cudaStream_t)cuda_stream, out);
-}
-
 kgs_status kgs_query(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, const kgs_params *pp,
                      void *cuda_stream, kgs_result **out) {
     if (!g || !kw_ids || !out) return fail(KGS_EINVAL, "null argument");
     *out = nullptr;
     kgs_params p;
     if (pp) p = *pp; else kgs_params_default(&p);
-    kgs_status st = check_params(g, p, q, k);
+    kgs_status st = check_params(p, k);
     if (st != KGS_OK) return st;
-    for (int i = 0; i < q; ++i) {
-        if (kw_ids[i] < 0 || kw_ids[i] >= g->n_kw) return fail(KGS_EINVAL, "keyword id out of range");
-        for (int j = 0; j < i; ++j)
-            if (kw_ids[j] == kw_ids[i]) return fail(KGS_EINVAL, "duplicate keyword id");
+    st = check_query(g, kw_ids, q);
+    if (st != KGS_OK) return st;
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    const int32_t qp[2] = {0, q};
+    st = stage_host(g, 1, qp, kw_ids, s);
+    if (st != KGS_OK) return st;
+    st = launch(g, 1, k, p, 1, s);
+    if (st != KGS_OK) return st;
+    return fetch(g, s, out);
+}
+
+kgs_status kgs_query_device(kgs_graph *g, const int32_t *kw_ids_dev, int32_t q, int32_t k, const kgs_params *pp,
+                            void *cuda_stream) {
+    if (!g || !kw_ids_dev) return fail(KGS_EINVAL, "null argument");
+    if (q < 1 || q > KGS_MAX_Q) return fail(KGS_EINVAL, "q must be in [1, 8]");
+    kgs_params p;
+    if (pp) p = *pp; else kgs_params_default(&p);
+    kgs_status st = check_params(p, k);
+    if (st != KGS_OK) return st;
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    CUDA_TRY(grow_dev(&g->d_kw, &g->d_kw_cap, (size_t)KGS_MAX_Q));
+    CUDA_TRY(grow_dev(&g->d_qlen, &g->d_qlen_cap, (size_t)1));
+    CUDA_TRY(cudaMemsetAsync(g->d_kw, 0xFF, sizeof(int32_t) * KGS_MAX_Q, s));
+    CUDA_TRY(cudaMemcpyAsync(g->d_kw, kw_ids_dev, sizeof(int32_t) * q, cudaMemcpyDeviceToDevice, s));
+    g->last_q.assign(1, q);
+    return launch(g, 1, k, p, 1, s, q);   // q travels as a kernel argument
+}
+
+kgs_status kgs_query_fetch(kgs_graph *g, void *cuda_stream, kgs_result **out) {
+    if (!g || !out) return fail(KGS_EINVAL, "null argument");
+    std::lock_guard<std::mutex> lk(g->mu);
+    CUDA_TRY(cudaSetDevice(g->device));
+    if (g->pending && g->last_nq != 1) return fail(KGS_EINVAL, "the pending launch is a batch: use kgs_query_batch_fetch");
+    return fetch(g, (cudaStream_t)cuda_stream, out);
+}
+
+kgs_status kgs_query_batch(kgs_graph *g, int32_t n_queries, const int32_t *q_ptr, const int32_t *kw_ids, int32_t k,
+                           const kgs_params *pp, int32_t n_groups, void *cuda_stream, kgs_result **results) {
+    if (!g || !q_ptr || !kw_ids || !results || n_queries < 1) return fail(KGS_EINVAL, "null argument / empty batch");
+    kgs_params p;
+    if (pp) p = *pp; else kgs_params_default(&p);
+    kgs_status st = check_params(p, k);
+    if (st != KGS_OK) return st;
+    if (q_ptr[0] != 0) return fail(KGS_EINVAL, "q_ptr[0] must be 0");
+    for (int j = 0; j < n_queries; ++j) {
+        st = check_query(g, kw_ids + q_ptr[j], q_ptr[j + 1] - q_ptr[j]);
+        if (st != KGS_OK) return fail(st, "query " + std::to_string(j) + ": " + g_err);
     }
     std::lock_guard<std::mutex> lk(g->mu);
     cudaStream_t s = (cudaStream_t)cuda_stream;
     CUDA_TRY(cudaSetDevice(g->device));
-    std::memcpy(g->h_kw, kw_ids, sizeof(int32_t) * q);
-    CUDA_TRY(cudaMemcpyAsync(g->w.kw_dev, g->h_kw, sizeof(int32_t) * q, cudaMemcpyHostToDevice, s));
-    st = enqueue(g, q, k, p, s);
+    st = stage_host(g, n_queries, q_ptr, kw_ids, s);
     if (st != KGS_OK) return st;
-    return fetch(g, s, out);
+    st = launch(g, n_queries, k, p, n_groups > 0 ? n_groups : 8, s);
+    if (st != KGS_OK) return st;
+    return fetch(g, s, results);
+}
+
+kgs_status kgs_query_batch_device(kgs_graph *g, int32_t n_queries, const int32_t *kw_dev, const int32_t *qlen_dev,
+                                  int32_t k, const kgs_params *pp, int32_t n_groups, void *cuda_stream) {
+    if (!g || !kw_dev || !qlen_dev || n_queries < 1) return fail(KGS_EINVAL, "null argument / empty batch");
+    kgs_params p;
+    if (pp) p = *pp; else kgs_params_default(&p);
+    kgs_status st = check_params(p, k);
+    if (st != KGS_OK) return st;
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    CUDA_TRY(grow_dev(&g->d_kw, &g->d_kw_cap, (size_t)n_queries * KGS_MAX_Q));
+    CUDA_TRY(grow_dev(&g->d_qlen, &g->d_qlen_cap, (size_t)n_queries));
+    CUDA_TRY(cudaMemcpyAsync(g->d_kw, kw_dev, sizeof(int32_t) * n_queries * KGS_MAX_Q, cudaMemcpyDeviceToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(g->d_qlen, qlen_dev, sizeof(int32_t) * n_queries, cudaMemcpyDeviceToDevice, s));
+    g->last_q.clear();
+    return launch(g, n_queries, k, p, n_groups > 0 ? n_groups : 8, s);
+}
+
+kgs_status kgs_query_batch_fetch(kgs_graph *g, void *cuda_stream, kgs_result **results) {
+    if (!g || !results) return fail(KGS_EINVAL, "null argument");
+    std::lock_guard<std::mutex> lk(g->mu);
+    CUDA_TRY(cudaSetDevice(g->device));
+    if (g->last_q.empty() && g->pending) {   // device batch: lengths come back from the device
+        std::vector<int32_t> ql(g->last_nq);
+        CUDA_TRY(cudaMemcpyAsync(ql.data(), g->d_qlen, sizeof(int32_t) * g->last_nq, cudaMemcpyDeviceToHost,
+                                 (cudaStream_t)cuda_stream));
+        CUDA_TRY(cudaStreamSynchronize((cudaStream_t)cuda_stream));
+        g->last_q.assign(ql.begin(), ql.end());
+    }
+    return fetch(g, (cudaStream_t)cuda_stream, results);
 }
 
 int32_t kgs_result_count(const kgs_result *r) { return r ? (int32_t)r->ans.size() : 0; }

@@ -1,0 +1,1394 @@
+// engine.cu — the query engine of libkgs on sm_100a (product CUDA path; shares nothing with oracle/).
+//
+// ONE persistent cooperative kernel answers a batch of queries.  Its CTAs are split into G groups; a
+// group pulls the next query index from a device counter and runs the whole hot path for it with
+// group-scoped barriers (no host round trip, no further launches):
+//
+//   search     Alg. 1 ln 1-7 + Alg. 2: reset, initialise M / sources (L254), then per
+//              level { enqueue frontiers = compact the level's bitmap, merge new hits, identify central
+//              nodes (L256-266, Lemma V.1); termination (Def. 4, Thm. V.3); expansion gated by the
+//              activation levels (L210) }.
+//   pre-pass   shared predecessor DAG: the Thm. V.4 arcs of the union of all Central Graphs, computed
+//              once, round by round, into a CSR keyed by successor.
+//   extract    per central node: per-keyword backward closure over the predecessor lists (Def. 2/3,
+//              Alg. 3, R11/R12), level-cover (L454, R13), Eq. 6 key (L464, R14/R15).
+//   select     top-k by (key, id) (L478, L496): one CTA sorts |C| <= 4096 candidates, else a group-wide
+//              radix select over the 96-bit composite key.
+//   emit       the winners' graphs as sorted node / unique sorted arc lists.
+//
+// G = 1 is the single-query latency mode (the whole GPU on one query); G > 1 runs G queries at a time
+// (the batch of BASELINE.json configs[3]).
+//
+// Data layout:
+//   st[v]   uint16: low byte = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of the level),
+//           high byte = gate (0 if v contains a query keyword, else a_v).  One 2-byte load per inspected arc.
+//   nm[v]   uint8 (packed in 32-bit words for atomicOr): bits newly hit during the current level.
+//   M[v*8+i] uint8 hitting level, written once per (v, i) by the thread that set the bit; never reset.
+//   fbits   one frontier bitmap per level slot (R = amax+2 slots): "FIdentifier[v] <- 1 for level L" is one
+//           bit set on a bitmap word, so pushes never contend on a queue counter.  A node is re-queued
+//           exactly at the level where it can make progress again: a_v if it is not yet active (Alg. 2
+//           ln 5-7), gate(n)-1 if a neighbour n is still gated (ln 18-19) (reading R22).
+//
+// Snapshot semantics (reading R10): expansion at level l reads hm as of the start of the level; new hits
+// accumulate in nm and are merged when the next level is compacted, so the result equals the sequential
+// Alg. 2 (Thm. V.2).  All writes are idempotent (bits OR-ed, level l+1 written once).
+#include "kgs_internal.h"
+
+namespace kgs {
+
+// ------------------------------------------------------------------------------------------ groups
+__device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Barrier over the CTAs of one group (all CTAs are co-resident: cooperative launch).
+__device__ __forceinline__ void group_sync(GroupBar *b, int gcount) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned gen = ld_acquire(&b->gen);
+        __threadfence();
+        if (atomicAdd(&b->arrive, 1u) == (unsigned)gcount - 1) {
+            atomicExch(&b->arrive, 0u);
+            __threadfence();
+            atomicAdd(&b->gen, 1u);
+        } else {
+            while (ld_acquire(&b->gen) == gen) __nanosleep(20);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+struct Grp {
+    int g, grank, gcount;
+    int64_t gtid, gsz;
+    GroupBar *bar;
+    __device__ __forceinline__ void sync() const { group_sync(bar, gcount); }
+};
+
+// ------------------------------------------------------------------------------------------ helpers
+__device__ __forceinline__ unsigned lane_id() { return threadIdx.x & 31u; }
+__device__ __forceinline__ unsigned lanemask_lt() {
+    unsigned r;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(r));
+    return r;
+}
+
+// Append to a list with one atomic per group of converged lanes sharing the same counter.
+__device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
+    const unsigned mask = __activemask();
+    const unsigned peers = __match_any_sync(mask, key);
+    const int leader = __ffs(peers) - 1;
+    const int rank = __popc(peers & lanemask_lt());
+    uint32_t base = 0;
+    if ((int)lane_id() == leader) base = atomicAdd(counter, (uint32_t)__popc(peers));
+    base = __shfl_sync(peers, base, leader);
+    return base + rank;
+}
+
+__device__ __forceinline__ long long block_excl_scan64(long long x, long long *total, long long *sh) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+    long long incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    __syncthreads();
+    if (lane == 31) sh[wid] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long acc = 0;
+        for (int w = 0; w < nw; ++w) { const long long t = sh[w]; sh[w] = acc; acc += t; }
+        sh[32] = acc;
+    }
+    __syncthreads();
+    const long long r = sh[wid] + incl - x;
+    *total = sh[32];
+    __syncthreads();
+    return r;
+}
+__device__ __forceinline__ int block_excl_scan(int x, int *total, long long *sh) {
+    long long t;
+    const long long r = block_excl_scan64((long long)x, &t, sh);
+    *total = (int)t;
+    return (int)r;
+}
+
+__device__ __forceinline__ uint64_t ldrow(const uint8_t *M, int32_t v) {
+    return __ldcg(reinterpret_cast<const unsigned long long *>(M) + v);
+}
+
+struct Q {   // the query a group is answering
+    int32_t qi;
+    int q;
+    uint32_t full;
+    int32_t kw[kMaxQ];
+};
+
+// phase timestamp of the current query (group leader only)
+__device__ __forceinline__ void stamp(const Grp &G, QOut *o, int tag) {
+    if (G.gtid == 0) {
+        const int i = o->n_stamp;
+        if (i < kMaxStamps) { o->stamp[i] = globaltimer_ns(); o->stamp_tag[i] = tag; o->n_stamp = i + 1; }
+    }
+}
+
+// ------------------------------------------------------------------------------------------ frontier
+// Set v's bit in bitmap `bits`; `flag` records that the bitmap is non-empty.  The bit is set with a
+// reduction (no return value); the flag is stored once per group of converged lanes, after a check.
+__device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t v) {
+    uint32_t *word = bits + (v >> 5);
+    const uint32_t bit = 1u << (v & 31);
+    if (__ldcg(word) & bit) return;
+    asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
+    const unsigned mask = __activemask();
+    if ((int)lane_id() == __ffs(mask) - 1 && !__ldcg(flag)) *flag = 1u;
+}
+
+struct Ctx {        // everything a group needs while answering one query
+    const EngineArgs &a;
+    const DevWork &w;
+    Ctl *ctl;
+    const Grp &G;
+    const Q &qq;
+};
+
+// Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
+__device__ __forceinline__ void push(const Ctx &c, int32_t v, int L) {
+    const int s = L % c.a.R;
+    set_bit(c.w.fbits + (int64_t)s * c.a.W, &c.ctl->slot_flag[s], v);
+}
+
+constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16-byte loads)
+
+// Enqueue frontiers: compact a bitmap (which is cleared) into the light / big queues.
+// on_node(v) runs once per set bit and returns whether v goes to the aux list; on_aux(v, pos) runs when
+// v is written there.  (A) extracts the node ids of a tile of words with stores only; (B) processes the
+// tile's nodes one per thread.  Appends cost one atomic per CTA per tile.
+template <class OnNode, class OnAux>
+__device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W, const uint8_t *cls, int32_t *ql,
+                                        uint32_t *nl, int32_t *qb, uint32_t *nb, int32_t *aux, uint32_t *naux,
+                                        long long *sh, OnNode on_node, OnAux on_aux) {
+    const int64_t step = (int64_t)blockDim.x * kWpt;
+    const int64_t cw = ((W + G.gcount - 1) / G.gcount + kWpt - 1) / kWpt * kWpt;
+    const int64_t w0 = (int64_t)G.grank * cw, w1 = w0 + cw < W ? w0 + cw : W;
+    for (int64_t base = w0; base < w1; base += step) {
+        const int64_t wi = base + (int64_t)threadIdx.x * kWpt;
+        uint32_t word[kWpt];
+        if (wi + kWpt <= w1) {
+            const uint4 x0 = __ldcg(reinterpret_cast<const uint4 *>(bits + wi));
+            const uint4 x1 = __ldcg(reinterpret_cast<const uint4 *>(bits + wi + 4));
+            word[0] = x0.x; word[1] = x0.y; word[2] = x0.z; word[3] = x0.w;
+            word[4] = x1.x; word[5] = x1.y; word[6] = x1.z; word[7] = x1.w;
+            if ((x0.x | x0.y | x0.z | x0.w) != 0u) *reinterpret_cast<uint4 *>(bits + wi) = make_uint4(0, 0, 0, 0);
+            if ((x1.x | x1.y | x1.z | x1.w) != 0u) *reinterpret_cast<uint4 *>(bits + wi + 4) = make_uint4(0, 0, 0, 0);
+        } else {
+#pragma unroll
+            for (int k = 0; k < kWpt; ++k) {
+                word[k] = (wi + k < w1) ? __ldcg(bits + wi + k) : 0u;
+                if (word[k]) bits[wi + k] = 0u;
+            }
+        }
+        int cnt = 0;
+#pragma unroll
+        for (int k = 0; k < kWpt; ++k) cnt += __popc(word[k]);
+        long long tot;
+        const long long ex = block_excl_scan64(cnt, &tot, sh);
+        if (threadIdx.x == 0) sh[34] = tot ? (long long)atomicAdd(nl, (uint32_t)tot) : 0;
+        __syncthreads();
+        const uint32_t seg0 = (uint32_t)sh[34];
+        uint32_t p = seg0 + (uint32_t)ex;
+#pragma unroll
+        for (int k = 0; k < kWpt; ++k)
+            for (uint32_t m = word[k]; m; m &= m - 1) ql[p++] = (int32_t)((wi + k) * 32 + __ffs(m) - 1);
+        __syncthreads();
+        for (long long c0 = 0; c0 < tot; c0 += blockDim.x) {
+            const long long j = c0 + threadIdx.x;
+            int32_t v = -1;
+            int flag = 0;
+            if (j < tot) {
+                v = ql[seg0 + j];
+                flag = on_node(v) ? 1 : 0;
+                if (cls[v] != CLS_LIGHT) { qb[atomicAdd(nb, 1u)] = v; ql[seg0 + j] = -1; }
+            }
+            long long atot;
+            const long long aex = block_excl_scan64(flag, &atot, sh);
+            if (threadIdx.x == 0) sh[35] = atot ? (long long)atomicAdd(naux, (uint32_t)atot) : 0;
+            __syncthreads();
+            if (flag) {
+                const uint32_t pos = (uint32_t)sh[35] + (uint32_t)aex;
+                aux[pos] = v;
+                on_aux(v, pos);
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------ expansion
+// One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
+// sx = st[x] gathered by the caller).
+__device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, int32_t x, uint32_t sx,
+                                          unsigned &hits) {
+    const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
+    if (!bits) return;
+    const uint32_t gate = sx >> 8;
+    if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
+        const uint32_t sh = (uint32_t)(x & 3) << 3;
+        uint32_t *nw = c.w.nm + (x >> 2);
+        const uint32_t cur = (__ldcg(nw) >> sh) & 0xFFu;
+        if (!(bits & ~cur)) return;
+        const uint32_t old = (atomicOr(nw, bits << sh) >> sh) & 0xFFu;
+        const uint32_t nb = bits & ~old;
+        if (nb) {
+            hits += __popc(nb);
+            uint8_t *row = c.w.M + (int64_t)x * 8;
+            const uint8_t lv = (uint8_t)(l + 1);
+#pragma unroll
+            for (int i = 0; i < kMaxQ; ++i)
+                if (nb & (1u << i)) row[i] = lv;          // ln 21: m_xi <- l+1
+            if (old == 0) push(c, x, l + 1);              // ln 22: FIdentifier[x] <- 1 (first new bit)
+        }
+    } else {
+        push(c, v, (int)gate - 1);                        // ln 19: v must retry when x opens
+    }
+}
+
+// Alg. 2 ln 2-7 for node v at level l: returns its expansion mask (0 = does not expand now).
+__device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool leader) {
+    const uint32_t hm = __ldcg(c.w.st + v) & 0xFFu;
+    if (c.a.block_central && hm == c.qq.full) return 0;   // ln 2-3: central nodes do not expand
+    const int av = c.a.act[v];
+    if (av > l) {                                          // ln 5-7: not yet active
+        if (leader) push(c, v, av);
+        return 0;
+    }
+    return hm;                                             // ln 8-11: every hit instance has m <= l
+}
+
+constexpr int kTileMax = kBlock;
+constexpr int kBigUnroll = 4;
+constexpr int kLightUnroll = 2;
+
+struct FwdNode {
+    int32_t v;
+    uint32_t hm;
+};
+
+struct PdNode {
+    uint32_t P;      // keyword bits to expand backwards
+    uint64_t hx;     // M row of the node
+    int gx;          // gate - 1
+    int32_t cidx;    // compact id
+};
+
+struct BigTile {
+    long long incl[kTileMax];
+    long long start[kTileMax];
+    PdNode node[kTileMax];   // FwdNode fits in a PdNode slot
+};
+
+// Big frontier nodes (> kBigDeg arcs) in tiles of blockDim entries: every CTA of the group computes the
+// same tile prefix of degrees in shared memory; the tile's arcs form one index space that all threads of
+// the group stride over (owner found by binary search), kBigUnroll arcs per thread per step with the
+// index and status gathers issued before any of them is processed.
+template <class NodeT, class Prep, class Visit>
+__device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint32_t cb, const int64_t *ptr,
+                                           const int32_t *idx, const uint16_t *st, BigTile &S, long long *sh,
+                                           Prep prep, Visit visit, unsigned long long &arcs) {
+    NodeT *node = reinterpret_cast<NodeT *>(S.node);
+    for (uint32_t t0 = 0; t0 < cb; t0 += blockDim.x) {
+        const int nt = (int)min((uint32_t)blockDim.x, cb - t0);
+        const int j = threadIdx.x;
+        long long deg = 0, s0 = 0;
+        if (j < nt) {
+            const int32_t v = __ldcg(qb + t0 + j);
+            NodeT nd;
+            if (prep(v, G.grank == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
+            node[j] = nd;
+            S.start[j] = s0;
+        }
+        long long T;
+        const long long ex = block_excl_scan64(deg, &T, sh);
+        S.incl[j] = ex + deg;
+        __syncthreads();
+        if (G.gtid == 0) arcs += (unsigned long long)T;
+        for (long long e = G.gtid; e < T; e += kBigUnroll * G.gsz) {
+            int own[kBigUnroll];
+            int32_t x[kBigUnroll];
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k) {
+                const long long ek = e + k * G.gsz;
+                own[k] = -1;
+                x[k] = 0;
+                if (ek < T) {
+                    int lo = 0, hi = nt - 1;
+                    while (lo < hi) {
+                        const int mid = (lo + hi) >> 1;
+                        if (S.incl[mid] > ek) hi = mid; else lo = mid + 1;
+                    }
+                    const long long exo = lo ? S.incl[lo - 1] : 0;
+                    own[k] = lo;
+                    x[k] = __ldcs(idx + S.start[lo] + (ek - exo));
+                }
+            }
+            uint32_t sx[kBigUnroll];
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k) sx[k] = own[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+#pragma unroll
+            for (int k = 0; k < kBigUnroll; ++k)
+                if (own[k] >= 0) visit(node[own[k]], x[k], sx[k]);
+        }
+        __syncthreads();
+    }
+}
+
+// Light frontier nodes: warp w of the group takes batches w, w + #warps, ... of B nodes each (no shared
+// counter); the batch's arcs are balanced over the 32 lanes by a warp scan and a shuffle binary search.
+// B = 32 when the frontier is large, fewer (down to 1) when it is small so that every warp gets work.
+template <class NodeT, class Prep, class Visit>
+__device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
+                                             const int32_t *idx, const uint16_t *st, Prep prep, Visit visit,
+                                             unsigned long long &arcs) {
+    const uint32_t warps = (uint32_t)(G.gsz >> 5);
+    uint32_t B = (c0 + 2 * warps - 1) / (2 * warps);
+    B = B < 1 ? 1u : (B > 32 ? 32u : B);
+    const uint32_t nbatch = (c0 + B - 1) / B;
+    const unsigned lane = lane_id();
+    for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi += warps) {
+        const uint32_t i = bi * B + lane;
+        NodeT nd{};
+        int64_t start = 0;
+        int deg = 0;
+        if (lane < B && i < c0) {
+            const int32_t v = __ldcg(ql + i);   // -1: a big node, expanded by expand_big
+            if (v >= 0 && prep(v, true, nd)) { start = ptr[v]; deg = (int)(ptr[v + 1] - start); }
+        }
+        int incl = deg;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if ((int)lane >= o) incl += t;
+        }
+        const int tot = __shfl_sync(0xffffffffu, incl, 31);
+        if (lane == 0) arcs += (unsigned long long)tot;
+        const int excl = incl - deg;
+        for (int e0 = 0; e0 < tot; e0 += 32 * kLightUnroll) {
+            NodeT no[kLightUnroll];
+            int32_t x[kLightUnroll];
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k) {
+                const int e = e0 + 32 * k + (int)lane;
+                int pos = 0;
+#pragma unroll
+                for (int bb = 16; bb > 0; bb >>= 1) {
+                    const int val = __shfl_sync(0xffffffffu, incl, pos + bb - 1);
+                    if (val <= e) pos += bb;
+                }
+                const int64_t st_o = __shfl_sync(0xffffffffu, start, pos);
+                const int ex_o = __shfl_sync(0xffffffffu, excl, pos);
+                const uint32_t *src = reinterpret_cast<const uint32_t *>(&nd);
+                uint32_t *dst = reinterpret_cast<uint32_t *>(&no[k]);
+#pragma unroll
+                for (int w = 0; w < (int)(sizeof(NodeT) / 4); ++w) dst[w] = __shfl_sync(0xffffffffu, src[w], pos);
+                x[k] = e < tot ? __ldcs(idx + st_o + (e - ex_o)) : -1;
+            }
+            uint32_t sx[kLightUnroll];
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k) sx[k] = x[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+#pragma unroll
+            for (int k = 0; k < kLightUnroll; ++k)
+                if (x[k] >= 0) visit(no[k], x[k], sx[k]);
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------ pre-pass
+// Thm. V.4 test of in-arc u -> x for the keyword bits P of x (hx = M row of x, gx = gate(x) - 1,
+// su = st[u] gathered by the caller): m_xi = 1 + max{a_u, m_ui, g_x}, and in exact mode with blocking
+// (reading R12) u was not central yet at level m_xi - 1.
+__device__ __forceinline__ uint32_t pred_test(const Ctx &c, bool exact_block, uint32_t P, uint64_t hx, int gx,
+                                              int32_t u, uint32_t su, uint32_t &zbu) {
+    const uint32_t hmu = su & 0xFFu;
+    const uint32_t cand = P & hmu;
+    if (!cand) return 0;
+    const int au = c.a.act[u];
+    const uint64_t Mu = ldrow(c.w.M, u);
+    uint32_t pb = 0, zb = 0;
+    int maxrow = 0;
+#pragma unroll
+    for (int i = 0; i < kMaxQ; ++i) {
+        if (!((hmu >> i) & 1u)) continue;
+        const int mu = (int)((Mu >> (8 * i)) & 0xFF);
+        maxrow = maxrow > mu ? maxrow : mu;
+        if (mu == 0) zb |= 1u << i;
+        if (!((cand >> i) & 1u)) continue;
+        int need = au > mu ? au : mu;
+        need = need > gx ? need : gx;
+        if ((int)((hx >> (8 * i)) & 0xFF) == need + 1) pb |= 1u << i;
+    }
+    if (pb && exact_block && hmu == c.qq.full) {
+#pragma unroll
+        for (int i = 0; i < kMaxQ; ++i)   // u central at depth maxrow: it only expanded at levels < maxrow
+            if (((pb >> i) & 1u) && maxrow <= (int)((hx >> (8 * i)) & 0xFF) - 1) pb &= ~(1u << i);
+    }
+    zbu = zb;
+    return pb;
+}
+
+__device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const PdNode &nd, int32_t u, uint32_t su,
+                                         uint32_t *nbits, uint32_t *nflag) {
+    uint32_t zbu = 0;
+    const uint32_t pb = pred_test(c, exact_block, nd.P, nd.hx, nd.gx, u, su, zbu);
+    if (!pb) return;
+    const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(c.w.pcnt + nd.cidx), (unsigned)nd.cidx);
+    const uint32_t ai = agg_slot(&c.ctl->n_parcs, 0xFFFFFFFFu);
+    if ((int64_t)ai < c.w.pcap) {
+        c.w.pa_u[ai] = u;
+        c.w.pa_x[ai] = nd.cidx;
+        c.w.pa_b[ai] = (uint16_t)(pb | (zbu << 8));
+        c.w.pa_slot[ai] = (int32_t)pos;
+    } else {
+        atomicExch(&c.ctl->fatal, 5);
+    }
+    const uint32_t nb = pb & ~zbu;        // sources (m = 0) have no predecessors
+    if (nb) {
+        const uint32_t old = atomicOr(c.w.pd_state + u, nb << 8);
+        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u);
+    }
+}
+
+__device__ __forceinline__ bool pd_prepare(const Ctx &c, int32_t x, PdNode &nd) {
+    nd.P = __ldcg(c.w.pd_state + x) & 0xFFu;
+    nd.hx = ldrow(c.w.M, x);
+    nd.gx = (int)(__ldcg(c.w.st + x) >> 8) - 1;
+    nd.cidx = __ldcg(c.w.pd_cid + x);
+    return nd.P != 0;
+}
+
+__device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
+    const Grp &G = c.G;
+    Ctl *ctl = c.ctl;
+    const bool exact_block = c.a.extract_mode == KGS_EXTRACT_EXACT && c.a.block_central;
+    const int64_t W = c.a.W;
+    // seeds (every central node, for every keyword it did not contain itself) were set when each central
+    // was identified (merge step of the search): round 0 starts from them.
+    unsigned long long my_arcs = 0;
+    int r = 0;
+    for (;; ++r) {
+        const int slot = r & 1;
+        if (!__ldcg(&ctl->pd_flag[slot])) break;
+        uint32_t *qn = ctl->pd_qn[slot];
+        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; }
+        compact(G, c.w.pd_bits + (int64_t)slot * W, W, c.a.g.cls_in, c.w.pd_qlight, &qn[0], c.w.pd_qbig, &qn[1],
+                c.w.pd_touched, &ctl->n_cid, sh,
+                [&](int32_t u) {
+                    const uint32_t s = __ldcg(c.w.pd_state + u);
+                    const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
+                    const uint32_t bits = nx & ~dn;
+                    c.w.pd_state[u] = bits | ((dn | bits) << 16);
+                    return bits != 0 && __ldcg(c.w.pd_cid + u) < 0;
+                },
+                [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; });
+        G.sync();
+        stamp(G, qo, TS_PD_MERGE);
+        const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
+        if (G.gtid == 0) ctl->pd_flag[slot] = 0u;
+        uint32_t *nbits = c.w.pd_bits + (int64_t)(slot ^ 1) * W;
+        uint32_t *nflag = &ctl->pd_flag[slot ^ 1];
+        auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
+        auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) { pd_visit(c, exact_block, nd, u, su, nbits, nflag); };
+        expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
+        expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
+        G.sync();
+        stamp(G, qo, TS_PD_EXPAND);
+    }
+    if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
+    if (G.gtid == 0) ctl->pd_rounds = r;
+    // CSR of the predecessor lists: exclusive scan of pcnt over compact ids, then scatter
+    const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
+    const int64_t chunk = (ncid + G.gcount - 1) / G.gcount;
+    const int64_t lo = (int64_t)G.grank * chunk, hi = lo + chunk < ncid ? lo + chunk : ncid;
+    int run = 0;
+    for (int64_t t0 = lo; t0 < lo + chunk; t0 += blockDim.x) {
+        const int64_t j = t0 + threadIdx.x;
+        const int v = j < hi ? __ldcg(c.w.pcnt + j) : 0;
+        int tot;
+        const int ex = block_excl_scan(v, &tot, sh);
+        if (j < hi) c.w.pred_ptr[j] = run + ex;
+        run += tot;
+    }
+    if (threadIdx.x == 0) c.w.scan_tmp[G.grank] = run;
+    G.sync();
+    if (G.grank == 0) {   // exclusive scan of the per-CTA sums
+        int carry = 0;
+        for (int b0 = 0; b0 < G.gcount; b0 += blockDim.x) {
+            const int b = b0 + threadIdx.x;
+            const int v = b < G.gcount ? __ldcg(c.w.scan_tmp + b) : 0;
+            int tot;
+            const int ex = block_excl_scan(v, &tot, sh);
+            if (b < G.gcount) c.w.scan_tmp[b] = carry + ex;
+            carry += tot;
+        }
+        if (threadIdx.x == 0) c.w.pred_ptr[ncid] = carry;
+    }
+    G.sync();
+    const int off = __ldcg(c.w.scan_tmp + G.grank);
+    for (int64_t j = lo + threadIdx.x; j < hi; j += blockDim.x) c.w.pred_ptr[j] += off;
+    G.sync();
+    const int64_t np = (int64_t)__ldcg(&ctl->n_parcs) < c.w.pcap ? (int64_t)__ldcg(&ctl->n_parcs) : c.w.pcap;
+    for (int64_t ai = G.gtid; ai < np; ai += G.gsz) {
+        const int64_t pos = (int64_t)__ldcg(c.w.pred_ptr + c.w.pa_x[ai]) + c.w.pa_slot[ai];
+        c.w.pred_u[pos] = c.w.pa_u[ai];
+        c.w.pred_b[pos] = c.w.pa_b[ai];
+    }
+    G.sync();
+    stamp(G, qo, TS_PD_CSR);
+}
+
+// ------------------------------------------------------------------------------------------ search
+__device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    const DevWork &w = c.w;
+    Ctl *ctl = c.ctl;
+    const int64_t n = a.g.n, W = a.W;
+    const int R = a.R, amax = R - 2;
+    const uint32_t full = c.qq.full;
+    uint8_t *st8 = reinterpret_cast<uint8_t *>(w.st);
+    uint8_t *nm8 = reinterpret_cast<uint8_t *>(w.nm);
+    const int64_t gtid = G.gtid, gsz = G.gsz;
+
+    // ---- reset the state the previous query of this group left behind
+    const uint32_t valid = __ldcg(w.gstate + 2), lastR = __ldcg(w.gstate + 3);
+    const uint32_t done = __ldcg(w.gstate + 1);
+    if (!valid || (int)lastR != R || done == 0) {
+        const int64_t n8 = n / 8;
+        for (int64_t j = gtid; j < n8; j += gsz) {
+            const uint2 av = *reinterpret_cast<const uint2 *>(a.act + j * 8);
+            uint4 o;
+            o.x = ((av.x & 0xFFu) << 8) | ((av.x & 0xFF00u) << 16);
+            o.y = ((av.x >> 8) & 0xFF00u) | ((av.x >> 24) << 24);
+            o.z = ((av.y & 0xFFu) << 8) | ((av.y & 0xFF00u) << 16);
+            o.w = ((av.y >> 8) & 0xFF00u) | ((av.y >> 24) << 24);
+            *reinterpret_cast<uint4 *>(w.st + j * 8) = o;
+        }
+        for (int64_t v = n8 * 8 + gtid; v < n; v += gsz) w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+        for (int64_t v = gtid; v < (n + 3) / 4; v += gsz) w.nm[v] = 0u;
+        for (int64_t j = gtid; j < (int64_t)R * W; j += gsz) w.fbits[j] = 0u;
+        for (int64_t j = gtid; j < 2 * W; j += gsz) w.pd_bits[j] = 0u;
+        for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
+    } else {
+        const Ctl *pv = w.ctl[(done + 1) & 1];   // the previous query's block
+        for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
+            const int32_t v = w.pd_touched[j];
+            w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[j] = 0;
+        }
+        const int64_t pt = (int64_t)pv->n_touched;
+        if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
+            const int64_t n8 = n / 8;
+            for (int64_t j = gtid; j < n8; j += gsz) {
+                const uint2 av = *reinterpret_cast<const uint2 *>(a.act + j * 8);
+                uint4 o;
+                o.x = ((av.x & 0xFFu) << 8) | ((av.x & 0xFF00u) << 16);
+                o.y = ((av.x >> 8) & 0xFF00u) | ((av.x >> 24) << 24);
+                o.z = ((av.y & 0xFFu) << 8) | ((av.y & 0xFF00u) << 16);
+                o.w = ((av.y >> 8) & 0xFF00u) | ((av.y >> 24) << 24);
+                *reinterpret_cast<uint4 *>(w.st + j * 8) = o;
+            }
+            for (int64_t v = n8 * 8 + gtid; v < n; v += gsz) w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+        } else {
+            for (int64_t j = gtid; j < pt; j += gsz) {
+                const int32_t v = w.touched[j];
+                w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+            }
+        }
+        for (int s = 0; s < R; ++s)   // level slots still pending when the previous query stopped
+            if (pv->slot_flag[s])
+                for (int64_t j = gtid; j < W; j += gsz) w.fbits[(int64_t)s * W + j] = 0u;
+    }
+    bool empty = false;
+    for (int i = 0; i < c.qq.q; ++i) {
+        const int32_t t = c.qq.kw[i];
+        if (a.g.kw_ptr[t + 1] == a.g.kw_ptr[t]) empty = true;
+    }
+    G.sync();
+    stamp(G, qo, TS_RESET);
+    // ---- initialisation: M = 0 on T_i, keyword nodes ungated, F_0 = K
+    {
+        int64_t kb[kMaxQ], ko[kMaxQ + 1];
+        ko[0] = 0;
+        for (int i = 0; i < c.qq.q; ++i) {
+            const int32_t t = c.qq.kw[i];
+            kb[i] = a.g.kw_ptr[t];
+            ko[i + 1] = ko[i] + (a.g.kw_ptr[t + 1] - kb[i]);
+        }
+        for (int64_t j = gtid; j < ko[c.qq.q]; j += gsz) {
+            int i = 0;
+            while (j >= ko[i + 1]) ++i;
+            const int32_t v = a.g.kw_nodes[kb[i] + (j - ko[i])];
+            w.M[(int64_t)v * 8 + i] = 0;
+            st8[2 * (int64_t)v + 1] = 0;                                  // keyword node: no gate (L210)
+            atomicOr(w.nm + (v >> 2), (1u << i) << ((v & 3) * 8));        // hit in B_i at level 0
+            push(c, v, 0);
+        }
+    }
+    G.sync();
+    stamp(G, qo, TS_SCATTER);
+
+    unsigned long long my_arcs = 0;
+    unsigned my_hits = 0;
+    for (int l = 0;; ++l) {
+        // ---- enqueue frontiers: anything pending at this or a later level?
+        __shared__ int s_pend;
+        if (threadIdx.x == 0) {
+            bool pend = false;
+            const int top = l > amax ? l : amax;
+            for (int L = l; L <= top; ++L) pend |= __ldcg(&ctl->slot_flag[L % R]) != 0u;
+            s_pend = pend;
+        }
+        __syncthreads();
+        if (!s_pend) {
+            if (gtid == 0) { ctl->stop_reason = empty ? KGS_STOP_EMPTY_KEYWORD : KGS_STOP_EXHAUSTED; ctl->levels = l; }
+            break;
+        }
+        const int s = l % R;
+        uint32_t *qn = ctl->qn[l & 1];
+        if (gtid == 0) { ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; }
+        // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
+        compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
+                &ctl->n_touched, sh,
+                [&](int32_t v) {
+                    const uint32_t b = nm8[v];
+                    if (!b) return false;
+                    nm8[v] = 0;
+                    const uint32_t old = st8[2 * (int64_t)v];
+                    const uint32_t nw = old | b;
+                    st8[2 * (int64_t)v] = (uint8_t)nw;
+                    if (nw == full && old != full) {                        // Lemma V.1: depth = l
+                        const uint32_t ci = agg_slot(&ctl->n_central, 1u);
+                        w.centrals[ci] = v;
+                        w.cdepth[ci] = (uint8_t)l;
+                        // seed of the top-down pre-pass: expand backwards every keyword v does not contain
+                        const uint64_t Mv = ldrow(w.M, v);
+                        uint32_t zb = 0;
+                        for (int i = 0; i < c.qq.q; ++i) if (((Mv >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
+                        if (full & ~zb) {
+                            w.pd_state[v] = (full & ~zb) << 8;
+                            set_bit(w.pd_bits, &ctl->pd_flag[0], v);
+                        }
+                    }
+                    return old == 0;
+                },
+                [&](int32_t, uint32_t) {});
+        G.sync();
+        stamp(G, qo, TS_MERGE);
+        __shared__ uint32_t s_ctl[3];
+        if (threadIdx.x == 0) { s_ctl[0] = __ldcg(&qn[0]); s_ctl[1] = __ldcg(&qn[1]); s_ctl[2] = __ldcg(&ctl->n_central); }
+        __syncthreads();
+        const uint32_t c0 = s_ctl[0], c1 = s_ctl[1], nc = s_ctl[2];
+        if (gtid == 0) ctl->frontier_total += (unsigned long long)c0 + c1;
+        // ---- termination (Def. 4 / Thm. V.3; reading R9: no expansion at d)
+        if (empty) {   // some T_i is empty: M holds the initialisation, nothing can be central (R17)
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_EMPTY_KEYWORD; ctl->levels = 0; }
+            break;
+        }
+        if (nc >= (uint32_t)a.k) {
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_K; ctl->levels = l; }
+            break;
+        }
+        if (l == a.max_depth) {
+            if (gtid == 0) { ctl->stop_reason = KGS_STOP_MAX_DEPTH; ctl->levels = l; }
+            break;
+        }
+        // ---- expansion (Alg. 2)
+        // slot s is consumed; nothing pushes to level l + R during this level (pushes reach <= max(l+1, amax))
+        if (gtid == 0) ctl->slot_flag[s] = 0u;
+        auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
+            nd.v = v;
+            nd.hm = prepare(c, l, v, leader);
+            return nd.hm != 0;
+        };
+        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(c, l, nd.v, nd.hm, x, sx, my_hits); };
+        expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
+        expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
+        G.sync();
+        stamp(G, qo, TS_EXPAND);
+    }
+    const unsigned wa = __reduce_add_sync(0xffffffffu, (unsigned)my_arcs);   // per-warp totals fit 32 bits
+    const unsigned wh = __reduce_add_sync(0xffffffffu, my_hits);
+    __shared__ unsigned long long s_sum[2];
+    if (threadIdx.x < 2) s_sum[threadIdx.x] = 0ull;
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0) {
+        if (wa) atomicAdd(&s_sum[0], (unsigned long long)wa);
+        if (wh) atomicAdd(&s_sum[1], (unsigned long long)wh);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {      // one global atomic per CTA
+        if (s_sum[0]) atomicAdd(&ctl->arcs_scanned, s_sum[0]);
+        if (s_sum[1]) atomicAdd(&ctl->hits, s_sum[1]);
+    }
+    G.sync();
+    stamp(G, qo, TS_END);
+    if (gtid == 0) qo->t_search_end = globaltimer_ns();
+}
+
+// ------------------------------------------------------------------------------------------ top-down
+struct WarpTeam {
+    __device__ __forceinline__ int rank() const { return threadIdx.x & 31; }
+    __device__ __forceinline__ int size() const { return 32; }
+    __device__ __forceinline__ void sync() const { __syncwarp(); }
+    __device__ __forceinline__ int scan_excl(int x, int *total) const {
+        int incl = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (rank() >= o) incl += t;
+        }
+        *total = __shfl_sync(0xffffffffu, incl, 31);
+        return incl - x;
+    }
+};
+
+struct BlockTeam {
+    long long *sh;   // block scan scratch (>= 40 entries)
+    __device__ __forceinline__ int rank() const { return threadIdx.x; }
+    __device__ __forceinline__ int size() const { return blockDim.x; }
+    __device__ __forceinline__ void sync() const { __syncthreads(); }
+    __device__ __forceinline__ int scan_excl(int x, int *total) const { return block_excl_scan(x, total, sh); }
+};
+
+enum { SC_NODES = 0, SC_ARCS, SC_HEAD, SC_TAIL, SC_OVF, SC_CHANGED, SC_COV, SC_SSTAR, SC_NOUT, SC_AOUT, SC_N };
+
+struct Arena {
+    int32_t *hkey;      // [hcap] node id or -1
+    int32_t *hval;      // [hcap] node index or -1
+    int32_t *id;        // [ncap]
+    uint32_t *inmask;   // [ncap] bit i: node in DAG_i(c)
+    uint32_t *zb;       // [ncap] bit i: m_vi == 0 (source of B_i)
+    uint32_t *pending;  // [ncap] bits still to expand backwards
+    uint32_t *keep;     // [ncap] bit i: kept in DAG_i after level-cover
+    int32_t *fifo;      // [ncap] ring of node indices with pending bits
+    int32_t *au, *ax;   // [acap] arc endpoints (node indices)
+    uint32_t *ab;       // [acap] keyword bits of the arc
+    int32_t *b_j;       // [team] batch: node index
+    int64_t *b_start;   // [team] batch: predecessor-list start
+    int32_t *b_incl;    // [team] batch: inclusive count
+    uint32_t *b_P;      // [team] batch: keywords to expand
+    unsigned long long *sortbuf;  // [2*acap]
+    int32_t *scal;      // [SC_N]
+    double *dsum;
+    int hcap, ncap, acap;
+};
+
+__host__ __device__ inline size_t arena_bytes(int hcap, int ncap, int acap, int team, bool with_sort) {
+    size_t b = 16 + sizeof(int64_t) * team + sizeof(double);
+    if (with_sort) b += sizeof(unsigned long long) * 2 * (size_t)acap;
+    b += sizeof(int32_t) * 2 * (size_t)hcap + sizeof(int32_t) * 6 * (size_t)ncap + sizeof(int32_t) * 3 * (size_t)acap;
+    b += sizeof(int32_t) * 3 * (size_t)team + sizeof(int32_t) * SC_N + 16;
+    return (b + 255) & ~size_t(255);
+}
+size_t arena_bytes_host(int hcap, int ncap, int acap, int team, bool with_sort) {
+    return arena_bytes(hcap, ncap, acap, team, with_sort);
+}
+
+__device__ __forceinline__ char *align8(char *p) {
+    return reinterpret_cast<char *>((reinterpret_cast<uintptr_t>(p) + 7) & ~uintptr_t(7));
+}
+
+__device__ Arena carve(char *p, int hcap, int ncap, int acap, int team, bool with_sort) {
+    Arena S;
+    S.hcap = hcap; S.ncap = ncap; S.acap = acap;
+    p = align8(p);
+    S.b_start = reinterpret_cast<int64_t *>(p); p += sizeof(int64_t) * team;
+    S.dsum = reinterpret_cast<double *>(p); p += sizeof(double);
+    if (with_sort) { S.sortbuf = reinterpret_cast<unsigned long long *>(p); p += sizeof(unsigned long long) * 2 * (size_t)acap; }
+    else S.sortbuf = nullptr;
+    S.hkey = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * hcap;
+    S.hval = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * hcap;
+    S.id = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * ncap;
+    S.inmask = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * ncap;
+    S.zb = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * ncap;
+    S.pending = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * ncap;
+    S.keep = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * ncap;
+    S.fifo = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * ncap;
+    S.au = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * acap;
+    S.ax = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * acap;
+    S.ab = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * acap;
+    S.b_j = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * team;
+    S.b_incl = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * team;
+    S.b_P = reinterpret_cast<uint32_t *>(p); p += sizeof(uint32_t) * team;
+    S.scal = reinterpret_cast<int32_t *>(p);
+    return S;
+}
+
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352dU; x ^= x >> 15; x *= 0x846ca68bU; x ^= x >> 16;
+    return x;
+}
+
+// insert (or find) node u; returns its index, -1 on overflow
+__device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu) {
+    uint32_t h = hash32((uint32_t)u) & (uint32_t)(S.hcap - 1);
+    for (int probe = 0; probe < S.hcap; ++probe) {
+        const int32_t k = atomicCAS(S.hkey + h, -1, u);
+        if (k == -1) {
+            const int idx = atomicAdd(S.scal + SC_NODES, 1);
+            if (idx >= S.ncap) { atomicExch(S.scal + SC_OVF, 1); atomicExch(S.hval + h, -2); return -1; }
+            S.id[idx] = u;
+            S.zb[idx] = zbu;
+            __threadfence_block();
+            atomicExch(S.hval + h, idx);
+            return idx;
+        }
+        if (k == u) {
+            int v;
+            while ((v = atomicAdd(S.hval + h, 0)) == -1) { }
+            return v >= 0 ? v : -1;
+        }
+        h = (h + 1) & (uint32_t)(S.hcap - 1);
+    }
+    atomicExch(S.scal + SC_OVF, 1);
+    return -1;
+}
+
+__device__ __forceinline__ void fifo_push(Arena &S, int j) {
+    const int pos = atomicAdd(S.scal + SC_TAIL, 1);
+    S.fifo[pos % S.ncap] = j;
+}
+
+// Closure (over the shared predecessor lists) + level-cover + Eq. 6 key of the Central Graph at c.
+// Returns false on arena overflow.
+template <class Team>
+__device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, int depth, double *key) {
+    const uint32_t full = c.qq.full;
+    const int r = T.rank(), ts = T.size();
+    for (int i = r; i < S.hcap; i += ts) { S.hkey[i] = -1; S.hval[i] = -1; }
+    for (int i = r; i < S.ncap; i += ts) { S.inmask[i] = 0; S.pending[i] = 0; S.keep[i] = 0; }
+    if (r < SC_N) S.scal[r] = 0;
+    if (r == 0) *S.dsum = 0.0;
+    T.sync();
+    if (r == 0) {
+        const uint64_t Mc = ldrow(c.w.M, cn);
+        uint32_t zbc = 0;
+        for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
+        const int j = arena_insert(S, cn, zbc);  // index 0
+        S.inmask[j] = full;
+        const uint32_t p = full & ~zbc;
+        if (p) { S.pending[j] = p; fifo_push(S, j); }
+    }
+    T.sync();
+    // ---- backward closure, batch by batch (all pending nodes of a round in parallel)
+    for (;;) {
+        const int head = S.scal[SC_HEAD], tail = S.scal[SC_TAIL];
+        if (head == tail || S.scal[SC_OVF]) break;
+        T.sync();
+        for (int b0 = head; b0 < tail; b0 += ts) {
+            int deg = 0;
+            if (b0 + r < tail) {
+                const int j = S.fifo[(b0 + r) % S.ncap];
+                const uint32_t P = atomicExch(S.pending + j, 0u);
+                const int32_t x = S.id[j];
+                S.b_j[r] = j;
+                S.b_P[r] = P;
+                const int32_t cid = __ldcg(c.w.pd_cid + x);   // predecessor list from the shared DAG
+                int64_t s0 = 0;
+                if (P && cid >= 0) { s0 = __ldcg(c.w.pred_ptr + cid); deg = (int)(__ldcg(c.w.pred_ptr + cid + 1) - s0); }
+                S.b_start[r] = s0;
+            }
+            int tot;
+            const int ex = T.scan_excl(deg, &tot);
+            S.b_incl[r] = ex + deg;
+            T.sync();
+            const int nb = min(ts, tail - b0);
+            for (int e = r; e < tot; e += ts) {
+                int lo = 0, hi = nb - 1;       // owner = first o with incl[o] > e
+                while (lo < hi) {
+                    const int mid = (lo + hi) >> 1;
+                    if (S.b_incl[mid] > e) hi = mid; else lo = mid + 1;
+                }
+                const int o = lo;
+                const int exo = o ? S.b_incl[o - 1] : 0;
+                const int64_t pi = S.b_start[o] + (e - exo);
+                const int32_t u = __ldcg(c.w.pred_u + pi);
+                const uint32_t bz = __ldcg(c.w.pred_b + pi);
+                const uint32_t pb = bz & S.b_P[o] & 0xFFu;   // Thm. V.4 arc for the keywords x needs here
+                if (!pb) continue;
+                const uint32_t zbu = bz >> 8;
+                const int j = arena_insert(S, u, zbu);
+                if (j < 0) continue;
+                const uint32_t old = atomicOr(S.inmask + j, pb);
+                const uint32_t nbits = pb & ~old & ~S.zb[j];
+                if (nbits) {
+                    const uint32_t oldp = atomicOr(S.pending + j, nbits);
+                    if (oldp == 0) fifo_push(S, j);
+                }
+                const int ai = atomicAdd(S.scal + SC_ARCS, 1);
+                if (ai >= S.acap) { atomicExch(S.scal + SC_OVF, 1); continue; }
+                S.au[ai] = j;
+                S.ax[ai] = S.b_j[o];
+                S.ab[ai] = pb;
+            }
+            T.sync();
+        }
+        if (r == 0) S.scal[SC_HEAD] = tail;
+        T.sync();
+    }
+    T.sync();
+    if (S.scal[SC_OVF]) return false;
+    const int nn = S.scal[SC_NODES];
+    const int na = S.scal[SC_ARCS] < S.acap ? S.scal[SC_ARCS] : S.acap;
+    // ---- level-cover
+    if (c.a.level_cover) {
+        const uint32_t cov0 = S.zb[0];
+        int sstar = c.qq.q + 1;
+        if (cov0 != full) {
+            if (r == 0) S.scal[SC_COV] = (int)cov0;
+            T.sync();
+            for (int s = c.qq.q; s >= 1; --s) {
+                for (int j = 1 + r; j < nn; j += ts) {
+                    const uint32_t con = S.inmask[j] & S.zb[j];
+                    if (__popc(con) == s) atomicOr(reinterpret_cast<unsigned *>(S.scal + SC_COV), con);
+                }
+                T.sync();
+                if ((uint32_t)S.scal[SC_COV] == full) { sstar = s; break; }
+                T.sync();
+            }
+        }
+        for (int j = r; j < nn; j += ts) {
+            const uint32_t con = S.inmask[j] & S.zb[j];
+            S.keep[j] = (j == 0 || __popc(con) >= sstar) ? con : 0u;
+        }
+        T.sync();
+        for (;;) {   // forward reachability from the kept sources inside each DAG_i
+            if (r == 0) S.scal[SC_CHANGED] = 0;
+            T.sync();
+            for (int e = r; e < na; e += ts) {
+                const uint32_t add = S.keep[S.au[e]] & S.ab[e];
+                if (add & ~S.keep[S.ax[e]]) { atomicOr(S.keep + S.ax[e], add); S.scal[SC_CHANGED] = 1; }
+            }
+            T.sync();
+            const int ch = S.scal[SC_CHANGED];
+            T.sync();
+            if (!ch) break;
+        }
+        if (r == 0) S.keep[0] = full;
+    } else {
+        for (int j = r; j < nn; j += ts) S.keep[j] = S.inmask[j];
+    }
+    T.sync();
+    // ---- Eq. 6
+    for (int j = r; j < nn; j += ts)
+        if (S.keep[j]) atomicAdd(S.dsum, (double)c.a.g.weight[S.id[j]]);
+    T.sync();
+    *key = __dmul_rn(c.a.dpow[depth], *S.dsum);
+    T.sync();
+    return true;
+}
+
+// team bitonic sort (ascending) of buf[0..len) padded to a power of two with ~0
+template <class Team>
+__device__ void team_sort(const Team &T, unsigned long long *buf, int len) {
+    int p2 = 1;
+    while (p2 < len) p2 <<= 1;
+    for (int i = len + T.rank(); i < p2; i += T.size()) buf[i] = ~0ull;
+    T.sync();
+    for (int k = 2; k <= p2; k <<= 1)
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int i = T.rank(); i < p2; i += T.size()) {
+                const int l = i ^ j;
+                if (l > i) {
+                    const unsigned long long x = buf[i], y = buf[l];
+                    const bool up = (i & k) == 0;
+                    if ((x > y) == up) { buf[i] = y; buf[l] = x; }
+                }
+            }
+            T.sync();
+        }
+}
+
+// write the kept nodes / arcs of the arena (after central_graph) sorted and unique, as answer `rank_i`
+template <class Team>
+__device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
+    const EngineArgs &a = c.a;
+    const int r = T.rank(), ts = T.size();
+    const int nn = S.scal[SC_NODES];
+    const int na = S.scal[SC_ARCS];
+    if (r == 0) { S.scal[SC_NOUT] = 0; S.scal[SC_AOUT] = 0; }
+    T.sync();
+    for (int j = r; j < nn; j += ts)
+        if (S.keep[j]) S.sortbuf[atomicAdd(S.scal + SC_NOUT, 1)] = (unsigned long long)(uint32_t)S.id[j];
+    T.sync();
+    const int kn = S.scal[SC_NOUT];
+    team_sort(T, S.sortbuf, kn);
+    const int64_t ans = (int64_t)c.qq.qi * a.k + rank_i;
+    if (r == 0) S.b_start[0] = (int64_t)atomicAdd(a.out_used + 0, (unsigned long long)kn);   // team broadcast
+    T.sync();
+    const long long no = S.b_start[0];
+    T.sync();
+    if (no + kn > a.out_nodes_cap) {
+        if (r == 0) atomicExch(&c.ctl->fatal, 1);
+        return false;
+    }
+    for (int i = r; i < kn; i += ts) a.out_nodes[no + i] = (int32_t)S.sortbuf[i];
+    T.sync();
+    if (r == 0) S.scal[SC_AOUT] = 0;
+    T.sync();
+    for (int e = r; e < na; e += ts)
+        if (S.keep[S.au[e]] & S.ab[e])
+            S.sortbuf[atomicAdd(S.scal + SC_AOUT, 1)] =
+                ((unsigned long long)(uint32_t)S.id[S.au[e]] << 32) | (uint32_t)S.id[S.ax[e]];
+    T.sync();
+    const int ka = S.scal[SC_AOUT];
+    team_sort(T, S.sortbuf, ka);
+    int kept = 0;
+    for (int b0 = 0; b0 < ka; b0 += ts) {
+        const int i = b0 + r;
+        const int flag = (i < ka && (i == 0 || S.sortbuf[i] != S.sortbuf[i - 1])) ? 1 : 0;
+        int tot;
+        const int ex = T.scan_excl(flag, &tot);
+        T.sync();
+        if (flag) S.sortbuf[ka + kept + ex] = S.sortbuf[i];
+        kept += tot;
+        T.sync();
+    }
+    if (r == 0) S.b_start[0] = (int64_t)atomicAdd(a.out_used + 1, (unsigned long long)kept);
+    T.sync();
+    const long long ao = S.b_start[0];
+    T.sync();
+    if (ao + kept > a.out_arcs_cap) {
+        if (r == 0) atomicExch(&c.ctl->fatal, 1);
+        return false;
+    }
+    for (int i = r; i < kept; i += ts) {
+        const unsigned long long key = S.sortbuf[ka + i];
+        a.out_arcs[2 * (ao + i)] = (int32_t)(key >> 32);
+        a.out_arcs[2 * (ao + i) + 1] = (int32_t)(key & 0xFFFFFFFFu);
+    }
+    if (r == 0) {
+        a.out_hdr[4 * ans + 2] = kn;
+        a.out_hdr[4 * ans + 3] = kept;
+        a.out_off[2 * ans] = no;
+        a.out_off[2 * ans + 1] = ao;
+    }
+    T.sync();
+    return true;
+}
+
+// ------------------------------------------------------------------------------------------ select
+__device__ __forceinline__ void comp_key(const Ctx &c, uint32_t i, uint64_t &hi, uint32_t &lo) {
+    hi = (uint64_t)__double_as_longlong(__ldcg(c.w.ckey + i));
+    lo = (uint32_t)__ldcg(c.w.centrals + i);
+}
+__device__ __forceinline__ uint32_t digit_of(uint64_t hi, uint32_t lo, int d) {
+    return d < 8 ? (uint32_t)((hi >> (56 - 8 * d)) & 0xFF) : (lo >> (24 - 8 * (d - 8))) & 0xFF;
+}
+__device__ __forceinline__ bool prefix_match(uint64_t hi, uint32_t lo, uint64_t phi, uint32_t plo, int d) {
+    if (d == 0) return true;
+    if (d <= 8) {
+        const uint64_t m = d == 8 ? ~0ull : (~0ull << (64 - 8 * d));
+        return (hi & m) == (phi & m);
+    }
+    if (hi != phi) return false;
+    const uint32_t m = d == 12 ? 0xFFFFFFFFu : (0xFFFFFFFFu << (32 - 8 * (d - 8)));
+    return (lo & m) == (plo & m);
+}
+
+// Top-k by (fp64 key asc, central id asc).  |C| <= KGS_MAX_K: one CTA sorts every candidate.
+// Otherwise a group-wide MSD radix select over the 96-bit composite (12 digits of 8 bits) keeps
+// exactly k candidates, which one CTA then sorts.  Result: sel[0..count), ctl->sel_count.
+__device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
+    const Grp &G = c.G;
+    Ctl *ctl = c.ctl;
+    const uint32_t nc = __ldcg(&ctl->n_central);
+    const uint32_t kk = (uint32_t)c.a.k < nc ? (uint32_t)c.a.k : nc;
+    if (nc > (uint32_t)KGS_MAX_K) {
+        __shared__ uint32_t hsh[256];
+        __shared__ uint32_t s_bucket, s_before;
+        uint64_t phi = 0;
+        uint32_t plo = 0, want = kk;
+        for (int d = 0; d < 12; ++d) {
+            for (int t = threadIdx.x; t < 256; t += blockDim.x) hsh[t] = 0;
+            __syncthreads();
+            for (int64_t i = G.gtid; i < nc; i += G.gsz) {
+                uint64_t hi; uint32_t lo;
+                comp_key(c, (uint32_t)i, hi, lo);
+                if (prefix_match(hi, lo, phi, plo, d)) atomicAdd(hsh + digit_of(hi, lo, d), 1u);
+            }
+            __syncthreads();
+            for (int t = threadIdx.x; t < 256; t += blockDim.x)
+                if (hsh[t]) atomicAdd(&ctl->hist[d][t], hsh[t]);
+            G.sync();
+            if (threadIdx.x == 0) {
+                uint32_t acc = 0, b = 0;
+                for (b = 0; b < 256; ++b) {
+                    const uint32_t h = __ldcg(&ctl->hist[d][b]);
+                    if (acc + h >= want) break;
+                    acc += h;
+                }
+                s_bucket = b; s_before = acc;
+            }
+            __syncthreads();
+            want -= s_before;
+            const uint64_t bk = s_bucket;
+            if (d < 8) phi |= bk << (56 - 8 * d);
+            else plo |= (uint32_t)bk << (24 - 8 * (d - 8));
+            __syncthreads();
+        }
+        for (int64_t i = G.gtid; i < nc; i += G.gsz) {   // exactly kk candidates are <= the threshold
+            uint64_t hi; uint32_t lo;
+            comp_key(c, (uint32_t)i, hi, lo);
+            if (hi < phi || (hi == phi && lo <= plo)) {
+                const uint32_t pos = atomicAdd(&ctl->sel_count, 1u);
+                if (pos < (uint32_t)KGS_MAX_K) c.w.sel[pos] = (int32_t)i;
+            }
+        }
+        G.sync();
+    }
+    if (G.grank == 0) {   // one CTA ranks (all candidates, or the radix-selected ones)
+        unsigned long long *khi = reinterpret_cast<unsigned long long *>(dsmem);
+        uint32_t *klo = reinterpret_cast<uint32_t *>(khi + KGS_MAX_K);
+        int32_t *kid = reinterpret_cast<int32_t *>(klo + KGS_MAX_K);
+        const bool small = nc <= (uint32_t)KGS_MAX_K;
+        const uint32_t cnt = small ? nc : __ldcg(&ctl->sel_count);
+        int p2 = 1;
+        while (p2 < (int)cnt) p2 <<= 1;
+        for (int i = threadIdx.x; i < p2; i += blockDim.x) {
+            if (i < (int)cnt) {
+                const int32_t idx = small ? i : __ldcg(c.w.sel + i);
+                uint64_t hi; uint32_t lo;
+                comp_key(c, (uint32_t)idx, hi, lo);
+                khi[i] = hi; klo[i] = lo; kid[i] = idx;
+            } else { khi[i] = ~0ull; klo[i] = 0xFFFFFFFFu; kid[i] = -1; }
+        }
+        __syncthreads();
+        for (int k = 2; k <= p2; k <<= 1)
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int i = threadIdx.x; i < p2; i += blockDim.x) {
+                    const int l = i ^ j;
+                    if (l > i) {
+                        const bool gt = khi[i] > khi[l] || (khi[i] == khi[l] && klo[i] > klo[l]);
+                        const bool up = (i & k) == 0;
+                        if (gt == up) {
+                            const unsigned long long th = khi[i]; khi[i] = khi[l]; khi[l] = th;
+                            const uint32_t tl = klo[i]; klo[i] = klo[l]; klo[l] = tl;
+                            const int32_t ti = kid[i]; kid[i] = kid[l]; kid[l] = ti;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        for (int i = threadIdx.x; i < (int)kk; i += blockDim.x) c.w.sel[i] = kid[i];
+        if (threadIdx.x == 0) ctl->sel_count = kk;
+    }
+    G.sync();
+}
+
+// ------------------------------------------------------------------------------------------ top-down driver
+__device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    Ctl *ctl = c.ctl;
+    const uint32_t nc = __ldcg(&ctl->n_central);
+    // extract: one warp per central node, arena in global memory (per warp of the grid)
+    {
+        const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
+        Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
+        WarpTeam T;
+        for (;;) {
+            uint32_t idx = 0;
+            if (T.rank() == 0) idx = atomicAdd(&ctl->work_ext, 1u);
+            idx = __shfl_sync(0xffffffffu, idx, 0);
+            if (idx >= nc) break;
+            const int32_t cn = __ldcg(c.w.centrals + idx);
+            double key = 0.0;
+            const bool ok = central_graph(T, S, c, cn, __ldcg(c.w.cdepth + idx), &key);
+            if (T.rank() == 0) {
+                if (ok) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
+                else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = (int32_t)idx; }
+            }
+            __syncwarp();
+        }
+    }
+    G.sync();
+    stamp(G, qo, TS_EXTRACT);
+    // overflowed candidates: one CTA each over the CTA's global arena
+    const uint32_t no = __ldcg(&ctl->n_overflow);
+    BlockTeam BT{sh};
+    if (no) {
+        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+        for (uint32_t t = G.grank; t < no; t += G.gcount) {
+            const int32_t idx = __ldcg(c.w.overflow + t);
+            double key = 0.0;
+            const bool ok = central_graph(BT, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+            if (threadIdx.x == 0) {
+                if (ok) c.w.ckey[idx] = key;
+                else atomicExch(&ctl->fatal, 2);
+            }
+            __syncthreads();
+        }
+        G.sync();
+    }
+    stamp(G, qo, TS_EXTRACT_BIG);
+    select_topk(c, sh, dsmem);
+    stamp(G, qo, TS_SELECT);
+    // emit: one warp per winner (per-warp arena), overflowed winners by a CTA
+    const uint32_t cnt = __ldcg(&ctl->sel_count);
+    {
+        const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
+        Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
+        WarpTeam T;
+        for (;;) {
+            uint32_t rk = 0;
+            if (T.rank() == 0) rk = atomicAdd(&ctl->work_emit, 1u);
+            rk = __shfl_sync(0xffffffffu, rk, 0);
+            if (rk >= cnt) break;
+            const int32_t idx = __ldcg(c.w.sel + rk);
+            const int64_t ans = (int64_t)c.qq.qi * a.k + rk;
+            if (T.rank() == 0) {
+                a.out_hdr[4 * ans + 0] = __ldcg(c.w.centrals + idx);
+                a.out_hdr[4 * ans + 1] = __ldcg(c.w.cdepth + idx);
+                a.out_key[ans] = __ldcg(c.w.ckey + idx);
+            }
+            if (__ldcg(c.w.cflag + idx)) {
+                if (T.rank() == 0) c.w.overflow[atomicAdd(&ctl->work_big, 1u)] = (int32_t)rk;   // reuse list
+                continue;
+            }
+            double key;
+            if (central_graph(T, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
+                emit_graph(T, S, c, (int)rk);
+            else if (T.rank() == 0) atomicExch(&ctl->fatal, 3);
+        }
+    }
+    G.sync();
+    const uint32_t nbig = __ldcg(&ctl->work_big);
+    if (nbig) {
+        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+        for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
+            const int rk = __ldcg(c.w.overflow + t);
+            const int32_t idx = __ldcg(c.w.sel + rk);
+            double key;
+            if (central_graph(BT, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
+                emit_graph(BT, S, c, rk);
+            else if (threadIdx.x == 0) atomicExch(&ctl->fatal, 4);
+            __syncthreads();
+        }
+        G.sync();
+    }
+    stamp(G, qo, TS_EMIT);
+}
+
+// ------------------------------------------------------------------------------------------ engine
+__global__ void __launch_bounds__(kBlock, 2) k_engine(EngineArgs a) {
+    extern __shared__ __align__(16) char dsmem[];
+    __shared__ BigTile s_big;
+    __shared__ long long sh[40];
+    __shared__ int32_t s_q[2 + kMaxQ];
+    // group of this CTA: contiguous ranges, sizes differ by at most one
+    Grp G;
+    {
+        const int nb = gridDim.x, gsz_b = nb / a.G, extra = nb % a.G;
+        const int b = blockIdx.x;
+        const int cut = extra * (gsz_b + 1);
+        if (b < cut) { G.g = b / (gsz_b + 1); G.grank = b % (gsz_b + 1); G.gcount = gsz_b + 1; }
+        else { G.g = extra + (b - cut) / gsz_b; G.grank = (b - cut) % gsz_b; G.gcount = gsz_b; }
+        G.gtid = (int64_t)G.grank * blockDim.x + threadIdx.x;
+        G.gsz = (int64_t)G.gcount * blockDim.x;
+        G.bar = a.bars + G.g;
+    }
+    const DevWork &w = a.works[G.g];
+    for (;;) {
+        // the group leader takes the next query of the batch
+        if (G.gtid == 0) {
+            const uint32_t qi = atomicAdd(a.next_query, 1u);
+            w.gstate[0] = qi;
+        }
+        G.sync();
+        if (threadIdx.x == 0) {
+            const uint32_t qi = __ldcg(w.gstate);
+            s_q[0] = (int32_t)qi;
+            if (qi < (uint32_t)a.nq) {
+                s_q[1] = a.qconst > 0 ? a.qconst : a.qlen[qi];
+                for (int i = 0; i < kMaxQ; ++i) s_q[2 + i] = a.kw[(int64_t)qi * kMaxQ + i];
+            }
+        }
+        __syncthreads();
+        if (s_q[0] >= a.nq) break;
+        Q qq;
+        qq.qi = s_q[0];
+        qq.q = s_q[1];
+        qq.full = (1u << qq.q) - 1u;
+        for (int i = 0; i < kMaxQ; ++i) qq.kw[i] = s_q[2 + i];
+        bool bad = qq.q < 1 || qq.q > kMaxQ;   // device-side validation (kgs_query_batch_device)
+        for (int i = 0; !bad && i < qq.q; ++i) {
+            if (qq.kw[i] < 0 || qq.kw[i] >= a.g.n_kw) bad = true;
+            for (int j = 0; j < i; ++j) if (qq.kw[j] == qq.kw[i]) bad = true;
+        }
+        if (bad) {
+            if (G.gtid == 0) {
+                QOut *qo = a.qout + qq.qi;
+                qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
+                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g;
+            }
+            G.sync();
+            continue;
+        }
+        const uint32_t done = __ldcg(w.gstate + 1);
+        Ctl *ctl = w.ctl[done & 1];
+        {   // zero this query's control block
+            uint32_t *cw = reinterpret_cast<uint32_t *>(ctl);
+            for (int64_t j = G.gtid; j < (int64_t)(sizeof(Ctl) / 4); j += G.gsz) cw[j] = 0u;
+        }
+        QOut *qo = a.qout + qq.qi;
+        if (G.gtid == 0) { qo->n_stamp = 0; qo->t_start = globaltimer_ns(); qo->group = G.g; }
+        G.sync();
+        stamp(G, qo, TS_START);
+        const Ctx c{a, w, ctl, G, qq};
+        search(c, s_big, sh, qo);
+        pred_dag(c, s_big, sh, qo);
+        topdown(c, sh, dsmem, qo);
+        if (G.gtid == 0) {
+            qo->levels = ctl->levels;
+            qo->stop_reason = ctl->stop_reason;
+            qo->count = (int32_t)ctl->sel_count;
+            qo->fatal = ctl->fatal;
+            qo->n_central = ctl->n_central;
+            qo->n_overflow = ctl->n_overflow;
+            qo->n_cid = ctl->n_cid;
+            qo->n_parcs = ctl->n_parcs;
+            qo->frontier_total = ctl->frontier_total;
+            qo->arcs_scanned = ctl->arcs_scanned;
+            qo->hits = ctl->hits;
+            qo->td_arcs = ctl->td_arcs;
+            qo->t_end = globaltimer_ns();
+            w.gstate[1] = done + 1;
+            w.gstate[2] = 1u;
+            w.gstate[3] = (uint32_t)a.R;
+        }
+        G.sync();
+    }
+}
+
+size_t engine_dyn_smem() { return (size_t)KGS_MAX_K * (8 + 4 + 4); }
+
+int engine_max_grid(int device) {
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_engine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)engine_dyn_smem());
+        attr = true;
+    }
+    int per_sm = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_engine, kBlock, engine_dyn_smem());
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    return per_sm * sms;
+}
+
+cudaError_t launch_engine(const EngineArgs &a, int grid, cudaStream_t s) {
+    void *args[] = {(void *)&a};
+    return cudaLaunchCooperativeKernel((const void *)k_engine, dim3(grid), dim3(kBlock), args, engine_dyn_smem(), s);
+}
+
+}  // namespace kgs

@@ -152,3 +152,48 @@ def test_device_resident_path():
         o = oracle.query(w.graph, kw, w.k)
         assert [a.central for a in r.answers] == [a.central for a in o.answers]
         assert [a.score_key for a in r.answers] == [a.key for a in o.answers]
+
+
+def test_batch_engine_groups():
+    """kgs_query_batch: one engine launch, queries spread over G groups of CTAs; every query's answers
+    equal the oracle's whatever G is (C1 all queries, C2 a sample, mixed q)."""
+    _gpu()
+    for name, count in (("C1", 100), ("C2", 40)):
+        w = synth.make_workload(name)
+        G = kgs.kgs_load_graph(w.graph)
+        qs = w.queries[:count] if name == "C1" else w.queries[::max(1, len(w.queries) // count)][:count]
+        exp = [oracle.query(w.graph, kw, w.k) for kw in qs]
+        for groups in (1, 3, 8, 64):
+            res = kgs.kgs_query_batch(G, qs, w.k, None, groups)
+            for kw, r, o in zip(qs, res, exp):
+                assert r.stats["stop_reason"] == o.stop_reason and r.stats["levels"] == o.levels, (name, groups, kw)
+                assert [a.central for a in r.answers] == [a.central for a in o.answers], (name, groups, kw)
+                for ra, oa in zip(r.answers, o.answers):
+                    assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist()
+                    assert ra.arcs.tolist() == oa.arcs.tolist()
+        G.close()
+
+
+def test_batch_device_invalid_queries():
+    """kgs_query_batch_device validates on the device: bad ids / repeated ids / bad q are reported per
+    query (KGS_STOP_INVALID_QUERY) and do not disturb the valid queries of the batch."""
+    _gpu()
+    import torch
+    w = synth.make_workload("C1")
+    G = kgs.kgs_load_graph(w.graph)
+    good = [list(q) for q in w.queries[:6]]
+    rows = [good[0], [0, 0, 1], good[1], [w.graph.n_keywords + 5, 1, 2], good[2], [1] * 9]
+    ql = [len(r) for r in rows]
+    kwp = torch.full((len(rows), 8), -1, dtype=torch.int32)
+    for i, r in enumerate(rows):
+        kwp[i, :min(8, len(r))] = torch.tensor(r[:8], dtype=torch.int32)
+    kwd = kwp.cuda()
+    qld = torch.tensor(ql, dtype=torch.int32, device="cuda")
+    s = torch.cuda.current_stream().cuda_stream
+    kgs.kgs_query_batch_device(G, len(rows), kwd.data_ptr(), qld.data_ptr(), w.k, None, 2, s)
+    res = kgs.kgs_query_batch_fetch(G, [min(8, x) for x in ql], s)
+    for i in (1, 3, 5):
+        assert res[i].stats["stop_reason"] == kgs.KGS_STOP_INVALID_QUERY and res[i].answers == []
+    for i, gi in ((0, 0), (2, 1), (4, 2)):
+        o = oracle.query(w.graph, good[gi], w.k)
+        assert [a.central for a in res[i].answers] == [a.central for a in o.answers]
