@@ -2,26 +2,26 @@
 """Benchmark of the Central Graph keyword-search hot path (BASELINE.json metric: p50 query latency,
 queries/s and GTEPS on the Wikidata-scale synthetic graph).
 
-A step = one query through the whole hot path (activation gate, search, central detection,
-extraction + level-cover + Eq. 6 score of every central graph, radix-select top-k, answer emit).
-
   python bench.py [--gpus N --steps K --warmup W]          CUDA path (libkgs), one rank per GPU
   python bench.py --impl reference [...]                   the CPU oracle on this box's host cores
 
-N = 1: workload C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keywords, top-20), the
-queries cycled from its 350-query latency set.  N > 1 (torchrun): workload C4 (configs[3]: the same
-graph, 4096 queries with q ~ U{2..8}) sharded round-robin over ranks, each rank holding a replicated
-graph; after the timed steps the ranks all-gather their top-k headers over NCCL (inside the timed
-region).  Scaling is weak (K queries per rank).
+Workload.  N = 1: C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keyword queries, top-20).
+N > 1 (torchrun): C4 (configs[3]: the same graph, 4096 queries with q ~ U{2..8}) dealt round-robin to
+ranks holding a replicated graph; one NCCL all-gather of the top-k headers per step (inside the timed
+region).  The per-rank step is the same size for every N (weak scaling).
 
-Timing: W warm-up steps; then K steps, each bracketed by CUDA events on the launching stream; between
-steps L2 is flushed (a 512 MiB write, outside the events); barrier + synchronize on both sides; the
-max over ranks.  `value` = queries / second of device time (graph and keyword ids resident in HBM);
-`e2e` = the same through kgs_query with host keyword ids and the answers copied back (wall clock).
+A step = one batch of queries through the whole hot path in ONE engine launch (activation gate, search,
+central detection, extraction + level-cover + Eq. 6 of every central graph, top-k, answer emit):
+the 350-query C3 latency set at N = 1 (each query once per step), 350 queries of the rank's C4 shard at
+N > 1.  `value` = queries/s of device time over K steps (CUDA events on the launching stream, L2 flushed
+with a 512 MiB write between steps, outside the events; max over ranks).  The single-query latency
+mode (one launch per query, the whole GPU on it) gives `p50_ms` / `p95_ms`.  `e2e` = the same batches
+through kgs_query_batch from host keyword ids to host answers (wall clock, H2D + D2H inside).
 """
 from __future__ import annotations
 
 import argparse
+import glob
 import json
 import os
 import statistics
@@ -36,6 +36,8 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "p50 query latency (ms) & queries/s, Wikidata-scale graph; GTEPS"
+BATCH = 350          # queries per step (the C3 latency set)
+GROUPS = 8           # engine groups in batch mode (queries answered at the same time)
 
 
 def _env_int(k, d):
@@ -60,7 +62,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                          "-i", str(self.index), "-lms", "100"], stdout=subprocess.PIPE,
+                                          "-i", str(self.index), "-lms", "50"], stdout=subprocess.PIPE,
                                          stderr=subprocess.DEVNULL, text=True)
         except OSError:
             self.proc = None
@@ -104,27 +106,27 @@ def load_peaks():
 
 
 def load_traffic():
-    """Mean DRAM bytes per k_search launch from the newest committed ncu capture (profiles/)."""
-    import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_k_search_traffic.json")))
+    """Mean DRAM bytes per query of the engine from the newest committed ncu capture (profiles/)."""
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_engine_traffic.json")))
     if not files:
         return None, None
     with open(files[-1]) as f:
         d = json.load(f)
-    return d.get("mean_dram_bytes_per_launch"), os.path.basename(files[-1])
+    return d, os.path.basename(files[-1])
 
 
-def bfs_algorithmic_bytes(st: dict) -> float:
-    """SURVEY.md §8(d) / DESIGN.md "Roofline": bytes the search must move for this query.
-    per expanded frontier entry: 16 B row_ptr + 2 B own status + 1 B activation + 4 B queue slot;
-    per inspected arc: 4 B col_idx + 2 B neighbour status;
-    per new (node, keyword) hit: 1 B M write + 1 B new-hit mask + 4 B next-queue slot (amortised);
-    per touched node: 2 B status reset."""
-    return (st["frontier_total"] * 23.0 + st["arcs_scanned"] * 6.0 + st.get("hits", 0) * 6.0)
+def algorithmic_bytes(st: dict) -> float:
+    """SURVEY.md §8(d) / DESIGN.md §7: bytes the hot path must move for one query.
+    search: per frontier entry 16 B row_ptr + 2 B own status + 1 B activation + 4 B queue slot; per
+    inspected out-arc 4 B col_idx + 2 B neighbour status; per new (node, keyword) hit 1 B M write +
+    1 B new-hit mask + 4 B next frontier (amortised).  top-down pre-pass: per inspected in-arc 4 B in_idx
+    + 2 B status; per predecessor arc 4 B node + 2 B bits written and read back."""
+    return (st["frontier_total"] * 23.0 + st["arcs_scanned"] * 6.0 + st.get("hits", 0) * 6.0 +
+            st.get("td_arcs", 0) * 6.0 + st.get("td_pred_arcs", 0) * 12.0)
 
 
 # ------------------------------------------------------------------------------------------ workloads
-def build_workload(name: str, rank: int, world: int):
+def build_workload(name: str):
     import synth
     t0 = time.time()
     w = synth.make_workload(name)
@@ -132,8 +134,6 @@ def build_workload(name: str, rank: int, world: int):
 
 
 class _RemoteGraph:
-    """Sizes of a graph received from rank 0 (host arrays stay on rank 0)."""
-
     def __init__(self, n, n_arcs):
         self.n, self.n_arcs = n, n_arcs
 
@@ -147,7 +147,7 @@ def load_replicated(name, rank, world, dev, kgs):
     t0 = time.time()
     cuda = f"cuda:{dev}"
     if rank == 0:
-        w, _ = build_workload(name, 0, 1)
+        w, _ = build_workload(name)
         g = w.graph
         qmax = max(len(q) for q in w.queries)
         meta = torch.tensor([g.n, g.n_arcs, g.n_keywords, g.kw_nodes.shape[0], len(w.queries), qmax, w.k],
@@ -188,13 +188,13 @@ def load_replicated(name, rank, world, dev, kgs):
 
 
 def run_reference(args):
-    """The oracle, as it stands, on host cores (bench.py --impl reference)."""
+    """The oracle, as it stands, on host cores (bench.py --impl reference): rank 0 only."""
     rank, world = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1)
     if rank != 0:
         return 0
     import oracle
     name = "C3" if world == 1 else "C4"
-    w, gen_s = build_workload(name, 0, 1)
+    w, gen_s = build_workload(name)
     order = np.random.default_rng(12345).permutation(len(w.queries))
     qs = [w.queries[i] for i in order]
     for i in range(args.warmup):
@@ -211,8 +211,9 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot * 1e3 / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": name, "graph": f"R-MAT scale 25 edge factor 8 ({w.graph.n} nodes, "
-                                                   f"{w.graph.n_arcs} arcs)", "k": w.k, "queries": len(qs)},
+            "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {w.graph.n} nodes, "
+                                                   f"{w.graph.n_arcs} arcs", "k": w.k, "queries": len(qs),
+                       "step": "one query (the oracle is single-threaded; a step of the GPU arm is a batch)"},
             "p50_ms": statistics.median(lat),
             "cpu_baseline": {"value": qps, "unit": "queries/s", "cores": 1, "kind": "oracle",
                              "sample": f"{args.steps} consecutive {name} queries after {args.warmup} warm-up"},
@@ -224,11 +225,13 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kgs", choices=["kgs", "reference"])
+    ap.add_argument("--groups", type=int, default=GROUPS)
+    ap.add_argument("--batch", type=int, default=BATCH)
+    ap.add_argument("--latency-steps", type=int, default=200)
     ap.add_argument("--cpu-sample-s", type=float, default=15.0)
-    ap.add_argument("--e2e-steps", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
@@ -244,137 +247,164 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = local
     torch.cuda.set_device(dev)
+    cuda = f"cuda:{dev}"
     import paper_conf_icde_yangajtw19_b200 as kgs
 
     name = "C3" if world == 1 else "C4"
     if world == 1:
-        w, gen_s = build_workload(name, rank, world)
+        w, gen_s = build_workload(name)
         g = w.graph
         t0 = time.time()
         G = kgs.kgs_load_graph(g, device=dev)
         load_s = time.time() - t0
     else:
         w, g, G, gen_s, load_s = load_replicated(name, rank, world, dev, kgs)
-    # a fixed permutation so every window of steps mixes all query sizes (the config lists them by q)
     order = np.random.default_rng(12345).permutation(len(w.queries))
     allq = [w.queries[i] for i in order]
-    queries = allq[rank::world] if world > 1 else allq
-    qdev = [torch.tensor(list(kw), dtype=torch.int32, device=f"cuda:{dev}") for kw in queries]
+    qids_all = [int(i) for i in order]
+    mine = list(range(rank, len(allq), world)) if world > 1 else list(range(len(allq)))
+    queries = [allq[i] for i in mine]
+    qids = [qids_all[i] for i in mine]
+    B = args.batch
     stream = torch.cuda.current_stream(dev)
     sh = stream.cuda_stream
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=f"cuda:{dev}")
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=cuda)
+
+    def batch_rows(step):
+        idx = [((step * B) + j) % len(queries) for j in range(B)]
+        kwp = torch.full((B, 8), -1, dtype=torch.int32)
+        for r, i in enumerate(idx):
+            kwp[r, :len(queries[i])] = torch.tensor(queries[i], dtype=torch.int32)
+        return idx, kwp.to(cuda), torch.tensor([len(queries[i]) for i in idx], dtype=torch.int32, device=cuda)
+
+    steps_in = [batch_rows(s) for s in range(args.warmup + args.steps)]
     p = kgs.kgs_params_default()
 
-    def step(i):
-        j = i % len(queries)
-        kgs.kgs_query_device(G, qdev[j].data_ptr(), len(queries[j]), w.k, p, sh)
-
-    # warm-up (also builds the activation cache for alpha)
-    for i in range(args.warmup):
-        step(i)
-        kgs.kgs_query_fetch(G, len(queries[i % len(queries)]), 0, sh)
+    # ---- batch mode (value): one engine launch per step, GROUPS queries at a time
+    for s in range(args.warmup):
+        _, kwd, qld = steps_in[s]
+        kgs.kgs_query_batch_device(G, B, kwd.data_ptr(), qld.data_ptr(), w.k, p, args.groups, sh)
+        kgs.kgs_query_batch_fetch(G, qld.tolist(), sh)
     torch.cuda.synchronize(dev)
-
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    stats = []
-    answers = []
+    stats, answers = [], []
     clk = ClockSampler(dev)
     clk.start()
     if dist:
         dist.barrier()
     torch.cuda.synchronize(dev)
-    t_wall = time.perf_counter()
     for i in range(args.steps):
+        idx, kwd, qld = steps_in[args.warmup + i]
         flush.fill_(i & 0xFF)                       # L2 flush between timed steps (outside the events)
         ev[i][0].record(stream)
-        step(args.warmup + i)
+        kgs.kgs_query_batch_device(G, B, kwd.data_ptr(), qld.data_ptr(), w.k, p, args.groups, sh)
         ev[i][1].record(stream)
-        r = kgs.kgs_query_fetch(G, len(queries[(args.warmup + i) % len(queries)]), 0, sh)  # after ev: not timed
-        stats.append(r.stats)
-        answers.append([(a.central, a.depth, a.score_key) for a in r.answers])
+        res = kgs.kgs_query_batch_fetch(G, qld.tolist(), sh)   # after the end event: not timed
+        stats += [r.stats for r in res]
+        if i == args.steps - 1:
+            answers = [(qids[j], [(a.central, a.depth, a.score_key) for a in r.answers]) for j, r in zip(idx, res)]
     gather_ms = 0.0
     if dist:
-        # NCCL all-gather of every rank's top-k headers (central, depth, key) (config C4)
+        # NCCL all-gather of every rank's top-k headers (central, depth, key) of the last step (config C4)
         from paper_conf_icde_yangajtw19_b200 import dist as kd
-        qids = [int(order[(rank + world * ((args.warmup + i) % len(queries))) % len(order)]) for i in range(args.steps)]
-        hdr = kd.pack_headers(qids, answers, w.k).to(f"cuda:{dev}")
+        hdr = kd.pack_headers([q for q, _ in answers], [a for _, a in answers], w.k).to(cuda)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        merged = kd.gather_headers(hdr, args.steps * world, world)
+        kd.gather_headers(hdr, len(answers) * world, world)
         e1.record(stream)
     torch.cuda.synchronize(dev)
     if dist:
         dist.barrier()
         gather_ms = e0.elapsed_time(e1)
-    wall = time.perf_counter() - t_wall
     clocks = clk.stop()
-    lat = [a.elapsed_time(b) for a, b in ev]
-    dev_ms = sum(lat) + gather_ms
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    dev_ms = sum(step_ms) + gather_ms
     if dist:
-        t = torch.tensor([dev_ms], dtype=torch.float64, device=f"cuda:{dev}")
+        t = torch.tensor([dev_ms], dtype=torch.float64, device=cuda)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dev_ms = float(t.item())
-    total_queries = args.steps * world
+    total_queries = args.steps * B * world
     value = total_queries / (dev_ms / 1e3)
-    arcs = sum(s["arcs_scanned"] for s in stats)
-    search_ms = sum(s["ms_search"] for s in stats)
-    td_ms = sum(s["ms_topdown"] for s in stats)
+    arcs = sum(s["arcs_scanned"] + s["td_arcs"] for s in stats)
+    alg = sum(algorithmic_bytes(s) for s in stats)
 
-    # e2e: host keyword ids -> kgs_query -> answers on the host (wall clock, includes H2D / D2H)
-    e2e_steps = args.e2e_steps or args.steps
-    e2e_lat = []
-    d2h = 0
-    for i in range(e2e_steps):
-        kw = list(queries[(args.warmup + i) % len(queries)])
+    # ---- single-query latency mode: the whole GPU on one query, one launch per query
+    lat = []
+    lat_stats = []
+    if rank == 0:
+        nlat = min(args.latency_steps, len(queries))
+        qdev = [torch.tensor(list(q), dtype=torch.int32, device=cuda) for q in queries[:nlat + args.warmup]]
+        for i in range(args.warmup):
+            kgs.kgs_query_device(G, qdev[i].data_ptr(), len(queries[i]), w.k, p, sh)
+            kgs.kgs_query_fetch(G, len(queries[i]), 0, sh)
+        for i in range(nlat):
+            j = args.warmup + i
+            flush.fill_(i & 0xFF)
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            kgs.kgs_query_device(G, qdev[j].data_ptr(), len(queries[j]), w.k, p, sh)
+            a1.record(stream)
+            r = kgs.kgs_query_fetch(G, len(queries[j]), 0, sh)
+            lat.append(a0.elapsed_time(a1))
+            lat_stats.append(r.stats)
+
+    # ---- e2e: host keyword ids -> kgs_query_batch -> answers on the host (wall clock)
+    e2e_ms, d2h = [], 0
+    for i in range(min(args.steps, 3)):
+        idx = [((i * B) + j) % len(queries) for j in range(B)]
+        hq = [queries[j] for j in idx]
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
-        r = kgs.kgs_query(G, kw, w.k, p, sh)
-        e2e_lat.append((time.perf_counter() - t0) * 1e3)
-        d2h += sum(16 + 8 + a.nodes.nbytes + a.arcs.nbytes for a in r.answers)
-    e2e_qps = e2e_steps / (sum(e2e_lat) / 1e3)
-    h2d = sum(4 * len(queries[(args.warmup + i) % len(queries)]) for i in range(e2e_steps)) / e2e_steps
+        res = kgs.kgs_query_batch(G, hq, w.k, p, args.groups, sh)
+        e2e_ms.append((time.perf_counter() - t0) * 1e3)
+        d2h += sum(32 + a.nodes.nbytes + a.arcs.nbytes + 24 for r in res for a in r.answers)
+    e2e_qps = len(e2e_ms) * B / (sum(e2e_ms) / 1e3)
+    h2d = B * (4 * 8 + 4)
 
     if rank != 0:
         if dist:
             dist.destroy_process_group()
         return 0
     peak, peak_kind = load_peaks()
-    traffic, traffic_src = load_traffic()
-    bfs_bytes = sum(bfs_algorithmic_bytes(s) for s in stats)
-    achieved = bfs_bytes / (search_ms / 1e3) / 1e9 if search_ms > 0 else 0.0
+    tr, tr_src = load_traffic()
+    achieved = alg / (sum(step_ms) / 1e3) / 1e9
+    lat_alg = sum(algorithmic_bytes(s) for s in lat_stats)
     line = {
         "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {g.n} nodes, {g.n_arcs} arcs",
-                   "k": w.k, "queries": len(w.queries), "alpha": 0.1, "lambda": 0.2,
-                   "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
-                   "load_s": round(load_s, 1), "parallelism": f"query-sharded x{world}" if world > 1 else "single"},
-        "p50_ms": statistics.median(lat), "p95_ms": float(np.percentile(lat, 95)),
-        "gteps": arcs / (dev_ms / 1e3) / 1e9 * (world if world > 1 else 1) if dev_ms else 0.0,
-        "phase_ms": {"search": search_ms / args.steps, "topdown": td_ms / args.steps},
-        "roofline": {"kernel": "k_search", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
-                     "peak_kind": peak_kind,
-                     "algorithmic_bytes_per_query": bfs_bytes / args.steps},
-        "e2e": {"value": e2e_qps, "unit": "queries/s", "p50_ms": statistics.median(e2e_lat),
-                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h / e2e_steps},
-        # ours per query: k_search, k_extract, k_extract_big, k_select, k_rank, k_emit
-        "gpu_launches": 6 * args.steps,
+                   "k": w.k, "queries_per_step": B * world, "engine_groups": args.groups, "alpha": 0.1,
+                   "lambda": 0.2, "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
+                   "load_s": round(load_s, 1),
+                   "parallelism": f"query-sharded x{world}" if world > 1 else "single GPU"},
+        "p50_ms": statistics.median(lat) if lat else None,
+        "p95_ms": float(np.percentile(lat, 95)) if lat else None,
+        "latency_mode": {"queries": len(lat), "qps": len(lat) / (sum(lat) / 1e3) if lat else None,
+                         "note": "one engine launch per query (G = 1), CUDA events per query"},
+        "gteps": arcs / (dev_ms / 1e3) / 1e9 * world,
+        "roofline": {"kernel": "k_engine", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "peak_kind": peak_kind,
+                     "traffic": (tr["mean_dram_bytes_per_query"] * B) if tr else None, "traffic_source": tr_src,
+                     "algorithmic_bytes_per_launch": alg / args.steps,
+                     "latency_mode_achieved": (lat_alg / (sum(lat) / 1e3) / 1e9) if lat else None},
+        "e2e": {"value": e2e_qps, "unit": "queries/s", "ms_per_step": statistics.median(e2e_ms),
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h / len(e2e_ms)},
+        "gpu_launches": args.steps,   # one k_engine launch per step
         "clocks": clocks,
         "stats_mean": {k: float(np.mean([s[k] for s in stats])) for k in
-                       ("levels", "n_centrals", "frontier_total", "arcs_scanned", "overflow")},
+                       ("levels", "n_centrals", "frontier_total", "arcs_scanned", "td_arcs", "overflow")},
     }
     if not args.no_cpu_baseline and world == 1:
         import oracle
         t0 = time.perf_counter()
         done = 0
         while time.perf_counter() - t0 < args.cpu_sample_s and done < len(queries):
-            oracle.query(g, queries[(args.warmup + done) % len(queries)], w.k)
+            oracle.query(g, queries[done], w.k)
             done += 1
         el = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
-                                "sample": f"the first {done} timed {name} queries ({el:.1f} s, single-threaded oracle)"}
+                                "sample": f"the first {done} {name} queries of a step ({el:.1f} s, single-threaded oracle)"}
     print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

@@ -441,7 +441,14 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
 
 // Enqueue one engine launch for nq queries whose padded keyword rows / lengths are in g->d_kw / d_qlen.
 kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaStream_t s, int qconst = 0) {
-    G = std::max(1, std::min(G, nq));
+    G = std::max(1, std::min({G, nq, g->grid}));
+    if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
+        size_t free_b = 0, total_b = 0;
+        cudaMemGetInfo(&free_b, &total_b);
+        const size_t per = (size_t)g->n * 64 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18;
+        const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
+        G = std::max(1, (int)g->works.size() + more);
+    }
     kgs_status st = prepare(g, p, G, s);
     if (st != KGS_OK) return st;
     CUDA_TRY(grow_dev(&g->d_qout, &g->d_qout_cap, (size_t)nq));

@@ -1,0 +1,40 @@
+"""Throughput of the query engine on a config's query set for several group counts G (one launch per
+batch, device-resident keyword ids, CUDA-event timing).  Usage: batch_sweep.py [config] [G,...] [batch]"""
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icde_yangajtw19_b200 as kgs  # noqa: E402
+import synth  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "C3"
+groups = [int(x) for x in (sys.argv[2] if len(sys.argv) > 2 else "1,2,4,8,16").split(",")]
+batch = int(sys.argv[3]) if len(sys.argv) > 3 else 0
+w = synth.make_workload(name)
+order = np.random.default_rng(12345).permutation(len(w.queries))
+qs = [w.queries[i] for i in order]
+if batch:
+    qs = (qs * ((batch + len(qs) - 1) // len(qs)))[:batch]
+G = kgs.kgs_load_graph(w.graph)
+kwp = torch.full((len(qs), 8), -1, dtype=torch.int32)
+for i, q in enumerate(qs):
+    kwp[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
+kwd = kwp.cuda()
+qld = torch.tensor([len(q) for q in qs], dtype=torch.int32, device="cuda")
+s = torch.cuda.current_stream()
+for g in groups:
+    for rep in range(3):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(s)
+        kgs.kgs_query_batch_device(G, len(qs), kwd.data_ptr(), qld.data_ptr(), w.k, None, g, s.cuda_stream)
+        e1.record(s)
+        res = kgs.kgs_query_batch_fetch(G, [len(q) for q in qs], s.cuda_stream)
+        ms = e0.elapsed_time(e1)
+        lat = sorted(r.stats["ms_total"] for r in res)
+    print(f"{name} G={g:3d} batch={len(qs)} launch {ms:8.2f} ms  {len(qs) / ms * 1e3:9.1f} q/s  "
+          f"query latency p50 {lat[len(lat) // 2]:.3f} ms p95 {lat[int(len(lat) * .95)]:.3f} ms", flush=True)
