@@ -43,20 +43,20 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     return v;
 }
 
-// Barrier over the CTAs of one group (all CTAs are co-resident: cooperative launch).
+// Barrier over the CTAs of one group (all CTAs are co-resident: cooperative launch).  Thread 0 of each
+// CTA arrives with a gpu-scope release and spins with acquire loads on the generation word.
 __device__ __forceinline__ void group_sync(GroupBar *b, int gcount) {
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned gen = ld_acquire(&b->gen);
-        __threadfence();
-        if (atomicAdd(&b->arrive, 1u) == (unsigned)gcount - 1) {
-            atomicExch(&b->arrive, 0u);
-            __threadfence();
-            atomicAdd(&b->gen, 1u);
+        unsigned prev;
+        asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(prev) : "l"(&b->arrive) : "memory");
+        if (prev == (unsigned)gcount - 1) {
+            asm volatile("st.relaxed.gpu.global.u32 [%0], 0;" ::"l"(&b->arrive) : "memory");
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&b->gen) : "memory");
         } else {
-            while (ld_acquire(&b->gen) == gen) __nanosleep(20);
+            while (ld_acquire(&b->gen) == gen) { }
         }
-        __threadfence();
     }
     __syncthreads();
 }
@@ -795,6 +795,14 @@ size_t arena_bytes_host(int hcap, int ncap, int acap, int team, bool with_sort) 
     return arena_bytes(hcap, ncap, acap, team, with_sort);
 }
 
+// tier-1 (shared-memory) extraction arena of one warp: most Central Graphs are small
+constexpr int kT1Hash = 256, kT1Nodes = 112, kT1Arcs = 160;
+constexpr int kSmemArena = 8192;
+constexpr int kExtWarps = 8;     // warps per CTA that extract (each owns one tier-1 arena)
+// tier-2: one CTA per Central Graph over the whole dynamic shared region
+constexpr int kT2Hash = 1024, kT2Nodes = 1024, kT2Arcs = 1536;
+static_assert(kSmemArena * kExtWarps <= KGS_MAX_K * 16, "tier-1 arenas must fit the dynamic shared region");
+
 __device__ __forceinline__ char *align8(char *p) {
     return reinterpret_cast<char *>((reinterpret_cast<uintptr_t>(p) + 7) & ~uintptr_t(7));
 }
@@ -1098,38 +1106,46 @@ __device__ __forceinline__ bool prefix_match(uint64_t hi, uint32_t lo, uint64_t 
 }
 
 // Top-k by (fp64 key asc, central id asc).  |C| <= KGS_MAX_K: one CTA sorts every candidate.
-// Otherwise a group-wide MSD radix select over the 96-bit composite (12 digits of 8 bits) keeps
-// exactly k candidates, which one CTA then sorts.  Result: sel[0..count), ctl->sel_count.
+// Otherwise an MSD radix select over the 96-bit composite (12 digits of 8 bits) keeps exactly k
+// candidates, which one CTA then sorts: by one CTA alone up to kCtaSelectMax candidates (no group
+// barrier), by the whole group beyond.  Result: sel[0..count), ctl->sel_count.
+constexpr uint32_t kCtaSelectMax = 1u << 18;
+
 __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const uint32_t nc = __ldcg(&ctl->n_central);
     const uint32_t kk = (uint32_t)c.a.k < nc ? (uint32_t)c.a.k : nc;
-    if (nc > (uint32_t)KGS_MAX_K) {
-        __shared__ uint32_t hsh[256];
-        __shared__ uint32_t s_bucket, s_before;
+    __shared__ uint32_t hsh[256];
+    __shared__ uint32_t s_bucket, s_before;
+    const bool group_wide = nc > kCtaSelectMax;
+    if (nc > (uint32_t)KGS_MAX_K && (group_wide || G.grank == 0)) {
+        const int64_t t0 = group_wide ? G.gtid : (int64_t)threadIdx.x;
+        const int64_t ts = group_wide ? G.gsz : (int64_t)blockDim.x;
         uint64_t phi = 0;
         uint32_t plo = 0, want = kk;
         for (int d = 0; d < 12; ++d) {
             for (int t = threadIdx.x; t < 256; t += blockDim.x) hsh[t] = 0;
             __syncthreads();
-            for (int64_t i = G.gtid; i < nc; i += G.gsz) {
+            for (int64_t i = t0; i < nc; i += ts) {
                 uint64_t hi; uint32_t lo;
                 comp_key(c, (uint32_t)i, hi, lo);
                 if (prefix_match(hi, lo, phi, plo, d)) atomicAdd(hsh + digit_of(hi, lo, d), 1u);
             }
             __syncthreads();
-            for (int t = threadIdx.x; t < 256; t += blockDim.x)
-                if (hsh[t]) atomicAdd(&ctl->hist[d][t], hsh[t]);
-            G.sync();
-            if (threadIdx.x == 0) {
-                uint32_t acc = 0, b = 0;
-                for (b = 0; b < 256; ++b) {
-                    const uint32_t h = __ldcg(&ctl->hist[d][b]);
-                    if (acc + h >= want) break;
-                    acc += h;
-                }
-                s_bucket = b; s_before = acc;
+            if (group_wide) {
+                for (int t = threadIdx.x; t < 256; t += blockDim.x)
+                    if (hsh[t]) atomicAdd(&ctl->hist[d][t], hsh[t]);
+                G.sync();
+                for (int t = threadIdx.x; t < 256; t += blockDim.x) hsh[t] = __ldcg(&ctl->hist[d][t]);
+                __syncthreads();
+            }
+            // the bucket holding the want-th smallest: parallel prefix over the 256 bins
+            const uint32_t hv = threadIdx.x < 256 ? hsh[threadIdx.x] : 0u;
+            int tot;
+            const int ex = block_excl_scan((int)hv, &tot, sh);
+            if (threadIdx.x < 256 && (uint32_t)ex < want && want <= (uint32_t)ex + hv) {
+                s_bucket = threadIdx.x; s_before = (uint32_t)ex;
             }
             __syncthreads();
             want -= s_before;
@@ -1138,7 +1154,7 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
             else plo |= (uint32_t)bk << (24 - 8 * (d - 8));
             __syncthreads();
         }
-        for (int64_t i = G.gtid; i < nc; i += G.gsz) {   // exactly kk candidates are <= the threshold
+        for (int64_t i = t0; i < nc; i += ts) {   // exactly kk candidates are <= the threshold
             uint64_t hi; uint32_t lo;
             comp_key(c, (uint32_t)i, hi, lo);
             if (hi < phi || (hi == phi && lo <= plo)) {
@@ -1146,8 +1162,9 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
                 if (pos < (uint32_t)KGS_MAX_K) c.w.sel[pos] = (int32_t)i;
             }
         }
-        G.sync();
     }
+    if (group_wide) G.sync();
+    else __syncthreads();
     if (G.grank == 0) {   // one CTA ranks (all candidates, or the radix-selected ones)
         unsigned long long *khi = reinterpret_cast<unsigned long long *>(dsmem);
         uint32_t *klo = reinterpret_cast<uint32_t *>(khi + KGS_MAX_K);
@@ -1193,10 +1210,9 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
     const EngineArgs &a = c.a;
     Ctl *ctl = c.ctl;
     const uint32_t nc = __ldcg(&ctl->n_central);
-    // extract: one warp per central node, arena in global memory (per warp of the grid)
-    {
-        const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
-        Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
+    // (A) one warp per central node, tier-1 arena in shared memory (most Central Graphs are small)
+    if ((threadIdx.x >> 5) < kExtWarps) {
+        Arena S1 = carve(dsmem + kSmemArena * (threadIdx.x >> 5), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
         WarpTeam T;
         for (;;) {
             uint32_t idx = 0;
@@ -1205,7 +1221,7 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
             if (idx >= nc) break;
             const int32_t cn = __ldcg(c.w.centrals + idx);
             double key = 0.0;
-            const bool ok = central_graph(T, S, c, cn, __ldcg(c.w.cdepth + idx), &key);
+            const bool ok = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key);
             if (T.rank() == 0) {
                 if (ok) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
                 else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = (int32_t)idx; }
@@ -1215,21 +1231,39 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
     }
     G.sync();
     stamp(G, qo, TS_EXTRACT);
-    // overflowed candidates: one CTA each over the CTA's global arena
+    // (B) the larger ones: a whole CTA per central node over the CTA's shared region; (C) beyond that,
+    // the CTA's global-memory arena
     const uint32_t no = __ldcg(&ctl->n_overflow);
     BlockTeam BT{sh};
     if (no) {
-        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+        Arena S2 = carve(dsmem, kT2Hash, kT2Nodes, kT2Arcs, kBlock, false);
         for (uint32_t t = G.grank; t < no; t += G.gcount) {
             const int32_t idx = __ldcg(c.w.overflow + t);
             double key = 0.0;
-            const bool ok = central_graph(BT, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+            const bool ok = central_graph(BT, S2, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
             if (threadIdx.x == 0) {
                 if (ok) c.w.ckey[idx] = key;
-                else atomicExch(&ctl->fatal, 2);
+                else c.w.overflow[no + atomicAdd(&ctl->work_big, 1u)] = idx;
             }
             __syncthreads();
         }
+        G.sync();
+        const uint32_t nbig = __ldcg(&ctl->work_big);
+        if (nbig) {
+            Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+            for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
+                const int32_t idx = __ldcg(c.w.overflow + no + t);
+                double key = 0.0;
+                const bool ok = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+                if (threadIdx.x == 0) {
+                    if (ok) c.w.ckey[idx] = key;
+                    else atomicExch(&ctl->fatal, 2);
+                }
+                __syncthreads();
+            }
+            G.sync();
+        }
+        if (G.gtid == 0) ctl->work_big = 0;
         G.sync();
     }
     stamp(G, qo, TS_EXTRACT_BIG);
@@ -1237,9 +1271,11 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
     stamp(G, qo, TS_SELECT);
     // emit: one warp per winner (per-warp arena), overflowed winners by a CTA
     const uint32_t cnt = __ldcg(&ctl->sel_count);
-    {
+    if ((threadIdx.x >> 5) < kExtWarps) {
         const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
         Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
+        Arena S1 = carve(dsmem + kSmemArena * ((threadIdx.x >> 5) % kExtWarps), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
+        S1.sortbuf = S.sortbuf;   // tier-1 closure in shared memory, its sort buffer in the global arena
         WarpTeam T;
         for (;;) {
             uint32_t rk = 0;
@@ -1258,8 +1294,10 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
                 continue;
             }
             double key;
-            if (central_graph(T, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
-                emit_graph(T, S, c, (int)rk);
+            const int32_t cn = __ldcg(c.w.centrals + idx);
+            const int dep = __ldcg(c.w.cdepth + idx);
+            if (central_graph(T, S1, c, cn, dep, &key)) emit_graph(T, S1, c, (int)rk);   // tier 1
+            else if (central_graph(T, S, c, cn, dep, &key)) emit_graph(T, S, c, (int)rk);
             else if (T.rank() == 0) atomicExch(&ctl->fatal, 3);
         }
     }
@@ -1267,12 +1305,16 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
     const uint32_t nbig = __ldcg(&ctl->work_big);
     if (nbig) {
         Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+        Arena S2 = carve(dsmem, kT2Hash, kT2Nodes, kT2Arcs, kBlock, false);
+        S2.sortbuf = S.sortbuf;   // tier-2 closure in shared memory, its sort buffer in the CTA's global arena
         for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
             const int rk = __ldcg(c.w.overflow + t);
             const int32_t idx = __ldcg(c.w.sel + rk);
+            const int32_t cn = __ldcg(c.w.centrals + idx);
+            const int dep = __ldcg(c.w.cdepth + idx);
             double key;
-            if (central_graph(BT, S, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
-                emit_graph(BT, S, c, rk);
+            if (central_graph(BT, S2, c, cn, dep, &key)) emit_graph(BT, S2, c, rk);
+            else if (central_graph(BT, S, c, cn, dep, &key)) emit_graph(BT, S, c, rk);
             else if (threadIdx.x == 0) atomicExch(&ctl->fatal, 4);
             __syncthreads();
         }
@@ -1283,8 +1325,10 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
 
 // ------------------------------------------------------------------------------------------ engine
 __global__ void __launch_bounds__(kBlock, 2) k_engine(EngineArgs a) {
+    // one dynamic shared region, reused phase by phase: expansion tiles (search, pre-pass), the per-warp
+    // tier-1 extraction arenas (top-down), the rank sort of the selection
     extern __shared__ __align__(16) char dsmem[];
-    __shared__ BigTile s_big;
+    BigTile &s_big = *reinterpret_cast<BigTile *>(dsmem);
     __shared__ long long sh[40];
     __shared__ int32_t s_q[2 + kMaxQ];
     // group of this CTA: contiguous ranges, sizes differ by at most one
