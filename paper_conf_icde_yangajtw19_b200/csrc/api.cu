@@ -468,6 +468,10 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
     a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
     a.level_cover = p.level_cover ? 1 : 0;
+    {
+        const char *e = std::getenv("KGS_TILE_LIGHT");   // ablation knob (nodes); default 8 tiles
+        a.tile_light = e ? std::atoi(e) : 8 * kBlock;
+    }
     a.qout = g->d_qout; a.out_hdr = g->d_hdr; a.out_key = g->d_key; a.out_off = g->d_off;
     a.out_nodes = g->d_nodes; a.out_arcs = g->d_arcs;
     a.out_nodes_cap = (long long)g->d_nodes_cap; a.out_arcs_cap = (long long)(g->d_arcs_cap / 2);

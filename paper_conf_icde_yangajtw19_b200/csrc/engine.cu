@@ -144,8 +144,9 @@ __device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t 
     const uint32_t bit = 1u << (v & 31);
     if (__ldcg(word) & bit) return;
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
-    const unsigned mask = __activemask();
-    if ((int)lane_id() == __ffs(mask) - 1 && !__ldcg(flag)) *flag = 1u;
+    // converged lanes may push to different bitmaps (level slots): one leader per flag address
+    const unsigned peers = __match_any_sync(__activemask(), (unsigned long long)flag);
+    if ((int)lane_id() == __ffs(peers) - 1 && !__ldcg(flag)) *flag = 1u;
 }
 
 struct Ctx {        // everything a group needs while answering one query
@@ -270,6 +271,7 @@ __device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool
 
 constexpr int kTileMax = kBlock;
 constexpr int kBigUnroll = 4;
+constexpr uint32_t kTileLight = 8;   // light frontiers of at most 8 tiles also go through the tile path
 constexpr int kLightUnroll = 2;
 
 struct FwdNode {
@@ -304,9 +306,9 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
         const int j = threadIdx.x;
         long long deg = 0, s0 = 0;
         if (j < nt) {
-            const int32_t v = __ldcg(qb + t0 + j);
-            NodeT nd;
-            if (prep(v, G.grank == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
+            const int32_t v = __ldcg(qb + t0 + j);   // -1: a big node listed in the light queue
+            NodeT nd{};
+            if (v >= 0 && prep(v, G.grank == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
             node[j] = nd;
             S.start[j] = s0;
         }
@@ -501,7 +503,10 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
         auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) { pd_visit(c, exact_block, nd, u, su, nbits, nflag); };
         expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
-        expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
+        if (c0 <= (uint32_t)c.a.tile_light)   // small frontier: tiles over the whole group
+            expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
+        else
+            expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
     }
@@ -713,7 +718,10 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         };
         auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(c, l, nd.v, nd.hm, x, sx, my_hits); };
         expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
-        expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
+        if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
+            expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
+        else
+            expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
         G.sync();
         stamp(G, qo, TS_EXPAND);
     }

@@ -150,6 +150,7 @@ struct EngineArgs {
     uint32_t *next_query;       // global query counter
     // parameters (shared by the batch)
     int k, max_depth, block_central, extract_mode, level_cover;
+    int tile_light;             // light frontiers up to this many nodes are expanded by group-wide tiles
     // outputs
     QOut *qout;                 // [nq]
     int32_t *out_hdr;           // [nq][k][4]: central, depth, n_nodes, n_arcs
