@@ -16,7 +16,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libkgs.so")
+LIB_PATH = os.environ.get("KGS_LIB", os.path.join(_HERE, "libkgs.so"))   # KGS_LIB: ablation builds
 
 KGS_OK, KGS_EINVAL, KGS_ENOMEM, KGS_ECUDA, KGS_ENCCL, KGS_EINTERNAL = 0, -1, -2, -3, -4, -5
 KGS_MAX_Q, KGS_MAX_K = 8, 4096

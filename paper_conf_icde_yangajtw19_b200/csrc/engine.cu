@@ -272,7 +272,10 @@ __device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool
 constexpr int kTileMax = kBlock;
 constexpr int kBigUnroll = 4;
 constexpr uint32_t kTileLight = 8;   // light frontiers of at most 8 tiles also go through the tile path
-constexpr int kLightUnroll = 2;
+#ifndef KGS_LIGHT_UNROLL
+#define KGS_LIGHT_UNROLL 4
+#endif
+constexpr int kLightUnroll = KGS_LIGHT_UNROLL;
 
 struct FwdNode {
     int32_t v;
@@ -1332,7 +1335,10 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
 }
 
 // ------------------------------------------------------------------------------------------ engine
-__global__ void __launch_bounds__(kBlock, 2) k_engine(EngineArgs a) {
+#ifndef KGS_MINB
+#define KGS_MINB 2   // CTAs per SM the register budget is sized for
+#endif
+__global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
     // one dynamic shared region, reused phase by phase: expansion tiles (search, pre-pass), the per-warp
     // tier-1 extraction arenas (top-down), the rank sort of the selection
     extern __shared__ __align__(16) char dsmem[];
