@@ -93,10 +93,20 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *   block_central  1 (default): a node identified as central no longer expands (Alg. 2 ln 2).
  *   extract_mode   KGS_EXTRACT_EXACT (default) or KGS_EXTRACT_LITERAL.
  *   level_cover    1 (default): apply level-cover pruning; 0 returns unpruned Central Graphs.
- *   want_levels    1: also copy M and the central list back (for parity checks); default 0. */
+ *   want_levels    1: also copy M and the central list back (for parity checks); default 0.
+ *   prune          exact lower-bound pruning of the top-down phase (Eq. 6 keys are computed only for the
+ *                  candidates whose (bound, id) can still beat the k-th exact (key, id); the answers are
+ *                  identical, only kgs_result_centrals' keys of skipped candidates are not computed, so
+ *                  want_levels = 1 forces prune = 0):
+ *                    0  off: every Central Graph is extracted (Alg. 3 as written);
+ *                    1  (default) bound d^lambda * w_c (the central node is always kept, weights >= 0);
+ *                    2  bound d^lambda * max_i (lightest Thm. V.4 path from T_i to c), computed by the
+ *                       search (an atomic min per hitting arc).  Tighter, costs search time.  Needs the
+ *                       Thm. V.4 DAG to consist of arcs the search traversed: with extract_mode = LITERAL
+ *                       and block_central = 1 it falls back to 1. */
 typedef struct {
     double alpha, lambda;
-    int32_t max_depth, block_central, extract_mode, level_cover, want_levels, reserved;
+    int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
 } kgs_params;
 
 /* One answer (a pruned Central Graph).  Pointers live until kgs_result_free. */
@@ -126,6 +136,7 @@ typedef struct {
     float ms_search, ms_topdown, ms_total;   /* this query: bottom-up search, top-down, total (device clock) */
     float ms_launch;       /* the whole engine launch that answered it (all queries of the batch) */
     int32_t group;         /* engine group (set of CTAs) that answered the query */
+    int32_t n_evaluated;   /* Central Graphs whose exact key was computed (|C| unless prune skipped some) */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index

@@ -42,7 +42,7 @@ class kgs_graph_desc(ctypes.Structure):
 class kgs_params(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("lambda_", ctypes.c_double), ("max_depth", ctypes.c_int32),
                 ("block_central", ctypes.c_int32), ("extract_mode", ctypes.c_int32),
-                ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("prune", ctypes.c_int32)]
 
 
 class kgs_answer(ctypes.Structure):
@@ -57,7 +57,8 @@ class kgs_stats(ctypes.Structure):
                 ("count", ctypes.c_int64), ("frontier_total", ctypes.c_int64), ("arcs_scanned", ctypes.c_int64),
                 ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("td_arcs", ctypes.c_int64),
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
-                ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32)]
+                ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
+                ("n_evaluated", ctypes.c_int32)]
 
 
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
@@ -135,11 +136,11 @@ def kgs_params_default() -> kgs_params:
 
 
 def make_params(alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=KGS_EXTRACT_EXACT,
-                level_cover=1, want_levels=0) -> kgs_params:
+                level_cover=1, want_levels=0, prune=1) -> kgs_params:
     p = kgs_params_default()
     p.alpha, p.lambda_, p.max_depth = float(alpha), float(lam), int(max_depth)
     p.block_central, p.extract_mode = int(block_central), int(extract_mode)
-    p.level_cover, p.want_levels = int(level_cover), int(want_levels)
+    p.level_cover, p.want_levels, p.prune = int(level_cover), int(want_levels), int(prune)
     return p
 
 

@@ -148,7 +148,7 @@ namespace {
 
 void free_work(DevWork &w) {
     void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.centrals, w.cdepth, w.ckey, w.overflow,
-                 w.cflag, w.sel, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
+                 w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
                  w.gstate};
     for (void *x : p) if (x) cudaFree(x);
@@ -172,6 +172,9 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.overflow, n));
     CUDA_TRY(dmalloc(&w.cflag, n));
     CUDA_TRY(dmalloc(&w.sel, KGS_MAX_K));
+    CUDA_TRY(dmalloc(&w.elist, n));
+    CUDA_TRY(dmalloc(&w.mw, n * 8));
+    CUDA_TRY(cudaMemset(w.mw, 0xFF, (size_t)n * 8 * sizeof(uint32_t)));
     CUDA_TRY(dmalloc(&w.ctl[0], 1));
     CUDA_TRY(dmalloc(&w.ctl[1], 1));
     CUDA_TRY(cudaMemset(w.ctl[0], 0, sizeof(Ctl)));
@@ -214,6 +217,7 @@ void kgs_params_default(kgs_params *p) {
     p->extract_mode = KGS_EXTRACT_EXACT;
     p->level_cover = 1;
     p->want_levels = 0;
+    p->prune = 1;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -368,6 +372,7 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.max_depth < 1 || p.max_depth > 254) return fail(KGS_EINVAL, "max_depth must be in [1, 254]");
     if (p.extract_mode != KGS_EXTRACT_EXACT && p.extract_mode != KGS_EXTRACT_LITERAL)
         return fail(KGS_EINVAL, "extract_mode");
+    if (p.prune < 0 || p.prune > 2) return fail(KGS_EINVAL, "prune must be 0, 1 or 2");
     return KGS_OK;
 }
 
@@ -445,7 +450,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        const size_t per = (size_t)g->n * 64 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18;
+        const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
         G = std::max(1, (int)g->works.size() + more);
     }
@@ -468,6 +473,14 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
     a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
     a.level_cover = p.level_cover ? 1 : 0;
+    // the parity view wants every central's key.  The path bound needs the Thm. V.4 DAG to be made of
+    // arcs the search traversed: exact extraction, or no central blocking.
+    a.prune = p.want_levels ? 0 : p.prune;
+    if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
+    {
+        const char *e = std::getenv("KGS_PRUNE_MIN");
+        a.prune_min = e ? std::max(1, std::atoi(e)) : 512;
+    }
     {
         const char *e = std::getenv("KGS_TILE_LIGHT");   // ablation knob (nodes); default 8 tiles
         a.tile_light = e ? std::atoi(e) : 8 * kBlock;
@@ -552,6 +565,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.hits = (int64_t)o.hits;
         st.td_arcs = (int64_t)o.td_arcs;
         st.td_pred_arcs = o.n_parcs;
+        st.n_evaluated = (int32_t)o.n_eval;
         st.group = o.group;
         if (o.stop_reason != KGS_STOP_INVALID_QUERY && o.t_end >= o.t_start) {
             st.ms_search = (float)((double)(o.t_search_end - o.t_start) * 1e-6);

@@ -229,6 +229,14 @@ __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W,
 }
 
 // ------------------------------------------------------------------------------------------ expansion
+// w in fixed point 2^-24, rounded down (weights are snapped to that grid at load, so this is exact).
+// Saturating, and the path sums wrap modulo 2^32: either way the value never exceeds the true sum, so
+// the pruning bound it feeds stays a lower bound.
+__device__ __forceinline__ uint32_t weight_fx(float wt) {
+    const double x = floor((double)wt * 16777216.0);
+    return x <= 0.0 ? 0u : (x >= 4294967295.0 ? 0xFFFFFFFFu : (uint32_t)x);
+}
+
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, int32_t x, uint32_t sx,
@@ -237,6 +245,12 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
     if (!bits) return;
     const uint32_t gate = sx >> 8;
     if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
+        if (c.a.prune == 2) {   // x is hit at l+1 for these keywords: v is a Thm. V.4 predecessor of (x, i)
+            for (uint32_t b = bits; b; b &= b - 1) {
+                const int i = __ffs(b) - 1;
+                atomicMin(c.w.mw + (int64_t)x * 8 + i, __ldcg(c.w.mw + (int64_t)v * 8 + i));
+            }
+        }
         const uint32_t sh = (uint32_t)(x & 3) << 3;
         uint32_t *nw = c.w.nm + (x >> 2);
         const uint32_t cur = (__ldcg(nw) >> sh) & 0xFFu;
@@ -478,8 +492,8 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     Ctl *ctl = c.ctl;
     const bool exact_block = c.a.extract_mode == KGS_EXTRACT_EXACT && c.a.block_central;
     const int64_t W = c.a.W;
-    // seeds (every central node, for every keyword it did not contain itself) were set when each central
-    // was identified (merge step of the search): round 0 starts from them.
+    // seeds (the candidates to extract, for every keyword they do not contain) were set by seed_pd: round 0
+    // starts from them.  A second call continues the same DAG: done bits persist, the CSR is rebuilt.
     unsigned long long my_arcs = 0;
     int r = 0;
     for (;; ++r) {
@@ -572,6 +586,15 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     // ---- reset the state the previous query of this group left behind
     const uint32_t valid = __ldcg(w.gstate + 2), lastR = __ldcg(w.gstate + 3);
     const uint32_t done = __ldcg(w.gstate + 1);
+    if (done > 0 && w.ctl[(done + 1) & 1]->mw_dirty) {   // the previous query's lightest-path rows
+        const Ctl *pv = w.ctl[(done + 1) & 1];
+        const int64_t pt = (int64_t)pv->n_touched;       // its touched list is complete
+        const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u);
+        for (int64_t j = gtid; j < 2 * pt; j += gsz) {
+            const int32_t v = w.touched[j >> 1];
+            reinterpret_cast<uint4 *>(w.mw + (int64_t)v * 8)[j & 1] = ones;
+        }
+    }
     if (!valid || (int)lastR != R || done == 0) {
         const int64_t n8 = n / 8;
         for (int64_t j = gtid; j < n8; j += gsz) {
@@ -622,6 +645,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int32_t t = c.qq.kw[i];
         if (a.g.kw_ptr[t + 1] == a.g.kw_ptr[t]) empty = true;
     }
+    if (gtid == 0) ctl->mw_dirty = a.prune == 2 ? 1u : 0u;
     G.sync();
     stamp(G, qo, TS_RESET);
     // ---- initialisation: M = 0 on T_i, keyword nodes ungated, F_0 = K
@@ -638,6 +662,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             while (j >= ko[i + 1]) ++i;
             const int32_t v = a.g.kw_nodes[kb[i] + (j - ko[i])];
             w.M[(int64_t)v * 8 + i] = 0;
+            if (a.prune == 2) w.mw[(int64_t)v * 8 + i] = 0u;              // the path {v}: w_v added at merge
             st8[2 * (int64_t)v + 1] = 0;                                  // keyword node: no gate (L210)
             atomicOr(w.nm + (v >> 2), (1u << i) << ((v & 3) * 8));        // hit in B_i at level 0
             push(c, v, 0);
@@ -675,18 +700,17 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                     const uint32_t old = st8[2 * (int64_t)v];
                     const uint32_t nw = old | b;
                     st8[2 * (int64_t)v] = (uint8_t)nw;
+                    if (a.prune == 2) {   // lightest path to v for keyword i = min over predecessors + w_v
+                        const uint32_t wv = weight_fx(__ldg(a.g.weight + v));
+                        for (uint32_t bb = b; bb; bb &= bb - 1) {
+                            uint32_t *p = w.mw + (int64_t)v * 8 + (__ffs(bb) - 1);
+                            *p = *p + wv;
+                        }
+                    }
                     if (nw == full && old != full) {                        // Lemma V.1: depth = l
                         const uint32_t ci = agg_slot(&ctl->n_central, 1u);
                         w.centrals[ci] = v;
                         w.cdepth[ci] = (uint8_t)l;
-                        // seed of the top-down pre-pass: expand backwards every keyword v does not contain
-                        const uint64_t Mv = ldrow(w.M, v);
-                        uint32_t zb = 0;
-                        for (int i = 0; i < c.qq.q; ++i) if (((Mv >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
-                        if (full & ~zb) {
-                            w.pd_state[v] = (full & ~zb) << 8;
-                            set_bit(w.pd_bits, &ctl->pd_flag[0], v);
-                        }
                     }
                     return old == 0;
                 },
@@ -1116,21 +1140,68 @@ __device__ __forceinline__ bool prefix_match(uint64_t hi, uint32_t lo, uint64_t 
     return (lo & m) == (plo & m);
 }
 
-// Top-k by (fp64 key asc, central id asc).  |C| <= KGS_MAX_K: one CTA sorts every candidate.
-// Otherwise an MSD radix select over the 96-bit composite (12 digits of 8 bits) keeps exactly k
-// candidates, which one CTA then sorts: by one CTA alone up to kCtaSelectMax candidates (no group
-// barrier), by the whole group beyond.  Result: sel[0..count), ctl->sel_count.
+// One CTA (group rank 0) ranks cnt <= KGS_MAX_K candidates by (fp64 key asc, central id asc) and keeps
+// the first kk in sel[0..kk), ctl->sel_count = kk.  list == nullptr: the candidates are 0..cnt-1.
+// Ends with a group barrier.
+__device__ void rank_list(const Ctx &c, char *dsmem, const int32_t *list, uint32_t cnt, uint32_t kk) {
+    const Grp &G = c.G;
+    if (G.grank == 0) {
+        unsigned long long *khi = reinterpret_cast<unsigned long long *>(dsmem);
+        uint32_t *klo = reinterpret_cast<uint32_t *>(khi + KGS_MAX_K);
+        int32_t *kid = reinterpret_cast<int32_t *>(klo + KGS_MAX_K);
+        int p2 = 1;
+        while (p2 < (int)cnt) p2 <<= 1;
+        for (int i = threadIdx.x; i < p2; i += blockDim.x) {
+            if (i < (int)cnt) {
+                const int32_t idx = list ? __ldcg(list + i) : i;
+                uint64_t hi; uint32_t lo;
+                comp_key(c, (uint32_t)idx, hi, lo);
+                khi[i] = hi; klo[i] = lo; kid[i] = idx;
+            } else { khi[i] = ~0ull; klo[i] = 0xFFFFFFFFu; kid[i] = -1; }
+        }
+        __syncthreads();
+        for (int k = 2; k <= p2; k <<= 1)
+            for (int j = k >> 1; j > 0; j >>= 1) {
+                for (int i = threadIdx.x; i < p2; i += blockDim.x) {
+                    const int l = i ^ j;
+                    if (l > i) {
+                        const bool gt = khi[i] > khi[l] || (khi[i] == khi[l] && klo[i] > klo[l]);
+                        const bool up = (i & k) == 0;
+                        if (gt == up) {
+                            const unsigned long long th = khi[i]; khi[i] = khi[l]; khi[l] = th;
+                            const uint32_t tl = klo[i]; klo[i] = klo[l]; klo[l] = tl;
+                            const int32_t ti = kid[i]; kid[i] = kid[l]; kid[l] = ti;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        for (int i = threadIdx.x; i < (int)kk; i += blockDim.x) c.w.sel[i] = kid[i];
+        if (threadIdx.x == 0) c.ctl->sel_count = kk;
+    }
+    G.sync();
+}
+
+// The kk smallest (key, id) of all |C| centrals, ranked, into sel[0..kk).  |C| <= KGS_MAX_K: one CTA
+// sorts every candidate.  Otherwise an MSD radix select over the 96-bit composite (12 digits of 8 bits)
+// keeps exactly kk candidates (in elist), which one CTA then sorts: the select runs on one CTA alone up
+// to kCtaSelectMax candidates (no group barrier), on the whole group beyond.
 constexpr uint32_t kCtaSelectMax = 1u << 18;
 
-__device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
+__device__ void select_topk(const Ctx &c, long long *sh, char *dsmem, uint32_t kk) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const uint32_t nc = __ldcg(&ctl->n_central);
-    const uint32_t kk = (uint32_t)c.a.k < nc ? (uint32_t)c.a.k : nc;
+    if (nc <= (uint32_t)KGS_MAX_K) { rank_list(c, dsmem, nullptr, nc, kk); return; }
     __shared__ uint32_t hsh[256];
-    __shared__ uint32_t s_bucket, s_before;
+    __shared__ uint32_t s_bucket, s_before, s_exact;
     const bool group_wide = nc > kCtaSelectMax;
-    if (nc > (uint32_t)KGS_MAX_K && (group_wide || G.grank == 0)) {
+    if (G.gtid == 0) ctl->sel_count = 0;
+    if (group_wide) {
+        for (int64_t j = G.gtid; j < 12 * 256; j += G.gsz) (&ctl->hist[0][0])[j] = 0u;
+        G.sync();
+    }
+    if (group_wide || G.grank == 0) {
         const int64_t t0 = group_wide ? G.gtid : (int64_t)threadIdx.x;
         const int64_t ts = group_wide ? G.gsz : (int64_t)blockDim.x;
         uint64_t phi = 0;
@@ -1156,94 +1227,83 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem) {
             int tot;
             const int ex = block_excl_scan((int)hv, &tot, sh);
             if (threadIdx.x < 256 && (uint32_t)ex < want && want <= (uint32_t)ex + hv) {
-                s_bucket = threadIdx.x; s_before = (uint32_t)ex;
+                s_bucket = threadIdx.x; s_before = (uint32_t)ex; s_exact = want == (uint32_t)ex + hv;
             }
             __syncthreads();
             want -= s_before;
             const uint64_t bk = s_bucket;
             if (d < 8) phi |= bk << (56 - 8 * d);
             else plo |= (uint32_t)bk << (24 - 8 * (d - 8));
+            const bool exact = s_exact;
             __syncthreads();
+            if (exact) {   // every candidate of the bucket is selected: the threshold is the bucket's top
+                if (d < 8) { phi |= (1ull << (56 - 8 * d)) - 1ull; plo = 0xFFFFFFFFu; }
+                else plo |= (1u << (24 - 8 * (d - 8))) - 1u;
+                break;
+            }
         }
         for (int64_t i = t0; i < nc; i += ts) {   // exactly kk candidates are <= the threshold
             uint64_t hi; uint32_t lo;
             comp_key(c, (uint32_t)i, hi, lo);
             if (hi < phi || (hi == phi && lo <= plo)) {
                 const uint32_t pos = atomicAdd(&ctl->sel_count, 1u);
-                if (pos < (uint32_t)KGS_MAX_K) c.w.sel[pos] = (int32_t)i;
+                if (pos < (uint32_t)KGS_MAX_K) c.w.elist[pos] = (int32_t)i;
             }
         }
     }
-    if (group_wide) G.sync();
-    else __syncthreads();
-    if (G.grank == 0) {   // one CTA ranks (all candidates, or the radix-selected ones)
-        unsigned long long *khi = reinterpret_cast<unsigned long long *>(dsmem);
-        uint32_t *klo = reinterpret_cast<uint32_t *>(khi + KGS_MAX_K);
-        int32_t *kid = reinterpret_cast<int32_t *>(klo + KGS_MAX_K);
-        const bool small = nc <= (uint32_t)KGS_MAX_K;
-        const uint32_t cnt = small ? nc : __ldcg(&ctl->sel_count);
-        int p2 = 1;
-        while (p2 < (int)cnt) p2 <<= 1;
-        for (int i = threadIdx.x; i < p2; i += blockDim.x) {
-            if (i < (int)cnt) {
-                const int32_t idx = small ? i : __ldcg(c.w.sel + i);
-                uint64_t hi; uint32_t lo;
-                comp_key(c, (uint32_t)idx, hi, lo);
-                khi[i] = hi; klo[i] = lo; kid[i] = idx;
-            } else { khi[i] = ~0ull; klo[i] = 0xFFFFFFFFu; kid[i] = -1; }
-        }
-        __syncthreads();
-        for (int k = 2; k <= p2; k <<= 1)
-            for (int j = k >> 1; j > 0; j >>= 1) {
-                for (int i = threadIdx.x; i < p2; i += blockDim.x) {
-                    const int l = i ^ j;
-                    if (l > i) {
-                        const bool gt = khi[i] > khi[l] || (khi[i] == khi[l] && klo[i] > klo[l]);
-                        const bool up = (i & k) == 0;
-                        if (gt == up) {
-                            const unsigned long long th = khi[i]; khi[i] = khi[l]; khi[l] = th;
-                            const uint32_t tl = klo[i]; klo[i] = klo[l]; klo[l] = tl;
-                            const int32_t ti = kid[i]; kid[i] = kid[l]; kid[l] = ti;
-                        }
-                    }
-                }
-                __syncthreads();
-            }
-        for (int i = threadIdx.x; i < (int)kk; i += blockDim.x) c.w.sel[i] = kid[i];
-        if (threadIdx.x == 0) ctl->sel_count = kk;
+    G.sync();
+    rank_list(c, dsmem, c.w.elist, kk, kk);
+}
+
+// ------------------------------------------------------------------------------------------ top-down driver
+// Seeds of the predecessor pre-pass: every candidate list[0..cnt) (nullptr: all centrals), for every
+// keyword it does not contain itself (those have m = 0 and no predecessors).
+__device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
+    const Grp &G = c.G;
+    if (G.gtid == 0) { c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; }   // round 0 of this call
+    for (int64_t j = G.gtid; j < cnt; j += G.gsz) {
+        const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;
+        const int32_t cn = __ldcg(c.w.centrals + idx);
+        const uint64_t Mc = ldrow(c.w.M, cn);
+        uint32_t zb = 0;
+        for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
+        const uint32_t bits = c.qq.full & ~zb;
+        if (bits) { atomicOr(c.w.pd_state + cn, bits << 8); set_bit(c.w.pd_bits, &c.ctl->pd_flag[0], cn); }
     }
     G.sync();
 }
 
-// ------------------------------------------------------------------------------------------ top-down driver
-__device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
+// Exact Eq. 6 key of every candidate list[0..cnt) (nullptr: all centrals): (A) one warp per candidate
+// over a tier-1 arena in shared memory (most Central Graphs are small); (B) the larger ones, a whole CTA
+// per candidate over the CTA's shared region; (C) beyond that, the CTA's global-memory arena.
+// cflag: 0 = key from tier 1, 1 = from tier 2/3 (emitted by a CTA).
+__device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int32_t *list, uint32_t cnt, QOut *qo) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
     Ctl *ctl = c.ctl;
-    const uint32_t nc = __ldcg(&ctl->n_central);
-    // (A) one warp per central node, tier-1 arena in shared memory (most Central Graphs are small)
+    if (G.gtid == 0) { ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->n_eval += cnt; }
+    G.sync();
     if ((threadIdx.x >> 5) < kExtWarps) {
         Arena S1 = carve(dsmem + kSmemArena * (threadIdx.x >> 5), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
         WarpTeam T;
         for (;;) {
-            uint32_t idx = 0;
-            if (T.rank() == 0) idx = atomicAdd(&ctl->work_ext, 1u);
-            idx = __shfl_sync(0xffffffffu, idx, 0);
-            if (idx >= nc) break;
+            uint32_t t = 0;
+            if (T.rank() == 0) t = atomicAdd(&ctl->work_ext, 1u);
+            t = __shfl_sync(0xffffffffu, t, 0);
+            if (t >= cnt) break;
+            const int32_t idx = list ? __ldcg(list + t) : (int32_t)t;
             const int32_t cn = __ldcg(c.w.centrals + idx);
             double key = 0.0;
             const bool ok = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key);
             if (T.rank() == 0) {
                 if (ok) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
-                else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = (int32_t)idx; }
+                else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = idx; }
             }
             __syncwarp();
         }
     }
     G.sync();
     stamp(G, qo, TS_EXTRACT);
-    // (B) the larger ones: a whole CTA per central node over the CTA's shared region; (C) beyond that,
-    // the CTA's global-memory arena
     const uint32_t no = __ldcg(&ctl->n_overflow);
     BlockTeam BT{sh};
     if (no) {
@@ -1272,16 +1332,20 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
                 }
                 __syncthreads();
             }
-            G.sync();
         }
-        if (G.gtid == 0) ctl->work_big = 0;
         G.sync();
+        stamp(G, qo, TS_EXTRACT_BIG);
     }
-    stamp(G, qo, TS_EXTRACT_BIG);
-    select_topk(c, sh, dsmem);
-    stamp(G, qo, TS_SELECT);
-    // emit: one warp per winner (per-warp arena), overflowed winners by a CTA
+}
+
+// Emit the ranked winners sel[0..sel_count): one warp per winner (per-warp arena), the winners that
+// overflowed tier 1 by a CTA.  work_emit and work_big are zero on entry.
+__device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    Ctl *ctl = c.ctl;
     const uint32_t cnt = __ldcg(&ctl->sel_count);
+    BlockTeam BT{sh};
     if ((threadIdx.x >> 5) < kExtWarps) {
         const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
         Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
@@ -1332,6 +1396,86 @@ __device__ void topdown(const Ctx &c, long long *sh, char *dsmem, QOut *qo) {
         G.sync();
     }
     stamp(G, qo, TS_EMIT);
+}
+
+// Top-down phase (Alg. 3 + Eq. 6): exact keys, top-k, answer subgraphs.
+// Without pruning every central is extracted.  With pruning (kgs_params.prune, DESIGN.md "Top-down
+// pruning"): key(c) = d^lambda (x) (sum of kept weights) >= LB(c) = d^lambda (x) w_c exactly in fp64
+// (c is always kept, weights are >= 0, rounded addition and multiplication are monotone).  Round 1
+// extracts the m smallest (LB, id); T = the k-th smallest exact (key, id) among them.  Every other
+// candidate has (LB, id) above the m-th (LB, id) B; if B >= T none of them can rank before T, else
+// round 2 extracts every remaining candidate with (LB, id) < T.  The top-k over the extracted
+// candidates is then the top-k over all of C.
+
+__device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QOut *qo) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    Ctl *ctl = c.ctl;
+    const uint32_t nc = __ldcg(&ctl->n_central);
+    const uint32_t kk = (uint32_t)a.k < nc ? (uint32_t)a.k : nc;
+    const uint32_t mcap = min((uint32_t)KGS_MAX_K, max(8u * kk, (uint32_t)a.prune_min));
+    if (!a.prune || nc <= mcap) {
+        seed_pd(c, nullptr, nc);
+        stamp(G, qo, TS_PD_SEED);
+        pred_dag(c, S, sh, qo);
+        extract_list(c, sh, dsmem, nullptr, nc, qo);
+        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }   // emit counters (read after the select)
+        select_topk(c, sh, dsmem, kk);
+    } else {
+        const uint32_t m = mcap;
+        for (int64_t i = G.gtid; i < nc; i += G.gsz) {   // lower bounds; cflag 2 = not extracted
+            const int32_t cn = __ldcg(c.w.centrals + i);
+            double lb;
+            if (a.prune == 2) {   // the kept graph holds a lightest-or-heavier path from T_i to c, every i
+                uint32_t mx = 0;
+                for (int j = 0; j < c.qq.q; ++j) mx = max(mx, __ldcg(c.w.mw + (int64_t)cn * 8 + j));
+                lb = (double)mx * (1.0 / 16777216.0);
+            } else {
+                lb = (double)__ldg(a.g.weight + cn);
+            }
+            c.w.ckey[i] = __dmul_rn(a.dpow[__ldcg(c.w.cdepth + i)], lb);
+            c.w.cflag[i] = 2;
+        }
+        G.sync();
+        select_topk(c, sh, dsmem, m);                          // sel[0..m): the m smallest (LB, id)
+        uint64_t bhi; uint32_t blo;
+        comp_key(c, (uint32_t)__ldcg(c.w.sel + m - 1), bhi, blo);
+        for (int64_t j = G.gtid; j < m; j += G.gsz) c.w.elist[j] = __ldcg(c.w.sel + j);
+        G.sync();
+        seed_pd(c, c.w.elist, m);
+        stamp(G, qo, TS_PD_SEED);
+        pred_dag(c, S, sh, qo);
+        extract_list(c, sh, dsmem, c.w.elist, m, qo);
+        rank_list(c, dsmem, c.w.elist, m, kk);                 // T = the kk-th exact (key, id)
+        uint64_t thi; uint32_t tlo;
+        comp_key(c, (uint32_t)__ldcg(c.w.sel + kk - 1), thi, tlo);
+        uint32_t n2 = 0;
+        if (bhi < thi || (bhi == thi && blo < tlo)) {
+            // round 2: every candidate not extracted yet whose (LB, id) still ranks before T
+            for (int64_t i = G.gtid; i < nc; i += G.gsz) {
+                if (__ldcg(c.w.cflag + i) != 2) continue;
+                uint64_t hi; uint32_t lo;
+                comp_key(c, (uint32_t)i, hi, lo);
+                if (hi < thi || (hi == thi && lo < tlo)) c.w.elist[m + agg_slot(&ctl->n_elist2, 7u)] = (int32_t)i;
+            }
+            G.sync();
+            n2 = __ldcg(&ctl->n_elist2);
+            seed_pd(c, c.w.elist + m, n2);
+            pred_dag(c, S, sh, qo);
+            extract_list(c, sh, dsmem, c.w.elist + m, n2, qo);
+        }
+        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }
+        if (m + n2 <= (uint32_t)KGS_MAX_K) {
+            rank_list(c, dsmem, c.w.elist, m + n2, kk);
+        } else {   // the candidates never extracted rank after every extracted one
+            for (int64_t i = G.gtid; i < nc; i += G.gsz)
+                if (__ldcg(c.w.cflag + i) == 2) c.w.ckey[i] = __longlong_as_double(0x7FF0000000000000ll);
+            G.sync();
+            select_topk(c, sh, dsmem, kk);
+        }
+    }
+    stamp(G, qo, TS_SELECT);
+    emit_answers(c, sh, dsmem, qo);
 }
 
 // ------------------------------------------------------------------------------------------ engine
@@ -1406,8 +1550,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         stamp(G, qo, TS_START);
         const Ctx c{a, w, ctl, G, qq};
         search(c, s_big, sh, qo);
-        pred_dag(c, s_big, sh, qo);
-        topdown(c, sh, dsmem, qo);
+        topdown(c, s_big, sh, dsmem, qo);
         if (G.gtid == 0) {
             qo->levels = ctl->levels;
             qo->stop_reason = ctl->stop_reason;
@@ -1417,6 +1560,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->n_overflow = ctl->n_overflow;
             qo->n_cid = ctl->n_cid;
             qo->n_parcs = ctl->n_parcs;
+            qo->n_eval = ctl->n_eval;
             qo->frontier_total = ctl->frontier_total;
             qo->arcs_scanned = ctl->arcs_scanned;
             qo->hits = ctl->hits;

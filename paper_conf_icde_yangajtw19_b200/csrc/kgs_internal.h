@@ -51,14 +51,16 @@ struct Ctl {
     uint32_t n_parcs;              // predecessor arcs found
     unsigned long long td_arcs;    // in-arcs inspected by the pre-pass
     int32_t pd_rounds;
-    int32_t pad3;
+    uint32_t n_eval;               // candidates whose exact key was computed (all of C without pruning)
+    uint32_t n_elist2;             // second pruning round: candidates whose bound still beats the threshold
+    uint32_t mw_dirty;             // this query wrote lightest-path rows (prune mode 2): the next one resets them
 };
 
 // Per-query summary written by the engine (device), read back by the host.
 constexpr int kMaxStamps = 48;
 struct QOut {
     int32_t levels, stop_reason, count, fatal;
-    uint32_t n_central, n_overflow, n_cid, n_parcs;
+    uint32_t n_central, n_overflow, n_cid, n_parcs, n_eval, pad;
     unsigned long long frontier_total, arcs_scanned, hits, td_arcs;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
@@ -104,6 +106,8 @@ struct DevWork {
     int32_t *overflow;  // [n] centrals whose graph exceeds the per-warp extractor
     uint8_t *cflag;     // [n] 1 = overflowed the per-warp extractor
     int32_t *sel;       // [KGS_MAX_K] ranked winners (index into centrals)
+    int32_t *elist;     // [n] candidates to extract (index into centrals)
+    uint32_t *mw;       // [n*8] lightest hitting path per (node, keyword), fixed point 2^-24; all-ones = unset
     Ctl *ctl[2];        // ping-pong: the previous query's block drives the sparse reset
     // shared predecessor DAG over the union of all Central Graphs
     uint32_t *pd_state; // [n] byte0 = bits to expand this round, byte1 = bits for the next round, byte2 = done
@@ -151,6 +155,8 @@ struct EngineArgs {
     // parameters (shared by the batch)
     int k, max_depth, block_central, extract_mode, level_cover;
     int tile_light;             // light frontiers up to this many nodes are expanded by group-wide tiles
+    int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
+    int prune_min;              // round 1 extracts max(8k, prune_min) candidates
     // outputs
     QOut *qout;                 // [nq]
     int32_t *out_hdr;           // [nq][k][4]: central, depth, n_nodes, n_arcs

@@ -1,0 +1,180 @@
+"""Exact lower-bound pruning of the top-down phase (kgs_params.prune).
+
+With pruning the engine computes the exact Eq. 6 key only for the candidates whose lower bound can
+still reach the top-k.  The answers must be those of the oracle
+(which extracts every Central Graph), and the number of candidates evaluated must be the one the
+two-round rule gives when it is replayed here on the oracle's own keys:
+
+  LB(c) = pow(d, lambda) * max_i (lightest Thm. V.4 path from T_i to c)   (exact extraction)
+
+  round 1: the m = min(KGS_MAX_K, max(8k, 512)) smallest (LB, id); T = the k-th smallest exact
+           (key, id) among them; B = the m-th (LB, id);
+  round 2 (only if B < T): every other candidate with (LB, id) < T.
+
+Graphs have several thousand Central Nodes so that both outcomes (round 2 or not) occur.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+kgs = pytest.importorskip("paper_conf_icde_yangajtw19_b200")
+
+KGS_MAX_K = 4096
+
+
+def _gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def medium_graph(seed, n=4000, deg=4, q=3, kw_size=300, wpow=1.0, zero_frac=0.0):
+    """Random undirected graph with many Central Nodes; weights on the 2^-24 grid, skewed by wpow."""
+    rng = np.random.default_rng(seed)
+    m = n * deg // 2
+    u = rng.integers(0, n, m)
+    v = rng.integers(0, n, m)
+    keep = u != v
+    edges = list(zip(u[keep].tolist(), v[keep].tolist()))
+    w = rng.random(n) ** wpow
+    w[rng.random(n) < zero_frac] = 0.0
+    w = (np.floor(w * (1 << 24) + 0.5) / (1 << 24)).astype(np.float32)
+    kws = [sorted(rng.choice(n, size=kw_size, replace=False).tolist()) for _ in range(q)]
+    return synth.from_edges(n, edges, w, kws, 2.0)
+
+
+def lightest_paths(g, kw, o):
+    """Per (node, keyword): the lightest weight (fixed point 2^-24) of a path from T_i to the node along
+    Thm. V.4 arcs (m_xi = 1 + max(a_u, m_ui, g_x - 1), u not a blocked central at m_xi - 1), by dynamic
+    programming over the oracle's hitting levels, level by level.  numpy, independent of the engine."""
+    n = len(g.row_ptr) - 1
+    q = len(kw)
+    src = np.repeat(np.arange(n, dtype=np.int64), np.diff(g.row_ptr))
+    dst = np.asarray(g.col_idx, np.int64)
+    W = np.floor(np.asarray(g.weight, np.float64) * (1 << 24)).astype(np.int64)
+    M = o.M.astype(np.int64)
+    a = o.a.astype(np.int64)
+    K = np.zeros(n, bool)
+    for t in kw:
+        K[g.kw_nodes[g.kw_ptr[t]:g.kw_ptr[t + 1]]] = True
+    gate = np.where(K, 0, a)
+    full = (M < 255).all(1)
+    maxrow = np.where(M < 255, M, 0).max(1)
+    big = np.int64(1) << 62
+    mw = np.full((n, q), big, np.int64)
+    for i in range(q):
+        lv = M[:, i]
+        mw[lv == 0, i] = W[lv == 0]
+        mu, mx = lv[src], lv[dst]
+        ok = (mu < 255) & (mx < 255) & (mx == 1 + np.maximum(np.maximum(a[src], mu), gate[dst] - 1))
+        ok &= ~(full[src] & (maxrow[src] <= mx - 1))
+        su, sx = src[ok], dst[ok]
+        top = int(lv[lv < 255].max()) if (lv < 255).any() else 0
+        for L in range(1, top + 1):
+            sel = lv[sx] == L
+            cand = np.full(n, big, np.int64)
+            np.minimum.at(cand, sx[sel], mw[su[sel], i])
+            hit = lv == L
+            mw[hit, i] = W[hit] + cand[hit]
+    return mw
+
+
+def expected_evaluated(g, o, k, lam, kw, pmin=512, bound="path"):
+    """Replay of the two-round rule on the oracle's exact keys (see the module docstring).  bound="path"
+    (exact extraction, the default): LB(c) = pow(d, lambda) * max_i lightest_i(c); bound="weight"
+    (literal extraction with central blocking): LB(c) = pow(d, lambda) * w_c."""
+    nc = len(o.centrals)
+    kk = min(k, nc)
+    mcap = min(KGS_MAX_K, max(8 * kk, pmin))
+    if nc <= mcap:
+        return nc
+    C = o.centrals.tolist()
+    if bound == "path":
+        mw = lightest_paths(g, kw, o)
+        lbw = [float(mw[c].max()) / (1 << 24) for c in C]
+    else:
+        lbw = [float(g.weight[c]) for c in C]
+    lb = [math.pow(float(d), lam) * x for x, d in zip(lbw, o.central_depth.tolist())]
+    keys = o.central_key.tolist()
+    assert all(x <= y for x, y in zip(lb, keys)), "the bound must not exceed the exact key"
+    ids = o.centrals.tolist()
+    order = sorted(range(nc), key=lambda i: (lb[i], ids[i]))
+    first = order[:mcap]
+    B = (lb[first[-1]], ids[first[-1]])
+    T = sorted((keys[i], ids[i]) for i in first)[kk - 1]
+    if not B < T:
+        return mcap
+    return mcap + sum(1 for i in order[mcap:] if (lb[i], ids[i]) < T)
+
+
+CASES = [  # seed, graph kwargs, k, lambda, round-1 minimum, extract mode, prune mode
+    (1, dict(), 20, 0.2, 512, 0, 1),                                            # |C| 35: no pruning
+    (6, dict(q=4, kw_size=250, deg=6), 300, 0.2, 512, 0, 2),                    # 1044 <= 8k: no pruning
+    (2, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 20, 0.2, 512, 0, 1),  # w_c bound, round 2
+    (12, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 5, 0.2, 64, 0, 1),   # w_c bound
+    (12, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 20, 0.2, 512, 0, 2), # path bound: 1078 -> 512
+    (10, dict(n=20000, deg=16, q=3, kw_size=20, zero_frac=0.9), 300, 0.0, 512, 0, 2),  # 16574 -> 2400
+    (2, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 20, 0.2, 1, 0, 2),    # 4239 -> 268: round 2
+    (12, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 20, 0.2, 1, 0, 2),   # 1078 -> 160
+    (2, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 20, 0.2, 512, 1, 2),  # literal: falls back to w_c
+    (12, dict(n=20000, deg=16, q=3, kw_size=20, wpow=4.0), 5, 0.2, 64, 1, 1),   # literal, w_c bound
+]
+
+
+def _outcome(exp, nc, mcap):
+    return "none" if nc <= mcap else ("round1" if exp == mcap else "round2")
+
+
+def test_pruned_answers_and_evaluated_counts(monkeypatch):
+    _gpu()
+    outcomes = set()
+    for seed, kwargs, k, lam, pmin, ext, mode in CASES:
+        monkeypatch.setenv("KGS_PRUNE_MIN", str(pmin))
+        g = medium_graph(seed, **kwargs)
+        G = kgs.kgs_load_graph(g)
+        kw = list(range(len(g.kw_ptr) - 1))
+        o = oracle.query(g, kw, k, lam=lam, extract_mode=ext)
+        ctx = f"seed={seed} k={k} lam={lam} pmin={pmin} ext={ext} mode={mode} |C|={len(o.centrals)}"
+        for prune in (mode, 0):
+            r = kgs.kgs_query(G, kw, k, kgs.make_params(lam=lam, prune=prune, extract_mode=ext))
+            assert r.stats["n_centrals"] == len(o.centrals), ctx
+            assert [a.central for a in r.answers] == [a.central for a in o.answers], (ctx, prune)
+            for ra, oa in zip(r.answers, o.answers):
+                assert ra.score_key == oa.key and ra.depth == oa.depth, (ctx, prune)
+                assert ra.nodes.tolist() == oa.nodes.tolist(), (ctx, prune)
+                assert ra.arcs.tolist() == oa.arcs.tolist(), (ctx, prune)
+            if prune:
+                exp = expected_evaluated(g, o, k, lam, kw, pmin, "path" if (ext == 0 and mode == 2) else "weight")
+                assert r.stats["n_evaluated"] == exp, (ctx, exp)
+                nc = len(o.centrals)
+                outcomes.add((mode, _outcome(exp, nc, min(KGS_MAX_K, max(8 * min(k, nc), pmin)))))
+            else:
+                assert r.stats["n_evaluated"] == len(o.centrals), ctx
+        G.close()
+    assert {(1, "round2"), (2, "round1"), (2, "round2")} <= outcomes, outcomes
+
+
+def test_batch_pruned_matches_oracle():
+    """The batch engine (several groups) prunes per query with the same result, in both bound modes;
+    a mode-2 batch followed by a mode-1 batch checks that the lightest-path rows are reset."""
+    _gpu()
+    g = medium_graph(10, n=20000, deg=16, q=3, kw_size=20, zero_frac=0.9)
+    G = kgs.kgs_load_graph(g)
+    rng = np.random.default_rng(3)
+    qs = [sorted(rng.choice(3, size=int(rng.integers(2, 4)), replace=False).tolist()) for _ in range(12)]
+    for mode in (2, 1, 2):
+        for k in (1, 20, 64):
+            exp = [oracle.query(g, kw, k) for kw in qs]
+            res = kgs.kgs_query_batch(G, qs, k, kgs.make_params(prune=mode), 4)
+            for kw, r, o in zip(qs, res, exp):
+                assert [a.central for a in r.answers] == [a.central for a in o.answers], (kw, k, mode)
+                assert [a.score_key for a in r.answers] == [a.key for a in o.answers], (kw, k, mode)
+                bound = "path" if mode == 2 else "weight"
+                assert r.stats["n_evaluated"] == expected_evaluated(g, o, k, 0.2, kw, 512, bound), (kw, k, mode)
+    G.close()
