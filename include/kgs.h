@@ -137,6 +137,7 @@ typedef struct {
     float ms_launch;       /* the whole engine launch that answered it (all queries of the batch) */
     int32_t group;         /* engine group (set of CTAs) that answered the query */
     int32_t n_evaluated;   /* Central Graphs whose exact key was computed (|C| unless prune skipped some) */
+    int64_t dag_arcs;      /* arcs the search traversed that hit their target: the Thm. V.4 arcs of all hit nodes */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index

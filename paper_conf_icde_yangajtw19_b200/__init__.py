@@ -58,7 +58,7 @@ class kgs_stats(ctypes.Structure):
                 ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("td_arcs", ctypes.c_int64),
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
-                ("n_evaluated", ctypes.c_int32)]
+                ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64)]
 
 
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",

@@ -563,6 +563,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.arcs_scanned = (int64_t)o.arcs_scanned;
         st.overflow = o.n_overflow;
         st.hits = (int64_t)o.hits;
+        st.dag_arcs = (int64_t)o.dag_arcs;
         st.td_arcs = (int64_t)o.td_arcs;
         st.td_pred_arcs = o.n_parcs;
         st.n_evaluated = (int32_t)o.n_eval;

@@ -240,11 +240,12 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, int32_t x, uint32_t sx,
-                                          unsigned &hits) {
+                                          unsigned &hits, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = sx >> 8;
     if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
+        ++dag;                                            // a Thm. V.4 arc (v -> x for these keywords)
         if (c.a.prune == 2) {   // x is hit at l+1 for these keywords: v is a Thm. V.4 predecessor of (x, i)
             for (uint32_t b = bits; b; b &= b - 1) {
                 const int i = __ffs(b) - 1;
@@ -672,7 +673,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     stamp(G, qo, TS_SCATTER);
 
     unsigned long long my_arcs = 0;
-    unsigned my_hits = 0;
+    unsigned my_hits = 0, my_dag = 0;
     for (int l = 0;; ++l) {
         // ---- enqueue frontiers: anything pending at this or a later level?
         __shared__ int s_pend;
@@ -743,7 +744,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             nd.hm = prepare(c, l, v, leader);
             return nd.hm != 0;
         };
-        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(c, l, nd.v, nd.hm, x, sx, my_hits); };
+        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(c, l, nd.v, nd.hm, x, sx, my_hits, my_dag); };
         expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
             expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
@@ -754,17 +755,20 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     }
     const unsigned wa = __reduce_add_sync(0xffffffffu, (unsigned)my_arcs);   // per-warp totals fit 32 bits
     const unsigned wh = __reduce_add_sync(0xffffffffu, my_hits);
-    __shared__ unsigned long long s_sum[2];
-    if (threadIdx.x < 2) s_sum[threadIdx.x] = 0ull;
+    const unsigned wd = __reduce_add_sync(0xffffffffu, my_dag);
+    __shared__ unsigned long long s_sum[3];
+    if (threadIdx.x < 3) s_sum[threadIdx.x] = 0ull;
     __syncthreads();
     if ((threadIdx.x & 31) == 0) {
         if (wa) atomicAdd(&s_sum[0], (unsigned long long)wa);
         if (wh) atomicAdd(&s_sum[1], (unsigned long long)wh);
+        if (wd) atomicAdd(&s_sum[2], (unsigned long long)wd);
     }
     __syncthreads();
     if (threadIdx.x == 0) {      // one global atomic per CTA
         if (s_sum[0]) atomicAdd(&ctl->arcs_scanned, s_sum[0]);
         if (s_sum[1]) atomicAdd(&ctl->hits, s_sum[1]);
+        if (s_sum[2]) atomicAdd(&ctl->dag_arcs, s_sum[2]);
     }
     G.sync();
     stamp(G, qo, TS_END);
@@ -1564,6 +1568,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->frontier_total = ctl->frontier_total;
             qo->arcs_scanned = ctl->arcs_scanned;
             qo->hits = ctl->hits;
+            qo->dag_arcs = ctl->dag_arcs;
             qo->td_arcs = ctl->td_arcs;
             qo->t_end = globaltimer_ns();
             w.gstate[1] = done + 1;

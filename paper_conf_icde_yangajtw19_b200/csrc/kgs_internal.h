@@ -54,6 +54,7 @@ struct Ctl {
     uint32_t n_eval;               // candidates whose exact key was computed (all of C without pruning)
     uint32_t n_elist2;             // second pruning round: candidates whose bound still beats the threshold
     uint32_t mw_dirty;             // this query wrote lightest-path rows (prune mode 2): the next one resets them
+    unsigned long long dag_arcs;   // arcs the search traversed that hit their target (the Thm. V.4 arcs)
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -61,7 +62,7 @@ constexpr int kMaxStamps = 48;
 struct QOut {
     int32_t levels, stop_reason, count, fatal;
     uint32_t n_central, n_overflow, n_cid, n_parcs, n_eval, pad;
-    unsigned long long frontier_total, arcs_scanned, hits, td_arcs;
+    unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
     unsigned long long stamp[kMaxStamps];

@@ -1,5 +1,5 @@
 """Aggregate ncu --page source --print-source=cuda,sass CSV by CUDA source line: warp-stall samples
-(total + top stall reasons) and L2 sectors.  Usage: ncu_hot.py report.ncu-rep [kernel-regex] [top]"""
+(total + top stall reasons) and L2 sectors.  Usage: ncu_hot.py report.ncu-rep [kernel-regex] [top] [samples|l2sec]"""
 import csv
 import collections
 import io
@@ -44,8 +44,11 @@ for r in rows:
     except ValueError:
         pass
 tot = sum(c["samples"] for c in agg.values()) or 1
-print(f"total samples {tot}")
-for key, c in sorted(agg.items(), key=lambda x: -x[1]["samples"])[:top]:
+tot_l2 = sum(c["l2sec"] for c in agg.values()) or 1
+order = sys.argv[4] if len(sys.argv) > 4 else "samples"   # or "l2sec"
+print(f"total samples {tot}, total L2 sectors {tot_l2}")
+for key, c in sorted(agg.items(), key=lambda x: -x[1][order])[:top]:
     stalls = sorted(((k, v) for k, v in c.items() if k.startswith("stall_")), key=lambda x: -x[1])[:3]
     s = ", ".join(f"{k[6:]}={v}" for k, v in stalls)
-    print(f"{c['samples']/tot*100:5.1f}% {key[0]}:{key[1]:>4s} l2sec={c['l2sec']:>9d} [{s}] {src.get(key, '')[:80]}")
+    print(f"{c['samples']/tot*100:5.1f}% {key[0]}:{key[1]:>4s} l2sec={c['l2sec']:>9d} ({c['l2sec']/tot_l2*100:4.1f}%) "
+          f"[{s}] {src.get(key, '')[:80]}")

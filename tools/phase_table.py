@@ -9,5 +9,5 @@ for line in open(sys.argv[1]):
     except (ValueError, SyntaxError):
         continue
     ph = {k: round(v) for k, v in d["phases_us"].items()}
-    print(i, "q=" + q, "C", d["n_centrals"], "lv", d["levels"], "arcs", d["arcs_scanned"],
+    print(i, "q=" + q, "C", d["n_centrals"], "lv", d["levels"], "arcs", d["arcs_scanned"], "dag", d.get("dag_arcs"), "td", d["td_arcs"],
           "search %.3f td %.3f" % (d["ms_search"], d["ms_topdown"]), ph)

@@ -1,0 +1,34 @@
+"""Driver for an ncu capture of ONE batch launch of the engine (the bench's launch shape): load a
+config's graph, run a warm batch (launch 1), then the captured batch (launch 2, `-s 1 -c 1`).
+Usage: profile_batch.py [config] [batch] [groups]"""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icde_yangajtw19_b200 as kgs  # noqa: E402
+import synth  # noqa: E402
+
+name = sys.argv[1] if len(sys.argv) > 1 else "C3"
+batch = int(sys.argv[2]) if len(sys.argv) > 2 else 128
+groups = int(sys.argv[3]) if len(sys.argv) > 3 else 8
+w = synth.make_workload(name)
+order = np.random.default_rng(12345).permutation(len(w.queries))
+qs = [w.queries[i] for i in order]
+G = kgs.kgs_load_graph(w.graph)
+s = torch.cuda.current_stream()
+for rep in range(2):
+    sub = [qs[(rep * batch + j) % len(qs)] for j in range(batch)]
+    kwp = torch.full((batch, 8), -1, dtype=torch.int32)
+    for i, q in enumerate(sub):
+        kwp[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
+    kwd = kwp.cuda()
+    qld = torch.tensor([len(q) for q in sub], dtype=torch.int32, device="cuda")
+    kgs.kgs_query_batch_device(G, batch, kwd.data_ptr(), qld.data_ptr(), w.k, None, groups, s.cuda_stream)
+    res = kgs.kgs_query_batch_fetch(G, [len(q) for q in sub], s.cuda_stream)
+    st = [r.stats for r in res]
+    print(f"launch {rep}: {batch} queries, G={groups}, ms_launch {st[0]['ms_launch']:.2f}, "
+          f"arcs {sum(x['arcs_scanned'] for x in st)}, td_arcs {sum(x['td_arcs'] for x in st)}, "
+          f"centrals {sum(x['n_centrals'] for x in st)}", flush=True)
