@@ -203,6 +203,50 @@ kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s);
 kgs_status kgs_result_phases(const kgs_result *r, int32_t *tags, uint64_t *t_ns, int32_t cap, int32_t *n);
 void kgs_result_free(kgs_result *r);
 
+/* ---- Vertex-partitioned search of ONE query over P ranks ----
+ * Every rank loads the whole graph (kgs_load_graph: the CSR is replicated) and owns the node rows
+ * [lo, hi) = [rank * slice, min((rank + 1) * slice, n)), slice = kgs_vp_slice(n, world).  The search is
+ * the level rule of Alg. 2 (reading R10) as a pull over the owned rows: at level l an owned x
+ * gets keyword i if some in-neighbour u expands i at l (a_u <= l, m_ui <= l, u not a blocked central) and
+ * x may be entered (x in K or a_x <= l + 1).  The caller owns the exchange buffers (device memory on the
+ * graph's device, n_pad = slice * world) and runs the collectives between the calls:
+ *   kgs_vp_begin          sources, owned level-0 centrals               then all_reduce(counts, sum)
+ *   kgs_vp_level(l)       one level over the owned rows                  then all_gather(hm <- hm_slice),
+ *                                                                             all_reduce(counts, sum)
+ *   kgs_vp_waiting(l)     only if the level made no mark, nothing waits for activation and
+ *                         l + 1 < amax: hit nodes waiting for a gated neighbour  then all_reduce(counts)
+ *   (host: the stop rules of kgs_query — |C| >= k, max_depth, and exhaustion when the work-list of
+ *    Alg. 2 is empty: no mark and nothing waiting, which stops at level l + 1)
+ *   after the search      all_gather(M <- owned rows), all_gather(central lists)
+ *   kgs_vp_topdown        Alg. 3 + level-cover + Eq. 6 + top-k on the replicated state -> kgs_result
+ * paper_conf_icde_yangajtw19_b200.dist.vp_query is that driver over torch.distributed.  The result equals
+ * kgs_query's.  Calls on one graph must not interleave with other queries between begin and topdown. */
+typedef struct {
+    uint8_t *hm;        /* [n_pad]     replicated hit masks (bit i = hit by keyword i); all_gather output */
+    uint8_t *hm_slice;  /* [slice]     this rank's hit masks after the level; all_gather input */
+    uint8_t *M;         /* [n_pad * 8] node-major hitting levels; this rank writes rows [lo, hi) */
+    int64_t *counts;    /* [3]         marks, new central nodes, waiting work-list nodes (all_reduce sum) */
+    int32_t *cent;      /* [slice]     this rank's central nodes (identification order) */
+    uint8_t *cdep;      /* [slice]     their depths */
+    int32_t *cent_n;    /* [1]         their count */
+} kgs_vp_buffers;
+/* ceil(n / world) rounded up to a multiple of 16 (0 for bad arguments). */
+int64_t kgs_vp_slice(int64_t n_nodes, int32_t world);
+/* Validation as kgs_query.  info[0] = amax (max activation level at alpha: the exhaustion rule needs it),
+ * info[1] = 1 if some T_i is empty (stop with KGS_STOP_EMPTY_KEYWORD, no level calls). */
+kgs_status kgs_vp_begin(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, const kgs_params *p, int32_t rank,
+                        int32_t world, const kgs_vp_buffers *b, void *cuda_stream, int32_t *info);
+/* Level l (0 <= l < 254) over the owned rows: reads hm (the state at the start of l), writes hm_slice,
+ * the owned M rows, the owned centrals (depth l + 1) and counts. */
+kgs_status kgs_vp_level(kgs_graph *g, int32_t level, void *cuda_stream);
+/* After a level l without marks (hm = the state after l): counts[2] = owned hit nodes, not blocked, active
+ * at l, with an out-neighbour gated at l + 1 that lacks one of their keywords (Alg. 2 ln 17-19). */
+kgs_status kgs_vp_waiting(kgs_graph *g, int32_t level, void *cuda_stream);
+/* Top-down on the replicated state: b.hm and b.M complete (all ranks' rows), centrals_dev / depth_dev the
+ * all-gathered central list (device, n_central entries), levels / stop_reason from the host loop. */
+kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centrals_dev, const uint8_t *depth_dev,
+                          int32_t levels, int32_t stop_reason, void *cuda_stream, kgs_result **out);
+
 /* Thread-local message describing the last non-OK status of this thread. */
 const char *kgs_last_error(void);
 

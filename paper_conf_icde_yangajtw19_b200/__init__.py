@@ -61,11 +61,18 @@ class kgs_stats(ctypes.Structure):
                 ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64)]
 
 
+class kgs_vp_buffers(ctypes.Structure):
+    _fields_ = [("hm", ctypes.c_void_p), ("hm_slice", ctypes.c_void_p), ("M", ctypes.c_void_p),
+                ("counts", ctypes.c_void_p), ("cent", ctypes.c_void_p), ("cdep", ctypes.c_void_p),
+                ("cent_n", ctypes.c_void_p)]
+
+
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
             "kgs_query_fetch", "kgs_result_count", "kgs_result_answer", "kgs_result_levels",
             "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_phases",
             "kgs_result_free", "kgs_last_error", "kgs_version", "kgs_query_batch", "kgs_query_batch_device",
-            "kgs_query_batch_fetch"]
+            "kgs_query_batch_fetch", "kgs_vp_slice", "kgs_vp_begin", "kgs_vp_level", "kgs_vp_waiting",
+            "kgs_vp_topdown"]
 
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
                "search_end", "extract", "extract_big", "select", "emit"]
@@ -118,6 +125,17 @@ def lib():
         L.kgs_result_free.restype = None
         L.kgs_last_error.argtypes = []
         L.kgs_last_error.restype = ctypes.c_char_p
+        L.kgs_vp_slice.argtypes = [i64, i32]
+        L.kgs_vp_slice.restype = i64
+        L.kgs_vp_begin.argtypes = [vp, vp, i32, i32, ctypes.POINTER(kgs_params), i32, i32,
+                                   ctypes.POINTER(kgs_vp_buffers), vp, vp]
+        L.kgs_vp_begin.restype = i32
+        L.kgs_vp_level.argtypes = [vp, i32, vp]
+        L.kgs_vp_level.restype = i32
+        L.kgs_vp_waiting.argtypes = [vp, i32, vp]
+        L.kgs_vp_waiting.restype = i32
+        L.kgs_vp_topdown.argtypes = [vp, i64, vp, vp, i32, i32, vp, ctypes.POINTER(vp)]
+        L.kgs_vp_topdown.restype = i32
         L.kgs_version.argtypes = []
         L.kgs_version.restype = ctypes.c_char_p
         _lib = L
@@ -314,3 +332,35 @@ def kgs_query_batch_fetch(graph: Graph, qlens, stream: int = 0) -> list:
 
 def kgs_version() -> str:
     return lib().kgs_version().decode()
+
+
+# ---- vertex-partitioned search of one query (driver: dist.vp_query) ----
+def kgs_vp_slice(n_nodes: int, world: int) -> int:
+    return int(lib().kgs_vp_slice(int(n_nodes), int(world)))
+
+
+def kgs_vp_begin(graph: Graph, kw_ids, k: int, params: kgs_params | None, rank: int, world: int,
+                 bufs: kgs_vp_buffers, stream: int = 0) -> tuple:
+    """Returns (amax, empty)."""
+    kw = np.ascontiguousarray(np.asarray(kw_ids, dtype=np.int32))
+    p = params if params is not None else kgs_params_default()
+    info = np.zeros(2, np.int32)
+    _check(lib().kgs_vp_begin(graph.handle, kw.ctypes.data, int(kw.shape[0]), int(k), ctypes.byref(p), int(rank),
+                              int(world), ctypes.byref(bufs), ctypes.c_void_p(stream), info.ctypes.data))
+    return int(info[0]), bool(info[1])
+
+
+def kgs_vp_level(graph: Graph, level: int, stream: int = 0) -> None:
+    _check(lib().kgs_vp_level(graph.handle, int(level), ctypes.c_void_p(stream)))
+
+
+def kgs_vp_waiting(graph: Graph, level: int, stream: int = 0) -> None:
+    _check(lib().kgs_vp_waiting(graph.handle, int(level), ctypes.c_void_p(stream)))
+
+
+def kgs_vp_topdown(graph: Graph, n_central: int, cent_ptr: int, dep_ptr: int, levels: int, stop_reason: int, q: int,
+                   want_levels: int = 0, stream: int = 0) -> Result:
+    h = ctypes.c_void_p()
+    _check(lib().kgs_vp_topdown(graph.handle, int(n_central), ctypes.c_void_p(cent_ptr), ctypes.c_void_p(dep_ptr),
+                                int(levels), int(stop_reason), ctypes.c_void_p(stream), ctypes.byref(h)))
+    return _read_result(h, graph.n, int(q), want_levels)

@@ -123,6 +123,17 @@ struct kgs_graph {
     uint32_t *h_amax = nullptr;
     cudaEvent_t ev[2];
     std::mutex mu;
+    // vertex-partitioned search of one query (vpart.cu)
+    uint8_t *vp_gate = nullptr, *vp_X = nullptr;
+    size_t vp_X_cap = 0;
+    int32_t *vp_big = nullptr, *vp_nbig_dev = nullptr;
+    int vp_nbig = 0;
+    int64_t vp_big_lo = -1, vp_big_hi = -1;
+    VpBufs vp{};
+    VpQuery vq{};
+    kgs_params vp_p{};
+    int vp_k = 0;
+    bool vp_active = false;
     // the last enqueued batch (for the fetch calls)
     int last_nq = 0, last_k = 0, last_G = 1;
     std::vector<int> last_q;
@@ -227,7 +238,8 @@ void kgs_free_graph(kgs_graph *g) {
     for (auto &w : g->works) free_work(w);
     void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->act, g->amax_dev, g->dpow,
                     g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
-                    g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr};
+                    g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr, g->vp_gate, g->vp_X, g->vp_big,
+                    g->vp_nbig_dev};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
     void *hp[] = {g->h_kw, g->h_qlen, g->h_qout, g->h_hdr, g->h_key, g->h_off, g->h_nodes, g->h_arcs, g->h_ctr,
@@ -445,7 +457,13 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
 }
 
 // Enqueue one engine launch for nq queries whose padded keyword rows / lengths are in g->d_kw / d_qlen.
-kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaStream_t s, int qconst = 0) {
+struct TdOnly {   // top-down-only launch over the state of a vertex-partitioned search
+    int levels, stop;
+    uint32_t n_central;
+};
+
+kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaStream_t s, int qconst = 0,
+                  const TdOnly *td = nullptr) {
     G = std::max(1, std::min({G, nq, g->grid}));
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
@@ -473,6 +491,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
     a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
     a.level_cover = p.level_cover ? 1 : 0;
+    if (td) { a.td_only = 1; a.td_levels = td->levels; a.td_stop = td->stop; a.td_ncentral = td->n_central; }
     // the parity view wants every central's key.  The path bound needs the Thm. V.4 DAG to be made of
     // arcs the search traversed: exact extraction, or no central blocking.
     a.prune = p.want_levels ? 0 : p.prune;
@@ -737,6 +756,132 @@ kgs_status kgs_query_batch_fetch(kgs_graph *g, void *cuda_stream, kgs_result **r
         g->last_q.assign(ql.begin(), ql.end());
     }
     return fetch(g, (cudaStream_t)cuda_stream, results);
+}
+
+// ------------------------------------------------------------------------------------------ vertex partition
+int64_t kgs_vp_slice(int64_t n_nodes, int32_t world) {
+    if (n_nodes < 0 || world < 1) return 0;
+    const int64_t s = (n_nodes + world - 1) / world;
+    return (s + 15) / 16 * 16;
+}
+
+kgs_status kgs_vp_begin(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, const kgs_params *pp, int32_t rank,
+                        int32_t world, const kgs_vp_buffers *b, void *cuda_stream, int32_t *info) {
+    if (!g || !kw_ids || !b || !info) return fail(KGS_EINVAL, "null argument");
+    if (world < 1 || rank < 0 || rank >= world) return fail(KGS_EINVAL, "rank / world out of range");
+    if (!b->hm || !b->hm_slice || !b->M || !b->counts || !b->cent || !b->cdep || !b->cent_n)
+        return fail(KGS_EINVAL, "null exchange buffer");
+    kgs_params p;
+    if (pp) p = *pp; else kgs_params_default(&p);
+    kgs_status st = check_params(p, k);
+    if (st != KGS_OK) return st;
+    st = check_query(g, kw_ids, q);
+    if (st != KGS_OK) return st;
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    st = prepare(g, p, 1, s);   // activation levels at alpha, one workspace for the top-down
+    if (st != KGS_OK) return st;
+    const int64_t slice = kgs_vp_slice(g->n, world), n_pad = slice * world;
+    if (!g->vp_gate) CUDA_TRY(dmalloc(&g->vp_gate, std::max<int64_t>(g->n, 1)));
+    CUDA_TRY(grow_dev(&g->vp_X, &g->vp_X_cap, (size_t)n_pad));
+    const int64_t lo = std::min<int64_t>((int64_t)rank * slice, g->n), hi = std::min<int64_t>(lo + slice, g->n);
+    if (lo != g->vp_big_lo || hi != g->vp_big_hi) {   // owned nodes pulled by a whole CTA
+        if (!g->vp_big) {
+            CUDA_TRY(dmalloc(&g->vp_big, std::max<int64_t>(g->n_big_in, 1)));
+            CUDA_TRY(dmalloc(&g->vp_nbig_dev, 1));
+        }
+        DevGraph dg{};
+        dg.in_ptr = g->in_ptr;
+        CUDA_TRY(launch_vp_biglist(dg, lo, hi, g->vp_big, g->vp_nbig_dev, s));
+        int32_t nb = 0;
+        CUDA_TRY(cudaMemcpyAsync(&nb, g->vp_nbig_dev, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+        g->vp_nbig = nb;
+        g->vp_big_lo = lo; g->vp_big_hi = hi;
+    }
+    VpQuery qd{};
+    qd.q = q;
+    qd.full = (1u << q) - 1u;
+    for (int i = 0; i < q; ++i) qd.kw[i] = kw_ids[i];
+    VpBufs vb{};
+    vb.hm = b->hm; vb.hm_slice = b->hm_slice; vb.M = b->M;
+    vb.counts = reinterpret_cast<unsigned long long *>(b->counts);
+    vb.cent = b->cent; vb.cdep = b->cdep; vb.cent_n = b->cent_n;
+    vb.n_pad = n_pad; vb.lo = lo; vb.hi = hi;
+    // an empty T_i: nothing can be central (reading R17)
+    std::vector<int64_t> kp(2 * q);
+    for (int i = 0; i < q; ++i)
+        CUDA_TRY(cudaMemcpyAsync(&kp[2 * i], g->kw_ptr + kw_ids[i], 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    bool empty = false;
+    for (int i = 0; i < q; ++i) empty |= kp[2 * i + 1] == kp[2 * i];
+    DevGraph dg{};
+    dg.n = g->n; dg.kw_ptr = g->kw_ptr; dg.kw_nodes = g->kw_nodes;
+    CUDA_TRY(launch_vp_begin(dg, qd, g->act, vb, g->vp_gate, s));
+    g->vp = vb; g->vq = qd; g->vp_p = p; g->vp_k = k; g->vp_active = true;
+    info[0] = g->amax;
+    info[1] = empty ? 1 : 0;
+    return KGS_OK;
+}
+
+kgs_status kgs_vp_level(kgs_graph *g, int32_t level, void *cuda_stream) {
+    if (!g) return fail(KGS_EINVAL, "null argument");
+    if (!g->vp_active) return fail(KGS_EINVAL, "kgs_vp_begin was not called");
+    if (level < 0 || level >= 254) return fail(KGS_EINVAL, "level out of range");
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    DevGraph dg{};
+    dg.n = g->n; dg.in_ptr = g->in_ptr; dg.in_idx = g->in_idx;
+    CUDA_TRY(launch_vp_level(dg, g->vq, g->act, g->vp, g->vp_gate, g->vp_X, g->vp_big, g->vp_nbig, level,
+                             g->vp_p.block_central ? 1 : 0, s));
+    return KGS_OK;
+}
+
+kgs_status kgs_vp_waiting(kgs_graph *g, int32_t level, void *cuda_stream) {
+    if (!g) return fail(KGS_EINVAL, "null argument");
+    if (!g->vp_active) return fail(KGS_EINVAL, "kgs_vp_begin was not called");
+    if (level < 0 || level >= 254) return fail(KGS_EINVAL, "level out of range");
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    DevGraph dg{};
+    dg.n = g->n; dg.row_ptr = g->row_ptr; dg.col_idx = g->col_idx;
+    CUDA_TRY(launch_vp_waiting(dg, g->vq, g->act, g->vp, g->vp_gate, level, g->vp_p.block_central ? 1 : 0, s));
+    return KGS_OK;
+}
+
+kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centrals_dev, const uint8_t *depth_dev,
+                          int32_t levels, int32_t stop_reason, void *cuda_stream, kgs_result **out) {
+    if (!g || !out) return fail(KGS_EINVAL, "null argument");
+    *out = nullptr;
+    if (!g->vp_active) return fail(KGS_EINVAL, "kgs_vp_begin was not called");
+    if (n_central < 0 || n_central > g->n || (n_central > 0 && (!centrals_dev || !depth_dev)))
+        return fail(KGS_EINVAL, "central list");
+    std::lock_guard<std::mutex> lk(g->mu);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    CUDA_TRY(cudaSetDevice(g->device));
+    kgs_params p = g->vp_p;
+    if (p.prune == 2) p.prune = 1;   // the lightest-path rows are written by the single-GPU search only
+    kgs_status st = prepare(g, p, 1, s);
+    if (st != KGS_OK) return st;
+    const DevWork &w = g->works[0];
+    // the replicated final state in the engine's layout (DevWork::st, M, centrals)
+    CUDA_TRY(launch_vp_pack_st(g->vp.hm, g->vp_gate, g->n, w.st, s));
+    CUDA_TRY(cudaMemcpyAsync(w.M, g->vp.M, (size_t)g->n * 8, cudaMemcpyDeviceToDevice, s));
+    if (n_central) {
+        CUDA_TRY(cudaMemcpyAsync(w.centrals, centrals_dev, sizeof(int32_t) * n_central, cudaMemcpyDeviceToDevice, s));
+        CUDA_TRY(cudaMemcpyAsync(w.cdepth, depth_dev, (size_t)n_central, cudaMemcpyDeviceToDevice, s));
+    }
+    const int32_t qp[2] = {0, g->vq.q};
+    st = stage_host(g, 1, qp, g->vq.kw, s);
+    if (st != KGS_OK) return st;
+    const TdOnly td{levels, stop_reason, (uint32_t)n_central};
+    st = launch(g, 1, g->vp_k, p, 1, s, 0, &td);
+    if (st != KGS_OK) return st;
+    g->vp_active = false;
+    return fetch(g, s, out);
 }
 
 int32_t kgs_result_count(const kgs_result *r) { return r ? (int32_t)r->ans.size() : 0; }

@@ -572,6 +572,47 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
 }
 
 // ------------------------------------------------------------------------------------------ search
+// The previous query's lightest-path rows (prune mode 2), through its touched list (always complete).
+__device__ void reset_mw_prev(const Ctx &c) {
+    const DevWork &w = c.w;
+    const uint32_t done = __ldcg(w.gstate + 1);
+    if (done == 0 || !w.ctl[(done + 1) & 1]->mw_dirty) return;
+    const Ctl *pv = w.ctl[(done + 1) & 1];
+    const int64_t pt = (int64_t)pv->n_touched;
+    const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u);
+    for (int64_t j = c.G.gtid; j < 2 * pt; j += c.G.gsz) {
+        const int32_t v = w.touched[j >> 1];
+        reinterpret_cast<uint4 *>(w.mw + (int64_t)v * 8)[j & 1] = ones;
+    }
+}
+
+// Top-down only (the state of a vertex-partitioned search, vpart.cu): clear what the previous query
+// left in the predecessor pre-pass state, then take |C|, the stop level and reason from the host.
+__device__ void td_only_prepare(const Ctx &c, QOut *qo) {
+    const DevWork &w = c.w;
+    const int64_t gtid = c.G.gtid, gsz = c.G.gsz, n = c.a.g.n;
+    reset_mw_prev(c);
+    const uint32_t valid = __ldcg(w.gstate + 2), done = __ldcg(w.gstate + 1);
+    if (!valid || done == 0) {
+        for (int64_t j = gtid; j < 2 * c.a.W; j += gsz) w.pd_bits[j] = 0u;
+        for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
+    } else {
+        const Ctl *pv = w.ctl[(done + 1) & 1];
+        for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
+            const int32_t v = w.pd_touched[j];
+            w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[j] = 0;
+        }
+    }
+    if (gtid == 0) {
+        c.ctl->n_central = c.a.td_ncentral;
+        c.ctl->levels = c.a.td_levels;
+        c.ctl->stop_reason = c.a.td_stop;
+        qo->t_search_end = globaltimer_ns();
+    }
+    c.G.sync();
+    stamp(c.G, qo, TS_END);
+}
+
 __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -587,15 +628,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     // ---- reset the state the previous query of this group left behind
     const uint32_t valid = __ldcg(w.gstate + 2), lastR = __ldcg(w.gstate + 3);
     const uint32_t done = __ldcg(w.gstate + 1);
-    if (done > 0 && w.ctl[(done + 1) & 1]->mw_dirty) {   // the previous query's lightest-path rows
-        const Ctl *pv = w.ctl[(done + 1) & 1];
-        const int64_t pt = (int64_t)pv->n_touched;       // its touched list is complete
-        const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u);
-        for (int64_t j = gtid; j < 2 * pt; j += gsz) {
-            const int32_t v = w.touched[j >> 1];
-            reinterpret_cast<uint4 *>(w.mw + (int64_t)v * 8)[j & 1] = ones;
-        }
-    }
+    reset_mw_prev(c);
     if (!valid || (int)lastR != R || done == 0) {
         const int64_t n8 = n / 8;
         for (int64_t j = gtid; j < n8; j += gsz) {
@@ -1553,7 +1586,8 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         G.sync();
         stamp(G, qo, TS_START);
         const Ctx c{a, w, ctl, G, qq};
-        search(c, s_big, sh, qo);
+        if (a.td_only) td_only_prepare(c, qo);
+        else search(c, s_big, sh, qo);
         topdown(c, s_big, sh, dsmem, qo);
         if (G.gtid == 0) {
             qo->levels = ctl->levels;
@@ -1572,7 +1606,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->td_arcs = ctl->td_arcs;
             qo->t_end = globaltimer_ns();
             w.gstate[1] = done + 1;
-            w.gstate[2] = 1u;
+            w.gstate[2] = a.td_only ? 0u : 1u;   // after a top-down-only query the next one resets densely
             w.gstate[3] = (uint32_t)a.R;
         }
         G.sync();

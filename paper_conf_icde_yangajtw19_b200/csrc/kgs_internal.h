@@ -156,6 +156,9 @@ struct EngineArgs {
     // parameters (shared by the batch)
     int k, max_depth, block_central, extract_mode, level_cover;
     int tile_light;             // light frontiers up to this many nodes are expanded by group-wide tiles
+    int td_only;                // 1: skip the search, the state comes from the vertex-partitioned search (vpart.cu)
+    int td_levels, td_stop;     //    its stop level / reason
+    uint32_t td_ncentral;       //    and |C| (works[0].centrals / cdepth hold the list)
     int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
     // outputs
@@ -174,6 +177,24 @@ struct EngineArgs {
     size_t cta_arena_bytes;
 };
 
+// ---- vertex-partitioned search of one query (vpart.cu) ----
+constexpr int64_t kVpBig = 4096;   // owned nodes with more in-arcs are pulled by a whole CTA
+struct VpQuery {
+    int q;
+    uint32_t full;
+    int32_t kw[kMaxQ];
+};
+struct VpBufs {                    // exchange buffers (caller-owned device memory, see kgs_vp_buffers)
+    uint8_t *hm;                   // [n_pad] replicated hit masks (all-gather output)
+    uint8_t *hm_slice;             // [slice] this rank's hit masks after the level (all-gather input)
+    uint8_t *M;                    // [n_pad * 8] node-major hitting levels; rows [lo, hi) are this rank's
+    unsigned long long *counts;    // [3] marks, new centrals, waiting work-list nodes (all-reduce sum)
+    int32_t *cent;                 // [slice] this rank's central nodes
+    uint8_t *cdep;                 // [slice] their depths
+    int32_t *cent_n;               // [1] their count
+    int64_t n_pad, lo, hi;
+};
+
 // ---- launchers (return cudaError_t) ----
 cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha, uint8_t *act, uint32_t *amax,
                               cudaStream_t s);
@@ -185,5 +206,14 @@ int engine_max_grid(int device);
 size_t engine_dyn_smem();
 size_t arena_bytes_host(int hcap, int ncap, int acap, int team, bool with_sort);
 cudaError_t launch_engine(const EngineArgs &a, int grid, cudaStream_t s);
+cudaError_t launch_vp_begin(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b, uint8_t *gate,
+                            cudaStream_t s);
+cudaError_t launch_vp_biglist(const DevGraph &g, int64_t lo, int64_t hi, int32_t *big, int32_t *nbig, cudaStream_t s);
+cudaError_t launch_vp_level(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
+                            const uint8_t *gate, uint8_t *X, const int32_t *big, int nbig, int l, int block_central,
+                            cudaStream_t s);
+cudaError_t launch_vp_waiting(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
+                              const uint8_t *gate, int l, int block_central, cudaStream_t s);
+cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, int64_t n, uint16_t *st, cudaStream_t s);
 
 }  // namespace kgs
