@@ -38,6 +38,7 @@ sys.path.insert(0, ROOT)
 METRIC = "p50 query latency (ms) & queries/s, Wikidata-scale graph; GTEPS"
 BATCH = 350          # queries per step (the C3 latency set)
 GROUPS = 8           # engine groups in batch mode (queries answered at the same time)
+RELABEL = os.environ.get("KGS_RELABEL", "1") != "0"   # ablation: 0 keeps the input node order internally
 
 
 def _env_int(k, d):
@@ -178,7 +179,7 @@ def load_replicated(name, rank, world, dev, kgs):
     gen_s = time.time() - t0
     t1 = time.time()
     G = kgs.kgs_load_graph_device(n, m, t[0].data_ptr(), t[1].data_ptr(), t[2].data_ptr(), V, t[3].data_ptr(),
-                                  t[4].data_ptr(), float(A.item()), True, dev)
+                                  t[4].data_ptr(), float(A.item()), True, dev, relabel=RELABEL)
     torch.cuda.synchronize(dev)
     load_s = time.time() - t1
     del t
@@ -255,7 +256,7 @@ def main():
         w, gen_s = build_workload(name)
         g = w.graph
         t0 = time.time()
-        G = kgs.kgs_load_graph(g, device=dev)
+        G = kgs.kgs_load_graph(g, device=dev, relabel=RELABEL)
         load_s = time.time() - t0
     else:
         w, g, G, gen_s, load_s = load_replicated(name, rank, world, dev, kgs)
@@ -376,7 +377,7 @@ def main():
         "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {g.n} nodes, {g.n_arcs} arcs",
                    "k": w.k, "queries_per_step": B * world, "engine_groups": args.groups, "alpha": 0.1,
                    "lambda": 0.2, "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
-                   "load_s": round(load_s, 1),
+                   "load_s": round(load_s, 1), "node_order": "degree (internal relabel)" if RELABEL else "input",
                    "parallelism": f"query-sharded x{world}" if world > 1 else "single GPU"},
         "p50_ms": statistics.median(lat) if lat else None,
         "p95_ms": float(np.percentile(lat, 95)) if lat else None,

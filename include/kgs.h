@@ -45,6 +45,8 @@ typedef enum {
 #define KGS_INF_LEVEL 255  /* "infinity" in the uint8 node-keyword matrix M */
 
 #define KGS_INPUT_DEVICE_PTRS 1  /* kgs_graph_desc arrays are device pointers (copied, not borrowed) */
+#define KGS_NO_RELABEL 2         /* keep the input node order internally (default: renumbered by degree for
+                                    L2 locality; every id at the ABI is the input id either way) */
 
 #define KGS_EXTRACT_EXACT 0    /* Thm. V.4 + "predecessor not yet central" (reading R12, default) */
 #define KGS_EXTRACT_LITERAL 1  /* Thm. V.4 exactly as printed */
@@ -68,7 +70,9 @@ typedef enum {
  *   symmetric   1: in-arcs == out-arcs (bi-directed KG).  0: the library builds the reverse CSR used
  *               by extraction (reading R1).
  *   device      CUDA device ordinal the graph lives on.
- *   flags       KGS_INPUT_DEVICE_PTRS or 0. */
+ *   flags       KGS_INPUT_DEVICE_PTRS | KGS_NO_RELABEL, or 0.  The library stores the graph with its
+ *               nodes renumbered by non-increasing degree (ties by input id) unless KGS_NO_RELABEL is
+ *               set; results are identical (every id returned is the input id, ties rank by input id). */
 typedef struct {
     int64_t n_nodes, n_arcs;
     const int64_t *row_ptr;

@@ -21,6 +21,7 @@ LIB_PATH = os.environ.get("KGS_LIB", os.path.join(_HERE, "libkgs.so"))   # KGS_L
 KGS_OK, KGS_EINVAL, KGS_ENOMEM, KGS_ECUDA, KGS_ENCCL, KGS_EINTERNAL = 0, -1, -2, -3, -4, -5
 KGS_MAX_Q, KGS_MAX_K = 8, 4096
 KGS_INPUT_DEVICE_PTRS = 1
+KGS_NO_RELABEL = 2
 KGS_EXTRACT_EXACT, KGS_EXTRACT_LITERAL = 0, 1
 KGS_STOP_K, KGS_STOP_EXHAUSTED, KGS_STOP_MAX_DEPTH, KGS_STOP_EMPTY_KEYWORD = 0, 1, 2, 3
 
@@ -182,9 +183,10 @@ class Graph:
             pass
 
 
-def kgs_load_graph(g, device: int = 0) -> Graph:
+def kgs_load_graph(g, device: int = 0, relabel: bool = True) -> Graph:
     """Load a graph given as host numpy arrays (attributes row_ptr, col_idx, weight, kw_ptr, kw_nodes,
-    A, symmetric — e.g. a synth.Graph)."""
+    A, symmetric — e.g. a synth.Graph).  relabel=False sets KGS_NO_RELABEL (keep the input node order
+    internally; results are identical either way)."""
     rp = np.ascontiguousarray(g.row_ptr, np.int64)
     ci = np.ascontiguousarray(g.col_idx, np.int32)
     w = np.ascontiguousarray(g.weight, np.float32)
@@ -192,19 +194,20 @@ def kgs_load_graph(g, device: int = 0) -> Graph:
     kn = np.ascontiguousarray(g.kw_nodes, np.int32)
     d = kgs_graph_desc(rp.shape[0] - 1, ci.shape[0], rp.ctypes.data, ci.ctypes.data, w.ctypes.data,
                        kp.shape[0] - 1, kp.ctypes.data, kn.ctypes.data if kn.size else None, float(g.A),
-                       1 if getattr(g, "symmetric", True) else 0, int(device), 0)
+                       1 if getattr(g, "symmetric", True) else 0, int(device), 0 if relabel else KGS_NO_RELABEL)
     h = ctypes.c_void_p()
     _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
     return Graph(h, rp.shape[0] - 1, kp.shape[0] - 1)
 
 
 def kgs_load_graph_device(n, n_arcs, row_ptr_ptr, col_idx_ptr, weight_ptr, n_keywords, kw_ptr_ptr, kw_nodes_ptr,
-                          A: float, symmetric: bool = True, device: int = 0) -> Graph:
+                          A: float, symmetric: bool = True, device: int = 0, relabel: bool = True) -> Graph:
     """Load a graph whose arrays already live in device memory (KGS_INPUT_DEVICE_PTRS): raw device
     pointers (e.g. torch CUDA tensors' data_ptr()), int64 row_ptr / kw_ptr, int32 col_idx / kw_nodes,
     float32 weight.  The library copies them; the caller keeps ownership."""
     d = kgs_graph_desc(int(n), int(n_arcs), row_ptr_ptr, col_idx_ptr, weight_ptr, int(n_keywords), kw_ptr_ptr,
-                       kw_nodes_ptr, float(A), 1 if symmetric else 0, int(device), KGS_INPUT_DEVICE_PTRS)
+                       kw_nodes_ptr, float(A), 1 if symmetric else 0, int(device),
+                       KGS_INPUT_DEVICE_PTRS | (0 if relabel else KGS_NO_RELABEL))
     h = ctypes.c_void_p()
     _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
     return Graph(h, int(n), int(n_keywords))

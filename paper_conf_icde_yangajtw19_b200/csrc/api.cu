@@ -73,6 +73,7 @@ struct kgs_graph {
     int32_t *col_idx = nullptr, *in_idx = nullptr, *kw_nodes = nullptr;
     float *weight = nullptr;
     uint8_t *cls = nullptr, *cls_in = nullptr;
+    int32_t *orig = nullptr, *perm = nullptr;   // internal <-> input ids (relabel.cu); null: identity
     int64_t n_big = 0, n_big_in = 0;   // nodes with more than kBigDeg out- / in-arcs
     // per-alpha / per-lambda caches
     uint8_t *act = nullptr;
@@ -158,7 +159,7 @@ struct kgs_result {
 namespace {
 
 void free_work(DevWork &w) {
-    void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.centrals, w.cdepth, w.ckey, w.overflow,
+    void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
                  w.gstate};
@@ -177,6 +178,7 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.qlight, n));
     CUDA_TRY(dmalloc(&w.qbig, g->n_big));
     CUDA_TRY(dmalloc(&w.touched, n));
+    CUDA_TRY(dmalloc(&w.qdef, n));
     CUDA_TRY(dmalloc(&w.centrals, n));
     CUDA_TRY(dmalloc(&w.cdepth, n));
     CUDA_TRY(dmalloc(&w.ckey, n));
@@ -239,7 +241,7 @@ void kgs_free_graph(kgs_graph *g) {
     void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->act, g->amax_dev, g->dpow,
                     g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
                     g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr, g->vp_gate, g->vp_X, g->vp_big,
-                    g->vp_nbig_dev};
+                    g->vp_nbig_dev, g->orig, g->perm};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
     void *hp[] = {g->h_kw, g->h_qlen, g->h_qout, g->h_hdr, g->h_key, g->h_off, g->h_nodes, g->h_arcs, g->h_ctr,
@@ -325,6 +327,8 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         return bail(fail(KGS_EINVAL, "invalid graph:" + why));
     }
     G_TRY(launch_snap_weights(g->weight, n, 0));
+    if (!(d->flags & KGS_NO_RELABEL))   // internal order: non-increasing degree (relabel.cu)
+        G_TRY(relabel_by_degree(n, m, P, &g->row_ptr, &g->col_idx, &g->weight, g->kw_nodes, &g->orig, &g->perm, 0));
     G_TRY(launch_degree_class(g->row_ptr, n, g->cls, 0));
     for (int64_t v = 0; v < n; ++v)
         if (rp[v + 1] - rp[v] > kBigDeg) ++g->n_big;
@@ -332,9 +336,9 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     if (g->symmetric) {
         g->in_ptr = g->row_ptr; g->in_idx = g->col_idx; g->cls_in = g->cls; g->n_big_in = g->n_big;
     } else {
-        std::vector<int32_t> ci(m);
-        if (on_dev) G_TRY(cudaMemcpy(ci.data(), d->col_idx, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
-        else std::memcpy(ci.data(), d->col_idx, sizeof(int32_t) * m);
+        std::vector<int32_t> ci(m);   // the stored (possibly renumbered) CSR
+        if (m) G_TRY(cudaMemcpy(ci.data(), g->col_idx, sizeof(int32_t) * m, cudaMemcpyDeviceToHost));
+        G_TRY(cudaMemcpy(rp.data(), g->row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost));
         std::vector<int64_t> ip(n + 1, 0);
         for (int64_t j = 0; j < m; ++j) ip[ci[j] + 1]++;
         for (int64_t v = 0; v < n; ++v) ip[v + 1] += ip[v];
@@ -485,6 +489,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx; a.g.in_ptr = g->in_ptr;
     a.g.in_idx = g->in_idx; a.g.weight = g->weight; a.g.cls = g->cls; a.g.cls_in = g->cls_in; a.g.n_kw = g->n_kw;
     a.g.kw_ptr = g->kw_ptr; a.g.kw_nodes = g->kw_nodes;
+    a.g.orig = g->orig;
     a.act = g->act; a.R = g->R; a.W = g->W; a.dpow = g->dpow;
     a.works = g->works_dev; a.bars = g->bars; a.G = G;
     a.nq = nq; a.kw = g->d_kw; a.qlen = g->d_qlen; a.qconst = qconst;
@@ -605,18 +610,22 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         const int64_t n = g->n, q = r->q;
         const DevWork &w = g->works[0];
         uint8_t *dM = nullptr;
-        CUDA_TRY(dmalloc(&dM, n * q));
-        CUDA_TRY(launch_levels_out(w.st, w.M, n, (int)q, dM, s));
+        const uint32_t nc = g->h_qout[0].n_central;
+        CUDA_TRY(dmalloc(&dM, std::max<int64_t>(n * q, (int64_t)nc * 4) + n));
+        uint8_t *dA = dM + std::max<int64_t>(n * q, (int64_t)nc * 4);
+        CUDA_TRY(launch_levels_out(w.st, w.M, g->perm, n, (int)q, dM, s));   // rows in input order
+        CUDA_TRY(launch_gather_u8(g->act, g->perm, n, dA, s));
         r->M.resize(n * q);
         r->act.resize(n);
         CUDA_TRY(cudaMemcpyAsync(r->M.data(), dM, n * q, cudaMemcpyDeviceToHost, s));
-        CUDA_TRY(cudaMemcpyAsync(r->act.data(), g->act, n, cudaMemcpyDeviceToHost, s));
-        const uint32_t nc = g->h_qout[0].n_central;
+        CUDA_TRY(cudaMemcpyAsync(r->act.data(), dA, n, cudaMemcpyDeviceToHost, s));
         std::vector<int32_t> ids(nc);
         std::vector<uint8_t> dep(nc);
         std::vector<double> key(nc);
         if (nc) {
-            CUDA_TRY(cudaMemcpyAsync(ids.data(), w.centrals, sizeof(int32_t) * nc, cudaMemcpyDeviceToHost, s));
+            int32_t *dI = reinterpret_cast<int32_t *>(dM);   // M was copied out above (stream order)
+            CUDA_TRY(launch_to_input_ids(w.centrals, g->orig, nc, dI, s));
+            CUDA_TRY(cudaMemcpyAsync(ids.data(), dI, sizeof(int32_t) * nc, cudaMemcpyDeviceToHost, s));
             CUDA_TRY(cudaMemcpyAsync(dep.data(), w.cdepth, nc, cudaMemcpyDeviceToHost, s));
             CUDA_TRY(cudaMemcpyAsync(key.data(), w.ckey, sizeof(double) * nc, cudaMemcpyDeviceToHost, s));
         }

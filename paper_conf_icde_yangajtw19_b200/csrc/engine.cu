@@ -157,6 +157,9 @@ struct Ctx {        // everything a group needs while answering one query
     const Q &qq;
 };
 
+// the input id of internal node v (every id leaving the engine, and the ranking tie-break, is an input id)
+__device__ __forceinline__ int32_t in_id(const EngineArgs &a, int32_t v) { return a.g.orig ? __ldg(a.g.orig + v) : v; }
+
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
 __device__ __forceinline__ void push(const Ctx &c, int32_t v, int L) {
     const int s = L % c.a.R;
@@ -168,11 +171,39 @@ constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16
 // Enqueue frontiers: compact a bitmap (which is cleared) into the light / big queues.
 // on_node(v) runs once per set bit and returns whether v goes to the aux list; on_aux(v, pos) runs when
 // v is written there.  (A) extracts the node ids of a tile of words with stores only; (B) processes the
-// tile's nodes one per thread.  Appends cost one atomic per CTA per tile.
+// tile's nodes one per thread.  Appends cost one atomic per CTA per tile.  A tile holding more than
+// kLocalNodes set bits (dense regions: the hubs of the degree order, relabel.cu) processes that many
+// locally and defers the rest to qdef (their queue positions); after the group barrier that follows,
+// compact_deferred spreads the deferred nodes over every thread of the group.
+constexpr int kLocalNodes = kBlock;
+
+template <class OnNode, class OnAux>
+__device__ __forceinline__ void compact_node(int32_t *ql, int64_t pos, const uint8_t *cls, int32_t *qb, uint32_t *nb,
+                                             int32_t *aux, uint32_t *naux, OnNode &on_node, OnAux &on_aux) {
+    const int32_t v = ql[pos];
+    const bool flag = on_node(v);
+    if (cls[v] != CLS_LIGHT) { qb[atomicAdd(nb, 1u)] = v; ql[pos] = -1; }
+    if (flag) {
+        const uint32_t p = agg_slot(naux, 0x5u);
+        aux[p] = v;
+        on_aux(v, p);
+    }
+}
+
+// The deferred nodes of compact(), strided over the group.  Call after a group barrier; returns whether
+// there were any (then the caller needs another barrier before reading the queues).
+template <class OnNode, class OnAux>
+__device__ __forceinline__ bool compact_deferred(const Grp &G, const int32_t *qdef, uint32_t nd, int32_t *ql,
+                                                 const uint8_t *cls, int32_t *qb, uint32_t *nb, int32_t *aux,
+                                                 uint32_t *naux, OnNode on_node, OnAux on_aux) {
+    for (int64_t j = G.gtid; j < nd; j += G.gsz) compact_node(ql, __ldcg(qdef + j), cls, qb, nb, aux, naux, on_node, on_aux);
+    return nd != 0;
+}
+
 template <class OnNode, class OnAux>
 __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W, const uint8_t *cls, int32_t *ql,
                                         uint32_t *nl, int32_t *qb, uint32_t *nb, int32_t *aux, uint32_t *naux,
-                                        long long *sh, OnNode on_node, OnAux on_aux) {
+                                        int32_t *qdef, uint32_t *ndef, long long *sh, OnNode on_node, OnAux on_aux) {
     const int64_t step = (int64_t)blockDim.x * kWpt;
     const int64_t cw = ((W + G.gcount - 1) / G.gcount + kWpt - 1) / kWpt * kWpt;
     const int64_t w0 = (int64_t)G.grank * cw, w1 = w0 + cw < W ? w0 + cw : W;
@@ -207,6 +238,14 @@ __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W,
             for (uint32_t m = word[k]; m; m &= m - 1) ql[p++] = (int32_t)((wi + k) * 32 + __ffs(m) - 1);
         __syncthreads();
         for (long long c0 = 0; c0 < tot; c0 += blockDim.x) {
+            if (c0 >= kLocalNodes) {   // dense tile: the rest goes to the group-wide pass
+                if (threadIdx.x == 0) sh[36] = (long long)atomicAdd(ndef, (uint32_t)(tot - c0));
+                __syncthreads();
+                const long long d0 = sh[36];
+                for (long long j = c0 + threadIdx.x; j < tot; j += blockDim.x) qdef[d0 + j - c0] = (int32_t)(seg0 + j);
+                __syncthreads();
+                break;
+            }
             const long long j = c0 + threadIdx.x;
             int32_t v = -1;
             int flag = 0;
@@ -368,6 +407,9 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 // Light frontier nodes: warp w of the group takes batches w, w + #warps, ... of B nodes each (no shared
 // counter); the batch's arcs are balanced over the 32 lanes by a warp scan and a shuffle binary search.
 // B = 32 when the frontier is large, fewer (down to 1) when it is small so that every warp gets work.
+// Batch bi holds the queue entries bi, bi + nbatch, bi + 2 nbatch, ...: the queue is in node-id order,
+// and in the degree order (relabel.cu) neighbouring ids have similar degrees, so strided batches mix
+// degrees and cost about the same.
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
                                              const int32_t *idx, const uint16_t *st, Prep prep, Visit visit,
@@ -378,7 +420,7 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
     const uint32_t nbatch = (c0 + B - 1) / B;
     const unsigned lane = lane_id();
     for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi += warps) {
-        const uint32_t i = bi * B + lane;
+        const uint32_t i = bi + lane * nbatch;
         NodeT nd{};
         int64_t start = 0;
         int deg = 0;
@@ -502,17 +544,21 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (!__ldcg(&ctl->pd_flag[slot])) break;
         uint32_t *qn = ctl->pd_qn[slot];
         if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; }
+        auto pd_node = [&](int32_t u) {
+            const uint32_t s = __ldcg(c.w.pd_state + u);
+            const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
+            const uint32_t bits = nx & ~dn;
+            c.w.pd_state[u] = bits | ((dn | bits) << 16);
+            return bits != 0 && __ldcg(c.w.pd_cid + u) < 0;
+        };
+        auto pd_aux = [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; };
+        if (G.gtid == 0) ctl->pd_ndef[slot ^ 1] = 0u;
         compact(G, c.w.pd_bits + (int64_t)slot * W, W, c.a.g.cls_in, c.w.pd_qlight, &qn[0], c.w.pd_qbig, &qn[1],
-                c.w.pd_touched, &ctl->n_cid, sh,
-                [&](int32_t u) {
-                    const uint32_t s = __ldcg(c.w.pd_state + u);
-                    const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
-                    const uint32_t bits = nx & ~dn;
-                    c.w.pd_state[u] = bits | ((dn | bits) << 16);
-                    return bits != 0 && __ldcg(c.w.pd_cid + u) < 0;
-                },
-                [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; });
+                c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, pd_node, pd_aux);
         G.sync();
+        if (compact_deferred(G, c.w.qdef, __ldcg(&ctl->pd_ndef[slot]), c.w.pd_qlight, c.a.g.cls_in, c.w.pd_qbig,
+                             &qn[1], c.w.pd_touched, &ctl->n_cid, pd_node, pd_aux))
+            G.sync();
         stamp(G, qo, TS_PD_MERGE);
         const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
         if (G.gtid == 0) ctl->pd_flag[slot] = 0u;
@@ -723,11 +769,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         }
         const int s = l % R;
         uint32_t *qn = ctl->qn[l & 1];
-        if (gtid == 0) { ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; }
+        if (gtid == 0) { ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; ctl->ndef[(l + 1) & 1] = 0u; }
         // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
-        compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
-                &ctl->n_touched, sh,
-                [&](int32_t v) {
+        auto merge_node = [&](int32_t v) {
                     const uint32_t b = nm8[v];
                     if (!b) return false;
                     nm8[v] = 0;
@@ -747,9 +791,14 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                         w.cdepth[ci] = (uint8_t)l;
                     }
                     return old == 0;
-                },
-                [&](int32_t, uint32_t) {});
+                };
+        auto merge_aux = [&](int32_t, uint32_t) {};
+        compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
+                &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
         G.sync();
+        if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.touched,
+                             &ctl->n_touched, merge_node, merge_aux))
+            G.sync();
         stamp(G, qo, TS_MERGE);
         __shared__ uint32_t s_ctl[3];
         if (threadIdx.x == 0) { s_ctl[0] = __ldcg(&qn[0]); s_ctl[1] = __ldcg(&qn[1]); s_ctl[2] = __ldcg(&ctl->n_central); }
@@ -1100,7 +1149,7 @@ __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
     if (r == 0) { S.scal[SC_NOUT] = 0; S.scal[SC_AOUT] = 0; }
     T.sync();
     for (int j = r; j < nn; j += ts)
-        if (S.keep[j]) S.sortbuf[atomicAdd(S.scal + SC_NOUT, 1)] = (unsigned long long)(uint32_t)S.id[j];
+        if (S.keep[j]) S.sortbuf[atomicAdd(S.scal + SC_NOUT, 1)] = (unsigned long long)(uint32_t)in_id(a, S.id[j]);
     T.sync();
     const int kn = S.scal[SC_NOUT];
     team_sort(T, S.sortbuf, kn);
@@ -1120,7 +1169,7 @@ __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
     for (int e = r; e < na; e += ts)
         if (S.keep[S.au[e]] & S.ab[e])
             S.sortbuf[atomicAdd(S.scal + SC_AOUT, 1)] =
-                ((unsigned long long)(uint32_t)S.id[S.au[e]] << 32) | (uint32_t)S.id[S.ax[e]];
+                ((unsigned long long)(uint32_t)in_id(a, S.id[S.au[e]]) << 32) | (uint32_t)in_id(a, S.id[S.ax[e]]);
     T.sync();
     const int ka = S.scal[SC_AOUT];
     team_sort(T, S.sortbuf, ka);
@@ -1161,7 +1210,7 @@ __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
 // ------------------------------------------------------------------------------------------ select
 __device__ __forceinline__ void comp_key(const Ctx &c, uint32_t i, uint64_t &hi, uint32_t &lo) {
     hi = (uint64_t)__double_as_longlong(__ldcg(c.w.ckey + i));
-    lo = (uint32_t)__ldcg(c.w.centrals + i);
+    lo = (uint32_t)in_id(c.a, __ldcg(c.w.centrals + i));   // ties rank by input id
 }
 __device__ __forceinline__ uint32_t digit_of(uint64_t hi, uint32_t lo, int d) {
     return d < 8 ? (uint32_t)((hi >> (56 - 8 * d)) & 0xFF) : (lo >> (24 - 8 * (d - 8))) & 0xFF;
@@ -1297,7 +1346,7 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem, uint32_t k
 // keyword it does not contain itself (those have m = 0 and no predecessors).
 __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
     const Grp &G = c.G;
-    if (G.gtid == 0) { c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; }   // round 0 of this call
+    if (G.gtid == 0) { c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; }   // round 0 of this call
     for (int64_t j = G.gtid; j < cnt; j += G.gsz) {
         const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;
         const int32_t cn = __ldcg(c.w.centrals + idx);
@@ -1397,7 +1446,7 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
             const int32_t idx = __ldcg(c.w.sel + rk);
             const int64_t ans = (int64_t)c.qq.qi * a.k + rk;
             if (T.rank() == 0) {
-                a.out_hdr[4 * ans + 0] = __ldcg(c.w.centrals + idx);
+                a.out_hdr[4 * ans + 0] = in_id(a, __ldcg(c.w.centrals + idx));
                 a.out_hdr[4 * ans + 1] = __ldcg(c.w.cdepth + idx);
                 a.out_key[ans] = __ldcg(c.w.ckey + idx);
             }

@@ -55,6 +55,8 @@ struct Ctl {
     uint32_t n_elist2;             // second pruning round: candidates whose bound still beats the threshold
     uint32_t mw_dirty;             // this query wrote lightest-path rows (prune mode 2): the next one resets them
     unsigned long long dag_arcs;   // arcs the search traversed that hit their target (the Thm. V.4 arcs)
+    uint32_t ndef[2];              // [level parity] compaction: nodes deferred to the group-wide pass
+    uint32_t pd_ndef[2];           // [round parity] the same for the predecessor pre-pass
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -90,6 +92,7 @@ struct DevGraph {
     int64_t n_kw;
     const int64_t *kw_ptr;
     const int32_t *kw_nodes;
+    const int32_t *orig;      // [n] internal id -> input id (relabel.cu); nullptr: ids are the input ids
 };
 
 // Per-group query workspace (all sized for n at load time).  One group answers one query at a time.
@@ -101,6 +104,7 @@ struct DevWork {
     int32_t *qlight;    // [n] compacted frontier of the current level (big nodes replaced by -1)
     int32_t *qbig;      // [n_big] compacted frontier, big nodes
     int32_t *touched;   // [n] nodes whose hm became non-zero (sparse reset of the next query)
+    int32_t *qdef;      // [n] compaction: queue positions deferred to the group-wide pass (dense tiles)
     int32_t *centrals;  // [n] central ids in identification order
     uint8_t *cdepth;    // [n] depth per central
     double *ckey;       // [n] Eq. 6 key per central
@@ -201,7 +205,12 @@ cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha,
 cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s);
 cudaError_t launch_snap_weights(float *w, int64_t n, cudaStream_t s);
 cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s);
-cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, int64_t n, int q, uint8_t *out, cudaStream_t s);
+cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
+                              uint8_t *out, cudaStream_t s);
+cudaError_t launch_gather_u8(const uint8_t *src, const int32_t *perm, int64_t n, uint8_t *out, cudaStream_t s);
+cudaError_t launch_to_input_ids(const int32_t *ids, const int32_t *orig, int64_t cnt, int32_t *out, cudaStream_t s);
+cudaError_t relabel_by_degree(int64_t n, int64_t m, int64_t P, int64_t **row_ptr, int32_t **col_idx, float **weight,
+                              int32_t *kw_nodes, int32_t **orig_out, int32_t **perm_out, cudaStream_t s);
 int engine_max_grid(int device);
 size_t engine_dyn_smem();
 size_t arena_bytes_host(int hcap, int ncap, int acap, int team, bool with_sort);

@@ -4,7 +4,6 @@
 //   k_degree_class light / big node classes for the engine's load balance.
 //   k_snap         weights onto the 2^-24 grid (reading R15).
 //   k_validate     CSR / index / weight checks of kgs_load_graph.
-//   k_levels_out   the n x q hitting-level matrix for the parity view (want_levels).
 #include "kgs_internal.h"
 
 namespace kgs {
@@ -101,19 +100,6 @@ __global__ void k_validate(DevGraph g, int32_t *err) {
 }
 cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s) {
     k_validate<<<148 * 8, 256, 0, s>>>(g, err);
-    return cudaGetLastError();
-}
-
-// M for the parity view: n*q bytes, 255 where the hit bit is clear
-__global__ void k_levels_out(const uint16_t *st, const uint8_t *M, int64_t n, int q, uint8_t *out) {
-    const int64_t gt = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gs = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = gt; v < n; v += gs) {
-        const uint32_t hm = st[v] & 0xFFu;
-        for (int i = 0; i < q; ++i) out[v * q + i] = ((hm >> i) & 1u) ? M[v * 8 + i] : (uint8_t)KGS_INF_LEVEL;
-    }
-}
-cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, int64_t n, int q, uint8_t *out, cudaStream_t s) {
-    k_levels_out<<<148 * 8, 256, 0, s>>>(st, M, n, q, out);
     return cudaGetLastError();
 }
 

@@ -82,7 +82,7 @@ def test_random_small_graphs_all_modes():
         q = int(rng.integers(1, 9))
         g = R.random_graph(rng, n, float(rng.uniform(0.03, 0.3)), directed, q, kw_size=(1, 5),
                            wmax=float(rng.choice([0.0, 0.2, 1.0])))
-        G = kgs.kgs_load_graph(g)
+        G = kgs.kgs_load_graph(g, relabel=bool(case % 2))   # internal degree order or input order
         kw = list(range(q))
         for _ in range(3):
             compare(G, g, kw, int(rng.choice([1, 2, 5, 40])), alpha=float(rng.choice([0.05, 0.1, 0.4])),
@@ -93,12 +93,15 @@ def test_random_small_graphs_all_modes():
 
 
 def test_c1_all_queries():
-    """Config C1 (BASELINE.json configs[0]): 100 three-keyword queries, top-5."""
+    """Config C1 (BASELINE.json configs[0]): 100 three-keyword queries, top-5, with the internal degree
+    order (default) and with the input order (KGS_NO_RELABEL)."""
     _gpu()
     w = synth.make_workload("C1")
-    G = kgs.kgs_load_graph(w.graph)
-    for kw in w.queries:
-        compare(G, w.graph, kw, w.k)
+    for relabel in (True, False):
+        G = kgs.kgs_load_graph(w.graph, relabel=relabel)
+        for kw in w.queries:
+            compare(G, w.graph, kw, w.k)
+        G.close()
 
 
 def test_c2_queries_and_state_reuse():

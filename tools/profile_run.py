@@ -14,11 +14,12 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C3")
 ap.add_argument("--warm", type=int, default=3)
 ap.add_argument("--queries", type=int, default=5)
+ap.add_argument("--relabel", type=int, default=1)
 args = ap.parse_args()
 w = synth.make_workload(args.config)
 order = np.random.default_rng(12345).permutation(len(w.queries))
 qs = [w.queries[i] for i in order]
-G = kgs.kgs_load_graph(w.graph)
+G = kgs.kgs_load_graph(w.graph, relabel=bool(args.relabel))
 for i in range(args.warm + args.queries):
     r = kgs.kgs_query(G, qs[i % len(qs)], w.k)
     print(i, len(qs[i % len(qs)]), r.stats, flush=True)
