@@ -515,6 +515,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.out_used = g->d_ctr + 1;
     a.warp_arenas = g->warp_arenas; a.warp_arena_bytes = g->warp_arena_bytes;
     a.cta_arenas = g->cta_arenas; a.cta_arena_bytes = g->cta_arena_bytes;
+    CUDA_TRY(cudaMemsetAsync(g->bars, 0, sizeof(GroupBar) * (size_t)G, s));   // monotonic group barriers
     CUDA_TRY(cudaEventRecord(g->ev[0], s));
     CUDA_TRY(launch_engine(a, g->grid, s));
     CUDA_TRY(cudaEventRecord(g->ev[1], s));
