@@ -326,7 +326,7 @@ def main():
         dev_ms = float(t.item())
     total_queries = args.steps * B * world
     value = total_queries / (dev_ms / 1e3)
-    arcs = sum(s["arcs_scanned"] + s["td_arcs"] for s in stats)
+    arcs = sum(s["arcs_scanned"] for s in stats)   # GTEPS: arcs the search expanded
     alg = sum(algorithmic_bytes(s) for s in stats)
 
     # ---- single-query latency mode: the whole GPU on one query, one launch per query

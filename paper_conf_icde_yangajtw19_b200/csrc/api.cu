@@ -427,9 +427,10 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
     }
     if ((int)g->works.size() < G) {
         CUDA_TRY(cudaStreamSynchronize(s));
-        // predecessor-arc capacity per group: 64 M for the single-query group, 16 M for the others
+        // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs): 64 M for the
+        // single-query group, 32 M for the others (20 B per arc)
         while ((int)g->works.size() < G) {
-            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, g->works.empty() ? (64ll << 20) : (16ll << 20)), 1 << 20);
+            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, g->works.empty() ? (64ll << 20) : (32ll << 20)), 1 << 20);
             DevWork w;
             kgs_status st = alloc_work(g, w, pcap);
             if (st != KGS_OK) { free_work(w); return st; }
@@ -504,6 +505,15 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     {
         const char *e = std::getenv("KGS_PRUNE_MIN");
         a.prune_min = e ? std::max(1, std::atoi(e)) : 512;
+    }
+    {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
+        // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass
+        // Default: on for the single-query (latency) launch, where the pre-pass's rounds of group barriers
+        // dominate; off for query groups, where the pre-pass's targeted work (closures of the top
+        // candidates only) is less total work than building every touched node's list.
+        const char *e = std::getenv("KGS_DAG_RECORD");   // ablation knob: 0 off, 1 on, unset auto
+        const bool on = e ? std::atoi(e) != 0 : G == 1;
+        a.dag_record = on && !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     }
     {
         const char *e = std::getenv("KGS_TILE_LIGHT");   // ablation knob (nodes); default 8 tiles

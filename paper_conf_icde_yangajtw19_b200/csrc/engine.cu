@@ -86,6 +86,16 @@ __device__ __forceinline__ uint32_t agg_slot(uint32_t *counter, unsigned key) {
     return base + rank;
 }
 
+// Append to one list from every active lane: one atomic per warp (ballot + popc).
+__device__ __forceinline__ uint32_t warp_slot(uint32_t *counter) {
+    const unsigned mask = __activemask();
+    const int leader = __ffs(mask) - 1;
+    uint32_t base = 0;
+    if ((int)lane_id() == leader) base = atomicAdd(counter, (uint32_t)__popc(mask));
+    base = __shfl_sync(mask, base, leader);
+    return base + __popc(mask & lanemask_lt());
+}
+
 __device__ __forceinline__ long long block_excl_scan64(long long x, long long *total, long long *sh) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
     long long incl = x;
@@ -146,6 +156,9 @@ __device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t 
     const unsigned peers = __match_any_sync(__activemask(), (unsigned long long)flag);
     if ((int)lane_id() == __ffs(peers) - 1 && !__ldcg(flag)) *flag = 1u;
 }
+
+// append regions of the recorded DAG used by a group: one per CTA, at most kRecStripes
+__device__ __forceinline__ int rec_stripes(const Grp &G) { return G.gcount < kRecStripes ? G.gcount : kRecStripes; }
 
 struct Ctx {        // everything a group needs while answering one query
     const EngineArgs &a;
@@ -276,13 +289,27 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
-__device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, int32_t x, uint32_t sx,
-                                          unsigned &hits, unsigned &dag) {
+__device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, uint32_t zbv, int32_t x,
+                                          uint32_t sx, unsigned &hits, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = sx >> 8;
     if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
         ++dag;                                            // a Thm. V.4 arc (v -> x for these keywords)
+        if (c.a.dag_record) {   // recorded predecessor arc
+            // one of kRecStripes append regions per CTA: a single counter would serialise millions of
+            // atomics per heavy query on one address
+            const int ns = rec_stripes(c.G);
+            const int stripe = c.G.grank % ns;
+            const uint32_t ai = warp_slot(&c.ctl->rec_cnt[stripe * kRecStride]);
+            const int64_t rcap = c.w.pcap / ns;
+            if ((int64_t)ai < rcap) {
+                const int64_t r = stripe * rcap + ai;
+                c.w.pa_u[r] = v;
+                c.w.pa_x[r] = x;
+                c.w.pa_b[r] = (uint16_t)(bits | (zbv << 8));
+            }
+        }
         if (c.a.prune == 2) {   // x is hit at l+1 for these keywords: v is a Thm. V.4 predecessor of (x, i)
             for (uint32_t b = bits; b; b &= b - 1) {
                 const int i = __ffs(b) - 1;
@@ -332,6 +359,7 @@ constexpr int kLightUnroll = KGS_LIGHT_UNROLL;
 struct FwdNode {
     int32_t v;
     uint32_t hm;
+    uint32_t zb;     // keywords for which v is a source (m = 0), recorded with its arcs
 };
 
 struct PdNode {
@@ -528,6 +556,38 @@ __device__ __forceinline__ bool pd_prepare(const Ctx &c, int32_t x, PdNode &nd) 
     return nd.P != 0;
 }
 
+// every recorded arc index (the kRecStripes append regions of visit_arc), strided over the group
+// (the region sizes are staged in shared memory once; a flat index finds its region by binary search)
+template <class F>
+__device__ __forceinline__ void for_each_record(const Ctx &c, F fn) {
+    const int ns = rec_stripes(c.G);
+    const int64_t rcap = c.w.pcap / ns;
+    __shared__ uint32_t s_pre[kRecStripes + 1];
+    static_assert(kRecStripes <= kBlock, "one thread per region");
+    __syncthreads();
+    if (threadIdx.x < kRecStripes) {
+        int64_t k = threadIdx.x < ns ? (int64_t)__ldcg(&c.ctl->rec_cnt[threadIdx.x * kRecStride]) : 0;
+        s_pre[threadIdx.x + 1] = (uint32_t)(k < rcap ? k : rcap);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        s_pre[0] = 0;
+        for (int r = 0; r < kRecStripes; ++r) s_pre[r + 1] += s_pre[r];
+    }
+    __syncthreads();
+    const int64_t T = s_pre[kRecStripes];
+    for (int64_t j = c.G.gtid; j < T; j += c.G.gsz) {
+        int lo = 0, hi = kRecStripes - 1;   // region r with s_pre[r] <= j < s_pre[r + 1]
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if ((int64_t)s_pre[mid] <= j) lo = mid; else hi = mid - 1;
+        }
+        fn(lo * rcap + (j - (int64_t)s_pre[lo]));
+    }
+}
+
+__device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo);
+
 __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
@@ -574,7 +634,14 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     }
     if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
     if (G.gtid == 0) ctl->pd_rounds = r;
-    // CSR of the predecessor lists: exclusive scan of pcnt over compact ids, then scatter
+    build_pred_csr(c, sh, qo);
+}
+
+// CSR of the predecessor lists: exclusive scan of pcnt over compact ids, then scatter of the arcs
+// (pa_u / pa_x = compact id of the successor / pa_b / pa_slot = position in its list).
+__device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
+    const Grp &G = c.G;
+    Ctl *ctl = c.ctl;
     const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
     const int64_t chunk = (ncid + G.gcount - 1) / G.gcount;
     const int64_t lo = (int64_t)G.grank * chunk, hi = lo + chunk < ncid ? lo + chunk : ncid;
@@ -605,11 +672,16 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const int off = __ldcg(c.w.scan_tmp + G.grank);
     for (int64_t j = lo + threadIdx.x; j < hi; j += blockDim.x) c.w.pred_ptr[j] += off;
     G.sync();
-    const int64_t np = (int64_t)__ldcg(&ctl->n_parcs) < c.w.pcap ? (int64_t)__ldcg(&ctl->n_parcs) : c.w.pcap;
-    for (int64_t ai = G.gtid; ai < np; ai += G.gsz) {
+    auto scatter = [&](int64_t ai) {
         const int64_t pos = (int64_t)__ldcg(c.w.pred_ptr + c.w.pa_x[ai]) + c.w.pa_slot[ai];
         c.w.pred_u[pos] = c.w.pa_u[ai];
         c.w.pred_b[pos] = c.w.pa_b[ai];
+    };
+    if (ctl->rec_used) {
+        for_each_record(c, scatter);
+    } else {
+        const int64_t np = (int64_t)__ldcg(&ctl->n_parcs) < c.w.pcap ? (int64_t)__ldcg(&ctl->n_parcs) : c.w.pcap;
+        for (int64_t ai = G.gtid; ai < np; ai += G.gsz) scatter(ai);
     }
     G.sync();
     stamp(G, qo, TS_PD_CSR);
@@ -691,11 +763,16 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
     } else {
         const Ctl *pv = w.ctl[(done + 1) & 1];   // the previous query's block
-        for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
-            const int32_t v = w.pd_touched[j];
-            w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[j] = 0;
-        }
+        // a recorded DAG gave compact ids to exactly the touched nodes (pd_state unused): one loop below
+        const bool prev_rec = pv->rec_used != 0;
+        if (!prev_rec)
+            for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
+                const int32_t v = w.pd_touched[j];
+                w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[j] = 0;
+            }
         const int64_t pt = (int64_t)pv->n_touched;
+        if (prev_rec && pt > n / 16)
+            for (int64_t j = gtid; j < pt; j += gsz) { w.pd_cid[w.touched[j]] = -1; w.pcnt[j] = 0; }
         if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
             const int64_t n8 = n / 8;
             for (int64_t j = gtid; j < n8; j += gsz) {
@@ -712,6 +789,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             for (int64_t j = gtid; j < pt; j += gsz) {
                 const int32_t v = w.touched[j];
                 w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+                if (prev_rec) { w.pd_cid[v] = -1; w.pcnt[j] = 0; }
             }
         }
         for (int s = 0; s < R; ++s)   // level slots still pending when the previous query stopped
@@ -790,7 +868,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                     }
                     return old == 0;
                 };
-        auto merge_aux = [&](int32_t, uint32_t) {};
+        auto merge_aux = [&](int32_t v, uint32_t pos) {   // recorded DAG: compact id = touched position
+            if (a.dag_record) { w.pd_touched[pos] = v; w.pd_cid[v] = (int32_t)pos; }
+        };
         compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
                 &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
         G.sync();
@@ -822,9 +902,19 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
             nd.v = v;
             nd.hm = prepare(c, l, v, leader);
+            nd.zb = 0;
+            if (a.dag_record && nd.hm) {
+                const uint64_t row = ldrow(w.M, v);
+                for (uint32_t b = nd.hm; b; b &= b - 1) {
+                    const int i = __ffs(b) - 1;
+                    if (((row >> (8 * i)) & 0xFF) == 0) nd.zb |= 1u << i;
+                }
+            }
             return nd.hm != 0;
         };
-        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) { visit_arc(c, l, nd.v, nd.hm, x, sx, my_hits, my_dag); };
+        auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) {
+            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_hits, my_dag);
+        };
         expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
             expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
@@ -853,6 +943,48 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     G.sync();
     stamp(G, qo, TS_END);
     if (gtid == 0) qo->t_search_end = globaltimer_ns();
+}
+
+// ------------------------------------------------------------------------------------------ recorded DAG
+// The search recorded every arc v -> x that hit x (Alg. 2 ln 16-21) with its keyword bits: exactly the
+// Thm. V.4 predecessor arcs of the exact reading R12 (a blocked central never expands, and every node
+// that can expand keyword i into x at level m_xi - 1 is scanned at that level).  Turn them
+// into the predecessor CSR keyed by the compact ids the merge gave the touched nodes.  Returns false
+// (and leaves the pre-pass state clean) when the record buffer overflowed.
+__device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
+    const Grp &G = c.G;
+    Ctl *ctl = c.ctl;
+    const DevWork &w = c.w;
+    const uint32_t nt = __ldcg(&ctl->n_touched);
+    __shared__ unsigned long long s_rec[2];
+    if (threadIdx.x == 0) {
+        unsigned long long tot = 0, over = 0;
+        const int ns = rec_stripes(G);
+        for (int r = 0; r < ns; ++r) {
+            const int64_t k = (int64_t)__ldcg(&ctl->rec_cnt[r * kRecStride]);
+            tot += (unsigned long long)k;
+            over |= k > w.pcap / ns;
+        }
+        s_rec[0] = tot; s_rec[1] = over;
+    }
+    __syncthreads();
+    if (s_rec[1]) {   // a region overflowed: forget the compact ids, use the pre-pass
+        for (int64_t j = G.gtid; j < nt; j += G.gsz) w.pd_cid[__ldcg(w.pd_touched + j)] = -1;
+        G.sync();
+        if (G.gtid == 0) { ctl->n_parcs = 0; ctl->n_cid = 0; ctl->rec_overflow = 1; }
+        G.sync();
+        return false;
+    }
+    for_each_record(c, [&](int64_t r) {
+        const int32_t cid = __ldcg(w.pd_cid + __ldcg(w.pa_x + r));
+        w.pa_x[r] = cid;
+        w.pa_slot[r] = atomicAdd(w.pcnt + cid, 1);
+    });
+    if (G.gtid == 0) { ctl->n_cid = nt; ctl->rec_used = 1; ctl->n_parcs = (uint32_t)s_rec[0]; }
+    G.sync();
+    stamp(G, qo, TS_PD_MERGE);
+    build_pred_csr(c, sh, qo);
+    return true;
 }
 
 // ------------------------------------------------------------------------------------------ top-down
@@ -1498,10 +1630,14 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
     const uint32_t nc = __ldcg(&ctl->n_central);
     const uint32_t kk = (uint32_t)a.k < nc ? (uint32_t)a.k : nc;
     const uint32_t mcap = min((uint32_t)KGS_MAX_K, max(8u * kk, (uint32_t)a.prune_min));
+    // predecessor lists: from the arcs the search recorded, else by the in-arc pre-pass (pred_dag)
+    const bool rec = a.dag_record && recorded_dag(c, sh, qo);
     if (!a.prune || nc <= mcap) {
-        seed_pd(c, nullptr, nc);
-        stamp(G, qo, TS_PD_SEED);
-        pred_dag(c, S, sh, qo);
+        if (!rec) {
+            seed_pd(c, nullptr, nc);
+            stamp(G, qo, TS_PD_SEED);
+            pred_dag(c, S, sh, qo);
+        }
         extract_list(c, sh, dsmem, nullptr, nc, qo);
         if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }   // emit counters (read after the select)
         select_topk(c, sh, dsmem, kk);
@@ -1526,9 +1662,11 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
         comp_key(c, (uint32_t)__ldcg(c.w.sel + m - 1), bhi, blo);
         for (int64_t j = G.gtid; j < m; j += G.gsz) c.w.elist[j] = __ldcg(c.w.sel + j);
         G.sync();
-        seed_pd(c, c.w.elist, m);
-        stamp(G, qo, TS_PD_SEED);
-        pred_dag(c, S, sh, qo);
+        if (!rec) {
+            seed_pd(c, c.w.elist, m);
+            stamp(G, qo, TS_PD_SEED);
+            pred_dag(c, S, sh, qo);
+        }
         extract_list(c, sh, dsmem, c.w.elist, m, qo);
         rank_list(c, dsmem, c.w.elist, m, kk);                 // T = the kk-th exact (key, id)
         uint64_t thi; uint32_t tlo;
@@ -1544,8 +1682,10 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             }
             G.sync();
             n2 = __ldcg(&ctl->n_elist2);
-            seed_pd(c, c.w.elist + m, n2);
-            pred_dag(c, S, sh, qo);
+            if (!rec) {
+                seed_pd(c, c.w.elist + m, n2);
+                pred_dag(c, S, sh, qo);
+            }
             extract_list(c, sh, dsmem, c.w.elist + m, n2, qo);
         }
         if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }

@@ -26,6 +26,10 @@ constexpr int kBigNodes = 1 << 16;
 constexpr int kBigArcs = 1 << 18;
 constexpr int kBigHash = 1 << 17;
 
+// Append regions of the recorded DAG (engine.cu visit_arc): one counter per region, 32 bytes apart.
+constexpr int kRecStripes = 128;
+constexpr int kRecStride = 8;
+
 // Query control block (one per query in flight, zeroed at the start of every query).
 struct Ctl {
     uint32_t slot_flag[256];       // level slot s has pending frontier bits
@@ -57,6 +61,9 @@ struct Ctl {
     unsigned long long dag_arcs;   // arcs the search traversed that hit their target (the Thm. V.4 arcs)
     uint32_t ndef[2];              // [level parity] compaction: nodes deferred to the group-wide pass
     uint32_t pd_ndef[2];           // [round parity] the same for the predecessor pre-pass
+    uint32_t rec_overflow;         // the recorded DAG overflowed pcap: the pre-pass was used
+    uint32_t rec_used;             // the predecessor lists came from the recorded DAG (compact ids = touched)
+    uint32_t rec_cnt[kRecStripes * kRecStride];   // recorded arcs per append region (stride 32 B)
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -165,6 +172,7 @@ struct EngineArgs {
     uint32_t td_ncentral;       //    and |C| (works[0].centrals / cdepth hold the list)
     int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
+    int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
     // outputs
     QOut *qout;                 // [nq]
     int32_t *out_hdr;           // [nq][k][4]: central, depth, n_nodes, n_arcs

@@ -19,7 +19,7 @@ order = np.random.default_rng(12345).permutation(len(w.queries))
 qs = [w.queries[i] for i in order]
 if batch:
     qs = (qs * ((batch + len(qs) - 1) // len(qs)))[:batch]
-G = kgs.kgs_load_graph(w.graph)
+G = kgs.kgs_load_graph(w.graph, relabel=os.environ.get("KGS_RELABEL", "1") != "0")
 kwp = torch.full((len(qs), 8), -1, dtype=torch.int32)
 for i, q in enumerate(qs):
     kwp[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
@@ -38,3 +38,10 @@ for g in groups:
         lat = sorted(r.stats["ms_total"] for r in res)
     print(f"{name} G={g:3d} batch={len(qs)} launch {ms:8.2f} ms  {len(qs) / ms * 1e3:9.1f} q/s  "
           f"query latency p50 {lat[len(lat) // 2]:.3f} ms p95 {lat[int(len(lat) * .95)]:.3f} ms", flush=True)
+    ph = {}
+    for r in res:
+        for k, v in r.stats["phases_us"].items():
+            ph[k] = ph.get(k, 0.0) + v
+    tot = sum(ph.values()) or 1.0
+    print("   group-time share: " + " ".join(f"{k}={v / tot:.1%}" for k, v in sorted(ph.items(), key=lambda x: -x[1])),
+          flush=True)
