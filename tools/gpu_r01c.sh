@@ -1,0 +1,10 @@
+#!/bin/bash
+# one gpurun call: build, GPU tests, full bench, ncu launch list of the bench command, per-query DRAM pass
+make -j8 all >/dev/null 2>&1 || { echo build failed; exit 1; }
+mkdir -p gpurun_out
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/smi.txt
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo rc=$? >> gpurun_out/pytest_gpu.log
+timeout 600 python bench.py > gpurun_out/bench_full.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:k_ --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > gpurun_out/bench_ncu.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_sector_hit_rate.pct,gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed --clock-control none -k regex:k_engine -s 3 -c 40 --csv --log-file gpurun_out/engine_dram.csv python tools/profile_run.py --warm 3 --queries 40 > gpurun_out/profile_queries.log 2>&1
+echo done

@@ -6,7 +6,7 @@ Inputs (produced on the GPU box):
                   lts__t_sector_hit_rate.pct,gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed
                   -k regex:k_engine over `profile_run.py --warm W --queries N`
   <queries.log>   the profile_run.py output of that run (per-query stats, same order)
-Usage: make_profile_summary.py tag dram.csv queries.log [skip]
+Usage: make_profile_summary.py tag dram.csv queries.log [skip queries] [skip launches]
 """
 import ast
 import collections
@@ -18,6 +18,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 tag, f_dram, f_q = sys.argv[1:4]
 skip = int(sys.argv[4]) if len(sys.argv) > 4 else 3
+lskip = int(sys.argv[5]) if len(sys.argv) > 5 else skip   # launches already skipped by ncu -s: 0
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1, "us": 1e3, "ms": 1e6, "%": 1}
 
 
@@ -32,9 +33,9 @@ def read_metrics(path):
             d = dict(zip(hdr, r))
             if "k_engine" not in d["Kernel Name"]:
                 continue
-            per.setdefault(d["ID"], {})[d["Metric Name"]] = float(d["Metric Value"].replace(",", "")) * SCALE.get(
+            per.setdefault(int(d["ID"]), {})[d["Metric Name"]] = float(d["Metric Value"].replace(",", "")) * SCALE.get(
                 d["Metric Unit"], 1)
-    return per
+    return collections.OrderedDict(sorted(per.items()))   # by launch id (numeric)
 
 
 def alg_bytes(s):   # bench.py algorithmic_bytes
@@ -50,7 +51,7 @@ for line in open(f_q):
         qs.append(ast.literal_eval(d))
     except (ValueError, SyntaxError):
         pass
-launches = list(per.values())[skip:]
+launches = list(per.values())[lskip:]
 qs = qs[skip:skip + len(launches)]
 n = min(len(launches), len(qs))
 traffic = [m["dram__bytes_read.sum"] + m["dram__bytes_write.sum"] for m in launches[:n]]
