@@ -145,16 +145,38 @@ __device__ __forceinline__ void stamp(const Grp &G, QOut *o, int tag) {
 }
 
 // ------------------------------------------------------------------------------------------ frontier
-// Set v's bit in bitmap `bits`; `flag` records that the bitmap is non-empty.  The bit is set with a
-// reduction (no return value); the flag is stored once per group of converged lanes, after a check.
-__device__ __forceinline__ void set_bit(uint32_t *bits, uint32_t *flag, int32_t v) {
+// Non-empty flags of the level-slot bitmaps (0..255) and of the pre-pass round bitmaps (kFlagPd + 0/1) are
+// kept per CTA in shared memory while a phase pushes, and published to the query's control block by
+// publish_flags() before the group barrier that ends the phase (a global check-then-store per push
+// stalled every pushing warp on an L2 round trip).
+constexpr int kFlagPd = 256;
+constexpr int kFlagSlots = kFlagPd + 2;
+__device__ __forceinline__ uint32_t *cta_flags() {
+    __shared__ uint32_t f[kFlagSlots];
+    return f;
+}
+
+// Set v's bit in bitmap `bits` and mark CTA flag `fi`.  The bit is set with a reduction (no return
+// value).  check: read the word first and skip the reduction when the bit is set (pushes that repeat:
+// Alg. 2 ln 19 re-queues v once per gated neighbour); the others are already unique per node.
+__device__ __forceinline__ void set_bit(uint32_t *bits, int fi, int32_t v, bool check) {
     uint32_t *word = bits + (v >> 5);
     const uint32_t bit = 1u << (v & 31);
-    if (__ldcg(word) & bit) return;
+    if (check && (__ldcg(word) & bit)) return;
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
-    // converged lanes may push to different bitmaps (level slots): one leader per flag address
-    const unsigned peers = __match_any_sync(__activemask(), (unsigned long long)flag);
-    if ((int)lane_id() == __ffs(peers) - 1 && !__ldcg(flag)) *flag = 1u;
+    uint32_t *f = cta_flags() + fi;
+    if (!*f) *f = 1u;
+}
+
+// All threads of the CTA: publish the CTA's flags (then the caller's group barrier makes them visible).
+__device__ __forceinline__ void publish_flags(Ctl *ctl) {
+    __syncthreads();
+    uint32_t *f = cta_flags();
+    for (int t = threadIdx.x; t < kFlagSlots; t += blockDim.x)
+        if (f[t]) {
+            f[t] = 0u;
+            if (t < kFlagPd) ctl->slot_flag[t] = 1u; else ctl->pd_flag[t - kFlagPd] = 1u;
+        }
 }
 
 // append regions of the recorded DAG used by a group: one per CTA, at most kRecStripes
@@ -172,9 +194,9 @@ struct Ctx {        // everything a group needs while answering one query
 __device__ __forceinline__ int32_t in_id(const EngineArgs &a, int32_t v) { return a.g.orig ? __ldg(a.g.orig + v) : v; }
 
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
-__device__ __forceinline__ void push(const Ctx &c, int32_t v, int L) {
+__device__ __forceinline__ void push(const Ctx &c, int32_t v, int L, bool check = false) {
     const int s = L % c.a.R;
-    set_bit(c.w.fbits + (int64_t)s * c.a.W, &c.ctl->slot_flag[s], v);
+    set_bit(c.w.fbits + (int64_t)s * c.a.W, s, v, check);
 }
 
 constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16-byte loads)
@@ -332,7 +354,7 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
             if (old == 0) push(c, x, l + 1);              // ln 22: FIdentifier[x] <- 1 (first new bit)
         }
     } else {
-        push(c, v, (int)gate - 1);                        // ln 19: v must retry when x opens
+        push(c, v, (int)gate - 1, true);                  // ln 19: v must retry when x opens
     }
 }
 
@@ -527,24 +549,29 @@ __device__ __forceinline__ uint32_t pred_test(const Ctx &c, bool exact_block, ui
 }
 
 __device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const PdNode &nd, int32_t u, uint32_t su,
-                                         uint32_t *nbits, uint32_t *nflag) {
+                                         uint32_t *nbits, int nflag) {
     uint32_t zbu = 0;
     const uint32_t pb = pred_test(c, exact_block, nd.P, nd.hx, nd.gx, u, su, zbu);
     if (!pb) return;
     const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(c.w.pcnt + nd.cidx), (unsigned)nd.cidx);
-    const uint32_t ai = agg_slot(&c.ctl->n_parcs, 0xFFFFFFFFu);
-    if ((int64_t)ai < c.w.pcap) {
-        c.w.pa_u[ai] = u;
-        c.w.pa_x[ai] = nd.cidx;
-        c.w.pa_b[ai] = (uint16_t)(pb | (zbu << 8));
-        c.w.pa_slot[ai] = (int32_t)pos;
+    // the CTA's append region (as the recorded DAG: one counter per CTA, not one per group)
+    const int ns = rec_stripes(c.G);
+    const int stripe = c.G.grank % ns;
+    const uint32_t ai = warp_slot(&c.ctl->pd_cnt[stripe * kRecStride]);
+    const int64_t rcap = c.w.pcap / ns;
+    if ((int64_t)ai < rcap) {
+        const int64_t r = stripe * rcap + ai;
+        c.w.pa_u[r] = u;
+        c.w.pa_x[r] = nd.cidx;
+        c.w.pa_b[r] = (uint16_t)(pb | (zbu << 8));
+        c.w.pa_slot[r] = (int32_t)pos;
     } else {
         atomicExch(&c.ctl->fatal, 5);
     }
     const uint32_t nb = pb & ~zbu;        // sources (m = 0) have no predecessors
     if (nb) {
         const uint32_t old = atomicOr(c.w.pd_state + u, nb << 8);
-        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u);
+        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u, false);
     }
 }
 
@@ -559,14 +586,14 @@ __device__ __forceinline__ bool pd_prepare(const Ctx &c, int32_t x, PdNode &nd) 
 // every recorded arc index (the kRecStripes append regions of visit_arc), strided over the group
 // (the region sizes are staged in shared memory once; a flat index finds its region by binary search)
 template <class F>
-__device__ __forceinline__ void for_each_record(const Ctx &c, F fn) {
+__device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cnt, F fn) {
     const int ns = rec_stripes(c.G);
     const int64_t rcap = c.w.pcap / ns;
     __shared__ uint32_t s_pre[kRecStripes + 1];
     static_assert(kRecStripes <= kBlock, "one thread per region");
     __syncthreads();
     if (threadIdx.x < kRecStripes) {
-        int64_t k = threadIdx.x < ns ? (int64_t)__ldcg(&c.ctl->rec_cnt[threadIdx.x * kRecStride]) : 0;
+        int64_t k = threadIdx.x < ns ? (int64_t)__ldcg(&cnt[threadIdx.x * kRecStride]) : 0;
         s_pre[threadIdx.x + 1] = (uint32_t)(k < rcap ? k : rcap);
     }
     __syncthreads();
@@ -621,7 +648,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
         if (G.gtid == 0) ctl->pd_flag[slot] = 0u;
         uint32_t *nbits = c.w.pd_bits + (int64_t)(slot ^ 1) * W;
-        uint32_t *nflag = &ctl->pd_flag[slot ^ 1];
+        const int nflag = kFlagPd + (slot ^ 1);
         auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
         auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) { pd_visit(c, exact_block, nd, u, su, nbits, nflag); };
         expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
@@ -629,11 +656,17 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         else
             expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
+        publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
     }
     if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
-    if (G.gtid == 0) ctl->pd_rounds = r;
+    if (G.gtid == 0) {
+        ctl->pd_rounds = r;
+        uint32_t np = 0;
+        for (int k = 0; k < rec_stripes(G); ++k) np += __ldcg(&ctl->pd_cnt[k * kRecStride]);
+        ctl->n_parcs = np;
+    }
     build_pred_csr(c, sh, qo);
 }
 
@@ -677,12 +710,7 @@ __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
         c.w.pred_u[pos] = c.w.pa_u[ai];
         c.w.pred_b[pos] = c.w.pa_b[ai];
     };
-    if (ctl->rec_used) {
-        for_each_record(c, scatter);
-    } else {
-        const int64_t np = (int64_t)__ldcg(&ctl->n_parcs) < c.w.pcap ? (int64_t)__ldcg(&ctl->n_parcs) : c.w.pcap;
-        for (int64_t ai = G.gtid; ai < np; ai += G.gsz) scatter(ai);
-    }
+    for_each_record(c, ctl->rec_used ? ctl->rec_cnt : ctl->pd_cnt, scatter);
     G.sync();
     stamp(G, qo, TS_PD_CSR);
 }
@@ -824,6 +852,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             push(c, v, 0);
         }
     }
+    publish_flags(ctl);
     G.sync();
     stamp(G, qo, TS_SCATTER);
 
@@ -920,6 +949,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         else
             expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
+        publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_EXPAND);
     }
@@ -975,7 +1005,7 @@ __device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
         G.sync();
         return false;
     }
-    for_each_record(c, [&](int64_t r) {
+    for_each_record(c, ctl->rec_cnt, [&](int64_t r) {
         const int32_t cid = __ldcg(w.pd_cid + __ldcg(w.pa_x + r));
         w.pa_x[r] = cid;
         w.pa_slot[r] = atomicAdd(w.pcnt + cid, 1);
@@ -1484,8 +1514,9 @@ __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
         uint32_t zb = 0;
         for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
         const uint32_t bits = c.qq.full & ~zb;
-        if (bits) { atomicOr(c.w.pd_state + cn, bits << 8); set_bit(c.w.pd_bits, &c.ctl->pd_flag[0], cn); }
+        if (bits) { atomicOr(c.w.pd_state + cn, bits << 8); set_bit(c.w.pd_bits, kFlagPd, cn, false); }
     }
+    publish_flags(c.ctl);
     G.sync();
 }
 
@@ -1726,6 +1757,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         G.bar = a.bars + G.g;
         G.episode = 0;
     }
+    for (int t = threadIdx.x; t < kFlagSlots; t += blockDim.x) cta_flags()[t] = 0u;   // (synced below)
     const DevWork &w = a.works[G.g];
     for (;;) {
         // the group leader takes the next query of the batch

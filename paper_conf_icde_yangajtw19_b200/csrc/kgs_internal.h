@@ -64,6 +64,7 @@ struct Ctl {
     uint32_t rec_overflow;         // the recorded DAG overflowed pcap: the pre-pass was used
     uint32_t rec_used;             // the predecessor lists came from the recorded DAG (compact ids = touched)
     uint32_t rec_cnt[kRecStripes * kRecStride];   // recorded arcs per append region (stride 32 B)
+    uint32_t pd_cnt[kRecStripes * kRecStride];    // pre-pass predecessor arcs per append region
 };
 
 // Per-query summary written by the engine (device), read back by the host.
