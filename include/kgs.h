@@ -107,11 +107,25 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *                    2  bound d^lambda * max_i (lightest Thm. V.4 path from T_i to c), computed by the
  *                       search (an atomic min per hitting arc).  Tighter, costs search time.  Needs the
  *                       Thm. V.4 DAG to consist of arcs the search traversed: with extract_mode = LITERAL
- *                       and block_central = 1 it falls back to 1. */
+ *                       and block_central = 1 it falls back to 1.
+ *   direction      expansion direction of Alg. 2 (the north star's push/pull switching):
+ *                    KGS_DIR_AUTO (0, default)  push; from the first level whose frontier has more than
+ *                                   m / pull_ratio and more than pull_min out-arcs (m = all arcs;
+ *                                   pull_ratio 14, pull_min 2^22 unless the environment variables
+ *                                   KGS_PULL_RATIO / KGS_PULL_MIN say otherwise) on, pull;
+ *                    KGS_DIR_PUSH (1)  push only: the frontier nodes scan their out-arcs (Alg. 2 as written);
+ *                    KGS_DIR_PULL (2)  pull at every level: every node x that still lacks a keyword and whose
+ *                                   gate is open scans its in-arcs for active neighbours (the level rule,
+ *                                   SURVEY.md §8(c) O3).
+ *                  M, the central set, depths and answers do not depend on it.  A pulling search is
+ *                  exhausted by the level rule (no new hit at a level l >= max a), so stats.levels of an
+ *                  exhausted search equals the oracle's level-rule form rather than the work-list form. */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
+    int32_t direction;
 } kgs_params;
+enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 
 /* One answer (a pruned Central Graph).  Pointers live until kgs_result_free. */
 typedef struct {
@@ -142,6 +156,8 @@ typedef struct {
     int32_t group;         /* engine group (set of CTAs) that answered the query */
     int32_t n_evaluated;   /* Central Graphs whose exact key was computed (|C| unless prune skipped some) */
     int64_t dag_arcs;      /* arcs the search traversed that hit their target: the Thm. V.4 arcs of all hit nodes */
+    int32_t pull_level;    /* first level expanded by pull (kgs_params.direction), -1: push throughout */
+    int32_t pad_;
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index

@@ -23,6 +23,7 @@ KGS_MAX_Q, KGS_MAX_K = 8, 4096
 KGS_INPUT_DEVICE_PTRS = 1
 KGS_NO_RELABEL = 2
 KGS_EXTRACT_EXACT, KGS_EXTRACT_LITERAL = 0, 1
+KGS_DIR_AUTO, KGS_DIR_PUSH, KGS_DIR_PULL = 0, 1, 2
 KGS_STOP_K, KGS_STOP_EXHAUSTED, KGS_STOP_MAX_DEPTH, KGS_STOP_EMPTY_KEYWORD = 0, 1, 2, 3
 
 
@@ -43,7 +44,8 @@ class kgs_graph_desc(ctypes.Structure):
 class kgs_params(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("lambda_", ctypes.c_double), ("max_depth", ctypes.c_int32),
                 ("block_central", ctypes.c_int32), ("extract_mode", ctypes.c_int32),
-                ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("prune", ctypes.c_int32)]
+                ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("prune", ctypes.c_int32),
+                ("direction", ctypes.c_int32)]
 
 
 class kgs_answer(ctypes.Structure):
@@ -59,7 +61,8 @@ class kgs_stats(ctypes.Structure):
                 ("overflow", ctypes.c_int64), ("hits", ctypes.c_int64), ("td_arcs", ctypes.c_int64),
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
-                ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64)]
+                ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64), ("pull_level", ctypes.c_int32),
+                ("pad_", ctypes.c_int32)]
 
 
 class kgs_vp_buffers(ctypes.Structure):
@@ -155,11 +158,12 @@ def kgs_params_default() -> kgs_params:
 
 
 def make_params(alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=KGS_EXTRACT_EXACT,
-                level_cover=1, want_levels=0, prune=1) -> kgs_params:
+                level_cover=1, want_levels=0, prune=1, direction=0) -> kgs_params:
     p = kgs_params_default()
     p.alpha, p.lambda_, p.max_depth = float(alpha), float(lam), int(max_depth)
     p.block_central, p.extract_mode = int(block_central), int(extract_mode)
     p.level_cover, p.want_levels, p.prune = int(level_cover), int(want_levels), int(prune)
+    p.direction = int(direction)
     return p
 
 
@@ -248,7 +252,7 @@ def _read_result(h, n, q, want_levels) -> Result:
             answers.append(Answer(a.central, a.depth, a.score, a.score_key, nodes, arcs))
         st = kgs_stats()
         _check(L.kgs_result_stats(h, ctypes.byref(st)))
-        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
+        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_ if f != "pad_"}
         tags = np.zeros(64, np.int32)
         tns = np.zeros(64, np.uint64)
         nph = ctypes.c_int32()

@@ -231,6 +231,7 @@ void kgs_params_default(kgs_params *p) {
     p->level_cover = 1;
     p->want_levels = 0;
     p->prune = 1;
+    p->direction = KGS_DIR_AUTO;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -389,6 +390,7 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.extract_mode != KGS_EXTRACT_EXACT && p.extract_mode != KGS_EXTRACT_LITERAL)
         return fail(KGS_EINVAL, "extract_mode");
     if (p.prune < 0 || p.prune > 2) return fail(KGS_EINVAL, "prune must be 0, 1 or 2");
+    if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     return KGS_OK;
 }
 
@@ -515,6 +517,13 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
         const bool on = e ? std::atoi(e) != 0 : G == 1;
         a.dag_record = on && !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     }
+    a.direction = p.direction;
+    {
+        const char *e = std::getenv("KGS_PULL_RATIO");   // auto direction: pull once frontier arcs > m / ratio
+        a.pull_ratio = e ? std::max(1, std::atoi(e)) : 14;
+        const char *f = std::getenv("KGS_PULL_MIN");     // ... and exceed this many (small graphs never pull)
+        a.pull_min = f ? std::atoll(f) : (1ll << 22);
+    }
     {
         const char *e = std::getenv("KGS_TILE_LIGHT");   // ablation knob (nodes); default 8 tiles
         a.tile_light = e ? std::atoi(e) : 8 * kBlock;
@@ -603,6 +612,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.td_pred_arcs = o.n_parcs;
         st.n_evaluated = (int32_t)o.n_eval;
         st.group = o.group;
+        st.pull_level = o.pull_level;
         if (o.stop_reason != KGS_STOP_INVALID_QUERY && o.t_end >= o.t_start) {
             st.ms_search = (float)((double)(o.t_search_end - o.t_start) * 1e-6);
             st.ms_topdown = (float)((double)(o.t_end - o.t_search_end) * 1e-6);

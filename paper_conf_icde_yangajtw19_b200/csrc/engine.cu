@@ -144,6 +144,18 @@ __device__ __forceinline__ void stamp(const Grp &G, QOut *o, int tag) {
     }
 }
 
+// Every thread of the CTA passes its x; one global atomic per CTA adds the sum to *dst.
+__device__ __forceinline__ void cta_add(unsigned long long x, unsigned long long *dst) {
+    __shared__ unsigned long long s_acc;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) x += __shfl_down_sync(0xffffffffu, x, o);
+    if (threadIdx.x == 0) s_acc = 0ull;
+    __syncthreads();
+    if ((threadIdx.x & 31) == 0 && x) atomicAdd(&s_acc, x);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_acc) atomicAdd(dst, s_acc);
+}
+
 // ------------------------------------------------------------------------------------------ frontier
 // Non-empty flags of the level-slot bitmaps (0..255) and of the pre-pass round bitmaps (kFlagPd + 0/1) are
 // kept per CTA in shared memory while a phase pushes, and published to the query's control block by
@@ -215,7 +227,7 @@ __device__ __forceinline__ void compact_node(int32_t *ql, int64_t pos, const uin
                                              int32_t *aux, uint32_t *naux, OnNode &on_node, OnAux &on_aux) {
     const int32_t v = ql[pos];
     const bool flag = on_node(v);
-    if (cls[v] != CLS_LIGHT) { qb[atomicAdd(nb, 1u)] = v; ql[pos] = -1; }
+    if (cls_big(cls[v])) { qb[atomicAdd(nb, 1u)] = v; ql[pos] = -1; }
     if (flag) {
         const uint32_t p = agg_slot(naux, 0x5u);
         aux[p] = v;
@@ -285,7 +297,7 @@ __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W,
             if (j < tot) {
                 v = ql[seg0 + j];
                 flag = on_node(v) ? 1 : 0;
-                if (cls[v] != CLS_LIGHT) { qb[atomicAdd(nb, 1u)] = v; ql[seg0 + j] = -1; }
+                if (cls_big(cls[v])) { qb[atomicAdd(nb, 1u)] = v; ql[seg0 + j] = -1; }
             }
             long long atot;
             const long long aex = block_excl_scan64(flag, &atot, sh);
@@ -384,6 +396,11 @@ struct FwdNode {
     uint32_t zb;     // keywords for which v is a source (m = 0), recorded with its arcs
 };
 
+struct PullNode {   // a node x pulling at level l: its status word (hit mask | gate << 8)
+    int32_t x;
+    uint32_t sx;
+};
+
 struct PdNode {
     uint32_t P;      // keyword bits to expand backwards
     uint64_t hx;     // M row of the node
@@ -457,7 +474,7 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 // B = 32 when the frontier is large, fewer (down to 1) when it is small so that every warp gets work.
 // Batch bi holds the queue entries bi, bi + nbatch, bi + 2 nbatch, ...: the queue is in node-id order,
 // and in the degree order (relabel.cu) neighbouring ids have similar degrees, so strided batches mix
-// degrees and cost about the same.
+// degrees and cost about the same.  ql = nullptr sweeps the nodes 0..c0-1 in contiguous batches (pull).
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
                                              const int32_t *idx, const uint16_t *st, Prep prep, Visit visit,
@@ -468,12 +485,12 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
     const uint32_t nbatch = (c0 + B - 1) / B;
     const unsigned lane = lane_id();
     for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi += warps) {
-        const uint32_t i = bi + lane * nbatch;
+        const uint32_t i = ql ? bi + lane * nbatch : bi * B + lane;   // no queue: nodes 0..c0-1, contiguous
         NodeT nd{};
         int64_t start = 0;
         int deg = 0;
         if (lane < B && i < c0) {
-            const int32_t v = __ldcg(ql + i);   // -1: a big node, expanded by expand_big
+            const int32_t v = ql ? __ldcg(ql + i) : (int32_t)i;   // -1: a big node, expanded by expand_big
             if (v >= 0 && prep(v, true, nd)) { start = ptr[v]; deg = (int)(ptr[v + 1] - start); }
         }
         int incl = deg;
@@ -757,6 +774,52 @@ __device__ void td_only_prepare(const Ctx &c, QOut *qo) {
     stamp(c.G, qo, TS_END);
 }
 
+// One pulled level l (kgs_params.direction; called by search()): light candidates by a contiguous sweep of
+// all nodes, the ones with more than kBigDeg in-arcs afterwards in group-wide tiles.  (Inlined: out of line, the
+// call spilled the push path's level-loop state, p50 0.35 -> 0.43 ms; tools/ab_perf.py.)
+__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh, unsigned &my_hits,
+                                         unsigned &my_dag, unsigned long long &my_arcs) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    const DevWork &w = c.w;
+    Ctl *ctl = c.ctl;
+    const int64_t n = a.g.n;
+    const uint32_t full = c.qq.full;
+    auto pprep = [&](int32_t x, bool, PullNode &nd) {
+        const uint32_t sx = __ldcg(w.st + x);
+        nd.x = x;
+        nd.sx = sx;
+        return (full & ~sx & 0xFFu) != 0u && (sx >> 8) <= (uint32_t)(l + 1);
+    };
+    auto plight = [&](int32_t x, bool leader, PullNode &nd) {
+        if (!pprep(x, leader, nd)) return false;
+        if (cls_big(a.g.cls_in[x])) {   // many in-arcs: tiles over the group, after the sweep
+            w.pd_qbig[warp_slot(&ctl->pull_nbig[l & 1])] = x;   // (sized for the big-in nodes; idle now)
+            return false;
+        }
+        return true;
+    };
+    auto pvisit = [&](const PullNode &nd, int32_t u, uint32_t su) {
+        const uint32_t hmu = su & 0xFFu;
+        if (!(hmu & ~nd.sx & 0xFFu)) return;                 // u has none of the keywords x lacks
+        if (a.block_central && hmu == full) return;           // ln 2-3
+        if ((int)__ldg(a.act + u) > l) return;               // ln 4-7
+        uint32_t zb = 0;
+        if (a.dag_record) {
+            const uint64_t row = ldrow(w.M, u);
+            for (uint32_t b = hmu; b; b &= b - 1) {
+                const int i = __ffs(b) - 1;
+                if (((row >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
+            }
+        }
+        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_hits, my_dag);
+    };
+    expand_light<PullNode>(G, nullptr, (uint32_t)n, a.g.in_ptr, a.g.in_idx, w.st, plight, pvisit, my_arcs);
+    G.sync();
+    expand_big<PullNode>(G, w.pd_qbig, __ldcg(&ctl->pull_nbig[l & 1]), a.g.in_ptr, a.g.in_idx, w.st, S, sh,
+                         pprep, pvisit, my_arcs);
+}
+
 __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -858,10 +921,17 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
 
     unsigned long long my_arcs = 0;
     unsigned my_hits = 0, my_dag = 0;
+    // push / pull (kgs_params.direction): once a level pulls, every later level pulls too; a pulling
+    // search ends by the level rule (no new hit at l >= amax) instead of the empty work-list
+    bool pulling = false;
+    const bool count_mf = a.direction == KGS_DIR_AUTO;
+    unsigned long long my_mf = 0;
     for (int l = 0;; ++l) {
         // ---- enqueue frontiers: anything pending at this or a later level?
         __shared__ int s_pend;
-        if (threadIdx.x == 0) {
+        if (pulling) {
+            if (threadIdx.x == 0) s_pend = 1;
+        } else if (threadIdx.x == 0) {
             bool pend = false;
             const int top = l > amax ? l : amax;
             for (int L = l; L <= top; ++L) pend |= __ldcg(&ctl->slot_flag[L % R]) != 0u;
@@ -874,9 +944,16 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         }
         const int s = l % R;
         uint32_t *qn = ctl->qn[l & 1];
-        if (gtid == 0) { ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; ctl->ndef[(l + 1) & 1] = 0u; }
+        if (gtid == 0) {
+            ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; ctl->ndef[(l + 1) & 1] = 0u;
+            ctl->mf[(l + 1) & 1] = 0ull; ctl->pull_nbig[(l + 1) & 1] = 0u;
+        }
         // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
         auto merge_node = [&](int32_t v) {
+                    // auto direction: out-arcs of the frontier nodes that can expand (a_v <= l, ln 4-7),
+                    // bounded by the power of two of the class byte (no row_ptr load)
+                    if (count_mf && !pulling && (int)a.act[v] <= l)
+                        my_mf += cls_deg_bound(a.g.cls[v]);
                     const uint32_t b = nm8[v];
                     if (!b) return false;
                     nm8[v] = 0;
@@ -902,10 +979,14 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         };
         compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
                 &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
+        if (count_mf && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
         G.sync();
         if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.touched,
-                             &ctl->n_touched, merge_node, merge_aux))
+                             &ctl->n_touched, merge_node, merge_aux)) {
+            if (count_mf && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
             G.sync();
+        }
+        if (gtid == 0) ctl->pull_marks[(l + 1) & 1] = 0ull;   // its last reader passed the barrier above
         stamp(G, qo, TS_MERGE);
         __shared__ uint32_t s_ctl[3];
         if (threadIdx.x == 0) { s_ctl[0] = __ldcg(&qn[0]); s_ctl[1] = __ldcg(&qn[1]); s_ctl[2] = __ldcg(&ctl->n_central); }
@@ -928,6 +1009,30 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         // ---- expansion (Alg. 2)
         // slot s is consumed; nothing pushes to level l + R during this level (pushes reach <= max(l+1, amax))
         if (gtid == 0) ctl->slot_flag[s] = 0u;
+        if (!pulling && (a.direction == KGS_DIR_PULL ||
+                         (count_mf && __ldcg(&ctl->mf[l & 1]) * (unsigned long long)a.pull_ratio > (unsigned long long)a.g.m &&
+                          __ldcg(&ctl->mf[l & 1]) > (unsigned long long)a.pull_min))) {
+            pulling = true;
+            if (gtid == 0) ctl->pull_at = l + 1;
+        }
+        if (pulling) {
+            // Pull (the level rule): every x that lacks a keyword and whose gate is open
+            // (x in K or a_x <= l+1, ln 16-17) scans its in-arcs u -> x; an active u (a_u <= l, not a
+            // blocked central, ln 2-7) hits x for the keywords it has and x lacks (ln 12-22).  The same
+            // visit_arc as the push, so the hits, the recorded Thm. V.4 arcs and the lightest-path rows
+            // are the same; no node is re-queued (ln 19): a pulling search has no work list.
+            const unsigned hits0 = my_hits;
+            pull_expand(c, l, S, sh, my_hits, my_dag, my_arcs);
+            cta_add((unsigned long long)(my_hits - hits0), &ctl->pull_marks[l & 1]);
+            publish_flags(ctl);
+            G.sync();
+            stamp(G, qo, TS_EXPAND);
+            if (__ldcg(&ctl->pull_marks[l & 1]) == 0ull && l >= amax) {   // level rule: nothing can change
+                if (gtid == 0) { ctl->stop_reason = KGS_STOP_EXHAUSTED; ctl->levels = l; }
+                break;
+            }
+            continue;
+        }
         auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
             nd.v = v;
             nd.hm = prepare(c, l, v, leader);
@@ -1790,7 +1895,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             if (G.gtid == 0) {
                 QOut *qo = a.qout + qq.qi;
                 qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
-                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g;
+                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1;
             }
             G.sync();
             continue;
@@ -1819,6 +1924,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->n_cid = ctl->n_cid;
             qo->n_parcs = ctl->n_parcs;
             qo->n_eval = ctl->n_eval;
+            qo->pull_level = ctl->pull_at - 1;
             qo->frontier_total = ctl->frontier_total;
             qo->arcs_scanned = ctl->arcs_scanned;
             qo->hits = ctl->hits;

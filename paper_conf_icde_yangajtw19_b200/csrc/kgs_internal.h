@@ -16,6 +16,9 @@ constexpr int kBlock = 512;            // threads per CTA of the engine kernel
 // expanded by warp batches, big ones (more than kBigDeg arcs) in tiles spread over the whole group.
 constexpr int64_t kBigDeg = 2048;
 enum : uint8_t { CLS_LIGHT = 0, CLS_BIG = 1 };
+// A class byte is (big flag) | (lg << 1): lg = 0 for no arcs, else 2^(lg-1) >= degree (auto direction).
+__host__ __device__ __forceinline__ bool cls_big(uint8_t c) { return (c & 1u) != 0; }
+__host__ __device__ __forceinline__ unsigned long long cls_deg_bound(uint8_t c) { return c >> 1 ? 1ull << ((c >> 1) - 1) : 0ull; }
 
 // Per-warp arena of the Central Graph extractor.
 constexpr int kExtNodes = 256;
@@ -65,6 +68,11 @@ struct Ctl {
     uint32_t rec_used;             // the predecessor lists came from the recorded DAG (compact ids = touched)
     uint32_t rec_cnt[kRecStripes * kRecStride];   // recorded arcs per append region (stride 32 B)
     uint32_t pd_cnt[kRecStripes * kRecStride];    // pre-pass predecessor arcs per append region
+    // push / pull direction (kgs_params.direction)
+    unsigned long long mf[2];      // [level parity] out-arcs of the compacted frontier (auto direction)
+    unsigned long long pull_marks[2];   // [level parity] new (node, keyword) hits of a pull level
+    uint32_t pull_nbig[2];         // [level parity] pull candidates with more than kBigDeg in-arcs
+    int32_t pull_at;               // first pulled level + 1 (0: push throughout)
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -75,6 +83,7 @@ struct QOut {
     unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
+    int32_t pull_level, pad2;      // first pulled level, -1: push throughout
     unsigned long long stamp[kMaxStamps];
     int32_t stamp_tag[kMaxStamps];
 };
@@ -174,6 +183,9 @@ struct EngineArgs {
     int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
     int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
+    int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
+    int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio
+    long long pull_min;         //       and pull_min
     // outputs
     QOut *qout;                 // [nq]
     int32_t *out_hdr;           // [nq][k][4]: central, depth, n_nodes, n_arcs

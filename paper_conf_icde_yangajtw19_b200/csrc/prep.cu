@@ -46,7 +46,11 @@ cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha,
 
 __global__ void k_degree_class(const int64_t *__restrict__ rp, int64_t n, uint8_t *__restrict__ cls) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        cls[v] = (rp[v + 1] - rp[v]) > kBigDeg ? CLS_BIG : CLS_LIGHT;
+    {
+        const int64_t d = rp[v + 1] - rp[v];
+        const int lg = d == 0 ? 0 : 1 + (d == 1 ? 0 : 64 - __clzll((unsigned long long)(d - 1)));   // 2^(lg-1) >= d
+        cls[v] = (uint8_t)((d > kBigDeg ? CLS_BIG : CLS_LIGHT) | (lg << 1));
+    }
 }
 cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s) {
     if (n > 0) {
