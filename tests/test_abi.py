@@ -39,11 +39,30 @@ def test_params_default_match_paper():
     assert p.max_depth == 254 and p.block_central == 1 and p.level_cover == 1
 
 
-def test_struct_layout_matches_header():
+def test_struct_layout_matches_header(tmp_path):
+    """The ctypes mirrors have the C compiler's size and field offsets for every struct in kgs.h."""
+    import subprocess
     import paper_conf_icde_yangajtw19_b200 as kgs
-    assert ctypes.sizeof(kgs.kgs_graph_desc) == 8 * 2 + 8 * 3 + 8 + 8 * 2 + 8 + 4 * 3 + 4
-    assert ctypes.sizeof(kgs.kgs_params) == 8 * 2 + 4 * 6
-    assert ctypes.sizeof(kgs.kgs_answer) == 4 * 3 + 4 + 8 + 8 + 8 + 8 + 8
+    structs = [kgs.kgs_graph_desc, kgs.kgs_params, kgs.kgs_answer, kgs.kgs_stats, kgs.kgs_vp_buffers]
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "kgs.h"', "int main(void) {"]
+    for st in structs:
+        nm = st.__name__
+        lines.append(f'printf("{nm} %zu\\n", sizeof({nm}));')
+        for f, _ in st._fields_:
+            cf = "lambda" if f == "lambda_" else f
+            lines.append(f'printf("{nm}.{f} %zu\\n", offsetof({nm}, {cf}));')
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    inc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include")
+    subprocess.run(["gcc", "-I", inc, str(src), "-o", str(exe)], check=True)
+    got = dict(l.split() for l in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split("\n") if l)
+    for st in structs:
+        nm = st.__name__
+        assert int(got[nm]) == ctypes.sizeof(st), nm
+        for f, _ in st._fields_:
+            assert int(got[f"{nm}.{f}"]) == getattr(st, f).offset, (nm, f)
 
 
 def test_no_cpu_fallback_without_gpu():
