@@ -1298,7 +1298,10 @@ __device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn,
             S.b_incl[r] = ex + deg;
             T.sync();
             const int nb = min(ts, tail - b0);
-            for (int e = r; e < tot; e += ts) {
+            for (int e = r, it = 0; e < tot; e += ts, ++it) {
+                // the arena overflowed: the next tier redoes this graph, stop scanning (a hub's list of
+                // millions of predecessors kept a tier-1 warp busy for milliseconds, C5)
+                if ((it & 31) == 0 && *reinterpret_cast<volatile int32_t *>(S.scal + SC_OVF)) break;
                 int lo = 0, hi = nb - 1;       // owner = first o with incl[o] > e
                 while (lo < hi) {
                     const int mid = (lo + hi) >> 1;
