@@ -352,8 +352,6 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
         }
         const uint32_t sh = (uint32_t)(x & 3) << 3;
         uint32_t *nw = c.w.nm + (x >> 2);
-        const uint32_t cur = (__ldcg(nw) >> sh) & 0xFFu;
-        if (!(bits & ~cur)) return;
         const uint32_t old = (atomicOr(nw, bits << sh) >> sh) & 0xFFu;
         const uint32_t nb = bits & ~old;
         if (nb) {
