@@ -117,9 +117,9 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *                    KGS_DIR_PULL (2)  pull at every level: every node x that still lacks a keyword and whose
  *                                   gate is open scans its in-arcs for active neighbours (the level rule,
  *                                   SURVEY.md §8(c) O3).
- *                  M, the central set, depths and answers do not depend on it.  A pulling search is
- *                  exhausted by the level rule (no new hit at a level l >= max a), so stats.levels of an
- *                  exhausted search equals the oracle's level-rule form rather than the work-list form. */
+ *                  Results do not depend on it (M, central set, depths, answers, stop level and reason):
+ *                  after a pulled level without hits the engine recomputes whether Alg. 2's work list
+ *                  would still hold a node (an inactive hit node, or one waiting for a gated neighbour). */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;

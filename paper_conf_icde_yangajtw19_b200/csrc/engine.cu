@@ -818,6 +818,44 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
                          pprep, pvisit, my_arcs);
 }
 
+// After a pulled level l without hits: would the work list of Alg. 2 (FIdentifier) still hold a node at
+// level l + 1?  The pull has no work list, so this recomputes membership: a hit node v (not a blocked
+// central) is re-queued at l iff it is inactive (a_v > l, ln 5-7) or it has an out-neighbour x that lacks
+// one of v's keywords behind a closed gate (gate(x) > l + 1, ln 17-20).  Both conditions can only turn
+// false as l grows unless v gains a keyword, which puts v on the list, so every node satisfying one is
+// on the list.  Sets ctl->pull_wait[l & 1]; nodes stop scanning once it is set.  Group-wide, ends with a
+// barrier.  Then the stop level of a pulling search is the work-list form's (the oracle's literal Alg. 2).
+__device__ __forceinline__ void pull_waiting(const Ctx &c, int l, BigTile &S, long long *sh) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    const DevWork &w = c.w;
+    Ctl *ctl = c.ctl;
+    const uint32_t full = c.qq.full;
+    volatile uint32_t *flag = &ctl->pull_wait[l & 1];
+    unsigned long long arcs = 0;
+    auto wprep = [&](int32_t v, bool, PullNode &nd) {
+        const uint32_t hm = __ldcg(w.st + v) & 0xFFu;
+        if (!hm || (a.block_central && hm == full) || *flag) return false;
+        if ((int)__ldg(a.act + v) > l) { *flag = 1u; return false; }
+        nd.x = v;
+        nd.sx = hm;
+        return true;
+    };
+    auto wlight = [&](int32_t v, bool leader, PullNode &nd) {
+        if (!wprep(v, leader, nd)) return false;
+        if (cls_big(a.g.cls[v])) { w.qbig[warp_slot(&ctl->pull_wbig[l & 1])] = v; return false; }
+        return true;
+    };
+    auto wvisit = [&](const PullNode &nd, int32_t x, uint32_t sx) {
+        if ((nd.sx & ~sx & 0xFFu) && (sx >> 8) > (uint32_t)(l + 1) && !*flag) *flag = 1u;
+    };
+    expand_light<PullNode>(G, nullptr, (uint32_t)a.g.n, a.g.row_ptr, a.g.col_idx, w.st, wlight, wvisit, arcs);
+    G.sync();
+    expand_big<PullNode>(G, w.qbig, __ldcg(&ctl->pull_wbig[l & 1]), a.g.row_ptr, a.g.col_idx, w.st, S, sh,
+                         wprep, wvisit, arcs);
+    G.sync();
+}
+
 __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -984,7 +1022,10 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             if (count_mf && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
             G.sync();
         }
-        if (gtid == 0) ctl->pull_marks[(l + 1) & 1] = 0ull;   // its last reader passed the barrier above
+        if (gtid == 0) {   // their last readers (level l - 1) passed the barrier above
+            ctl->pull_marks[(l + 1) & 1] = 0ull;
+            ctl->pull_wait[(l + 1) & 1] = 0u; ctl->pull_wbig[(l + 1) & 1] = 0u;
+        }
         stamp(G, qo, TS_MERGE);
         __shared__ uint32_t s_ctl[3];
         if (threadIdx.x == 0) { s_ctl[0] = __ldcg(&qn[0]); s_ctl[1] = __ldcg(&qn[1]); s_ctl[2] = __ldcg(&ctl->n_central); }
@@ -1018,16 +1059,25 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             // (x in K or a_x <= l+1, ln 16-17) scans its in-arcs u -> x; an active u (a_u <= l, not a
             // blocked central, ln 2-7) hits x for the keywords it has and x lacks (ln 12-22).  The same
             // visit_arc as the push, so the hits, the recorded Thm. V.4 arcs and the lightest-path rows
-            // are the same; no node is re-queued (ln 19): a pulling search has no work list.
+            // are the same; no node is re-queued (ln 19): a pulling search has no work list (a level
+            // without hits asks pull_waiting whether the list would still be non-empty).
             const unsigned hits0 = my_hits;
             pull_expand(c, l, S, sh, my_hits, my_dag, my_arcs);
             cta_add((unsigned long long)(my_hits - hits0), &ctl->pull_marks[l & 1]);
             publish_flags(ctl);
             G.sync();
             stamp(G, qo, TS_EXPAND);
-            if (__ldcg(&ctl->pull_marks[l & 1]) == 0ull && l >= amax) {   // level rule: nothing can change
-                if (gtid == 0) { ctl->stop_reason = KGS_STOP_EXHAUSTED; ctl->levels = l; }
-                break;
+            if (__ldcg(&ctl->pull_marks[l & 1]) == 0ull) {
+                // no hit at l: the work list at l + 1 holds only re-queued nodes (none once l >= amax)
+                bool waiting = false;
+                if (l < amax) {
+                    pull_waiting(c, l, S, sh);
+                    waiting = __ldcg(&ctl->pull_wait[l & 1]) != 0u;
+                }
+                if (!waiting) {
+                    if (gtid == 0) { ctl->stop_reason = KGS_STOP_EXHAUSTED; ctl->levels = l + 1; }
+                    break;
+                }
             }
             continue;
         }

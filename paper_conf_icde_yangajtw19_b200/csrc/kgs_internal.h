@@ -73,6 +73,8 @@ struct Ctl {
     unsigned long long pull_marks[2];   // [level parity] new (node, keyword) hits of a pull level
     uint32_t pull_nbig[2];         // [level parity] pull candidates with more than kBigDeg in-arcs
     int32_t pull_at;               // first pulled level + 1 (0: push throughout)
+    uint32_t pull_wait[2];         // [level parity] a pulled level without hits: some node is still on Alg. 2's work list
+    uint32_t pull_wbig[2];         // [level parity] ... big nodes to check after the sweep
 };
 
 // Per-query summary written by the engine (device), read back by the host.

@@ -1,12 +1,11 @@
 """Push / pull direction of the expansion (kgs_params.direction, the north star's "push/pull direction
 switching") against the oracle, through the C-ABI.
 
-Pull at every level is the frontier-free level rule (oracle BFS_LEVEL_RULE): M, the
-central set, depths, keys and answers must equal the oracle bit for bit, and so must the stop level,
-which for an exhausted search is the level rule's (the work-list form can stop a level earlier or
-later; the two forms agree on everything else, tests/test_oracle_search.py).  The automatic switch
-(push first, pull from the first level whose frontier has more than m / KGS_PULL_RATIO out-arcs) is
-exercised mid-search with small thresholds: the stop level then follows the form that was running.
+Pull at every level computes the frontier-free level rule; after a level without
+hits it recomputes whether Alg. 2's work list would still be non-empty, so M, the central set, depths,
+keys, answers AND the stop level equal the oracle's literal form bit for bit whatever the direction.
+The automatic switch (push first, pull from the first level whose active frontier has more than
+m / KGS_PULL_RATIO out-arcs) is exercised mid-search with small thresholds.
 """
 import os
 
@@ -39,9 +38,8 @@ def compare(G, g, kw, k, direction, *, alpha=0.1, lam=0.2, max_depth=254, block_
         assert r.stats["pull_level"] == 0 or (r.stats["pull_level"] == -1 and r.stats["levels"] == 0)
     if direction == kgs.KGS_DIR_PUSH:
         assert not pulled
-    form = oracle.BFS_LEVEL_RULE if pulled else oracle.BFS_LITERAL
     o = oracle.query(g, kw, k, alpha=alpha, lam=lam, max_depth=max_depth, block_central=block_central,
-                     extract_mode=extract_mode, level_cover=level_cover, bfs_form=form)
+                     extract_mode=extract_mode, level_cover=level_cover)
     ctx = f"kw={list(kw)} k={k} dir={direction} pulled_at={r.stats['pull_level']} blk={block_central} ext={extract_mode}"
     if full:
         assert (r.M == o.M).all(), ctx
@@ -138,7 +136,7 @@ def test_batch_groups_pull():
     w = synth.make_workload("C1")
     G = kgs.kgs_load_graph(w.graph)
     qs = w.queries[:60]
-    exp = [oracle.query(w.graph, kw, w.k, bfs_form=oracle.BFS_LEVEL_RULE) for kw in qs]
+    exp = [oracle.query(w.graph, kw, w.k) for kw in qs]
     p = kgs.make_params(direction=kgs.KGS_DIR_PULL)
     for groups in (1, 3, 8):
         res = kgs.kgs_query_batch(G, qs, w.k, p, groups)
