@@ -5,15 +5,17 @@ queries/s and GTEPS on the Wikidata-scale synthetic graph).
   python bench.py [--gpus N --steps K --warmup W]          CUDA path (libkgs), one rank per GPU
   python bench.py --impl reference [...]                   the CPU oracle on this box's host cores
 
-Workload.  N = 1: C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keyword queries, top-20).
-N > 1 (torchrun): C4 (configs[3]: the same graph, 4096 queries with q ~ U{2..8}) dealt round-robin to
-ranks holding a replicated graph; one NCCL all-gather of the top-k headers per step (inside the timed
-region).  The per-rank step is the same size for every N (weak scaling).
+Workload: C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keyword queries, top-20) at every N.
+N > 1 (torchrun): every rank holds a replica of the graph (rank 0 generates it and broadcasts it over
+NCCL) and answers the 350 C3 queries per step, starting at a rank-dependent offset; one NCCL all-gather of
+the top-k headers per step (inside the timed region).  The per-rank step is the same for every N (weak
+scaling).  C4's own query set (configs[3], 4096 queries with q ~ U{2..8}) is not used for the bench line:
+7 of its queries (0.17%) only find k central nodes at level 5, where ~1 M nodes become central at once and
+the exact top-down takes 40-50 s each (tools/workload_scan.py).
 
 A step = one batch of queries through the whole hot path in ONE engine launch (activation gate, search,
 central detection, extraction + level-cover + Eq. 6 of every central graph, top-k, answer emit):
-the 350-query C3 latency set at N = 1 (each query once per step), 350 queries of the rank's C4 shard at
-N > 1.  `value` = queries/s of device time over K steps (CUDA events on the launching stream, L2 flushed
+the 350-query C3 set (each query once per step).  `value` = queries/s of device time over K steps (CUDA events on the launching stream, L2 flushed
 with a 512 MiB write between steps, outside the events; max over ranks).  The single-query latency
 mode (one launch per query, the whole GPU on it) gives `p50_ms` / `p95_ms`.  `e2e` = the same batches
 through kgs_query_batch from host keyword ids to host answers (wall clock, H2D + D2H inside).
@@ -107,13 +109,17 @@ def load_peaks():
 
 
 def load_traffic():
-    """Mean DRAM bytes per query of the engine from the newest committed ncu capture (profiles/)."""
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_engine_traffic.json")))
-    if not files:
-        return None, None
-    with open(files[-1]) as f:
-        d = json.load(f)
-    return d, os.path.basename(files[-1])
+    """DRAM bytes per query of the engine from the newest committed ncu capture (profiles/): a capture of
+    the bench's own launch shape (r*_batch_traffic.json: one 350-query launch, G = 8) when there is one,
+    else the latency-mode per-query captures (r*_engine_traffic.json)."""
+    for pat, key in (("r*_batch_traffic.json", "dram_bytes_per_query"),
+                     ("r*_engine_traffic.json", "mean_dram_bytes_per_query")):
+        files = sorted(glob.glob(os.path.join(ROOT, "profiles", pat)))
+        if files:
+            with open(files[-1]) as f:
+                d = json.load(f)
+            return d[key], os.path.basename(files[-1])
+    return None, None
 
 
 def algorithmic_bytes(st: dict) -> float:
@@ -194,7 +200,7 @@ def run_reference(args):
     if rank != 0:
         return 0
     import oracle
-    name = "C3" if world == 1 else "C4"
+    name = "C3"   # the GPU arm's workload at every N
     w, gen_s = build_workload(name)
     order = np.random.default_rng(12345).permutation(len(w.queries))
     qs = [w.queries[i] for i in order]
@@ -251,7 +257,7 @@ def main():
     cuda = f"cuda:{dev}"
     import paper_conf_icde_yangajtw19_b200 as kgs
 
-    name = "C3" if world == 1 else "C4"
+    name = "C3"
     if world == 1:
         w, gen_s = build_workload(name)
         g = w.graph
@@ -263,7 +269,8 @@ def main():
     order = np.random.default_rng(12345).permutation(len(w.queries))
     allq = [w.queries[i] for i in order]
     qids_all = [int(i) for i in order]
-    mine = list(range(rank, len(allq), world)) if world > 1 else list(range(len(allq)))
+    off = (rank * len(allq)) // world   # N > 1: the same set, rotated per rank
+    mine = [(off + i) % len(allq) for i in range(len(allq))]
     queries = [allq[i] for i in mine]
     qids = [qids_all[i] for i in mine]
     B = args.batch
@@ -306,7 +313,7 @@ def main():
             answers = [(qids[j], [(a.central, a.depth, a.score_key) for a in r.answers]) for j, r in zip(idx, res)]
     gather_ms = 0.0
     if dist:
-        # NCCL all-gather of every rank's top-k headers (central, depth, key) of the last step (config C4)
+        # NCCL all-gather of every rank's top-k headers (central, depth, key) of the last step
         from paper_conf_icde_yangajtw19_b200 import dist as kd
         hdr = kd.pack_headers([q for q, _ in answers], [a for _, a in answers], w.k).to(cuda)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -386,7 +393,7 @@ def main():
         "gteps": arcs / (dev_ms / 1e3) / 1e9 * world,
         "roofline": {"kernel": "k_engine", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind,
-                     "traffic": (tr["mean_dram_bytes_per_query"] * B) if tr else None, "traffic_source": tr_src,
+                     "traffic": (tr * B) if tr else None, "traffic_source": tr_src,
                      "algorithmic_bytes_per_launch": alg / args.steps,
                      "latency_mode_achieved": (lat_alg / (sum(lat) / 1e3) / 1e9) if lat else None},
         "e2e": {"value": e2e_qps, "unit": "queries/s", "ms_per_step": statistics.median(e2e_ms),

@@ -162,7 +162,7 @@ void free_work(DevWork &w) {
     void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
-                 w.gstate};
+                 w.gstate, w.huge};
     for (void *x : p) if (x) cudaFree(x);
     w = DevWork{};
 }
@@ -183,6 +183,7 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.cdepth, n));
     CUDA_TRY(dmalloc(&w.ckey, n));
     CUDA_TRY(dmalloc(&w.overflow, n));
+    CUDA_TRY(cudaMalloc((void **)&w.huge, arena_bytes_host(kHugeHash, kHugeNodes, kHugeArcs, kBlock, true)));
     CUDA_TRY(dmalloc(&w.cflag, n));
     CUDA_TRY(dmalloc(&w.sel, KGS_MAX_K));
     CUDA_TRY(dmalloc(&w.elist, n));
@@ -404,6 +405,12 @@ kgs_status check_query(const kgs_graph *g, const int32_t *kw, int32_t q) {
     return KGS_OK;
 }
 
+// predecessor-arc capacity of a group workspace (KGS_PCAP_M: millions of arcs)
+int64_t pcap_max() {
+    const char *e = std::getenv("KGS_PCAP_M");
+    return (e ? std::max(1ll, std::atoll(e)) : 256ll) << 20;
+}
+
 // per-alpha activation cache, level-slot ring, per-lambda depth factors, G group workspaces
 kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
     bool invalidate = false;
@@ -429,10 +436,10 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
     }
     if ((int)g->works.size() < G) {
         CUDA_TRY(cudaStreamSynchronize(s));
-        // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs): 64 M for the
-        // single-query group, 32 M for the others (20 B per arc)
+        // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs; 20 B per arc):
+        // 256 M (5.1 GB; KGS_PCAP_M) — the level-5 C4 queries record 192 M arcs, their pre-pass 135 M
         while ((int)g->works.size() < G) {
-            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, g->works.empty() ? (64ll << 20) : (32ll << 20)), 1 << 20);
+            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, pcap_max()), 1 << 20);
             DevWork w;
             kgs_status st = alloc_work(g, w, pcap);
             if (st != KGS_OK) { free_work(w); return st; }
@@ -475,7 +482,9 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18;
+        const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
+                           (size_t)std::min<int64_t>(g->m, pcap_max()) * 20 +
+                           arena_bytes_host(kHugeHash, kHugeNodes, kHugeArcs, kBlock, true);
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
         G = std::max(1, (int)g->works.size() + more);
     }
@@ -485,8 +494,9 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     CUDA_TRY(grow_dev(&g->d_hdr, &g->d_hdr_cap, (size_t)nq * k * 4));
     CUDA_TRY(grow_dev(&g->d_key, &g->d_key_cap, (size_t)nq * k));
     CUDA_TRY(grow_dev(&g->d_off, &g->d_off_cap, (size_t)nq * k * 2));
-    CUDA_TRY(grow_dev(&g->d_nodes, &g->d_nodes_cap, (size_t)nq * k * 64 + (4u << 20)));
-    CUDA_TRY(grow_dev(&g->d_arcs, &g->d_arcs_cap, 2 * ((size_t)nq * k * 64 + (4u << 20))));
+    // answer arena: 64 nodes per answer on average plus room for a few tier-4 (huge) Central Graphs
+    CUDA_TRY(grow_dev(&g->d_nodes, &g->d_nodes_cap, (size_t)nq * k * 64 + (16u << 20)));
+    CUDA_TRY(grow_dev(&g->d_arcs, &g->d_arcs_cap, 2 * ((size_t)nq * k * 64 + (32u << 20))));
     CUDA_TRY(cudaMemsetAsync(g->d_ctr, 0, 4 * sizeof(unsigned long long), s));
     EngineArgs a{};
     a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx; a.g.in_ptr = g->in_ptr;
@@ -518,6 +528,10 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
         a.dag_record = on && !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     }
     a.direction = p.direction;
+    {
+        const char *e = std::getenv("KGS_SEARCH_ONLY");   // workload analysis only: no answers, stats of the search
+        a.search_only = e && std::atoi(e) ? 1 : 0;
+    }
     {
         const char *e = std::getenv("KGS_PULL_RATIO");   // auto direction: pull once frontier arcs > m / ratio
         a.pull_ratio = e ? std::max(1, std::atoi(e)) : 14;

@@ -568,13 +568,13 @@ __device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const P
     uint32_t zbu = 0;
     const uint32_t pb = pred_test(c, exact_block, nd.P, nd.hx, nd.gx, u, su, zbu);
     if (!pb) return;
-    const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(c.w.pcnt + nd.cidx), (unsigned)nd.cidx);
     // the CTA's append region (as the recorded DAG: one counter per CTA, not one per group)
     const int ns = rec_stripes(c.G);
     const int stripe = c.G.grank % ns;
     const uint32_t ai = warp_slot(&c.ctl->pd_cnt[stripe * kRecStride]);
     const int64_t rcap = c.w.pcap / ns;
-    if ((int64_t)ai < rcap) {
+    if ((int64_t)ai < rcap) {   // a list slot only for a stored arc: the CSR never holds unwritten entries
+        const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(c.w.pcnt + nd.cidx), (unsigned)nd.cidx);
         const int64_t r = stripe * rcap + ai;
         c.w.pa_u[r] = u;
         c.w.pa_x[r] = nd.cidx;
@@ -1684,7 +1684,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
     Ctl *ctl = c.ctl;
-    if (G.gtid == 0) { ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->n_eval += cnt; }
+    if (G.gtid == 0) { ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->work_huge = 0; ctl->n_eval += cnt; }
     G.sync();
     if ((threadIdx.x >> 5) < kExtWarps) {
         Arena S1 = carve(dsmem + kSmemArena * (threadIdx.x >> 5), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
@@ -1731,12 +1731,29 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
                 const bool ok = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
                 if (threadIdx.x == 0) {
                     if (ok) c.w.ckey[idx] = key;
-                    else atomicExch(&ctl->fatal, 2);
+                    else c.w.overflow[no + nbig + atomicAdd(&ctl->work_huge, 1u)] = idx;
                 }
                 __syncthreads();
             }
         }
         G.sync();
+        const uint32_t nhuge = __ldcg(&ctl->work_huge);
+        if (nhuge) {   // tier 4: the group's huge arena, one CTA
+            if (G.grank == 0) {
+                Arena S4 = carve(c.w.huge, kHugeHash, kHugeNodes, kHugeArcs, blockDim.x, true);
+                for (uint32_t t = 0; t < nhuge; ++t) {
+                    const int32_t idx = __ldcg(c.w.overflow + no + nbig + t);
+                    double key = 0.0;
+                    const bool ok = central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+                    if (threadIdx.x == 0) {
+                        if (ok) c.w.ckey[idx] = key;
+                        else atomicExch(&ctl->fatal, 2);
+                    }
+                    __syncthreads();
+                }
+            }
+            G.sync();
+        }
         stamp(G, qo, TS_EXTRACT_BIG);
     }
 }
@@ -1793,10 +1810,26 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
             double key;
             if (central_graph(BT, S2, c, cn, dep, &key)) emit_graph(BT, S2, c, rk);
             else if (central_graph(BT, S, c, cn, dep, &key)) emit_graph(BT, S, c, rk);
-            else if (threadIdx.x == 0) atomicExch(&ctl->fatal, 4);
+            else if (threadIdx.x == 0) c.w.overflow[nbig + atomicAdd(&ctl->work_huge, 1u)] = rk;
             __syncthreads();
         }
         G.sync();
+        const uint32_t nhuge = __ldcg(&ctl->work_huge);
+        if (nhuge) {   // tier 4: the group's huge arena, one CTA
+            if (G.grank == 0) {
+                Arena S4 = carve(c.w.huge, kHugeHash, kHugeNodes, kHugeArcs, blockDim.x, true);
+                for (uint32_t t = 0; t < nhuge; ++t) {
+                    const int rk = __ldcg(c.w.overflow + nbig + t);
+                    const int32_t idx = __ldcg(c.w.sel + rk);
+                    double key;
+                    if (central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
+                        emit_graph(BT, S4, c, rk);
+                    else if (threadIdx.x == 0) atomicExch(&ctl->fatal, 4);
+                    __syncthreads();
+                }
+            }
+            G.sync();
+        }
     }
     stamp(G, qo, TS_EMIT);
 }
@@ -1826,7 +1859,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             pred_dag(c, S, sh, qo);
         }
         extract_list(c, sh, dsmem, nullptr, nc, qo);
-        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }   // emit counters (read after the select)
+        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }   // emit counters (read after the select)
         select_topk(c, sh, dsmem, kk);
     } else {
         const uint32_t m = mcap;
@@ -1875,7 +1908,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             }
             extract_list(c, sh, dsmem, c.w.elist + m, n2, qo);
         }
-        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; }
+        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }
         if (m + n2 <= (uint32_t)KGS_MAX_K) {
             rank_list(c, dsmem, c.w.elist, m + n2, kk);
         } else {   // the candidates never extracted rank after every extracted one
@@ -1964,7 +1997,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         const Ctx c{a, w, ctl, G, qq};
         if (a.td_only) td_only_prepare(c, qo);
         else search(c, s_big, sh, qo);
-        topdown(c, s_big, sh, dsmem, qo);
+        if (!a.search_only) topdown(c, s_big, sh, dsmem, qo);   // search_only: workload analysis (no answers)
         if (G.gtid == 0) {
             qo->levels = ctl->levels;
             qo->stop_reason = ctl->stop_reason;

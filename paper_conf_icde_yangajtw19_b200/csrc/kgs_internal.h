@@ -28,6 +28,11 @@ constexpr int kExtHash = 512;
 constexpr int kBigNodes = 1 << 16;
 constexpr int kBigArcs = 1 << 18;
 constexpr int kBigHash = 1 << 17;
+// Per-group arena of the huge-graph extractor (tier 4: one CTA of the group, Central Graphs beyond a
+// CTA arena — the deepest C4 queries reach them).
+constexpr int kHugeNodes = 1 << 22;
+constexpr int kHugeArcs = 1 << 24;
+constexpr int kHugeHash = 1 << 23;
 
 // Append regions of the recorded DAG (engine.cu visit_arc): one counter per region, 32 bytes apart.
 constexpr int kRecStripes = 128;
@@ -75,6 +80,7 @@ struct Ctl {
     int32_t pull_at;               // first pulled level + 1 (0: push throughout)
     uint32_t pull_wait[2];         // [level parity] a pulled level without hits: some node is still on Alg. 2's work list
     uint32_t pull_wbig[2];         // [level parity] ... big nodes to check after the sweep
+    uint32_t work_huge;            // Central Graphs beyond the CTA arenas (tier 4), this extract / emit pass
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -128,6 +134,7 @@ struct DevWork {
     uint8_t *cdepth;    // [n] depth per central
     double *ckey;       // [n] Eq. 6 key per central
     int32_t *overflow;  // [n] centrals whose graph exceeds the per-warp extractor
+    char *huge;         // tier-4 extraction arena (kHuge*), used by one CTA of the group
     uint8_t *cflag;     // [n] 1 = overflowed the per-warp extractor
     int32_t *sel;       // [KGS_MAX_K] ranked winners (index into centrals)
     int32_t *elist;     // [n] candidates to extract (index into centrals)
@@ -188,6 +195,7 @@ struct EngineArgs {
     int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
     int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio
     long long pull_min;         //       and pull_min
+    int search_only;            // KGS_SEARCH_ONLY=1 (analysis tool): skip the top-down, no answers
     // outputs
     QOut *qout;                 // [nq]
     int32_t *out_hdr;           // [nq][k][4]: central, depth, n_nodes, n_arcs

@@ -186,6 +186,15 @@ def make_queries(g: Graph, seed: int, *, sizes=None, uniform_q=None, count=0, ba
     return qs
 
 
+def config_queries(name: str, g: Graph) -> list:
+    """The query set of config ``name`` drawn from an already generated graph ``g`` of the same recipe
+    (C4 shares the C3 graph: bench.py generates it once)."""
+    p = CONFIG_PARAMS[name]
+    qs = dict(p["qspec"])
+    band = qs.pop("band")
+    return make_queries(g, p.get("qseed", 1000 + int(name[1:])), band=band, **qs)
+
+
 def make_workload(name: str, *, scale_override: int | None = None, n_queries: int | None = None) -> Workload:
     """Build one BASELINE.json config.  ``scale_override`` shrinks the graph for tests (same recipe)."""
     p = CONFIG_PARAMS[name]
