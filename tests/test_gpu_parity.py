@@ -200,3 +200,22 @@ def test_batch_device_invalid_queries():
     for i, gi in ((0, 0), (2, 1), (4, 2)):
         o = oracle.query(w.graph, good[gi], w.k)
         assert [a.central for a in res[i].answers] == [a.central for a in o.answers]
+
+
+def test_huge_central_graph_tier4():
+    """A Central Graph beyond the per-CTA arena (64 K nodes): a hub c joined to 150 000 nodes holding
+    keyword 0 and to one node holding keyword 1 — G(c) has 150 002 nodes, so extraction and emit reach
+    the per-group tier-4 arena; latency mode (recorded DAG) and query groups (pre-pass)."""
+    _gpu()
+    n0 = 150_000
+    a, c = n0, n0 + 1
+    edges = [(v, c) for v in range(n0)] + [(a, c)]
+    g = synth.from_edges(n0 + 2, edges, [0.0] * (n0 + 2), [list(range(n0)), [a]], 2.0)
+    G = kgs.kgs_load_graph(g)
+    r, o = compare(G, g, [0, 1], 1)
+    assert len(r.answers) == 1 and r.answers[0].central == c and len(r.answers[0].nodes) == n0 + 2
+    res = kgs.kgs_query_batch(G, [[0, 1], [1, 0], [0, 1]], 1, None, 3)
+    for rr in res:
+        assert rr.answers[0].central == c and rr.answers[0].nodes.tolist() == o.answers[0].nodes.tolist()
+        assert rr.answers[0].arcs.tolist() == o.answers[0].arcs.tolist()
+    G.close()
