@@ -200,6 +200,9 @@ struct Ctx {        // everything a group needs while answering one query
     Ctl *ctl;
     const Grp &G;
     const Q &qq;
+    int rec_ns;         // append regions of the recorded DAG / pre-pass used by the group
+    int rec_stripe;     // this CTA's region
+    int64_t rec_cap;    // arcs per region
 };
 
 // the input id of internal node v (every id leaving the engine, and the ranking tie-break, is an input id)
@@ -207,7 +210,7 @@ __device__ __forceinline__ int32_t in_id(const EngineArgs &a, int32_t v) { retur
 
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
 __device__ __forceinline__ void push(const Ctx &c, int32_t v, int L, bool check = false) {
-    const int s = L % c.a.R;
+    const int s = L < c.a.R ? L : L % c.a.R;   // L < R except for new hits past level R - 1 (no division)
     set_bit(c.w.fbits + (int64_t)s * c.a.W, s, v, check);
 }
 
@@ -333,10 +336,9 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
         if (c.a.dag_record) {   // recorded predecessor arc
             // one of kRecStripes append regions per CTA: a single counter would serialise millions of
             // atomics per heavy query on one address
-            const int ns = rec_stripes(c.G);
-            const int stripe = c.G.grank % ns;
+            const int stripe = c.rec_stripe;
             const uint32_t ai = warp_slot(&c.ctl->rec_cnt[stripe * kRecStride]);
-            const int64_t rcap = c.w.pcap / ns;
+            const int64_t rcap = c.rec_cap;
             if ((int64_t)ai < rcap) {
                 const int64_t r = stripe * rcap + ai;
                 c.w.pa_u[r] = v;
@@ -569,10 +571,9 @@ __device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const P
     const uint32_t pb = pred_test(c, exact_block, nd.P, nd.hx, nd.gx, u, su, zbu);
     if (!pb) return;
     // the CTA's append region (as the recorded DAG: one counter per CTA, not one per group)
-    const int ns = rec_stripes(c.G);
-    const int stripe = c.G.grank % ns;
+    const int stripe = c.rec_stripe;
     const uint32_t ai = warp_slot(&c.ctl->pd_cnt[stripe * kRecStride]);
-    const int64_t rcap = c.w.pcap / ns;
+    const int64_t rcap = c.rec_cap;
     if ((int64_t)ai < rcap) {   // a list slot only for a stored arc: the CSR never holds unwritten entries
         const uint32_t pos = agg_slot(reinterpret_cast<uint32_t *>(c.w.pcnt + nd.cidx), (unsigned)nd.cidx);
         const int64_t r = stripe * rcap + ai;
@@ -602,8 +603,8 @@ __device__ __forceinline__ bool pd_prepare(const Ctx &c, int32_t x, PdNode &nd) 
 // (the region sizes are staged in shared memory once; a flat index finds its region by binary search)
 template <class F>
 __device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cnt, F fn) {
-    const int ns = rec_stripes(c.G);
-    const int64_t rcap = c.w.pcap / ns;
+    const int ns = c.rec_ns;
+    const int64_t rcap = c.rec_cap;
     __shared__ uint32_t s_pre[kRecStripes + 1];
     static_assert(kRecStripes <= kBlock, "one thread per region");
     __syncthreads();
@@ -1994,7 +1995,8 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         if (G.gtid == 0) { qo->n_stamp = 0; qo->t_start = globaltimer_ns(); qo->group = G.g; }
         G.sync();
         stamp(G, qo, TS_START);
-        const Ctx c{a, w, ctl, G, qq};
+        const int rns = rec_stripes(G);
+        const Ctx c{a, w, ctl, G, qq, rns, G.grank % rns, w.pcap / rns};
         if (a.td_only) td_only_prepare(c, qo);
         else search(c, s_big, sh, qo);
         if (!a.search_only) topdown(c, s_big, sh, dsmem, qo);   // search_only: workload analysis (no answers)
