@@ -90,8 +90,11 @@ struct kgs_graph {
     int works_dev_n = 0;
     GroupBar *bars = nullptr;
     int grid = 0;
-    char *warp_arenas = nullptr, *cta_arenas = nullptr;
-    size_t warp_arena_bytes = 0, cta_arena_bytes = 0;
+    char *warp_arenas = nullptr, *cta_arenas = nullptr, *large_arenas = nullptr;
+    size_t warp_arena_bytes = 0, cta_arena_bytes = 0, large_arena_bytes = 0;
+    int large_hash = 0, large_nodes = 0, large_arcs = 0;
+    int big_hash = 0, big_nodes = 0, big_arcs = 0, huge_hash = 0, huge_nodes = 0, huge_arcs = 0;
+    size_t huge_arena_bytes = 0;
     // batch buffers
     int32_t *d_kw = nullptr, *d_qlen = nullptr;
     size_t d_kw_cap = 0, d_qlen_cap = 0;
@@ -183,7 +186,7 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.cdepth, n));
     CUDA_TRY(dmalloc(&w.ckey, n));
     CUDA_TRY(dmalloc(&w.overflow, n));
-    CUDA_TRY(cudaMalloc((void **)&w.huge, arena_bytes_host(kHugeHash, kHugeNodes, kHugeArcs, kBlock, true)));
+    CUDA_TRY(cudaMalloc((void **)&w.huge, g->huge_arena_bytes));
     CUDA_TRY(dmalloc(&w.cflag, n));
     CUDA_TRY(dmalloc(&w.sel, KGS_MAX_K));
     CUDA_TRY(dmalloc(&w.elist, n));
@@ -241,7 +244,7 @@ void kgs_free_graph(kgs_graph *g) {
     cudaDeviceSynchronize();
     for (auto &w : g->works) free_work(w);
     void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->act, g->amax_dev, g->dpow,
-                    g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
+                    g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->large_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
                     g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr, g->vp_gate, g->vp_X, g->vp_big,
                     g->vp_nbig_dev, g->orig, g->perm};
     for (void *p : ptrs) if (p) cudaFree(p);
@@ -369,9 +372,30 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     g->grid = engine_max_grid(g->device);
     if (g->grid <= 0) return bail(fail(KGS_ECUDA, "engine occupancy query failed"));
     g->warp_arena_bytes = arena_bytes_host(kExtHash, kExtNodes, kExtArcs, 32, true);
-    g->cta_arena_bytes = arena_bytes_host(kBigHash, kBigNodes, kBigArcs, kBlock, true);
+    {   // tiers 3, 3b and 4 sized to the graph (a Central Graph has at most n nodes; its arena arcs are the
+        // predecessor entries, at most q per arc): small graphs do not pay for Wikidata-scale arenas
+        auto pow2 = [](int64_t x) { int64_t p = 1; while (p < x) p <<= 1; return p; };
+        const int64_t pn = pow2(std::max<int64_t>(g->n, 1024)), pm = pow2(std::max<int64_t>(8 * g->m, 4096));
+        g->big_nodes = (int)std::min<int64_t>(kBigNodes, pn);
+        g->big_arcs = (int)std::min<int64_t>(kBigArcs, pm);
+        g->big_hash = 2 * g->big_nodes;
+        g->huge_nodes = (int)std::min<int64_t>(kHugeNodes, pn);
+        g->huge_arcs = (int)std::min<int64_t>(kHugeArcs, pm);
+        g->huge_hash = 2 * g->huge_nodes;
+        g->huge_arena_bytes = arena_bytes_host(g->huge_hash, g->huge_nodes, g->huge_arcs, kBlock, true);
+    }
+    g->cta_arena_bytes = arena_bytes_host(g->big_hash, g->big_nodes, g->big_arcs, kBlock, true);
     G_TRY(cudaMalloc(&g->warp_arenas, g->warp_arena_bytes * (size_t)g->grid * (kBlock / 32)));
     G_TRY(cudaMalloc(&g->cta_arenas, g->cta_arena_bytes * (size_t)g->grid));
+    {   // tier 3b: per-CTA arenas for Central Graphs beyond 64 K nodes, sized to the graph (at most 1 M nodes /
+        // 4 M arcs, 88 MB per CTA at C3 scale)
+        auto pow2 = [](int64_t x) { int64_t p = 1; while (p < x) p <<= 1; return p; };
+        g->large_nodes = (int)std::min<int64_t>(1 << 20, pow2(std::max<int64_t>(g->n, 1024)));
+        g->large_arcs = (int)std::min<int64_t>(1 << 22, pow2(std::max<int64_t>(8 * g->m, 4096)));
+        g->large_hash = 2 * g->large_nodes;
+        g->large_arena_bytes = arena_bytes_host(g->large_hash, g->large_nodes, g->large_arcs, kBlock, false);
+        G_TRY(cudaMalloc(&g->large_arenas, g->large_arena_bytes * (size_t)g->grid));
+    }
     G_TRY(cudaDeviceSynchronize());
 #undef G_TRY
     *out = g;
@@ -484,7 +508,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
         cudaMemGetInfo(&free_b, &total_b);
         const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
                            (size_t)std::min<int64_t>(g->m, pcap_max()) * 20 +
-                           arena_bytes_host(kHugeHash, kHugeNodes, kHugeArcs, kBlock, true);
+                           g->huge_arena_bytes;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
         G = std::max(1, (int)g->works.size() + more);
     }
@@ -548,6 +572,10 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.out_used = g->d_ctr + 1;
     a.warp_arenas = g->warp_arenas; a.warp_arena_bytes = g->warp_arena_bytes;
     a.cta_arenas = g->cta_arenas; a.cta_arena_bytes = g->cta_arena_bytes;
+    a.large_arenas = g->large_arenas; a.large_arena_bytes = g->large_arena_bytes;
+    a.large_hash = g->large_hash; a.large_nodes = g->large_nodes; a.large_arcs = g->large_arcs;
+    a.big_hash = g->big_hash; a.big_nodes = g->big_nodes; a.big_arcs = g->big_arcs;
+    a.huge_hash = g->huge_hash; a.huge_nodes = g->huge_nodes; a.huge_arcs = g->huge_arcs;
     CUDA_TRY(cudaMemsetAsync(g->bars, 0, sizeof(GroupBar) * (size_t)G, s));   // monotonic group barriers
     CUDA_TRY(cudaEventRecord(g->ev[0], s));
     CUDA_TRY(launch_engine(a, g->grid, s));

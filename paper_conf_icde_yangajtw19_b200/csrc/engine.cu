@@ -993,6 +993,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                         my_mf += cls_deg_bound(a.g.cls[v]);
                     const uint32_t b = nm8[v];
                     if (!b) return false;
+                    if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
                     nm8[v] = 0;
                     const uint32_t old = st8[2 * (int64_t)v];
                     const uint32_t nw = old | b;
@@ -1216,11 +1217,12 @@ struct Arena {
     unsigned long long *sortbuf;  // [2*acap]
     int32_t *scal;      // [SC_N]
     double *dsum;
+    unsigned long long *wsum;     // closure weight so far, 2^-24 fixed point (key cut-off)
     int hcap, ncap, acap;
 };
 
 __host__ __device__ inline size_t arena_bytes(int hcap, int ncap, int acap, int team, bool with_sort) {
-    size_t b = 16 + sizeof(int64_t) * team + sizeof(double);
+    size_t b = 16 + sizeof(int64_t) * team + sizeof(double) + sizeof(unsigned long long);
     if (with_sort) b += sizeof(unsigned long long) * 2 * (size_t)acap;
     b += sizeof(int32_t) * 2 * (size_t)hcap + sizeof(int32_t) * 6 * (size_t)ncap + sizeof(int32_t) * 3 * (size_t)acap;
     b += sizeof(int32_t) * 3 * (size_t)team + sizeof(int32_t) * SC_N + 16;
@@ -1248,6 +1250,7 @@ __device__ Arena carve(char *p, int hcap, int ncap, int acap, int team, bool wit
     p = align8(p);
     S.b_start = reinterpret_cast<int64_t *>(p); p += sizeof(int64_t) * team;
     S.dsum = reinterpret_cast<double *>(p); p += sizeof(double);
+    S.wsum = reinterpret_cast<unsigned long long *>(p); p += sizeof(unsigned long long);
     if (with_sort) { S.sortbuf = reinterpret_cast<unsigned long long *>(p); p += sizeof(unsigned long long) * 2 * (size_t)acap; }
     else S.sortbuf = nullptr;
     S.hkey = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * hcap;
@@ -1274,7 +1277,8 @@ __device__ __forceinline__ uint32_t hash32(uint32_t x) {
 }
 
 // insert (or find) node u; returns its index, -1 on overflow
-__device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu) {
+__device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu, bool &fresh) {
+    fresh = false;
     uint32_t h = hash32((uint32_t)u) & (uint32_t)(S.hcap - 1);
     for (int probe = 0; probe < S.hcap; ++probe) {
         const int32_t k = atomicCAS(S.hkey + h, -1, u);
@@ -1285,6 +1289,7 @@ __device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu) {
             S.zb[idx] = zbu;
             __threadfence_block();
             atomicExch(S.hval + h, idx);
+            fresh = true;
             return idx;
         }
         if (k == u) {
@@ -1304,30 +1309,47 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
 }
 
 // Closure (over the shared predecessor lists) + level-cover + Eq. 6 key of the Central Graph at c.
-// Returns false on arena overflow.
+// Returns CG_OK, CG_OVERFLOW (arena too small: the next tier redoes it) or CG_CUT.
+// cut (pruning round 2, exact): the key is known to exceed `cut` (the k-th exact key so far), so c cannot
+// rank in the top-k — stop.  Valid when the pruned graph is the whole closure, i.e. when level-cover
+// keeps every source (s* = 1): no set of sources holding two or more query keywords can cover Q together
+// with c's own keywords (multi = union of the keyword sets of all such nodes of the graph), or
+// level_cover = 0.  Then the closure weight so far, times d^lambda, is a lower bound of the key.
+enum { CG_OVERFLOW = 0, CG_OK = 1, CG_CUT = 2 };
+constexpr double kNoCut = __builtin_huge_val();
 template <class Team>
-__device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, int depth, double *key) {
+__device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, int depth, double *key,
+                             double cut = kNoCut, uint32_t multi = 0u) {
     const uint32_t full = c.qq.full;
     const int r = T.rank(), ts = T.size();
     for (int i = r; i < S.hcap; i += ts) { S.hkey[i] = -1; S.hval[i] = -1; }
     for (int i = r; i < S.ncap; i += ts) { S.inmask[i] = 0; S.pending[i] = 0; S.keep[i] = 0; }
     if (r < SC_N) S.scal[r] = 0;
-    if (r == 0) *S.dsum = 0.0;
+    if (r == 0) { *S.dsum = 0.0; *S.wsum = 0ull; }
     T.sync();
+    const uint64_t Mc = ldrow(c.w.M, cn);
+    uint32_t zbc = 0;
+    for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
+    const bool cut_on = cut < kNoCut &&
+                        (!c.a.level_cover || ((multi | zbc) & full) != full);
     if (r == 0) {
-        const uint64_t Mc = ldrow(c.w.M, cn);
-        uint32_t zbc = 0;
-        for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
-        const int j = arena_insert(S, cn, zbc);  // index 0
+        bool fresh;
+        const int j = arena_insert(S, cn, zbc, fresh);  // index 0
         S.inmask[j] = full;
         const uint32_t p = full & ~zbc;
         if (p) { S.pending[j] = p; fifo_push(S, j); }
+        if (cut_on) *S.wsum = weight_fx(__ldg(c.a.g.weight + cn));
     }
     T.sync();
     // ---- backward closure, batch by batch (all pending nodes of a round in parallel)
     for (;;) {
         const int head = S.scal[SC_HEAD], tail = S.scal[SC_TAIL];
         if (head == tail || S.scal[SC_OVF]) break;
+        if (cut_on && __dmul_rn(c.a.dpow[depth], (double)*reinterpret_cast<volatile unsigned long long *>(S.wsum) *
+                                                     (1.0 / 16777216.0)) > cut) {
+            T.sync();
+            return CG_CUT;
+        }
         T.sync();
         for (int b0 = head; b0 < tail; b0 += ts) {
             int deg = 0;
@@ -1364,8 +1386,10 @@ __device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn,
                 const uint32_t pb = bz & S.b_P[o] & 0xFFu;   // Thm. V.4 arc for the keywords x needs here
                 if (!pb) continue;
                 const uint32_t zbu = bz >> 8;
-                const int j = arena_insert(S, u, zbu);
+                bool fresh;
+                const int j = arena_insert(S, u, zbu, fresh);
                 if (j < 0) continue;
+                if (fresh && cut_on) atomicAdd(S.wsum, (unsigned long long)weight_fx(__ldg(c.a.g.weight + u)));
                 const uint32_t old = atomicOr(S.inmask + j, pb);
                 const uint32_t nbits = pb & ~old & ~S.zb[j];
                 if (nbits) {
@@ -1384,7 +1408,7 @@ __device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn,
         T.sync();
     }
     T.sync();
-    if (S.scal[SC_OVF]) return false;
+    if (S.scal[SC_OVF]) return CG_OVERFLOW;
     const int nn = S.scal[SC_NODES];
     const int na = S.scal[SC_ARCS] < S.acap ? S.scal[SC_ARCS] : S.acap;
     // ---- level-cover
@@ -1432,7 +1456,7 @@ __device__ bool central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn,
     T.sync();
     *key = __dmul_rn(c.a.dpow[depth], *S.dsum);
     T.sync();
-    return true;
+    return CG_OK;
 }
 
 // team bitonic sort (ascending) of buf[0..len) padded to a power of two with ~0
@@ -1681,11 +1705,17 @@ __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
 // over a tier-1 arena in shared memory (most Central Graphs are small); (B) the larger ones, a whole CTA
 // per candidate over the CTA's shared region; (C) beyond that, the CTA's global-memory arena.
 // cflag: 0 = key from tier 1, 1 = from tier 2/3 (emitted by a CTA).
-__device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int32_t *list, uint32_t cnt, QOut *qo) {
+__device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int32_t *list, uint32_t cnt, QOut *qo,
+                             double cut = kNoCut) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
     Ctl *ctl = c.ctl;
-    if (G.gtid == 0) { ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->work_huge = 0; ctl->n_eval += cnt; }
+    const uint32_t multi = __ldcg(&ctl->multi_kw);
+    const double kInf = __longlong_as_double(0x7FF0000000000000ll);
+    if (G.gtid == 0) {
+        ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->work_huge = 0; ctl->work_huge2 = 0;
+        ctl->n_eval += cnt;
+    }
     G.sync();
     if ((threadIdx.x >> 5) < kExtWarps) {
         Arena S1 = carve(dsmem + kSmemArena * (threadIdx.x >> 5), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
@@ -1698,9 +1728,10 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
             const int32_t idx = list ? __ldcg(list + t) : (int32_t)t;
             const int32_t cn = __ldcg(c.w.centrals + idx);
             double key = 0.0;
-            const bool ok = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key);
+            const int st = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key, cut, multi);
             if (T.rank() == 0) {
-                if (ok) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
+                if (st == CG_OK) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
+                else if (st == CG_CUT) { c.w.ckey[idx] = kInf; c.w.cflag[idx] = 0; atomicAdd(&ctl->n_cut, 1u); }
                 else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = idx; }
             }
             __syncwarp();
@@ -1715,9 +1746,10 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         for (uint32_t t = G.grank; t < no; t += G.gcount) {
             const int32_t idx = __ldcg(c.w.overflow + t);
             double key = 0.0;
-            const bool ok = central_graph(BT, S2, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+            const int st = central_graph(BT, S2, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
             if (threadIdx.x == 0) {
-                if (ok) c.w.ckey[idx] = key;
+                if (st == CG_OK) c.w.ckey[idx] = key;
+                else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
                 else c.w.overflow[no + atomicAdd(&ctl->work_big, 1u)] = idx;
             }
             __syncthreads();
@@ -1725,29 +1757,49 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         G.sync();
         const uint32_t nbig = __ldcg(&ctl->work_big);
         if (nbig) {
-            Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+            Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true);
             for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
                 const int32_t idx = __ldcg(c.w.overflow + no + t);
                 double key = 0.0;
-                const bool ok = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+                const int st = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
                 if (threadIdx.x == 0) {
-                    if (ok) c.w.ckey[idx] = key;
+                    if (st == CG_OK) c.w.ckey[idx] = key;
+                    else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
                     else c.w.overflow[no + nbig + atomicAdd(&ctl->work_huge, 1u)] = idx;
                 }
                 __syncthreads();
             }
         }
         G.sync();
-        const uint32_t nhuge = __ldcg(&ctl->work_huge);
+        const uint32_t nlarge = __ldcg(&ctl->work_huge);
+        uint32_t nhuge = 0;
+        if (nlarge) {   // tier 3b: every CTA of the group over its large arena
+            Arena SL = carve(a.large_arenas + a.large_arena_bytes * blockIdx.x, a.large_hash, a.large_nodes,
+                             a.large_arcs, blockDim.x, false);
+            for (uint32_t t = G.grank; t < nlarge; t += G.gcount) {
+                const int32_t idx = __ldcg(c.w.overflow + no + nbig + t);
+                double key = 0.0;
+                const int st = central_graph(BT, SL, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
+                if (threadIdx.x == 0) {
+                    if (st == CG_OK) c.w.ckey[idx] = key;
+                    else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
+                    else c.w.overflow[no + nbig + nlarge + atomicAdd(&ctl->work_huge2, 1u)] = idx;
+                }
+                __syncthreads();
+            }
+            G.sync();
+            nhuge = __ldcg(&ctl->work_huge2);
+        }
         if (nhuge) {   // tier 4: the group's huge arena, one CTA
             if (G.grank == 0) {
-                Arena S4 = carve(c.w.huge, kHugeHash, kHugeNodes, kHugeArcs, blockDim.x, true);
+                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true);
                 for (uint32_t t = 0; t < nhuge; ++t) {
-                    const int32_t idx = __ldcg(c.w.overflow + no + nbig + t);
+                    const int32_t idx = __ldcg(c.w.overflow + no + nbig + nlarge + t);
                     double key = 0.0;
-                    const bool ok = central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key);
+                    const int st = central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
                     if (threadIdx.x == 0) {
-                        if (ok) c.w.ckey[idx] = key;
+                        if (st == CG_OK) c.w.ckey[idx] = key;
+                        else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
                         else atomicExch(&ctl->fatal, 2);
                     }
                     __syncthreads();
@@ -1792,15 +1844,15 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
             double key;
             const int32_t cn = __ldcg(c.w.centrals + idx);
             const int dep = __ldcg(c.w.cdepth + idx);
-            if (central_graph(T, S1, c, cn, dep, &key)) emit_graph(T, S1, c, (int)rk);   // tier 1
-            else if (central_graph(T, S, c, cn, dep, &key)) emit_graph(T, S, c, (int)rk);
+            if (central_graph(T, S1, c, cn, dep, &key) == CG_OK) emit_graph(T, S1, c, (int)rk);   // tier 1
+            else if (central_graph(T, S, c, cn, dep, &key) == CG_OK) emit_graph(T, S, c, (int)rk);
             else if (T.rank() == 0) atomicExch(&ctl->fatal, 3);
         }
     }
     G.sync();
     const uint32_t nbig = __ldcg(&ctl->work_big);
     if (nbig) {
-        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, kBigHash, kBigNodes, kBigArcs, blockDim.x, true);
+        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true);
         Arena S2 = carve(dsmem, kT2Hash, kT2Nodes, kT2Arcs, kBlock, false);
         S2.sortbuf = S.sortbuf;   // tier-2 closure in shared memory, its sort buffer in the CTA's global arena
         for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
@@ -1809,8 +1861,8 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
             const int32_t cn = __ldcg(c.w.centrals + idx);
             const int dep = __ldcg(c.w.cdepth + idx);
             double key;
-            if (central_graph(BT, S2, c, cn, dep, &key)) emit_graph(BT, S2, c, rk);
-            else if (central_graph(BT, S, c, cn, dep, &key)) emit_graph(BT, S, c, rk);
+            if (central_graph(BT, S2, c, cn, dep, &key) == CG_OK) emit_graph(BT, S2, c, rk);
+            else if (central_graph(BT, S, c, cn, dep, &key) == CG_OK) emit_graph(BT, S, c, rk);
             else if (threadIdx.x == 0) c.w.overflow[nbig + atomicAdd(&ctl->work_huge, 1u)] = rk;
             __syncthreads();
         }
@@ -1818,12 +1870,12 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
         const uint32_t nhuge = __ldcg(&ctl->work_huge);
         if (nhuge) {   // tier 4: the group's huge arena, one CTA
             if (G.grank == 0) {
-                Arena S4 = carve(c.w.huge, kHugeHash, kHugeNodes, kHugeArcs, blockDim.x, true);
+                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true);
                 for (uint32_t t = 0; t < nhuge; ++t) {
                     const int rk = __ldcg(c.w.overflow + nbig + t);
                     const int32_t idx = __ldcg(c.w.sel + rk);
                     double key;
-                    if (central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key))
+                    if (central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key) == CG_OK)
                         emit_graph(BT, S4, c, rk);
                     else if (threadIdx.x == 0) atomicExch(&ctl->fatal, 4);
                     __syncthreads();
@@ -1907,7 +1959,9 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
                 seed_pd(c, c.w.elist + m, n2);
                 pred_dag(c, S, sh, qo);
             }
-            extract_list(c, sh, dsmem, c.w.elist + m, n2, qo);
+            // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union)
+            const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
+            extract_list(c, sh, dsmem, c.w.elist + m, n2, qo, cut);
         }
         if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }
         if (m + n2 <= (uint32_t)KGS_MAX_K) {

@@ -81,6 +81,9 @@ struct Ctl {
     uint32_t pull_wait[2];         // [level parity] a pulled level without hits: some node is still on Alg. 2's work list
     uint32_t pull_wbig[2];         // [level parity] ... big nodes to check after the sweep
     uint32_t work_huge;            // Central Graphs beyond the CTA arenas (tier 4), this extract / emit pass
+    uint32_t multi_kw;             // union of the keyword sets of the nodes holding >= 2 query keywords
+    uint32_t n_cut;                // candidates stopped by the exact key cut-off (pruning round 2)
+    uint32_t work_huge2;           // ... beyond the per-CTA large arenas too (tier 4, one CTA of the group)
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -209,6 +212,11 @@ struct EngineArgs {
     char *warp_arenas;          // one per warp of the grid
     size_t warp_arena_bytes;
     char *cta_arenas;           // one per CTA (large-graph path)
+    char *large_arenas;         // one per CTA (tier 3b: up to large_nodes / large_arcs, no sort buffer)
+    size_t large_arena_bytes;
+    int large_hash, large_nodes, large_arcs;
+    int big_hash, big_nodes, big_arcs;      // tier 3 (cta_arenas), sized to the graph (at most kBig*)
+    int huge_hash, huge_nodes, huge_arcs;   // tier 4 (DevWork::huge), sized to the graph (at most kHuge*)
     size_t cta_arena_bytes;
 };
 

@@ -11,7 +11,7 @@ w = synth.make_workload("C4")
 G = kgs.kgs_load_graph(w.graph)
 for i in (int(x) for x in sys.argv[1:]):
     kw = w.queries[i]
-    for rec in ("1", "0"):
+    for rec in os.environ.get("RECS", "1,0").split(","):
         os.environ["KGS_DAG_RECORD"] = rec
         try:
             r = kgs.kgs_query(G, kw, w.k, kgs.make_params(prune=int(os.environ.get("PRUNE", "1"))))
