@@ -157,7 +157,7 @@ typedef struct {
     int32_t n_evaluated;   /* Central Graphs whose exact key was computed (|C| unless prune skipped some) */
     int64_t dag_arcs;      /* arcs the search traversed that hit their target: the Thm. V.4 arcs of all hit nodes */
     int32_t pull_level;    /* first level expanded by pull (kgs_params.direction), -1: push throughout */
-    int32_t pad_;
+    int32_t n_cut;         /* candidates whose extraction stopped at the exact key cut-off (prune round 2) */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index

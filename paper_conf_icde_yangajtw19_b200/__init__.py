@@ -62,7 +62,7 @@ class kgs_stats(ctypes.Structure):
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
                 ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64), ("pull_level", ctypes.c_int32),
-                ("pad_", ctypes.c_int32)]
+                ("n_cut", ctypes.c_int32)]
 
 
 class kgs_vp_buffers(ctypes.Structure):
@@ -252,7 +252,7 @@ def _read_result(h, n, q, want_levels) -> Result:
             answers.append(Answer(a.central, a.depth, a.score, a.score_key, nodes, arcs))
         st = kgs_stats()
         _check(L.kgs_result_stats(h, ctypes.byref(st)))
-        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_ if f != "pad_"}
+        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
         tags = np.zeros(64, np.int32)
         tns = np.zeros(64, np.uint64)
         nph = ctypes.c_int32()

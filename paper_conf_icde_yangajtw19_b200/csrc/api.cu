@@ -655,6 +655,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.n_evaluated = (int32_t)o.n_eval;
         st.group = o.group;
         st.pull_level = o.pull_level;
+        st.n_cut = o.n_cut;
         if (o.stop_reason != KGS_STOP_INVALID_QUERY && o.t_end >= o.t_start) {
             st.ms_search = (float)((double)(o.t_search_end - o.t_start) * 1e-6);
             st.ms_topdown = (float)((double)(o.t_end - o.t_search_end) * 1e-6);

@@ -2034,7 +2034,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             if (G.gtid == 0) {
                 QOut *qo = a.qout + qq.qi;
                 qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
-                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1;
+                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1; qo->n_cut = 0;
             }
             G.sync();
             continue;
@@ -2065,6 +2065,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->n_parcs = ctl->n_parcs;
             qo->n_eval = ctl->n_eval;
             qo->pull_level = ctl->pull_at - 1;
+            qo->n_cut = (int32_t)ctl->n_cut;
             qo->frontier_total = ctl->frontier_total;
             qo->arcs_scanned = ctl->arcs_scanned;
             qo->hits = ctl->hits;

@@ -94,7 +94,7 @@ struct QOut {
     unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
-    int32_t pull_level, pad2;      // first pulled level, -1: push throughout
+    int32_t pull_level, n_cut;     // first pulled level (-1: push throughout); key cut-offs
     unsigned long long stamp[kMaxStamps];
     int32_t stamp_tag[kMaxStamps];
 };

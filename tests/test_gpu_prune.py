@@ -178,3 +178,33 @@ def test_batch_pruned_matches_oracle():
                 bound = "path" if mode == 2 else "weight"
                 assert r.stats["n_evaluated"] == expected_evaluated(g, o, k, 0.2, kw, 512, bound), (kw, k, mode)
     G.close()
+
+
+def test_key_cutoff_in_round_two(monkeypatch):
+    """Round 2 stops a candidate's extraction once its closure weight times d^lambda exceeds the k-th
+    exact key (kgs_stats.n_cut).  Valid when level-cover must keep every source: no node holds two query
+    keywords (disjoint keyword sets here), or level_cover = 0.  Answers must be the oracle's."""
+    _gpu()
+    monkeypatch.setenv("KGS_PRUNE_MIN", "40")
+    cuts = 0
+    for seed, deg, k in ((0, 16, 5), (0, 16, 20), (1, 16, 5), (1, 16, 20), (0, 8, 50)):
+        rng = np.random.default_rng(500 + seed)
+        n, q = 6000, 3
+        g0 = medium_graph(500 + seed, n=n, deg=deg, q=q, kw_size=10, wpow=3.0)
+        perm = rng.permutation(n)
+        kws = [sorted(perm[i * 100:(i + 1) * 100].tolist()) for i in range(q)]   # disjoint
+        edges = [(u, int(v)) for u in range(n) for v in g0.col_idx[g0.row_ptr[u]:g0.row_ptr[u + 1]] if u < v]
+        g = synth.from_edges(n, edges, g0.weight, kws, 2.0)
+        G = kgs.kgs_load_graph(g)
+        kw = list(range(q))
+        for lc in (1, 0):
+            o = oracle.query(g, kw, k, level_cover=lc)
+            r = kgs.kgs_query(G, kw, k, kgs.make_params(prune=1, level_cover=lc))
+            ctx = f"seed={seed} deg={deg} k={k} lc={lc} |C|={len(o.centrals)}"
+            assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
+            for ra, oa in zip(r.answers, o.answers):
+                assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist(), ctx
+                assert ra.arcs.tolist() == oa.arcs.tolist(), ctx
+            cuts += r.stats["n_cut"]
+        G.close()
+    assert cuts > 0
