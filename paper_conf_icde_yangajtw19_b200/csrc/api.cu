@@ -187,6 +187,7 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.ckey, n));
     CUDA_TRY(dmalloc(&w.overflow, n));
     CUDA_TRY(cudaMalloc((void **)&w.huge, g->huge_arena_bytes));
+    CUDA_TRY(cudaMemset(w.huge, 0, g->huge_arena_bytes));   // persistent arena: not yet in a known state
     CUDA_TRY(dmalloc(&w.cflag, n));
     CUDA_TRY(dmalloc(&w.sel, KGS_MAX_K));
     CUDA_TRY(dmalloc(&w.elist, n));
@@ -387,6 +388,9 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     g->cta_arena_bytes = arena_bytes_host(g->big_hash, g->big_nodes, g->big_arcs, kBlock, true);
     G_TRY(cudaMalloc(&g->warp_arenas, g->warp_arena_bytes * (size_t)g->grid * (kBlock / 32)));
     G_TRY(cudaMalloc(&g->cta_arenas, g->cta_arena_bytes * (size_t)g->grid));
+    // persistent arenas (engine.cu carve): zero = "not yet reset", the first use resets fully
+    G_TRY(cudaMemset(g->warp_arenas, 0, g->warp_arena_bytes * (size_t)g->grid * (kBlock / 32)));
+    G_TRY(cudaMemset(g->cta_arenas, 0, g->cta_arena_bytes * (size_t)g->grid));
     {   // tier 3b: per-CTA arenas for Central Graphs beyond 64 K nodes, sized to the graph (at most 1 M nodes /
         // 4 M arcs, 88 MB per CTA at C3 scale)
         auto pow2 = [](int64_t x) { int64_t p = 1; while (p < x) p <<= 1; return p; };
@@ -395,6 +399,7 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         g->large_hash = 2 * g->large_nodes;
         g->large_arena_bytes = arena_bytes_host(g->large_hash, g->large_nodes, g->large_arcs, kBlock, false);
         G_TRY(cudaMalloc(&g->large_arenas, g->large_arena_bytes * (size_t)g->grid));
+        G_TRY(cudaMemset(g->large_arenas, 0, g->large_arena_bytes * (size_t)g->grid));
     }
     G_TRY(cudaDeviceSynchronize());
 #undef G_TRY

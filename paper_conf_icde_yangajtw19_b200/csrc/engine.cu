@@ -1218,18 +1218,24 @@ struct Arena {
     int32_t *scal;      // [SC_N]
     double *dsum;
     unsigned long long *wsum;     // closure weight so far, 2^-24 fixed point (key cut-off)
+    int32_t *hslot;     // [ncap] hash slot of node j (persistent arenas: lazy reset of the next use)
+    int32_t *magic;     // kArenaMagic once the arena has been fully reset (persistent arenas)
     int hcap, ncap, acap;
 };
 
-__host__ __device__ inline size_t arena_bytes(int hcap, int ncap, int acap, int team, bool with_sort) {
+// persistent: a global-memory arena that keeps its state between uses (and launches): the next use
+// resets only the hash slots and node rows the previous one touched, unless it overflowed.
+__host__ __device__ inline size_t arena_bytes(int hcap, int ncap, int acap, int team, bool with_sort,
+                                              bool persistent = false) {
     size_t b = 16 + sizeof(int64_t) * team + sizeof(double) + sizeof(unsigned long long);
+    if (persistent) b += sizeof(int32_t) * (size_t)ncap + 16;
     if (with_sort) b += sizeof(unsigned long long) * 2 * (size_t)acap;
     b += sizeof(int32_t) * 2 * (size_t)hcap + sizeof(int32_t) * 6 * (size_t)ncap + sizeof(int32_t) * 3 * (size_t)acap;
     b += sizeof(int32_t) * 3 * (size_t)team + sizeof(int32_t) * SC_N + 16;
     return (b + 255) & ~size_t(255);
 }
 size_t arena_bytes_host(int hcap, int ncap, int acap, int team, bool with_sort) {
-    return arena_bytes(hcap, ncap, acap, team, with_sort);
+    return arena_bytes(hcap, ncap, acap, team, with_sort, true);   // host-allocated arenas are persistent
 }
 
 // tier-1 (shared-memory) extraction arena of one warp: most Central Graphs are small
@@ -1244,10 +1250,17 @@ __device__ __forceinline__ char *align8(char *p) {
     return reinterpret_cast<char *>((reinterpret_cast<uintptr_t>(p) + 7) & ~uintptr_t(7));
 }
 
-__device__ Arena carve(char *p, int hcap, int ncap, int acap, int team, bool with_sort) {
+__device__ Arena carve(char *p, int hcap, int ncap, int acap, int team, bool with_sort, bool persistent = false) {
     Arena S;
     S.hcap = hcap; S.ncap = ncap; S.acap = acap;
     p = align8(p);
+    if (persistent) {
+        S.magic = reinterpret_cast<int32_t *>(p); p += 16;
+        S.hslot = reinterpret_cast<int32_t *>(p); p += sizeof(int32_t) * (size_t)ncap;
+    } else {
+        S.magic = nullptr;
+        S.hslot = nullptr;
+    }
     S.b_start = reinterpret_cast<int64_t *>(p); p += sizeof(int64_t) * team;
     S.dsum = reinterpret_cast<double *>(p); p += sizeof(double);
     S.wsum = reinterpret_cast<unsigned long long *>(p); p += sizeof(unsigned long long);
@@ -1287,6 +1300,7 @@ __device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu, b
             if (idx >= S.ncap) { atomicExch(S.scal + SC_OVF, 1); atomicExch(S.hval + h, -2); return -1; }
             S.id[idx] = u;
             S.zb[idx] = zbu;
+            if (S.hslot) S.hslot[idx] = (int32_t)h;
             __threadfence_block();
             atomicExch(S.hval + h, idx);
             fresh = true;
@@ -1316,14 +1330,30 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
 // with c's own keywords (multi = union of the keyword sets of all such nodes of the graph), or
 // level_cover = 0.  Then the closure weight so far, times d^lambda, is a lower bound of the key.
 enum { CG_OVERFLOW = 0, CG_OK = 1, CG_CUT = 2 };
+constexpr int32_t kArenaMagic = 0x4B475341;   // "KGSA": a persistent arena in a known state
 constexpr double kNoCut = __builtin_huge_val();
 template <class Team>
 __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, int depth, double *key,
                              double cut = kNoCut, uint32_t multi = 0u) {
     const uint32_t full = c.qq.full;
     const int r = T.rank(), ts = T.size();
-    for (int i = r; i < S.hcap; i += ts) { S.hkey[i] = -1; S.hval[i] = -1; }
-    for (int i = r; i < S.ncap; i += ts) { S.inmask[i] = 0; S.pending[i] = 0; S.keep[i] = 0; }
+    // reset: only what the previous use of a persistent arena touched (its node count is still in scal),
+    // everything after an overflow (its claimed slots were not recorded) or on first use
+    const int prev_nodes = S.magic ? S.scal[SC_NODES] : 0;
+    const bool lazy = S.magic && *S.magic == kArenaMagic && S.scal[SC_OVF] == 0 && prev_nodes <= S.ncap;
+    T.sync();
+    if (lazy) {
+        for (int j = r; j < prev_nodes; j += ts) {
+            const int h = S.hslot[j];
+            S.hkey[h] = -1; S.hval[h] = -1;
+            S.inmask[j] = 0; S.pending[j] = 0; S.keep[j] = 0;
+        }
+    } else {
+        for (int i = r; i < S.hcap; i += ts) { S.hkey[i] = -1; S.hval[i] = -1; }
+        for (int i = r; i < S.ncap; i += ts) { S.inmask[i] = 0; S.pending[i] = 0; S.keep[i] = 0; }
+        if (r == 0 && S.magic) *S.magic = kArenaMagic;
+    }
+    T.sync();
     if (r < SC_N) S.scal[r] = 0;
     if (r == 0) { *S.dsum = 0.0; *S.wsum = 0ull; }
     T.sync();
@@ -1757,7 +1787,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         G.sync();
         const uint32_t nbig = __ldcg(&ctl->work_big);
         if (nbig) {
-            Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true);
+            Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true, true);
             for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
                 const int32_t idx = __ldcg(c.w.overflow + no + t);
                 double key = 0.0;
@@ -1775,7 +1805,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         uint32_t nhuge = 0;
         if (nlarge) {   // tier 3b: every CTA of the group over its large arena
             Arena SL = carve(a.large_arenas + a.large_arena_bytes * blockIdx.x, a.large_hash, a.large_nodes,
-                             a.large_arcs, blockDim.x, false);
+                             a.large_arcs, blockDim.x, false, true);
             for (uint32_t t = G.grank; t < nlarge; t += G.gcount) {
                 const int32_t idx = __ldcg(c.w.overflow + no + nbig + t);
                 double key = 0.0;
@@ -1792,7 +1822,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         }
         if (nhuge) {   // tier 4: the group's huge arena, one CTA
             if (G.grank == 0) {
-                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true);
+                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true, true);
                 for (uint32_t t = 0; t < nhuge; ++t) {
                     const int32_t idx = __ldcg(c.w.overflow + no + nbig + nlarge + t);
                     double key = 0.0;
@@ -1821,7 +1851,7 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
     BlockTeam BT{sh};
     if ((threadIdx.x >> 5) < kExtWarps) {
         const int gwarp = (int)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5));
-        Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true);
+        Arena S = carve(a.warp_arenas + a.warp_arena_bytes * gwarp, kExtHash, kExtNodes, kExtArcs, 32, true, true);
         Arena S1 = carve(dsmem + kSmemArena * ((threadIdx.x >> 5) % kExtWarps), kT1Hash, kT1Nodes, kT1Arcs, 32, false);
         S1.sortbuf = S.sortbuf;   // tier-1 closure in shared memory, its sort buffer in the global arena
         WarpTeam T;
@@ -1852,7 +1882,7 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
     G.sync();
     const uint32_t nbig = __ldcg(&ctl->work_big);
     if (nbig) {
-        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true);
+        Arena S = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x, true, true);
         Arena S2 = carve(dsmem, kT2Hash, kT2Nodes, kT2Arcs, kBlock, false);
         S2.sortbuf = S.sortbuf;   // tier-2 closure in shared memory, its sort buffer in the CTA's global arena
         for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
@@ -1870,7 +1900,7 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
         const uint32_t nhuge = __ldcg(&ctl->work_huge);
         if (nhuge) {   // tier 4: the group's huge arena, one CTA
             if (G.grank == 0) {
-                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true);
+                Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true, true);
                 for (uint32_t t = 0; t < nhuge; ++t) {
                     const int rk = __ldcg(c.w.overflow + nbig + t);
                     const int32_t idx = __ldcg(c.w.sel + rk);
