@@ -295,7 +295,7 @@ def main():
         kgs.kgs_query_batch_fetch(G, qld.tolist(), sh)
     torch.cuda.synchronize(dev)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    stats, answers = [], []
+    stats, answers, subgraphs = [], [], []
     clk = ClockSampler(dev)
     clk.start()
     if dist:
@@ -311,14 +311,19 @@ def main():
         stats += [r.stats for r in res]
         if i == args.steps - 1:
             answers = [(qids[j], [(a.central, a.depth, a.score_key) for a in r.answers]) for j, r in zip(idx, res)]
+            subgraphs = [(qids[j], [(a.nodes, a.arcs) for a in r.answers]) for j, r in zip(idx, res)]
     gather_ms = 0.0
     if dist:
-        # NCCL all-gather of every rank's top-k headers (central, depth, key) of the last step
+        # NCCL all-gather of every rank's top-k headers (central, depth, key) and answer subgraphs
+        # (sizes, then a padded gather of the variable payloads) of the last step
         from paper_conf_icde_yangajtw19_b200 import dist as kd
         hdr = kd.pack_headers([q for q, _ in answers], [a for _, a in answers], w.k).to(cuda)
+        pidx, pdat = kd.pack_payloads([q for q, _ in subgraphs], [s_ for _, s_ in subgraphs])
+        pidx, pdat = pidx.to(cuda), pdat.to(cuda)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         kd.gather_headers(hdr, len(answers) * world, world)
+        kd.gather_payloads(pidx, pdat)
         e1.record(stream)
     torch.cuda.synchronize(dev)
     if dist:

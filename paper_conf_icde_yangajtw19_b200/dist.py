@@ -64,6 +64,52 @@ def merge_headers(gathered: torch.Tensor, k: int) -> dict:
     return res
 
 
+def pack_payloads(query_ids, answers_per_query) -> tuple:
+    """The answer subgraphs of this rank's queries as two flat int32 tensors: `index` rows (query id,
+    answer rank, #nodes, #arcs) and `data` = for each answer its nodes then its (pred, succ) arc pairs."""
+    idx, parts = [], []
+    for qid, answers in zip(query_ids, answers_per_query):
+        for j, (nodes, arcs) in enumerate(answers):
+            nodes = np.asarray(nodes, np.int32).reshape(-1)
+            arcs = np.asarray(arcs, np.int32).reshape(-1)
+            idx.append((int(qid), j, nodes.size, arcs.size // 2))
+            parts += [nodes, arcs]
+    index = torch.tensor(np.asarray(idx, np.int32).reshape(-1, 4))
+    data = torch.from_numpy(np.concatenate(parts) if parts else np.zeros(0, np.int32))
+    return index, data
+
+
+def gather_payloads(index: torch.Tensor, data: torch.Tensor, group=None) -> dict:
+    """Variable-size all-gather of every rank's packed subgraphs (sizes first, then one padded
+    all-gather of each tensor), unpacked to {query id: [(nodes, arcs), ...] in answer order}."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    dev = index.device
+    sizes = torch.tensor([index.shape[0], data.shape[0]], dtype=torch.int64, device=dev)
+    all_sizes = [torch.empty_like(sizes) for _ in range(world)]
+    dist.all_gather(all_sizes, sizes, group=group)
+    all_sizes = [tuple(int(x) for x in t.tolist()) for t in all_sizes]
+    mi, md = max(max(a for a, _ in all_sizes), 1), max(max(b for _, b in all_sizes), 1)
+    ipad = torch.zeros((mi, 4), dtype=torch.int32, device=dev)
+    dpad = torch.zeros(md, dtype=torch.int32, device=dev)
+    ipad[: index.shape[0]] = index
+    dpad[: data.shape[0]] = data
+    iout = [torch.empty_like(ipad) for _ in range(world)]
+    dout = [torch.empty_like(dpad) for _ in range(world)]
+    dist.all_gather(iout, ipad, group=group)
+    dist.all_gather(dout, dpad, group=group)
+    res = {}
+    for (ni, _), it, dt in zip(all_sizes, iout, dout):
+        it, dt = it.cpu().numpy(), dt.cpu().numpy()
+        off = 0
+        for qid, j, nn, na in it[:ni]:
+            nodes = dt[off: off + nn]
+            arcs = dt[off + nn: off + nn + 2 * na].reshape(-1, 2)
+            off += nn + 2 * na
+            res.setdefault(int(qid), []).append((int(j), nodes, arcs))
+    return {q: [(n, a) for _, n, a in sorted(v, key=lambda t: t[0])] for q, v in res.items()}
+
+
 def run_sharded(graph, queries, k: int, rank: int, world: int, params=None, group=None, device="cuda"):
     """Answer this rank's share of `queries` with libkgs and all-gather every rank's top-k headers.
     Returns (merged dict query id -> answers, local results)."""

@@ -1,5 +1,5 @@
 """World-size-2 gloo test (CPU) of the multi-GPU host logic: round-robin sharding, header packing,
-the all-gather and the merge by query id.  The per-query answers come from the oracle (test
+the all-gather and the merge by query id, and the variable-size gather of the answer subgraphs.  The per-query answers come from the oracle (test
 infrastructure), standing in for libkgs which needs a GPU."""
 import os
 import socket
@@ -39,8 +39,12 @@ def _worker(rank, world, port, out_q):
         local.append([(a.central, a.depth, a.key) for a in r.answers])
     hdr = kd.pack_headers(mine.tolist(), local, w.k)
     merged = kd.merge_headers(kd.gather_headers(hdr, len(qs), world), w.k)
+    # the answer subgraphs: sizes first, then a padded all-gather (variable payloads)
+    subs = [[(a.nodes, a.arcs) for a in oracle.query(w.graph, qs[qi], w.k).answers] for qi in mine]
+    index, data = kd.pack_payloads(mine.tolist(), subs)
+    payloads = kd.gather_payloads(index, data)
     if rank == 0:
-        out_q.put(merged)
+        out_q.put((merged, {q: [(n.tolist(), a.tolist()) for n, a in v] for q, v in payloads.items()}))
     dist.barrier()
     dist.destroy_process_group()
 
@@ -58,7 +62,7 @@ def test_sharded_gather_equals_single_process():
     procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
     for p in procs:
         p.start()
-    merged = q.get(timeout=300)
+    merged, payloads = q.get(timeout=300)
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
@@ -68,3 +72,6 @@ def test_sharded_gather_equals_single_process():
     for qi, kw in enumerate(qs):
         r = oracle.query(w.graph, kw, w.k)
         assert merged[qi] == [(a.central, a.depth, a.key) for a in r.answers]
+        got = payloads.get(qi, [])
+        assert [n for n, _ in got] == [a.nodes.tolist() for a in r.answers]
+        assert [x for _, x in got] == [a.arcs.reshape(-1, 2).tolist() for a in r.answers]
