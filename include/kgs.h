@@ -56,6 +56,9 @@ typedef enum {
 #define KGS_STOP_MAX_DEPTH 2      /* level reached params.max_depth (truncated) */
 #define KGS_STOP_EMPTY_KEYWORD 3  /* some T_i is empty: nothing can be central (reading R17) */
 #define KGS_STOP_INVALID_QUERY (-1) /* device batch only: q out of range, keyword id out of range or repeated */
+#define KGS_STOP_CAPACITY (-2)    /* batch only: the query exceeded an internal capacity (predecessor arcs,
+                                     extraction or answer arena); no answers, the rest of the batch is valid
+                                     (a single kgs_query returns KGS_EINTERNAL instead) */
 
 /* Graph description for kgs_load_graph (node-weighted graph stored as CSR).
  *   n_nodes     number of nodes, 0 <= n < 2^31.

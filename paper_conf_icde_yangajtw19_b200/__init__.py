@@ -81,6 +81,7 @@ EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
                "search_end", "extract", "extract_big", "select", "emit"]
 KGS_STOP_INVALID_QUERY = -1
+KGS_STOP_CAPACITY = -2
 
 _lib = None
 

@@ -434,8 +434,9 @@ kgs_status check_query(const kgs_graph *g, const int32_t *kw, int32_t q) {
     return KGS_OK;
 }
 
-// predecessor-arc capacity of a group workspace (KGS_PCAP_M: millions of arcs)
+// predecessor-arc capacity of a group workspace (KGS_PCAP_M: millions of arcs; KGS_PCAP_ARCS: arcs, tests)
 int64_t pcap_max() {
+    if (const char *a = std::getenv("KGS_PCAP_ARCS")) return std::max(1024ll, std::atoll(a));
     const char *e = std::getenv("KGS_PCAP_M");
     return (e ? std::max(1ll, std::atoll(e)) : 256ll) << 20;
 }
@@ -468,7 +469,8 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
         // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs; 20 B per arc):
         // 256 M (5.1 GB; KGS_PCAP_M) — the level-5 C4 queries record 192 M arcs, their pre-pass 135 M
         while ((int)g->works.size() < G) {
-            const int64_t pcap = std::max<int64_t>(std::min<int64_t>(g->m, pcap_max()), 1 << 20);
+            const int64_t pcap = std::getenv("KGS_PCAP_ARCS") ? pcap_max()
+                                                              : std::max<int64_t>(std::min<int64_t>(g->m, pcap_max()), 1 << 20);
             DevWork w;
             kgs_status st = alloc_work(g, w, pcap);
             if (st != KGS_OK) { free_work(w); return st; }
@@ -613,16 +615,14 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
     CUDA_TRY(cudaStreamSynchronize(s));
     float ms_all = 0.f;
     cudaEventElapsedTime(&ms_all, g->ev[0], g->ev[1]);
+    // a capacity overflow fails a single query; in a batch it marks that query (KGS_STOP_CAPACITY, no
+    // answers) and leaves the others
+    if (nq == 1 && g->h_qout[0].fatal)
+        return fail(KGS_EINTERNAL, "a query exceeded an internal capacity (code " +
+                                       std::to_string(g->h_qout[0].fatal) + ")");
     for (int j = 0; j < nq; ++j) {
-        const QOut &o = g->h_qout[j];
-        if (o.fatal) {
-            for (int t = 0; t < j; ++t) { delete results[t]; results[t] = nullptr; }
-            return fail(KGS_EINTERNAL, "a Central Graph exceeded the large-graph extractor capacity (query " +
-                                           std::to_string(j) + ", code " + std::to_string(o.fatal) + ")");
-        }
-    }
-    for (int j = 0; j < nq; ++j) {
-        const QOut &o = g->h_qout[j];
+        QOut &o = g->h_qout[j];
+        if (o.fatal) { o.stop_reason = KGS_STOP_CAPACITY; o.count = 0; }
         kgs_result *r = new kgs_result();
         r->n = g->n;
         r->q = g->last_q.empty() ? 0 : g->last_q[j];

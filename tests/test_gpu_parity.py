@@ -219,3 +219,30 @@ def test_huge_central_graph_tier4():
         assert rr.answers[0].central == c and rr.answers[0].nodes.tolist() == o.answers[0].nodes.tolist()
         assert rr.answers[0].arcs.tolist() == o.answers[0].arcs.tolist()
     G.close()
+
+
+def test_batch_capacity_overflow_is_per_query(monkeypatch):
+    """A query that exceeds an internal capacity (here the predecessor-arc regions, shrunk to 64 K arcs
+    with KGS_PCAP_ARCS, against a Central Graph of 150 000 predecessor arcs) is reported per query in a
+    batch (KGS_STOP_CAPACITY, no answers); the other queries of the batch keep their exact answers.
+    A single kgs_query reports KGS_EINTERNAL."""
+    _gpu()
+    monkeypatch.setenv("KGS_PCAP_ARCS", str(1 << 16))
+    n0 = 150_000
+    a, c = n0, n0 + 1
+    g = synth.from_edges(n0 + 2, [(v, c) for v in range(n0)] + [(a, c)], [0.0] * (n0 + 2),
+                         [list(range(n0)), [a]], 2.0)
+    G = kgs.kgs_load_graph(g)
+    qs = [[0, 1], [1], [1, 0], [1]]
+    res = kgs.kgs_query_batch(G, qs, 1, None, 2)
+    assert [r.stats["stop_reason"] for r in res] == [kgs.KGS_STOP_CAPACITY, kgs.KGS_STOP_K] * 2
+    for kw, r in zip(qs, res):
+        if kw == [1]:
+            o = oracle.query(g, kw, 1)
+            assert [(x.central, x.score_key, x.nodes.tolist()) for x in r.answers] == \
+                [(x.central, x.key, x.nodes.tolist()) for x in o.answers]
+        else:
+            assert r.answers == []
+    with pytest.raises(kgs.KgsError):
+        kgs.kgs_query(G, [0, 1], 1)
+    G.close()
