@@ -962,6 +962,11 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     // search ends by the level rule (no new hit at l >= amax) instead of the empty work-list
     bool pulling = false;
     const bool count_mf = a.direction == KGS_DIR_AUTO;
+    // the frontier's arcs are counted (two byte loads per frontier node in the merge, 2-3% of a query)
+    // only at levels that follow a frontier of more than n / (4 pull_ratio) nodes: a level cannot reach
+    // m / pull_ratio out-arcs from a frontier much smaller than that (the graph's mean degree is m / n),
+    // and level 0 (the keyword nodes) is never pulled in the automatic mode
+    bool count_lvl = false;
     unsigned long long my_mf = 0;
     for (int l = 0;; ++l) {
         // ---- enqueue frontiers: anything pending at this or a later level?
@@ -989,7 +994,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         auto merge_node = [&](int32_t v) {
                     // auto direction: out-arcs of the frontier nodes that can expand (a_v <= l, ln 4-7),
                     // bounded by the power of two of the class byte (no row_ptr load)
-                    if (count_mf && !pulling && (int)a.act[v] <= l)
+                    if (count_lvl && !pulling && (int)a.act[v] <= l)
                         my_mf += cls_deg_bound(a.g.cls[v]);
                     const uint32_t b = nm8[v];
                     if (!b) return false;
@@ -1017,11 +1022,11 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         };
         compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
                 &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
-        if (count_mf && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
+        if (count_lvl && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
         G.sync();
         if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.touched,
                              &ctl->n_touched, merge_node, merge_aux)) {
-            if (count_mf && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
+            if (count_lvl && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
             G.sync();
         }
         if (gtid == 0) {   // their last readers (level l - 1) passed the barrier above
@@ -1034,6 +1039,8 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         __syncthreads();
         const uint32_t c0 = s_ctl[0], c1 = s_ctl[1], nc = s_ctl[2];
         if (gtid == 0) ctl->frontier_total += (unsigned long long)c0 + c1;
+        const bool count_this = count_lvl;
+        count_lvl = count_mf && ((unsigned long long)c0 + c1) * 4ull * (unsigned long long)a.pull_ratio > (unsigned long long)n;
         // ---- termination (Def. 4 / Thm. V.3; reading R9: no expansion at d)
         if (empty) {   // some T_i is empty: M holds the initialisation, nothing can be central (R17)
             if (gtid == 0) { ctl->stop_reason = KGS_STOP_EMPTY_KEYWORD; ctl->levels = 0; }
@@ -1051,7 +1058,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         // slot s is consumed; nothing pushes to level l + R during this level (pushes reach <= max(l+1, amax))
         if (gtid == 0) ctl->slot_flag[s] = 0u;
         if (!pulling && (a.direction == KGS_DIR_PULL ||
-                         (count_mf && __ldcg(&ctl->mf[l & 1]) * (unsigned long long)a.pull_ratio > (unsigned long long)a.g.m &&
+                         (count_this && __ldcg(&ctl->mf[l & 1]) * (unsigned long long)a.pull_ratio > (unsigned long long)a.g.m &&
                           __ldcg(&ctl->mf[l & 1]) > (unsigned long long)a.pull_min))) {
             pulling = true;
             if (gtid == 0) ctl->pull_at = l + 1;
