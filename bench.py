@@ -250,8 +250,15 @@ def main():
     dist = None
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        # KGS_BENCH_ONE_GPU=1 (test of the multi-rank path on a one-GPU box): every rank on cuda:0 over
+        # gloo (NCCL refuses two ranks on one device); the collectives of dist.py stage through the host
+        if os.environ.get("KGS_BENCH_ONE_GPU") == "1":
+            local = 0
+            torch.cuda.set_device(0)
+            dist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = local
     torch.cuda.set_device(dev)
     cuda = f"cuda:{dev}"

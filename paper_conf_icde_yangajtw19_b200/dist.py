@@ -39,6 +39,8 @@ def gather_headers(local: torch.Tensor, n_total: int, world: int, group=None) ->
     padded to the same row count (query id -1) so one all_gather suffices."""
     import torch.distributed as dist
     rows = (n_total + world - 1) // world
+    if not _is_nccl(group):   # gloo: collectives on host tensors
+        local = local.cpu()
     pad = torch.full((rows, local.shape[1]), -1.0, dtype=local.dtype, device=local.device)
     pad[: local.shape[0]] = local
     outs = [torch.empty_like(pad) for _ in range(world)]
@@ -84,6 +86,8 @@ def gather_payloads(index: torch.Tensor, data: torch.Tensor, group=None) -> dict
     all-gather of each tensor), unpacked to {query id: [(nodes, arcs), ...] in answer order}."""
     import torch.distributed as dist
     world = dist.get_world_size(group)
+    if not _is_nccl(group):   # gloo: collectives on host tensors
+        index, data = index.cpu(), data.cpu()
     dev = index.device
     sizes = torch.tensor([index.shape[0], data.shape[0]], dtype=torch.int64, device=dev)
     all_sizes = [torch.empty_like(sizes) for _ in range(world)]
