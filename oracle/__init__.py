@@ -56,6 +56,8 @@ def _load():
         L.oracle_stats.argtypes = [vp, vp]
         L.oracle_answer.argtypes = [vp, i64] + [vp] * 8
         L.oracle_free.argtypes = [vp]
+        L.oracle_pair_distances.argtypes = [i64, vp, vp, i64, vp, vp, i32, vp, vp]
+        L.oracle_summary_weights.argtypes = [i64, vp, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -144,3 +146,27 @@ def query(g, kw_ids, k: int, *, alpha: float = 0.1, lam: float = 0.2, max_depth:
         return res
     finally:
         L.oracle_free(h)
+
+
+def pair_distances(row_ptr, col_idx, src, dst, max_hops: int = 254):
+    """P1: hop distance of each sampled pair by a plain BFS; (dist, mean)."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    ci = np.ascontiguousarray(col_idx, dtype=np.int32)
+    s = np.ascontiguousarray(src, dtype=np.int32)
+    d = np.ascontiguousarray(dst, dtype=np.int32)
+    out = np.empty(s.shape[0], np.int32)
+    mean = ctypes.c_double(0.0)
+    _load().oracle_pair_distances(int(rp.shape[0] - 1), rp.ctypes.data, ci.ctypes.data, int(s.shape[0]),
+                                  s.ctypes.data, d.ctypes.data, int(max_hops), out.ctypes.data, ctypes.byref(mean))
+    return out, float(mean.value)
+
+
+def summary_weights(in_row_ptr, in_label):
+    """P2, Eq. 2 + min-max normalisation; (w_norm float32, w_raw float64)."""
+    rp = np.ascontiguousarray(in_row_ptr, dtype=np.int64)
+    lab = np.ascontiguousarray(in_label, dtype=np.int32)
+    n = int(rp.shape[0] - 1)
+    wn = np.empty(n, np.float32)
+    wr = np.empty(n, np.float64)
+    _load().oracle_summary_weights(n, rp.ctypes.data, lab.ctypes.data, wn.ctypes.data, wr.ctypes.data)
+    return wn, wr
