@@ -6,7 +6,7 @@ NVFLAGS := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC \
 PKG := paper_conf_icde_yangajtw19_b200
 CSRC := $(PKG)/csrc
 LIB := $(PKG)/libkgs.so
-OBJS := $(CSRC)/api.o $(CSRC)/prep.o $(CSRC)/engine.o $(CSRC)/vpart.o $(CSRC)/relabel.o
+OBJS := $(CSRC)/api.o $(CSRC)/prep.o $(CSRC)/engine.o $(CSRC)/vpart.o $(CSRC)/relabel.o $(CSRC)/load.o
 
 all: $(LIB) oracle/liboracle.so synth/libkgs_synth.so
 

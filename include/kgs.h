@@ -270,6 +270,32 @@ kgs_status kgs_vp_waiting(kgs_graph *g, int32_t level, void *cuda_stream);
 kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centrals_dev, const uint8_t *depth_dev,
                           int32_t levels, int32_t stop_reason, void *cuda_stream, kgs_result **out);
 
+/* ---- Load-time preprocessing: the steps that produce kgs_load_graph's inputs.
+ * Both run on the raw CSR before kgs_load_graph, on `device`, on `cuda_stream` (NULL = default),
+ * and return when their host outputs are written.  Inputs are host pointers (copied) unless
+ * flags & KGS_INPUT_DEVICE_PTRS (borrowed device pointers).  KGS_EINVAL for malformed sizes.     */
+
+/* A, "the average shortest distance (hops) between two nodes ... by sampling" (Table II and
+ * 10^4 sampled pairs).  dist[j] = number of arcs of a shortest src[j] -> dst[j] path along
+ * out-arcs (0 when src == dst), or -1 when dst is not reached within max_hops (1..254) hops.
+ * *mean = the mean of the reachable dist[j] (fp64), or NaN when none is.  row_ptr [n+1] int64,
+ * col_idx [n_arcs] int32 (out-arcs), src/dst [n_pairs] int32 in [0, n); dist [n_pairs] host output,
+ * mean host output (may be NULL).  Pairs are answered 64 at a time by one bit-parallel BFS.      */
+kgs_status kgs_prep_pair_distances(int64_t n_nodes, int64_t n_arcs, const int64_t *row_ptr,
+                                   const int32_t *col_idx, int32_t n_pairs, const int32_t *src,
+                                   const int32_t *dst, int32_t max_hops, int32_t device, int32_t flags,
+                                   void *cuda_stream, int32_t *dist, double *mean);
+
+/* Eq. 2 degree of summary: for node v with in-arc label multiset R_v, where n_r is
+ * the number of in-arcs of label r,  w_v = sum_r n_r log2(1 + n_r) / sum_r n_r  (fp64; 0 for a node
+ * without in-arcs, reading R25), then w'_v = (w_v - min w) / (max w - min w) (0 for every
+ * node when max = min, reading R26).  in_row_ptr [n+1] int64, in_label [n_in_arcs] int32 (any order within a
+ * row).  w_norm [n] host output (float, the kgs_graph_desc.weight input); w_raw [n] host output
+ * (fp64, may be NULL).                                                                            */
+kgs_status kgs_prep_summary_weights(int64_t n_nodes, int64_t n_in_arcs, const int64_t *in_row_ptr,
+                                    const int32_t *in_label, int32_t device, int32_t flags,
+                                    void *cuda_stream, float *w_norm, double *w_raw);
+
 /* Thread-local message describing the last non-OK status of this thread. */
 const char *kgs_last_error(void);
 

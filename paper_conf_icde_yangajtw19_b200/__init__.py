@@ -76,7 +76,7 @@ EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query
             "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_phases",
             "kgs_result_free", "kgs_last_error", "kgs_version", "kgs_query_batch", "kgs_query_batch_device",
             "kgs_query_batch_fetch", "kgs_vp_slice", "kgs_vp_begin", "kgs_vp_level", "kgs_vp_waiting",
-            "kgs_vp_topdown"]
+            "kgs_vp_topdown", "kgs_prep_pair_distances", "kgs_prep_summary_weights"]
 
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
                "search_end", "extract", "extract_big", "select", "emit"]
@@ -141,6 +141,10 @@ def lib():
         L.kgs_vp_waiting.restype = i32
         L.kgs_vp_topdown.argtypes = [vp, i64, vp, vp, i32, i32, vp, ctypes.POINTER(vp)]
         L.kgs_vp_topdown.restype = i32
+        L.kgs_prep_pair_distances.argtypes = [i64, i64, vp, vp, i32, vp, vp, i32, i32, i32, vp, vp, vp]
+        L.kgs_prep_pair_distances.restype = i32
+        L.kgs_prep_summary_weights.argtypes = [i64, i64, vp, vp, i32, i32, vp, vp, vp]
+        L.kgs_prep_summary_weights.restype = i32
         L.kgs_version.argtypes = []
         L.kgs_version.restype = ctypes.c_char_p
         _lib = L
@@ -372,3 +376,35 @@ def kgs_vp_topdown(graph: Graph, n_central: int, cent_ptr: int, dep_ptr: int, le
     _check(lib().kgs_vp_topdown(graph.handle, int(n_central), ctypes.c_void_p(cent_ptr), ctypes.c_void_p(dep_ptr),
                                 int(levels), int(stop_reason), ctypes.c_void_p(stream), ctypes.byref(h)))
     return _read_result(h, graph.n, int(q), want_levels)
+
+
+# ---- load-time preprocessing: the inputs kgs_load_graph takes ----
+def kgs_prep_pair_distances(row_ptr, col_idx, src, dst, max_hops: int = 254, device: int = 0,
+                            stream: int = 0) -> tuple:
+    """Hop distances of sampled (src, dst) pairs along out-arcs, and their mean over the reachable
+    pairs: A of P:L184 / P:L524.  Returns (dist int32 [n_pairs], -1 = unreachable; mean)."""
+    rp = np.ascontiguousarray(np.asarray(row_ptr, dtype=np.int64))
+    ci = np.ascontiguousarray(np.asarray(col_idx, dtype=np.int32))
+    s = np.ascontiguousarray(np.asarray(src, dtype=np.int32))
+    d = np.ascontiguousarray(np.asarray(dst, dtype=np.int32))
+    if s.shape != d.shape:
+        raise ValueError("src and dst differ in length")
+    out = np.empty(s.shape[0], np.int32)
+    mean = ctypes.c_double(0.0)
+    _check(lib().kgs_prep_pair_distances(int(rp.shape[0] - 1), int(ci.shape[0]), rp.ctypes.data, ci.ctypes.data,
+                                         int(s.shape[0]), s.ctypes.data, d.ctypes.data, int(max_hops), int(device),
+                                         0, ctypes.c_void_p(stream), out.ctypes.data, ctypes.byref(mean)))
+    return out, float(mean.value)
+
+
+def kgs_prep_summary_weights(in_row_ptr, in_label, device: int = 0, stream: int = 0) -> tuple:
+    """Eq. 2 degree of summary from the in-arc labels, min-max normalised.
+    Returns (w_norm float32 [n], w_raw float64 [n])."""
+    rp = np.ascontiguousarray(np.asarray(in_row_ptr, dtype=np.int64))
+    lab = np.ascontiguousarray(np.asarray(in_label, dtype=np.int32))
+    n = int(rp.shape[0] - 1)
+    wn = np.empty(n, np.float32)
+    wr = np.empty(n, np.float64)
+    _check(lib().kgs_prep_summary_weights(n, int(lab.shape[0]), rp.ctypes.data, lab.ctypes.data, int(device), 0,
+                                          ctypes.c_void_p(stream), wn.ctypes.data, wr.ctypes.data))
+    return wn, wr

@@ -220,6 +220,10 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
 
 }  // namespace
 
+namespace kgs {
+kgs_status set_error(kgs_status s, const std::string &msg) { return fail(s, msg); }
+}  // namespace kgs
+
 extern "C" {
 
 const char *kgs_last_error(void) { return g_err.c_str(); }
