@@ -2,8 +2,8 @@
 // with oracle/).  Produces the inputs kgs_load_graph takes: the normalised node weight w' (Eq. 2 and
 // min-max) and the sampled average distance A (Table II).
 //
-//   k_dist_push / k_dist_update   bit-parallel BFS: 64 (src, dst) pairs per pass, one bit of a
-//                                 uint64 per pair in the visited / frontier words of every node.
+//   k_dist_push / k_dist_update   bit-parallel BFS: 128 (src, dst) pairs per pass, one bit per pair
+//                                 in a node's visited / next words (one 32-byte sector per node).
 //   k_summary                     Eq. 2 per node over its in-arc labels sorted per row (cub segmented
 //                                 sort), one warp per node, runs of equal labels found by ballots.
 //   k_normalise                   w' = (w - min) / (max - min).
@@ -35,65 +35,84 @@ namespace {
 
 // ---------------------------------------------------------------- pair distances (A by sampling)
 
+// Node state of a pass: one 32-byte sector per node, {visited[2], next[2]} (128 pair bits each), so
+// the per-arc gather of the push touches one sector; the frontier words cur[2] are read sequentially.
+struct alignas(32) PairState {
+    unsigned long long vis0, vis1, nxt0, nxt1;
+};
+
 // Push one level: every node u with frontier bits f = cur[u] ORs f & ~vis[x] into nxt[x] for each
 // out-arc u -> x.  A warp takes 32 consecutive nodes and scans the arcs of each active one together
 // (coalesced col_idx reads; hubs do not serialise a thread).
 __global__ void k_dist_push(const int64_t *__restrict__ rp, const int32_t *__restrict__ ci, int64_t n,
-                            const unsigned long long *__restrict__ cur, const unsigned long long *__restrict__ vis,
-                            unsigned long long *__restrict__ nxt) {
+                            const ulonglong2 *__restrict__ cur, PairState *__restrict__ st) {
     const int lane = threadIdx.x & 31;
     const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t base = warp0 * 32; base < n; base += nwarps * 32) {
         const int64_t v = base + lane;
-        const unsigned long long f = v < n ? cur[v] : 0ull;
-        unsigned act = __ballot_sync(0xffffffffu, f != 0ull);
+        const ulonglong2 f = v < n ? cur[v] : make_ulonglong2(0ull, 0ull);
+        unsigned act = __ballot_sync(0xffffffffu, (f.x | f.y) != 0ull);
         while (act) {
             const int src = __ffs(act) - 1;
             act &= act - 1;
-            const unsigned long long fu = __shfl_sync(0xffffffffu, f, src);
+            const unsigned long long f0 = __shfl_sync(0xffffffffu, f.x, src);
+            const unsigned long long f1 = __shfl_sync(0xffffffffu, f.y, src);
             const int64_t u = base + src;
             const int64_t b = rp[u], e = rp[u + 1];
             for (int64_t j = b + lane; j < e; j += 32) {
-                const int32_t x = ci[j];
-                const unsigned long long m = fu & ~vis[x];
-                if (m && (nxt[x] & m) != m) atomicOr(&nxt[x], m);
+                PairState *px = st + ci[j];
+                const ulonglong2 vn = *reinterpret_cast<const ulonglong2 *>(&px->vis0);
+                const ulonglong2 nx = *reinterpret_cast<const ulonglong2 *>(&px->nxt0);
+                const unsigned long long m0 = f0 & ~vn.x, m1 = f1 & ~vn.y;
+                if (m0 && (nx.x & m0) != m0) atomicOr(&px->nxt0, m0);
+                if (m1 && (nx.y & m1) != m1) atomicOr(&px->nxt1, m1);
             }
         }
     }
 }
 
-// New frontier = nxt & ~vis; vis |= it; nxt cleared.  any = 1 if some bit is new.
-__global__ void k_dist_update(int64_t n, unsigned long long *__restrict__ cur, unsigned long long *__restrict__ vis,
-                              unsigned long long *__restrict__ nxt, int32_t *any) {
+// New frontier = next & ~visited; visited |= it; next cleared.  any = 1 if some bit is new.
+__global__ void k_dist_update(int64_t n, ulonglong2 *__restrict__ cur, PairState *__restrict__ st, int32_t *any) {
     int found = 0;
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned long long x = nxt[v];
-        const unsigned long long nw = x & ~vis[v];
-        cur[v] = nw;
-        if (x) nxt[v] = 0ull;
-        if (nw) { vis[v] |= nw; found = 1; }
+        PairState p = st[v];
+        const unsigned long long n0 = p.nxt0 & ~p.vis0, n1 = p.nxt1 & ~p.vis1;
+        cur[v] = make_ulonglong2(n0, n1);
+        if (p.nxt0 | p.nxt1) {
+            p.vis0 |= n0;
+            p.vis1 |= n1;
+            p.nxt0 = p.nxt1 = 0ull;
+            st[v] = p;
+            found |= (n0 | n1) != 0ull;
+        }
     }
     if (__syncthreads_or(found) && threadIdx.x == 0) *any = 1;
+}
+
+__device__ __forceinline__ bool pair_bit(const PairState &p, int j) {
+    return j < 64 ? ((p.vis0 >> j) & 1ull) : ((p.vis1 >> (j - 64)) & 1ull);
 }
 
 // Pair j of the batch (bit j): when its target's visited word first shows bit j, its distance is l.
 // done counts the resolved pairs.
 __global__ void k_dist_check(const int32_t *__restrict__ dst, int32_t cnt, int32_t level,
-                             const unsigned long long *__restrict__ vis, int32_t *__restrict__ dist, int32_t *done) {
+                             const PairState *__restrict__ st, int32_t *__restrict__ dist, int32_t *done) {
     const int j = threadIdx.x;
-    if (j < cnt && dist[j] < 0 && ((vis[dst[j]] >> j) & 1ull)) {
+    if (j < cnt && dist[j] < 0 && pair_bit(st[dst[j]], j)) {
         dist[j] = level;
         atomicAdd(done, 1);
     }
 }
 
-__global__ void k_dist_seed(const int32_t *__restrict__ src, int32_t cnt, unsigned long long *cur,
-                            unsigned long long *vis) {
+__global__ void k_dist_seed(const int32_t *__restrict__ src, int32_t cnt, ulonglong2 *cur, PairState *st) {
     const int j = threadIdx.x;
     if (j < cnt) {
-        atomicOr(&cur[src[j]], 1ull << j);
-        atomicOr(&vis[src[j]], 1ull << j);
+        const unsigned long long bit = 1ull << (j & 63);
+        unsigned long long *c = j < 64 ? &cur[src[j]].x : &cur[src[j]].y;
+        unsigned long long *vz = j < 64 ? &st[src[j]].vis0 : &st[src[j]].vis1;
+        atomicOr(c, bit);
+        atomicOr(vz, bit);
     }
 }
 
@@ -109,6 +128,8 @@ __global__ void k_check_rows(const int64_t *__restrict__ rp, int64_t n, int64_t 
         if (v < n && rp[v + 1] < rp[v]) atomicOr(err, 1);
     }
 }
+
+constexpr int kPairs = 128;   // pairs per bit-parallel BFS pass
 
 int grid_for(int64_t items, int block) {
     int64_t g = (items + block - 1) / block;
@@ -196,7 +217,8 @@ kgs_status kgs_prep_pair_distances(int64_t n, int64_t m, const int64_t *row_ptr,
     cudaStream_t s = (cudaStream_t)cuda_stream;
     int64_t *d_rp = nullptr, *o_rp = nullptr;
     int32_t *d_ci = nullptr, *o_ci = nullptr, *d_src = nullptr, *o_src = nullptr, *d_dst = nullptr, *o_dst = nullptr;
-    unsigned long long *cur = nullptr, *vis = nullptr, *nxt = nullptr;
+    ulonglong2 *cur = nullptr;
+    PairState *pst = nullptr;
     int32_t *ctl = nullptr, *h_ctl = nullptr, *d_dist = nullptr;   // ctl: [0] err, [1] any, [2] done
     std::vector<int32_t> out((size_t)n_pairs, -1);
     double sum = 0.0;
@@ -208,7 +230,7 @@ kgs_status kgs_prep_pair_distances(int64_t n, int64_t m, const int64_t *row_ptr,
     LD_TRY(stage(dst, (int64_t)n_pairs, dev, s, &d_dst, &o_dst));
     LD_TRY(cudaMallocAsync((void **)&ctl, 4 * sizeof(int32_t), s));
     LD_TRY(cudaMallocHost((void **)&h_ctl, 4 * sizeof(int32_t)));
-    LD_TRY(cudaMallocAsync((void **)&d_dist, 64 * sizeof(int32_t), s));
+    LD_TRY(cudaMallocAsync((void **)&d_dist, kPairs * sizeof(int32_t), s));
     LD_TRY(cudaMemsetAsync(ctl, 0, 4 * sizeof(int32_t), s));
     k_check_rows<<<grid_for(n + 1, 256), 256, 0, s>>>(d_rp, n, m, ctl);
     if (m > 0) k_check_ids<<<grid_for(m, 256), 256, 0, s>>>(d_ci, m, n, ctl);
@@ -221,30 +243,28 @@ kgs_status kgs_prep_pair_distances(int64_t n, int64_t m, const int64_t *row_ptr,
     LD_TRY(cudaStreamSynchronize(s));
     if (h_ctl[0]) { st = set_error(KGS_EINVAL, "kgs_prep_pair_distances: malformed row_ptr or id out of range"); goto done; }
     if (n_pairs > 0) {
-        LD_TRY(cudaMallocAsync((void **)&cur, sizeof(unsigned long long) * (size_t)n, s));
-        LD_TRY(cudaMallocAsync((void **)&vis, sizeof(unsigned long long) * (size_t)n, s));
-        LD_TRY(cudaMallocAsync((void **)&nxt, sizeof(unsigned long long) * (size_t)n, s));
-        LD_TRY(cudaMemsetAsync(nxt, 0, sizeof(unsigned long long) * (size_t)n, s));
+        LD_TRY(cudaMallocAsync((void **)&cur, sizeof(ulonglong2) * (size_t)n, s));
+        LD_TRY(cudaMallocAsync((void **)&pst, sizeof(PairState) * (size_t)n, s));
     }
-    for (int32_t p0 = 0; p0 < n_pairs; p0 += 64) {
-        const int32_t cnt = n_pairs - p0 < 64 ? n_pairs - p0 : 64;
-        LD_TRY(cudaMemsetAsync(cur, 0, sizeof(unsigned long long) * (size_t)n, s));
-        LD_TRY(cudaMemsetAsync(vis, 0, sizeof(unsigned long long) * (size_t)n, s));
-        LD_TRY(cudaMemsetAsync(d_dist, 0xFF, 64 * sizeof(int32_t), s));
+    for (int32_t p0 = 0; p0 < n_pairs; p0 += kPairs) {
+        const int32_t cnt = n_pairs - p0 < kPairs ? n_pairs - p0 : kPairs;
+        LD_TRY(cudaMemsetAsync(cur, 0, sizeof(ulonglong2) * (size_t)n, s));
+        LD_TRY(cudaMemsetAsync(pst, 0, sizeof(PairState) * (size_t)n, s));
+        LD_TRY(cudaMemsetAsync(d_dist, 0xFF, kPairs * sizeof(int32_t), s));
         LD_TRY(cudaMemsetAsync(ctl + 2, 0, sizeof(int32_t), s));
-        k_dist_seed<<<1, 64, 0, s>>>(d_src + p0, cnt, cur, vis);
-        k_dist_check<<<1, 64, 0, s>>>(d_dst + p0, cnt, 0, vis, d_dist, ctl + 2);
+        k_dist_seed<<<1, kPairs, 0, s>>>(d_src + p0, cnt, cur, pst);
+        k_dist_check<<<1, kPairs, 0, s>>>(d_dst + p0, cnt, 0, pst, d_dist, ctl + 2);
         for (int32_t l = 1; l <= max_hops; ++l) {
             LD_TRY(cudaMemsetAsync(ctl + 1, 0, sizeof(int32_t), s));
-            k_dist_push<<<grid_for(n, 256), 256, 0, s>>>(d_rp, d_ci, n, cur, vis, nxt);
-            k_dist_update<<<grid_for(n, 256), 256, 0, s>>>(n, cur, vis, nxt, ctl + 1);
-            k_dist_check<<<1, 64, 0, s>>>(d_dst + p0, cnt, l, vis, d_dist, ctl + 2);
+            k_dist_push<<<grid_for(n, 256), 256, 0, s>>>(d_rp, d_ci, n, cur, pst);
+            k_dist_update<<<grid_for(n, 256), 256, 0, s>>>(n, cur, pst, ctl + 1);
+            k_dist_check<<<1, kPairs, 0, s>>>(d_dst + p0, cnt, l, pst, d_dist, ctl + 2);
             LD_TRY(cudaGetLastError());
             LD_TRY(cudaMemcpyAsync(h_ctl + 1, ctl + 1, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, s));
             LD_TRY(cudaStreamSynchronize(s));
             if (!h_ctl[1] || h_ctl[2] == cnt) break;   // frontier empty or every pair of the batch answered
         }
-        // a batch that stopped early leaves nxt clean (update cleared it) and cur/vis are reset above
+        // every pass starts from zeroed cur / state (reset above)
         LD_TRY(cudaMemcpyAsync(out.data() + p0, d_dist, sizeof(int32_t) * (size_t)cnt, cudaMemcpyDeviceToHost, s));
         LD_TRY(cudaStreamSynchronize(s));
     }
@@ -255,8 +275,7 @@ kgs_status kgs_prep_pair_distances(int64_t n, int64_t m, const int64_t *row_ptr,
     if (mean) *mean = reach ? sum / (double)reach : NAN;
 done:
     if (cur) cudaFreeAsync(cur, s);
-    if (vis) cudaFreeAsync(vis, s);
-    if (nxt) cudaFreeAsync(nxt, s);
+    if (pst) cudaFreeAsync(pst, s);
     if (ctl) cudaFreeAsync(ctl, s);
     if (d_dist) cudaFreeAsync(d_dist, s);
     if (o_rp) cudaFreeAsync(o_rp, s);

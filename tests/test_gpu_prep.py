@@ -1,7 +1,8 @@
 """Load-time preprocessing through the C-ABI vs the oracle.
 
 kgs_prep_pair_distances: bit-exact integer distances (and the mean computed from them) on small
-graphs with ragged batches (not a multiple of the 64 pairs one BFS pass carries), unreachable pairs,
+graphs with ragged batches (not a multiple of the 128 pairs one BFS pass carries; bits 0-63 and
+64-127 live in different words), unreachable pairs,
 src == dst, duplicate pairs, a max_hops cut-off, and a 1M-node R-MAT graph (config C2's) with 150
 sampled pairs.  kgs_prep_summary_weights: Eq. 2 in fp64 — the raw w within 1e-13 relative (log2 is
 1-ulp on both sides, the run sums are exact integers) and w' within 1e-6 absolute — on random
@@ -36,7 +37,8 @@ def _rand_graph(rng, n, p, directed=True):
 
 
 @pytest.mark.parametrize("seed,n,p,pairs", [(0, 50, 0.04, 1), (1, 300, 0.01, 64), (2, 200, 0.02, 65),
-                                            (3, 500, 0.005, 201)])
+                                            (3, 500, 0.005, 201), (4, 400, 0.008, 128), (5, 400, 0.008, 129),
+                                            (6, 600, 0.004, 300)])
 def test_pair_distances_small(seed, n, p, pairs):
     _gpu()
     rng = np.random.default_rng(seed)
