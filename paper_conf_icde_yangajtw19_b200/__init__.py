@@ -408,3 +408,27 @@ def kgs_prep_summary_weights(in_row_ptr, in_label, device: int = 0, stream: int 
     _check(lib().kgs_prep_summary_weights(n, int(lab.shape[0]), rp.ctypes.data, lab.ctypes.data, int(device), 0,
                                           ctypes.c_void_p(stream), wn.ctypes.data, wr.ctypes.data))
     return wn, wr
+
+
+def kgs_prep_pair_distances_device(n_nodes: int, n_arcs: int, row_ptr_ptr: int, col_idx_ptr: int, n_pairs: int,
+                                   src_ptr: int, dst_ptr: int, max_hops: int = 254, device: int = 0,
+                                   stream: int = 0) -> tuple:
+    """kgs_prep_pair_distances with borrowed device inputs (KGS_INPUT_DEVICE_PTRS)."""
+    out = np.empty(int(n_pairs), np.int32)
+    mean = ctypes.c_double(0.0)
+    _check(lib().kgs_prep_pair_distances(int(n_nodes), int(n_arcs), ctypes.c_void_p(row_ptr_ptr),
+                                         ctypes.c_void_p(col_idx_ptr), int(n_pairs), ctypes.c_void_p(src_ptr),
+                                         ctypes.c_void_p(dst_ptr), int(max_hops), int(device), KGS_INPUT_DEVICE_PTRS,
+                                         ctypes.c_void_p(stream), out.ctypes.data, ctypes.byref(mean)))
+    return out, float(mean.value)
+
+
+def kgs_prep_summary_weights_device(n_nodes: int, n_in_arcs: int, in_row_ptr_ptr: int, in_label_ptr: int,
+                                    device: int = 0, stream: int = 0) -> tuple:
+    """kgs_prep_summary_weights with borrowed device inputs (KGS_INPUT_DEVICE_PTRS)."""
+    wn = np.empty(int(n_nodes), np.float32)
+    wr = np.empty(int(n_nodes), np.float64)
+    _check(lib().kgs_prep_summary_weights(int(n_nodes), int(n_in_arcs), ctypes.c_void_p(in_row_ptr_ptr),
+                                          ctypes.c_void_p(in_label_ptr), int(device), KGS_INPUT_DEVICE_PTRS,
+                                          ctypes.c_void_p(stream), wn.ctypes.data, wr.ctypes.data))
+    return wn, wr

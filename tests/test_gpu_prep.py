@@ -117,3 +117,26 @@ def test_summary_weights_c2_and_hub():
     assert np.allclose(wr, wr_o, rtol=1e-13, atol=0)
     assert np.abs(wn - wn_o).max() <= 1e-6
     assert wn[-1] == wn_o[-1]
+
+
+def test_device_pointer_inputs():
+    """KGS_INPUT_DEVICE_PTRS: the same answers from borrowed device buffers, on a non-default stream."""
+    _gpu()
+    import torch
+    rng = np.random.default_rng(9)
+    rp, ci = _rand_graph(rng, 400, 0.01, directed=False)
+    s = rng.integers(0, 400, 150).astype(np.int32)
+    t = rng.integers(0, 400, 150).astype(np.int32)
+    want, wmean = oracle.pair_distances(rp, ci, s, t)
+    dev = [torch.from_numpy(x).cuda() for x in (rp, ci, s, t)]
+    st = torch.cuda.Stream()
+    got, gmean = kgs.kgs_prep_pair_distances_device(400, ci.shape[0], dev[0].data_ptr(), dev[1].data_ptr(), 150,
+                                                    dev[2].data_ptr(), dev[3].data_ptr(), stream=st.cuda_stream)
+    assert got.tolist() == want.tolist() and gmean == wmean
+    lab = _labels(rng, ci.shape[0], 7)
+    wn_o, wr_o = oracle.summary_weights(rp, lab)
+    dl = torch.from_numpy(lab).cuda()
+    wn, wr = kgs.kgs_prep_summary_weights_device(400, lab.shape[0], dev[0].data_ptr(), dl.data_ptr(),
+                                                 stream=st.cuda_stream)
+    assert np.allclose(wr, wr_o, rtol=1e-13, atol=0) and np.abs(wn - wn_o).max() <= 1e-6
+    assert (dev[1].cpu().numpy() == ci).all()          # borrowed inputs are not modified
