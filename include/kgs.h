@@ -75,7 +75,10 @@ typedef enum {
  *   device      CUDA device ordinal the graph lives on.
  *   flags       KGS_INPUT_DEVICE_PTRS | KGS_NO_RELABEL, or 0.  The library stores the graph with its
  *               nodes renumbered by non-increasing degree (ties by input id) unless KGS_NO_RELABEL is
- *               set; results are identical (every id returned is the input id, ties rank by input id). */
+ *               set; results are identical (every id returned is the input id, ties rank by input id).
+ *   pred_arc_cap  capacity, in arcs, of each query workspace's predecessor-arc buffers (the Thm. V.4 arcs
+ *               of the top-down, 20 B each); 0 = min(n_arcs, 2^28), at least 2^20.  A query whose
+ *               predecessor DAG exceeds it reports KGS_STOP_CAPACITY (batch) / KGS_EINTERNAL (single). */
 typedef struct {
     int64_t n_nodes, n_arcs;
     const int64_t *row_ptr;
@@ -88,6 +91,7 @@ typedef struct {
     int32_t symmetric;
     int32_t device;
     int32_t flags;
+    int64_t pred_arc_cap;
 } kgs_graph_desc;
 
 typedef struct kgs_graph kgs_graph;   /* opaque: device CSR (+ reverse), weights, index, workspace */
@@ -113,20 +117,30 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *                       and block_central = 1 it falls back to 1.
  *   direction      expansion direction of Alg. 2 (the north star's push/pull switching):
  *                    KGS_DIR_AUTO (0, default)  push; from the first level whose frontier has more than
- *                                   m / pull_ratio and more than pull_min out-arcs (m = all arcs;
- *                                   pull_ratio 14, pull_min 2^22 unless the environment variables
- *                                   KGS_PULL_RATIO / KGS_PULL_MIN say otherwise) on, pull;
+ *                                   m / pull_ratio and more than pull_min out-arcs (m = all arcs) on, pull;
  *                    KGS_DIR_PUSH (1)  push only: the frontier nodes scan their out-arcs (Alg. 2 as written);
  *                    KGS_DIR_PULL (2)  pull at every level: every node x that still lacks a keyword and whose
  *                                   gate is open scans its in-arcs for active neighbours (the level rule,
  *                                   SURVEY.md §8(c) O3).
  *                  Results do not depend on it (M, central set, depths, answers, stop level and reason):
  *                  after a pulled level without hits the engine recomputes whether Alg. 2's work list
- *                  would still hold a node (an inactive hit node, or one waiting for a gated neighbour). */
+ *                  would still hold a node (an inactive hit node, or one waiting for a gated neighbour).
+ * Engine tuning (results never depend on these; kgs_params_default sets the defaults in brackets):
+ *   pull_ratio     >= 1 [14]: the auto direction pulls once the frontier's out-arcs exceed m / pull_ratio
+ *   pull_min       >= 0 [2^22]: ... and exceed pull_min
+ *   prune_min      >= 1 [512]: pruning round 1 extracts min(4096, max(8k, prune_min)) candidates
+ *   tile_light     >= 0 [4096]: light frontiers of at most this many nodes are expanded by group-wide tiles
+ *   dag_record     -1 [auto: on for single-query launches] / 0 / 1: the top-down's predecessor lists come
+ *                  from the arcs the search recorded (1) or from the in-arc pre-pass (0); the recorded DAG
+ *                  is used only where it is exact (extract_mode EXACT, or block_central 0)
+ *   search_only    0 [0] / 1: workload analysis — stop after the search (no top-down, no answers) */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
     int32_t direction;
+    int32_t pull_ratio;
+    int64_t pull_min;
+    int32_t prune_min, tile_light, dag_record, search_only;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 
@@ -161,6 +175,7 @@ typedef struct {
     int64_t dag_arcs;      /* arcs the search traversed that hit their target: the Thm. V.4 arcs of all hit nodes */
     int32_t pull_level;    /* first level expanded by pull (kgs_params.direction), -1: push throughout */
     int32_t n_cut;         /* candidates whose extraction stopped at the exact key cut-off (prune round 2) */
+    int32_t n_tier4;       /* Central Graphs extracted in the per-group tier-4 arena (beyond the per-CTA arenas) */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index
@@ -280,18 +295,20 @@ kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centra
  * out-arcs (0 when src == dst), or -1 when dst is not reached within max_hops (1..254) hops.
  * *mean = the mean of the reachable dist[j] (fp64), or NaN when none is.  row_ptr [n+1] int64,
  * col_idx [n_arcs] int32 (out-arcs), src/dst [n_pairs] int32 in [0, n); dist [n_pairs] host output,
- * mean host output (may be NULL).  Pairs are answered 64 at a time by one bit-parallel BFS.      */
+ * mean host output (may be NULL).  Pairs are answered 128 at a time by one bit-parallel BFS.     */
 kgs_status kgs_prep_pair_distances(int64_t n_nodes, int64_t n_arcs, const int64_t *row_ptr,
                                    const int32_t *col_idx, int32_t n_pairs, const int32_t *src,
                                    const int32_t *dst, int32_t max_hops, int32_t device, int32_t flags,
                                    void *cuda_stream, int32_t *dist, double *mean);
 
 /* Eq. 2 degree of summary: for node v with in-arc label multiset R_v, where n_r is
- * the number of in-arcs of label r,  w_v = sum_r n_r log2(1 + n_r) / sum_r n_r  (fp64; 0 for a node
- * without in-arcs, reading R25), then w'_v = (w_v - min w) / (max w - min w) (0 for every
- * node when max = min, reading R26).  in_row_ptr [n+1] int64, in_label [n_in_arcs] int32 (any order within a
- * row).  w_norm [n] host output (float, the kgs_graph_desc.weight input); w_raw [n] host output
- * (fp64, may be NULL).                                                                            */
+ * the number of in-arcs of label r,  w_v = sum_r n_r log2(1 + n_r) / sum_r n_r  (fp64, the terms added
+ * in ascending label order), then w'_v = (w_v - min w) / (max w - min w) over the nodes WITH in-arcs
+ * (P:L184).  A node without in-arcs summarises nothing: w' = 0, raw w reported as 0, and it takes no
+ * part in the min / max (reading R6).  Every w' is 0 when max = min (R26).  w' is produced on the
+ * 2^-24 grid: the nearest grid point of the fp64 value, ties up (R27), so kgs_load_graph's snap keeps it.
+ * in_row_ptr [n+1] int64, in_label [n_in_arcs] int32 (any order within a row).  w_norm [n] host output
+ * (float, the kgs_graph_desc.weight input); w_raw [n] host output (fp64, may be NULL).              */
 kgs_status kgs_prep_summary_weights(int64_t n_nodes, int64_t n_in_arcs, const int64_t *in_row_ptr,
                                     const int32_t *in_label, int32_t device, int32_t flags,
                                     void *cuda_stream, float *w_norm, double *w_raw);

@@ -42,8 +42,10 @@ def _load():
         L = ctypes.CDLL(_LIB_PATH)
         vp, i64, i32, dbl = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_double
         L.oracle_query.restype = vp
-        L.oracle_query.argtypes = [i64, vp, vp, vp, i64, vp, vp, dbl, i32, vp, i32, i64, dbl, dbl, i32, i32, i32, i32, i32]
+        L.oracle_query.argtypes = [i64, vp, vp, vp, i64, vp, vp, dbl, i32, vp, i32, i64, dbl, dbl, i32, i32, i32, i32, i32,
+                                   vp, i64]
         L.oracle_activation.argtypes = [i64, vp, dbl, dbl, vp]
+        L.oracle_snap_weights.argtypes = [i64, vp, vp]
         for f in ("oracle_a", "oracle_M", "oracle_centrals", "oracle_central_depth", "oracle_central_key"):
             getattr(L, f).restype = vp
             getattr(L, f).argtypes = [vp]
@@ -60,6 +62,16 @@ def _load():
         L.oracle_summary_weights.argtypes = [i64, vp, vp, vp, vp]
         _lib = L
     return _lib
+
+
+def snap_weights(weight: np.ndarray) -> np.ndarray:
+    """O0 (reading R15): every weight to the nearest point of the 2^-24 grid, ties up.  ``query`` applies
+    it before the activation map and the score."""
+    L = _load()
+    w = np.ascontiguousarray(weight, np.float32)
+    out = np.empty(w.shape[0], np.float32)
+    L.oracle_snap_weights(w.shape[0], w.ctypes.data, out.ctypes.data)
+    return out
 
 
 def activation(weight: np.ndarray, A: float, alpha: float) -> np.ndarray:
@@ -96,9 +108,11 @@ class Result:
 
 def query(g, kw_ids, k: int, *, alpha: float = 0.1, lam: float = 0.2, max_depth: int = 254,
           block_central: int = 1, extract_mode: int = EXTRACT_EXACT, bfs_form: int = BFS_LITERAL,
-          level_cover: int = 1) -> Result:
+          level_cover: int = 1, eval_ids=None) -> Result:
     """One query through the oracle.  ``g`` is a synth.Graph-like object (row_ptr, col_idx, weight,
-    kw_ptr, kw_nodes, A, symmetric)."""
+    kw_ptr, kw_nodes, A, symmetric).  ``eval_ids`` (test sampling at sizes where scoring every central
+    node is out of reach): only these central nodes are extracted and scored (the others' keys are NaN)
+    and the answers rank them alone."""
     L = _load()
     kw = np.ascontiguousarray(np.asarray(kw_ids, dtype=np.int32))
     q = int(kw.shape[0])
@@ -108,10 +122,12 @@ def query(g, kw_ids, k: int, *, alpha: float = 0.1, lam: float = 0.2, max_depth:
     kp = np.ascontiguousarray(g.kw_ptr, np.int64)
     kn = np.ascontiguousarray(g.kw_nodes, np.int32)
     n = rp.shape[0] - 1
+    ev = None if eval_ids is None else np.ascontiguousarray(np.asarray(eval_ids, dtype=np.int32))
     h = L.oracle_query(n, rp.ctypes.data, ci.ctypes.data, w.ctypes.data, kp.shape[0] - 1, kp.ctypes.data,
                        kn.ctypes.data, float(g.A), 1 if g.symmetric else 0, kw.ctypes.data, q, int(k),
                        float(alpha), float(lam), int(max_depth), int(block_central), int(extract_mode),
-                       int(bfs_form), int(level_cover))
+                       int(bfs_form), int(level_cover), None if ev is None else ev.ctypes.data,
+                       0 if ev is None else int(ev.shape[0]))
     try:
         st = L.oracle_status(h)
         if st != 0:

@@ -38,14 +38,16 @@ class kgs_graph_desc(ctypes.Structure):
                 ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("weight", ctypes.c_void_p),
                 ("n_keywords", ctypes.c_int64), ("kw_ptr", ctypes.c_void_p), ("kw_nodes", ctypes.c_void_p),
                 ("avg_dist_A", ctypes.c_double), ("symmetric", ctypes.c_int32), ("device", ctypes.c_int32),
-                ("flags", ctypes.c_int32)]
+                ("flags", ctypes.c_int32), ("pred_arc_cap", ctypes.c_int64)]
 
 
 class kgs_params(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_double), ("lambda_", ctypes.c_double), ("max_depth", ctypes.c_int32),
                 ("block_central", ctypes.c_int32), ("extract_mode", ctypes.c_int32),
                 ("level_cover", ctypes.c_int32), ("want_levels", ctypes.c_int32), ("prune", ctypes.c_int32),
-                ("direction", ctypes.c_int32)]
+                ("direction", ctypes.c_int32), ("pull_ratio", ctypes.c_int32), ("pull_min", ctypes.c_int64),
+                ("prune_min", ctypes.c_int32), ("tile_light", ctypes.c_int32), ("dag_record", ctypes.c_int32),
+                ("search_only", ctypes.c_int32)]
 
 
 class kgs_answer(ctypes.Structure):
@@ -62,7 +64,7 @@ class kgs_stats(ctypes.Structure):
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
                 ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64), ("pull_level", ctypes.c_int32),
-                ("n_cut", ctypes.c_int32)]
+                ("n_cut", ctypes.c_int32), ("n_tier4", ctypes.c_int32)]
 
 
 class kgs_vp_buffers(ctypes.Structure):
@@ -163,12 +165,19 @@ def kgs_params_default() -> kgs_params:
 
 
 def make_params(alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=KGS_EXTRACT_EXACT,
-                level_cover=1, want_levels=0, prune=1, direction=0) -> kgs_params:
+                level_cover=1, want_levels=0, prune=1, direction=0, **tuning) -> kgs_params:
+    """kgs_params from the defaults; ``tuning`` sets engine-tuning fields by name (pull_ratio, pull_min,
+    prune_min, tile_light, dag_record, search_only)."""
     p = kgs_params_default()
     p.alpha, p.lambda_, p.max_depth = float(alpha), float(lam), int(max_depth)
     p.block_central, p.extract_mode = int(block_central), int(extract_mode)
     p.level_cover, p.want_levels, p.prune = int(level_cover), int(want_levels), int(prune)
     p.direction = int(direction)
+    names = {f for f, _ in kgs_params._fields_}
+    for k, v in tuning.items():
+        if k not in names:
+            raise TypeError(f"unknown kgs_params field {k}")
+        setattr(p, k, int(v))
     return p
 
 
@@ -192,7 +201,7 @@ class Graph:
             pass
 
 
-def kgs_load_graph(g, device: int = 0, relabel: bool = True) -> Graph:
+def kgs_load_graph(g, device: int = 0, relabel: bool = True, pred_arc_cap: int = 0) -> Graph:
     """Load a graph given as host numpy arrays (attributes row_ptr, col_idx, weight, kw_ptr, kw_nodes,
     A, symmetric — e.g. a synth.Graph).  relabel=False sets KGS_NO_RELABEL (keep the input node order
     internally; results are identical either way)."""
@@ -203,20 +212,22 @@ def kgs_load_graph(g, device: int = 0, relabel: bool = True) -> Graph:
     kn = np.ascontiguousarray(g.kw_nodes, np.int32)
     d = kgs_graph_desc(rp.shape[0] - 1, ci.shape[0], rp.ctypes.data, ci.ctypes.data, w.ctypes.data,
                        kp.shape[0] - 1, kp.ctypes.data, kn.ctypes.data if kn.size else None, float(g.A),
-                       1 if getattr(g, "symmetric", True) else 0, int(device), 0 if relabel else KGS_NO_RELABEL)
+                       1 if getattr(g, "symmetric", True) else 0, int(device), 0 if relabel else KGS_NO_RELABEL,
+                       int(pred_arc_cap))
     h = ctypes.c_void_p()
     _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
     return Graph(h, rp.shape[0] - 1, kp.shape[0] - 1)
 
 
 def kgs_load_graph_device(n, n_arcs, row_ptr_ptr, col_idx_ptr, weight_ptr, n_keywords, kw_ptr_ptr, kw_nodes_ptr,
-                          A: float, symmetric: bool = True, device: int = 0, relabel: bool = True) -> Graph:
+                          A: float, symmetric: bool = True, device: int = 0, relabel: bool = True,
+                          pred_arc_cap: int = 0) -> Graph:
     """Load a graph whose arrays already live in device memory (KGS_INPUT_DEVICE_PTRS): raw device
     pointers (e.g. torch CUDA tensors' data_ptr()), int64 row_ptr / kw_ptr, int32 col_idx / kw_nodes,
     float32 weight.  The library copies them; the caller keeps ownership."""
     d = kgs_graph_desc(int(n), int(n_arcs), row_ptr_ptr, col_idx_ptr, weight_ptr, int(n_keywords), kw_ptr_ptr,
                        kw_nodes_ptr, float(A), 1 if symmetric else 0, int(device),
-                       KGS_INPUT_DEVICE_PTRS | (0 if relabel else KGS_NO_RELABEL))
+                       KGS_INPUT_DEVICE_PTRS | (0 if relabel else KGS_NO_RELABEL), int(pred_arc_cap))
     h = ctypes.c_void_p()
     _check(lib().kgs_load_graph(ctypes.byref(d), ctypes.byref(h)))
     return Graph(h, int(n), int(n_keywords))

@@ -75,6 +75,7 @@ struct kgs_graph {
     uint8_t *cls = nullptr, *cls_in = nullptr;
     int32_t *orig = nullptr, *perm = nullptr;   // internal <-> input ids (relabel.cu); null: identity
     int64_t n_big = 0, n_big_in = 0;   // nodes with more than kBigDeg out- / in-arcs
+    int64_t pred_arc_cap = 0;          // kgs_graph_desc.pred_arc_cap (0 = default)
     // per-alpha / per-lambda caches
     uint8_t *act = nullptr;
     uint32_t *amax_dev = nullptr;
@@ -170,14 +171,15 @@ void free_work(DevWork &w) {
     w = DevWork{};
 }
 
-// one group's workspace, sized for the graph (fbits for the current R)
+// one group's workspace, sized for the graph (fbits for the largest level ring any group was given:
+// every workspace of the graph holds R_alloc slots, so a later alpha with R <= R_alloc fits all of them)
 kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     const int64_t n = g->n;
     w = DevWork{};
     CUDA_TRY(dmalloc(&w.st, n));
     CUDA_TRY(dmalloc(&w.nm, (n + 3) / 4));
     CUDA_TRY(dmalloc(&w.M, n * 8));
-    CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max(g->R, 2) * (size_t)g->W));
+    CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max({g->R_alloc, g->R, 2}) * (size_t)g->W));
     CUDA_TRY(dmalloc(&w.qlight, n));
     CUDA_TRY(dmalloc(&w.qbig, g->n_big));
     CUDA_TRY(dmalloc(&w.touched, n));
@@ -241,6 +243,12 @@ void kgs_params_default(kgs_params *p) {
     p->want_levels = 0;
     p->prune = 1;
     p->direction = KGS_DIR_AUTO;
+    p->pull_ratio = 14;
+    p->pull_min = 1ll << 22;
+    p->prune_min = 512;
+    p->tile_light = 8 * kBlock;
+    p->dag_record = -1;
+    p->search_only = 0;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -268,6 +276,7 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
         d->n_keywords < 1 || !(d->avg_dist_A > 0.0) || !std::isfinite(d->avg_dist_A))
         return fail(KGS_EINVAL, "n_nodes / n_arcs / n_keywords / avg_dist_A out of range");
     if (d->n_nodes > 0 && (!d->row_ptr || !d->weight)) return fail(KGS_EINVAL, "missing row_ptr / weight");
+    if (d->pred_arc_cap < 0) return fail(KGS_EINVAL, "pred_arc_cap must be >= 0");
     if (d->n_arcs > 0 && !d->col_idx) return fail(KGS_EINVAL, "missing col_idx");
     if (!d->kw_ptr || !d->row_ptr) return fail(KGS_EINVAL, "missing kw_ptr / row_ptr");
     int ndev = 0;
@@ -297,6 +306,7 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     kgs_graph *g = new kgs_graph();
     g->device = d->device; g->n = n; g->m = m; g->n_kw = V; g->A = d->avg_dist_A;
     g->symmetric = d->symmetric ? 1 : 0;
+    g->pred_arc_cap = d->pred_arc_cap;
     auto bail = [&](kgs_status s) { kgs_free_graph(g); return s; };
 #define G_TRY(expr)                                                                          \
     do {                                                                                     \
@@ -425,6 +435,10 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
         return fail(KGS_EINVAL, "extract_mode");
     if (p.prune < 0 || p.prune > 2) return fail(KGS_EINVAL, "prune must be 0, 1 or 2");
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
+    if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
+        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1))
+        return fail(KGS_EINVAL, "tuning parameters out of range (pull_ratio >= 1, pull_min >= 0, prune_min >= 1, "
+                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1)");
     return KGS_OK;
 }
 
@@ -438,11 +452,11 @@ kgs_status check_query(const kgs_graph *g, const int32_t *kw, int32_t q) {
     return KGS_OK;
 }
 
-// predecessor-arc capacity of a group workspace (KGS_PCAP_M: millions of arcs; KGS_PCAP_ARCS: arcs, tests)
-int64_t pcap_max() {
-    if (const char *a = std::getenv("KGS_PCAP_ARCS")) return std::max(1024ll, std::atoll(a));
-    const char *e = std::getenv("KGS_PCAP_M");
-    return (e ? std::max(1ll, std::atoll(e)) : 256ll) << 20;
+// predecessor-arc capacity of a group workspace (kgs_graph_desc.pred_arc_cap; default min(m, 2^28),
+// at least 2^20: the level-5 C4 queries record 192 M arcs, their pre-pass 135 M)
+int64_t pcap_of(const kgs_graph *g) {
+    if (g->pred_arc_cap > 0) return std::max<int64_t>(1024, g->pred_arc_cap);
+    return std::max<int64_t>(std::min<int64_t>(g->m, 1ll << 28), 1 << 20);
 }
 
 // per-alpha activation cache, level-slot ring, per-lambda depth factors, G group workspaces
@@ -458,29 +472,26 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
         g->R = g->amax + 2;
         invalidate = true;
     }
-    if (g->R > g->R_alloc) {   // bigger ring: reallocate every group's bitmaps
+    if (std::max(g->R, 2) > g->R_alloc) {   // bigger ring: reallocate every group's bitmaps
         CUDA_TRY(cudaStreamSynchronize(s));
+        g->R_alloc = std::max(g->R, 2);
         for (auto &w : g->works) {
             cudaFree(w.fbits);
             w.fbits = nullptr;
-            CUDA_TRY(dmalloc(&w.fbits, (size_t)g->R * (size_t)g->W));
+            CUDA_TRY(dmalloc(&w.fbits, (size_t)g->R_alloc * (size_t)g->W));
         }
-        g->R_alloc = g->R;
         invalidate = true;
     }
     if ((int)g->works.size() < G) {
         CUDA_TRY(cudaStreamSynchronize(s));
-        // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs; 20 B per arc):
-        // 256 M (5.1 GB; KGS_PCAP_M) — the level-5 C4 queries record 192 M arcs, their pre-pass 135 M
+        // predecessor-arc capacity per group (recorded search arcs, or pre-pass arcs; 20 B per arc)
         while ((int)g->works.size() < G) {
-            const int64_t pcap = std::getenv("KGS_PCAP_ARCS") ? pcap_max()
-                                                              : std::max<int64_t>(std::min<int64_t>(g->m, pcap_max()), 1 << 20);
+            const int64_t pcap = pcap_of(g);
             DevWork w;
             kgs_status st = alloc_work(g, w, pcap);
             if (st != KGS_OK) { free_work(w); return st; }
             g->works.push_back(w);
         }
-        g->R_alloc = std::max(g->R_alloc, std::max(g->R, 2));
         if (g->works_dev) cudaFree(g->works_dev);
         if (g->bars) cudaFree(g->bars);
         CUDA_TRY(dmalloc(&g->works_dev, g->works.size()));
@@ -518,7 +529,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
         const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
-                           (size_t)std::min<int64_t>(g->m, pcap_max()) * 20 +
+                           (size_t)pcap_of(g) * 20 +
                            g->huge_arena_bytes;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
         G = std::max(1, (int)g->works.size() + more);
@@ -549,34 +560,20 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     // arcs the search traversed: exact extraction, or no central blocking.
     a.prune = p.want_levels ? 0 : p.prune;
     if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
-    {
-        const char *e = std::getenv("KGS_PRUNE_MIN");
-        a.prune_min = e ? std::max(1, std::atoi(e)) : 512;
-    }
+    a.prune_min = p.prune_min;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
-        // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass
-        // Default: on for the single-query (latency) launch, where the pre-pass's rounds of group barriers
+        // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass.
+        // Auto: on for the single-query (latency) launch, where the pre-pass's rounds of group barriers
         // dominate; off for query groups, where the pre-pass's targeted work (closures of the top
         // candidates only) is less total work than building every touched node's list.
-        const char *e = std::getenv("KGS_DAG_RECORD");   // ablation knob: 0 off, 1 on, unset auto
-        const bool on = e ? std::atoi(e) != 0 : G == 1;
+        const bool on = p.dag_record < 0 ? G == 1 : p.dag_record != 0;
         a.dag_record = on && !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     }
     a.direction = p.direction;
-    {
-        const char *e = std::getenv("KGS_SEARCH_ONLY");   // workload analysis only: no answers, stats of the search
-        a.search_only = e && std::atoi(e) ? 1 : 0;
-    }
-    {
-        const char *e = std::getenv("KGS_PULL_RATIO");   // auto direction: pull once frontier arcs > m / ratio
-        a.pull_ratio = e ? std::max(1, std::atoi(e)) : 14;
-        const char *f = std::getenv("KGS_PULL_MIN");     // ... and exceed this many (small graphs never pull)
-        a.pull_min = f ? std::atoll(f) : (1ll << 22);
-    }
-    {
-        const char *e = std::getenv("KGS_TILE_LIGHT");   // ablation knob (nodes); default 8 tiles
-        a.tile_light = e ? std::atoi(e) : 8 * kBlock;
-    }
+    a.search_only = p.search_only;
+    a.pull_ratio = p.pull_ratio;
+    a.pull_min = p.pull_min;
+    a.tile_light = p.tile_light;
     a.qout = g->d_qout; a.out_hdr = g->d_hdr; a.out_key = g->d_key; a.out_off = g->d_off;
     a.out_nodes = g->d_nodes; a.out_arcs = g->d_arcs;
     a.out_nodes_cap = (long long)g->d_nodes_cap; a.out_arcs_cap = (long long)(g->d_arcs_cap / 2);
@@ -611,7 +608,9 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
     CUDA_TRY(cudaMemcpyAsync(g->h_ctr, g->d_ctr, 4 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     g->pending = false;
-    const size_t used_n = (size_t)g->h_ctr[1], used_a = (size_t)g->h_ctr[2];
+    // the arena counters never pass their capacity (engine.cu arena_reserve); clamp anyway
+    const size_t used_n = std::min<size_t>((size_t)g->h_ctr[1], g->d_nodes_cap);
+    const size_t used_a = std::min<size_t>((size_t)g->h_ctr[2], g->d_arcs_cap / 2);
     CUDA_TRY(grow_pinned(&g->h_nodes, &g->h_nodes_cap, std::max<size_t>(used_n, 1)));
     CUDA_TRY(grow_pinned(&g->h_arcs, &g->h_arcs_cap, std::max<size_t>(2 * used_a, 1)));
     if (used_n) CUDA_TRY(cudaMemcpyAsync(g->h_nodes, g->d_nodes, sizeof(int32_t) * used_n, cudaMemcpyDeviceToHost, s));
@@ -662,6 +661,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.td_arcs = (int64_t)o.td_arcs;
         st.td_pred_arcs = o.n_parcs;
         st.n_evaluated = (int32_t)o.n_eval;
+        st.n_tier4 = (int32_t)o.n_tier4;
         st.group = o.group;
         st.pull_level = o.pull_level;
         st.n_cut = o.n_cut;

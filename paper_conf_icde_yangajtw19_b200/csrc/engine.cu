@@ -384,7 +384,6 @@ __device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool
 
 constexpr int kTileMax = kBlock;
 constexpr int kBigUnroll = 4;
-constexpr uint32_t kTileLight = 8;   // light frontiers of at most 8 tiles also go through the tile path
 #ifndef KGS_LIGHT_UNROLL
 #define KGS_LIGHT_UNROLL 4
 #endif
@@ -1517,6 +1516,19 @@ __device__ void team_sort(const Team &T, unsigned long long *buf, int len) {
         }
 }
 
+// Reserve cnt entries of an answer arena without ever moving its counter past cap: a reservation that
+// does not fit fails (-1) and leaves the counter as it was, so later (smaller) answers still fit and only
+// the overflowing query is marked (KGS_STOP_CAPACITY).
+__device__ __forceinline__ long long arena_reserve(unsigned long long *ctr, unsigned long long cnt, long long cap) {
+    unsigned long long cur = atomicAdd(ctr, 0ull);
+    for (;;) {
+        if (cur + cnt > (unsigned long long)cap) return -1;
+        const unsigned long long prev = atomicCAS(ctr, cur, cur + cnt);
+        if (prev == cur) return (long long)cur;
+        cur = prev;
+    }
+}
+
 // write the kept nodes / arcs of the arena (after central_graph) sorted and unique, as answer `rank_i`
 template <class Team>
 __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
@@ -1532,11 +1544,11 @@ __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
     const int kn = S.scal[SC_NOUT];
     team_sort(T, S.sortbuf, kn);
     const int64_t ans = (int64_t)c.qq.qi * a.k + rank_i;
-    if (r == 0) S.b_start[0] = (int64_t)atomicAdd(a.out_used + 0, (unsigned long long)kn);   // team broadcast
+    if (r == 0) S.b_start[0] = arena_reserve(a.out_used + 0, (unsigned long long)kn, a.out_nodes_cap);   // team broadcast
     T.sync();
     const long long no = S.b_start[0];
     T.sync();
-    if (no + kn > a.out_nodes_cap) {
+    if (no < 0) {
         if (r == 0) atomicExch(&c.ctl->fatal, 1);
         return false;
     }
@@ -1562,11 +1574,11 @@ __device__ bool emit_graph(const Team &T, Arena &S, const Ctx &c, int rank_i) {
         kept += tot;
         T.sync();
     }
-    if (r == 0) S.b_start[0] = (int64_t)atomicAdd(a.out_used + 1, (unsigned long long)kept);
+    if (r == 0) S.b_start[0] = arena_reserve(a.out_used + 1, (unsigned long long)kept, a.out_arcs_cap);
     T.sync();
     const long long ao = S.b_start[0];
     T.sync();
-    if (ao + kept > a.out_arcs_cap) {
+    if (ao < 0) {
         if (r == 0) atomicExch(&c.ctl->fatal, 1);
         return false;
     }
@@ -1830,6 +1842,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         if (nhuge) {   // tier 4: the group's huge arena, one CTA
             if (G.grank == 0) {
                 Arena S4 = carve(c.w.huge, a.huge_hash, a.huge_nodes, a.huge_arcs, blockDim.x, true, true);
+                if (threadIdx.x == 0) ctl->n_tier4 += nhuge;
                 for (uint32_t t = 0; t < nhuge; ++t) {
                     const int32_t idx = __ldcg(c.w.overflow + no + nbig + nlarge + t);
                     double key = 0.0;
@@ -2101,6 +2114,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->n_cid = ctl->n_cid;
             qo->n_parcs = ctl->n_parcs;
             qo->n_eval = ctl->n_eval;
+            qo->n_tier4 = ctl->n_tier4;
             qo->pull_level = ctl->pull_at - 1;
             qo->n_cut = (int32_t)ctl->n_cut;
             qo->frontier_total = ctl->frontier_total;
@@ -2120,11 +2134,8 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
 size_t engine_dyn_smem() { return (size_t)KGS_MAX_K * (8 + 4 + 4); }
 
 int engine_max_grid(int device) {
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_engine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)engine_dyn_smem());
-        attr = true;
-    }
+    // the dynamic shared-memory attribute is per device: set it on every device the engine runs on
+    cudaFuncSetAttribute(k_engine, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)engine_dyn_smem());
     int per_sm = 0, sms = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_engine, kBlock, engine_dyn_smem());
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);

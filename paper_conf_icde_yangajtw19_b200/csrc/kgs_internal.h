@@ -84,13 +84,14 @@ struct Ctl {
     uint32_t multi_kw;             // union of the keyword sets of the nodes holding >= 2 query keywords
     uint32_t n_cut;                // candidates stopped by the exact key cut-off (pruning round 2)
     uint32_t work_huge2;           // ... beyond the per-CTA large arenas too (tier 4, one CTA of the group)
+    uint32_t n_tier4;              // Central Graphs this query extracted in the tier-4 arena (all passes)
 };
 
 // Per-query summary written by the engine (device), read back by the host.
 constexpr int kMaxStamps = 48;
 struct QOut {
     int32_t levels, stop_reason, count, fatal;
-    uint32_t n_central, n_overflow, n_cid, n_parcs, n_eval, pad;
+    uint32_t n_central, n_overflow, n_cid, n_parcs, n_eval, n_tier4;
     unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
@@ -237,6 +238,9 @@ struct VpBufs {                    // exchange buffers (caller-owned device memo
     int32_t *cent_n;               // [1] their count
     int64_t n_pad, lo, hi;
 };
+
+// SM count of the current device (cached per device): grids are sized in multiples of it.
+int device_sm_count();
 
 // ---- launchers (return cudaError_t) ----
 cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha, uint8_t *act, uint32_t *amax,

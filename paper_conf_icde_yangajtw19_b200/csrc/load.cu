@@ -6,7 +6,7 @@
 //                                 in a node's visited / next words (one 32-byte sector per node).
 //   k_summary                     Eq. 2 per node over its in-arc labels sorted per row (cub segmented
 //                                 sort), one warp per node, runs of equal labels found by ballots.
-//   k_normalise                   w' = (w - min) / (max - min).
+//   k_normalise                   w' = (w - min) / (max - min) over the nodes with in-arcs, on the 2^-24 grid.
 #include <cub/device/device_segmented_sort.cuh>
 
 #include <cmath>
@@ -133,7 +133,7 @@ constexpr int kPairs = 128;   // pairs per bit-parallel BFS pass
 
 int grid_for(int64_t items, int block) {
     int64_t g = (items + block - 1) / block;
-    if (g > 148 * 16) g = 148 * 16;
+    if (g > device_sm_count() * 16) g = device_sm_count() * 16;
     return g < 1 ? 1 : (int)g;
 }
 
@@ -151,8 +151,10 @@ cudaError_t stage(const T *p, int64_t cnt, bool dev, cudaStream_t s, T **out, T 
 
 // One warp per node over its sorted labels: a run of equal labels r has n_r entries and adds
 // n_r log2(1 + n_r); w = that sum / deg.  Run starts inside a 32-label chunk come from
-// a ballot; a run that started in an earlier chunk carries its start.  Also min/max of w (w >= 0, so
-// the IEEE bit patterns order like the values).
+// a ballot; a run that started in an earlier chunk carries its start.  The terms are added in label
+// order (the run ends of a chunk, lowest lane first, chunk after chunk), the order Eq. 2's sum is
+// written in.  Also min/max of w over the nodes with in-arcs (reading R6; w >= 0, so the IEEE bit
+// patterns order like the values).
 __global__ void k_summary(const int64_t *__restrict__ rp, const int32_t *__restrict__ lab, int64_t n,
                           double *__restrict__ w, unsigned long long *wmin, unsigned long long *wmax) {
     const int lane = threadIdx.x & 31;
@@ -161,7 +163,7 @@ __global__ void k_summary(const int64_t *__restrict__ rp, const int32_t *__restr
     unsigned long long lmin = ~0ull, lmax = 0ull;
     for (int64_t v = warp0; v < n; v += nwarps) {
         const int64_t b = rp[v], e = rp[v + 1];
-        double acc = 0.0;
+        double acc = 0.0;    // the same value in every lane
         int64_t carry = b;   // start of the run open at the chunk boundary
         for (int64_t c = b; c < e; c += 32) {
             const int64_t j = c + lane;
@@ -170,21 +172,27 @@ __global__ void k_summary(const int64_t *__restrict__ rp, const int32_t *__restr
             const bool start = in && (j == b || lab[j - 1] != l);
             const bool end = in && (j + 1 == e || lab[j + 1] != l);
             const unsigned starts = __ballot_sync(0xffffffffu, start);
+            double term = 0.0;
             if (end) {
                 const unsigned upto = starts & (0xffffffffu >> (31 - lane));
                 const int64_t s0 = upto ? c + (31 - __clz(upto)) : carry;
                 const double nr = (double)(j - s0 + 1);
-                acc += nr * log2(1.0 + nr);
+                term = nr * log2(1.0 + nr);
             }
+            for (unsigned ends = __ballot_sync(0xffffffffu, end); ends; ends &= ends - 1)
+                acc += __shfl_sync(0xffffffffu, term, __ffs(ends) - 1);
             if (starts) carry = c + (31 - __clz(starts));
         }
-        for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-        const double wv = e > b ? acc / (double)(e - b) : 0.0;   // R25: no in-arcs -> 0
-        if (lane == 0) {
-            w[v] = wv;
-            const unsigned long long bits = (unsigned long long)__double_as_longlong(wv);
-            lmin = bits < lmin ? bits : lmin;
-            lmax = bits > lmax ? bits : lmax;
+        if (e > b) {
+            const double wv = acc / (double)(e - b);
+            if (lane == 0) {
+                w[v] = wv;
+                const unsigned long long bits = (unsigned long long)__double_as_longlong(wv);
+                lmin = bits < lmin ? bits : lmin;
+                lmax = bits > lmax ? bits : lmax;
+            }
+        } else if (lane == 0) {
+            w[v] = 0.0;   // no in-arcs: summarises nothing, out of the min / max (R6)
         }
     }
     if (lane == 0) {
@@ -193,12 +201,18 @@ __global__ void k_summary(const int64_t *__restrict__ rp, const int32_t *__restr
     }
 }
 
-__global__ void k_normalise(const double *__restrict__ w, int64_t n, const unsigned long long *wmin,
-                            const unsigned long long *wmax, float *__restrict__ out) {
-    const double lo = __longlong_as_double((long long)*wmin), hi = __longlong_as_double((long long)*wmax);
+// w' = (w - min) / (max - min) over the nodes with in-arcs, 0 for the others (R6) and for every node when
+// max = min (R26); produced on the 2^-24 grid, nearest point of the fp64 value, ties up (R27).
+__global__ void k_normalise(const double *__restrict__ w, const int64_t *__restrict__ rp, int64_t n,
+                            const unsigned long long *wmin, const unsigned long long *wmax, float *__restrict__ out) {
+    const unsigned long long bmin = *wmin, bmax = *wmax;
+    const bool any = bmin != ~0ull;
+    const double lo = __longlong_as_double((long long)bmin), hi = __longlong_as_double((long long)bmax);
     const double span = hi - lo;
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        out[v] = span > 0.0 ? (float)((w[v] - lo) / span) : 0.0f;   // R26: max = min -> 0
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        const double x = (any && span > 0.0 && rp[v + 1] > rp[v]) ? (w[v] - lo) / span : 0.0;
+        out[v] = (float)(floor(x * 16777216.0 + 0.5) * (1.0 / 16777216.0));
+    }
 }
 
 }  // namespace
@@ -325,7 +339,7 @@ kgs_status kgs_prep_summary_weights(int64_t n, int64_t m, const int64_t *in_row_
     LD_TRY(cudaMemsetAsync(mm, 0xFF, sizeof(unsigned long long), s));
     LD_TRY(cudaMemsetAsync(mm + 1, 0, sizeof(unsigned long long), s));
     k_summary<<<grid_for(n * 32, 256), 256, 0, s>>>(d_rp, sorted, n, w, mm, mm + 1);
-    k_normalise<<<grid_for(n, 256), 256, 0, s>>>(w, n, mm, mm + 1, d_out);
+    k_normalise<<<grid_for(n, 256), 256, 0, s>>>(w, d_rp, n, mm, mm + 1, d_out);
     LD_TRY(cudaGetLastError());
     LD_TRY(cudaMemcpyAsync(w_norm, d_out, sizeof(float) * (size_t)n, cudaMemcpyDeviceToHost, s));
     if (w_raw) LD_TRY(cudaMemcpyAsync(w_raw, w, sizeof(double) * (size_t)n, cudaMemcpyDeviceToHost, s));

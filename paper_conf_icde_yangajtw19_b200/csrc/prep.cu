@@ -4,9 +4,26 @@
 //   k_degree_class light / big node classes for the engine's load balance.
 //   k_snap         weights onto the 2^-24 grid (reading R15).
 //   k_validate     CSR / index / weight checks of kgs_load_graph.
+#include <atomic>
+
 #include "kgs_internal.h"
 
 namespace kgs {
+
+int device_sm_count() {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) dev = 0;
+    const int slot = dev >= 0 && dev < 64 ? dev : -1;
+    if (slot >= 0) {
+        const int c = cache[slot].load(std::memory_order_relaxed);
+        if (c > 0) return c;
+    }
+    int sms = 0;
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || sms < 1) sms = 1;
+    if (slot >= 0) cache[slot].store(sms, std::memory_order_relaxed);
+    return sms;
+}
 
 __global__ void k_activation(const float *__restrict__ w, int64_t n, double A, double alpha,
                              uint8_t *__restrict__ act, uint32_t *amax) {
@@ -38,7 +55,7 @@ cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha,
     cudaMemsetAsync(amax, 0, sizeof(uint32_t), s);
     if (n > 0) {
         int grid = (int)((n + 255) / 256);
-        if (grid > 148 * 16) grid = 148 * 16;
+        if (grid > device_sm_count() * 16) grid = device_sm_count() * 16;
         k_activation<<<grid, 256, 0, s>>>(w, n, A, alpha, act, amax);
     }
     return cudaGetLastError();
@@ -55,7 +72,7 @@ __global__ void k_degree_class(const int64_t *__restrict__ rp, int64_t n, uint8_
 cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s) {
     if (n > 0) {
         int grid = (int)((n + 255) / 256);
-        if (grid > 148 * 16) grid = 148 * 16;
+        if (grid > device_sm_count() * 16) grid = device_sm_count() * 16;
         k_degree_class<<<grid, 256, 0, s>>>(row_ptr, n, cls);
     }
     return cudaGetLastError();
@@ -70,7 +87,7 @@ __global__ void k_snap(float *w, int64_t n) {
 cudaError_t launch_snap_weights(float *w, int64_t n, cudaStream_t s) {
     if (n > 0) {
         int grid = (int)((n + 255) / 256);
-        if (grid > 148 * 16) grid = 148 * 16;
+        if (grid > device_sm_count() * 16) grid = device_sm_count() * 16;
         k_snap<<<grid, 256, 0, s>>>(w, n);
     }
     return cudaGetLastError();
@@ -103,7 +120,7 @@ __global__ void k_validate(DevGraph g, int32_t *err) {
     }
 }
 cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s) {
-    k_validate<<<148 * 8, 256, 0, s>>>(g, err);
+    k_validate<<<device_sm_count() * 8, 256, 0, s>>>(g, err);
     return cudaGetLastError();
 }
 

@@ -76,7 +76,7 @@ __global__ void k_map(int32_t *__restrict__ ids, int64_t cnt, const int32_t *__r
 
 int grid_for(int64_t n) {
     int64_t g = (n + 255) / 256;
-    if (g > 148 * 16) g = 148 * 16;
+    if (g > device_sm_count() * 16) g = device_sm_count() * 16;
     return g < 1 ? 1 : (int)g;
 }
 
@@ -125,7 +125,7 @@ cudaError_t relabel_by_degree(int64_t n, int64_t m, int64_t P, int64_t **row_ptr
         RL_TRY(cudaGetLastError());
         RL_TRY(cudaMemsetAsync(rp_new, 0, sizeof(int64_t), s));
         RL_TRY(cub::DeviceScan::InclusiveSum(tmp, tb_scan, deg64, rp_new + 1, (int)n, s));
-        k_rows<<<148 * 16, 256, 0, s>>>(*row_ptr, *col_idx, rp_new, orig, perm, n, ci_new);
+        k_rows<<<device_sm_count() * 16, 256, 0, s>>>(*row_ptr, *col_idx, rp_new, orig, perm, n, ci_new);
         RL_TRY(cudaGetLastError());
         if (P > 0) {
             k_map<<<grid_for(P), 256, 0, s>>>(kw_nodes, P, perm);
@@ -166,7 +166,7 @@ __global__ void k_gather_i32(const int32_t *ids, const int32_t *orig, int64_t cn
 
 cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
                               uint8_t *out, cudaStream_t s) {
-    k_levels_out_perm<<<148 * 8, 256, 0, s>>>(st, M, perm, n, q, out);
+    k_levels_out_perm<<<device_sm_count() * 8, 256, 0, s>>>(st, M, perm, n, q, out);
     return cudaGetLastError();
 }
 cudaError_t launch_gather_u8(const uint8_t *src, const int32_t *perm, int64_t n, uint8_t *out, cudaStream_t s) {

@@ -201,7 +201,7 @@ __global__ void k_vp_pack_st(const uint8_t *__restrict__ hm, const uint8_t *__re
 
 static int vp_grid(int64_t items, int per_block) {
     int64_t g = (items + per_block - 1) / per_block;
-    if (g > 148 * 16) g = 148 * 16;
+    if (g > device_sm_count() * 16) g = device_sm_count() * 16;
     return g < 1 ? 1 : (int)g;
 }
 
@@ -211,7 +211,7 @@ cudaError_t launch_vp_begin(const DevGraph &g, const VpQuery &qd, const uint8_t 
     cudaMemcpyAsync(gate, act, (size_t)g.n, cudaMemcpyDeviceToDevice, s);
     cudaMemsetAsync(b.counts, 0, 3 * sizeof(unsigned long long), s);
     cudaMemsetAsync(b.cent_n, 0, sizeof(int32_t), s);
-    k_vp_init<<<148 * 4, kVpBlock, 0, s>>>(g.kw_ptr, g.kw_nodes, qd, b.hm, gate, b.M);
+    k_vp_init<<<device_sm_count() * 4, kVpBlock, 0, s>>>(g.kw_ptr, g.kw_nodes, qd, b.hm, gate, b.M);
     k_vp_ident0<<<vp_grid(b.hi - b.lo, kVpBlock), kVpBlock, 0, s>>>(b.hm, b.lo, b.hi, qd.full, b.cent, b.cdep,
                                                                        b.cent_n, b.counts);
     return cudaGetLastError();
@@ -234,7 +234,7 @@ cudaError_t launch_vp_level(const DevGraph &g, const VpQuery &qd, const uint8_t 
             g.in_ptr, g.in_idx, b.hm, X, gate, act, block_central, b.lo, b.hi, l, qd.full, b.hm_slice, b.M, b.cent,
             b.cdep, b.cent_n, b.counts);
     if (nbig)
-        k_vp_pull_big<<<nbig < 148 * 4 ? nbig : 148 * 4, kVpBlock, 0, s>>>(
+        k_vp_pull_big<<<nbig < device_sm_count() * 4 ? nbig : device_sm_count() * 4, kVpBlock, 0, s>>>(
             g.in_ptr, g.in_idx, b.hm, X, gate, big, nbig, b.lo, l, qd.full, b.hm_slice, b.M, b.cent, b.cdep, b.cent_n,
             b.counts);
     return cudaGetLastError();

@@ -43,6 +43,7 @@ def _load():
         lib.synth_A.argtypes = [ctypes.c_void_p]
         lib.synth_copy.argtypes = [ctypes.c_void_p] + [ctypes.c_void_p] * 5
         lib.synth_free.argtypes = [ctypes.c_void_p]
+        lib.synth_arc_labels.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
         lib.synth_num_threads.restype = ctypes.c_int
         _lib = lib
     return _lib
@@ -79,8 +80,10 @@ class Graph:
 def rmat_graph(scale: int, edge_factor: int, seed: int, *, n_hubs: int = 0, hub_arcs: int = 0,
                weight_mode: int = 0, n_labels: int = 1024, label_s: float = 1.2, vocab: int = 1 << 17,
                word_s: float = 1.0, words_mean_extra: float = 2.0, a_sources: int = 16,
-               a_pairs_per_source: int = 625) -> Graph:
-    """R-MAT(.57,.19,.19,.05) symmetric CSR with Eq.2 (weight_mode=0) or uniform (1) weights."""
+               a_pairs_per_source: int = 625, labels: bool = False) -> Graph:
+    """R-MAT(.57,.19,.19,.05) symmetric CSR with Eq.2 (weight_mode=0) or uniform (1) weights.
+    labels=True also returns the per-arc edge labels the Eq. 2 weights were computed from, in
+    ``meta["arc_labels"]`` (int32 [arcs])."""
     lib = _load()
     h = lib.synth_build(scale, edge_factor, seed, n_hubs, hub_arcs, weight_mode, n_labels, label_s, vocab,
                         word_s, words_mean_extra, a_sources, a_pairs_per_source)
@@ -95,11 +98,17 @@ def rmat_graph(scale: int, edge_factor: int, seed: int, *, n_hubs: int = 0, hub_
         kn = np.empty(post, np.int32)
         lib.synth_copy(h, rp.ctypes.data, ci.ctypes.data, w.ctypes.data, kp.ctypes.data, kn.ctypes.data)
         A = float(lib.synth_A(h))
+        lab = None
+        if labels:
+            lab = np.empty(arcs, np.int32)
+            lib.synth_arc_labels(h, lab.ctypes.data)
     finally:
         lib.synth_free(h)
     meta = dict(scale=scale, edge_factor=edge_factor, seed=seed, n_hubs=n_hubs, hub_arcs=hub_arcs,
                 weight_mode=weight_mode, n_labels=n_labels, vocab=vocab, max_degree=maxd, isolated=iso,
                 gen_threads=int(lib.synth_num_threads()))
+    if lab is not None:
+        meta["arc_labels"] = lab
     return Graph(rp, ci, w, kp, kn, A, True, meta)
 
 

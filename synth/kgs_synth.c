@@ -49,6 +49,12 @@ typedef struct {
     int32_t *kw_nodes;
     double A;
     int64_t max_degree, n_isolated;
+    /* what the edge labels were drawn from (synth_arc_labels recomputes them) */
+    uint64_t seed;
+    int64_t n_labels;
+    double label_s;
+    int32_t hubs[64];
+    int n_hubs;
 } synth_graph;
 
 static int cmp_i32(const void *a, const void *b) {
@@ -197,6 +203,15 @@ static void build_csr(synth_graph *g, int scale, int64_t edge_factor, uint64_t s
     g->max_degree = mx; g->n_isolated = iso;
 }
 
+/* Label of the edge {v, u} (both arcs get the same one): hub edges share label R, the others are a
+ * Zipf(label_s) draw keyed by the unordered pair. */
+static int32_t edge_label(uint64_t seed, const double *cdf, int64_t R, const int32_t *hubs, int n_hubs, int vh,
+                          int32_t v, int32_t u) {
+    if (vh || is_hub(hubs, n_hubs, u)) return (int32_t)R;
+    uint64_t lo = (uint64_t)(v < u ? v : u), hi = (uint64_t)(v < u ? u : v);
+    return (int32_t)zipf_draw(cdf, R, u01(rng3(seed, ST_LABEL, (lo << 32) | hi)));
+}
+
 /* Node weights.  mode 0: paper Eq. 2 over Zipf(label_s) edge labels (R labels, hub edges share label R),
  * then min-max normalised over non-isolated nodes (isolated -> 0; max==min -> all 0), snapped to 2^-24.
  * mode 1: uniform random on the 2^-24 grid. */
@@ -223,12 +238,8 @@ static void build_weights(synth_graph *g, uint64_t seed, int mode, int64_t R, do
             int64_t b = g->row_ptr[v], e = g->row_ptr[v + 1], len = e - b;
             if (len == 0) { raw[v] = -1.0; continue; }
             int vh = is_hub(hubs, n_hubs, (int32_t)v);
-            for (int64_t j = 0; j < len; ++j) {
-                int32_t u = g->col_idx[b + j];
-                if (vh || is_hub(hubs, n_hubs, u)) { lab[j] = (int32_t)R; continue; }
-                uint64_t lo = (uint64_t)(v < u ? v : u), hi = (uint64_t)(v < u ? u : v);
-                lab[j] = (int32_t)zipf_draw(cdf, R, u01(rng3(seed, ST_LABEL, (lo << 32) | hi)));
-            }
+            for (int64_t j = 0; j < len; ++j)
+                lab[j] = edge_label(seed, cdf, R, hubs, n_hubs, vh, (int32_t)v, g->col_idx[b + j]);
             sort_i32(lab, len);
             double num = 0.0, den = 0.0;
             int64_t i = 0;
@@ -358,6 +369,8 @@ synth_graph *synth_build(int scale, int64_t edge_factor, uint64_t seed, int n_hu
     int32_t hubs[64];
     if (n_hubs > 64) n_hubs = 64;
     build_csr(g, scale, edge_factor, seed, n_hubs, hub_arcs, hubs);
+    g->seed = seed; g->n_labels = n_labels; g->label_s = label_s; g->n_hubs = n_hubs;
+    memcpy(g->hubs, hubs, sizeof(int32_t) * (size_t)n_hubs);
     build_weights(g, seed, weight_mode, n_labels, label_s, hubs, n_hubs);
     build_keywords(g, seed, vocab, word_s, words_mean_extra);
     g->A = estimate_A(g, seed, a_sources, a_pairs_per_source);
@@ -377,6 +390,19 @@ void synth_copy(const synth_graph *g, int64_t *row_ptr, int32_t *col_idx, float 
     memcpy(kw_ptr, g->kw_ptr, sizeof(int64_t) * (size_t)(g->n_keywords + 1));
     memcpy(kw_nodes, g->kw_nodes, sizeof(int32_t) * (size_t)g->n_postings);
 }
+/* The edge labels behind the Eq. 2 weights (weight_mode 0), one per CSR arc (in-arcs = out-arcs: the
+ * graph is symmetric), so that the load-time preprocessing can be checked against the generator. */
+void synth_arc_labels(const synth_graph *g, int32_t *out) {
+    double *cdf = zipf_cdf(g->n_labels, g->label_s);
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t v = 0; v < g->n; ++v) {
+        int vh = is_hub(g->hubs, g->n_hubs, (int32_t)v);
+        for (int64_t j = g->row_ptr[v]; j < g->row_ptr[v + 1]; ++j)
+            out[j] = edge_label(g->seed, cdf, g->n_labels, g->hubs, g->n_hubs, vh, (int32_t)v, g->col_idx[j]);
+    }
+    free(cdf);
+}
+
 void synth_free(synth_graph *g) {
     if (!g) return;
     free(g->row_ptr); free(g->col_idx); free(g->weight); free(g->kw_ptr); free(g->kw_nodes);

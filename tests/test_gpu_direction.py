@@ -5,7 +5,7 @@ Pull at every level computes the frontier-free level rule (SURVEY.md §8(c) O3);
 hits it recomputes whether Alg. 2's work list would still be non-empty, so M, the central set, depths,
 keys, answers AND the stop level equal the oracle's literal form bit for bit whatever the direction.
 The automatic switch (push first, pull from the first level whose active frontier has more than
-m / KGS_PULL_RATIO out-arcs) is exercised mid-search with small thresholds.
+m / pull_ratio out-arcs, kgs_params) is exercised mid-search with small thresholds.
 """
 import os
 
@@ -28,10 +28,10 @@ def _gpu():
 
 
 def compare(G, g, kw, k, direction, *, alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=0,
-            level_cover=1, full=True, prune=1):
+            level_cover=1, full=True, prune=1, pull_ratio=14, pull_min=1 << 22):
     p = kgs.make_params(alpha=alpha, lam=lam, max_depth=max_depth, block_central=block_central,
                         extract_mode=extract_mode, level_cover=level_cover, want_levels=1 if full else 0,
-                        prune=prune, direction=direction)
+                        prune=prune, direction=direction, pull_ratio=pull_ratio, pull_min=pull_min)
     r = kgs.kgs_query(G, kw, k, p)
     pulled = r.stats["pull_level"] >= 0
     if direction == kgs.KGS_DIR_PULL:   # -1: stopped at level 0, before any expansion
@@ -58,18 +58,6 @@ def compare(G, g, kw, k, direction, *, alpha=0.1, lam=0.2, max_depth=254, block_
     return r
 
 
-@pytest.fixture
-def small_thresholds():
-    old = {k: os.environ.get(k) for k in ("KGS_PULL_RATIO", "KGS_PULL_MIN")}
-    os.environ["KGS_PULL_MIN"] = "0"
-    yield
-    for k, v in old.items():
-        if v is None:
-            os.environ.pop(k, None)
-        else:
-            os.environ[k] = v
-
-
 def test_golden_examples_pull():
     _gpu()
     d = R.load_golden("fig2_examples_1_3.json")
@@ -87,7 +75,7 @@ def test_golden_examples_pull():
         assert r.answers[0].nodes.tolist() == d["answer"]["nodes"]
 
 
-def test_random_small_graphs_pull_and_switch(small_thresholds):
+def test_random_small_graphs_pull_and_switch():
     """Forced pull, forced push and the automatic switch at several thresholds, on random directed and
     undirected graphs with gates (weights), every extraction / blocking / pruning mode."""
     _gpu()
@@ -103,8 +91,8 @@ def test_random_small_graphs_pull_and_switch(small_thresholds):
         kw = list(range(q))
         for j in range(3):
             direction = (kgs.KGS_DIR_PULL, kgs.KGS_DIR_PUSH, kgs.KGS_DIR_AUTO)[j]
-            os.environ["KGS_PULL_RATIO"] = str(int(rng.choice([1, 2, 4, 14])))
-            r = compare(G, g, kw, int(rng.choice([1, 2, 5, 40])), direction,
+            ratio = int(rng.choice([1, 2, 4, 14]))
+            r = compare(G, g, kw, int(rng.choice([1, 2, 5, 40])), direction, pull_ratio=ratio, pull_min=0,
                         alpha=float(rng.choice([0.05, 0.1, 0.4])), lam=float(rng.choice([0.0, 0.2, 1.0])),
                         max_depth=int(rng.choice([1, 3, 254])), block_central=int(rng.integers(0, 2)),
                         extract_mode=int(rng.integers(0, 2)), level_cover=int(rng.integers(0, 2)),
@@ -114,7 +102,7 @@ def test_random_small_graphs_pull_and_switch(small_thresholds):
     assert switched > 0   # some searches switched after at least one push level
 
 
-def test_c1_c2_pull(small_thresholds):
+def test_c1_c2_pull():
     """C1 (all queries) and a C2 sample with pull at every level; C2 also with the automatic switch."""
     _gpu()
     w = synth.make_workload("C1")
@@ -124,9 +112,9 @@ def test_c1_c2_pull(small_thresholds):
     G.close()
     w = synth.make_workload("C2")
     G = kgs.kgs_load_graph(w.graph)
-    os.environ["KGS_PULL_RATIO"] = "40"
     for j, kw in enumerate(w.queries[::25]):
-        compare(G, w.graph, kw, w.k, (kgs.KGS_DIR_PULL, kgs.KGS_DIR_AUTO)[j % 2], full=(j % 3 == 0))
+        compare(G, w.graph, kw, w.k, (kgs.KGS_DIR_PULL, kgs.KGS_DIR_AUTO)[j % 2], full=(j % 3 == 0), pull_ratio=40,
+                pull_min=0)
     G.close()
 
 

@@ -1,10 +1,17 @@
-"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times.
+"""Parity at BASELINE.json's full sizes, including the exact launch configuration bench.py times.
 
-C3 (configs[2]: 2^25 nodes, 5.3e8 arcs): the bench's query order (fixed permutation), queries run
-through kgs_query_device + kgs_query_fetch exactly as bench.py does, then the whole hitting-level
-matrix M (n x q), the central set with depths and Eq. 6 keys, and the ranked answers with their
-subgraphs are compared with the oracle element by element.  A sample of queries keeps the oracle
-(seconds per query at this size) within a few minutes.
+* C3 (configs[2]: 2^25 nodes, 5.3e8 arcs), the bench's timed step: ONE kgs_query_batch_device launch of
+  the 350 queries in bench order, G = 8 groups, kgs_params_default() (prune = 1, the round-2 key cut-off,
+  the in-arc pre-pass DAG of query groups) — answers compared with the oracle query by query on a sample
+  spanning q = 2..8.
+* C3 latency mode (one launch per query, G = 1, recorded DAG) with the full state view (want_levels:
+  the whole M, every central with its depth and key).
+* C4 (configs[3]: the C3 graph, 4096 queries, q ~ U{2..8}): a 64-query sample in one G = 8 launch that
+  includes level-5 queries (about 10^6 central nodes each).  Where the oracle cannot score every central
+  node in minutes, it scores the engine's k answers plus every central node among 20000 seeded random
+  node ids (oracle.query eval_ids, ~650 of them central): its top-k over that set must be the engine's answers exactly.
+* C5 (configs[4]: C3 + 16 hubs of 2^21 arcs, q = 8, k = 100): 10 queries, batch launch.
+* Tier-4 extraction: a Central Graph beyond the per-CTA arenas (1.1 M nodes > 2^20).
 """
 import numpy as np
 import pytest
@@ -16,36 +23,75 @@ pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 
 kgs = pytest.importorskip("paper_conf_icde_yangajtw19_b200")
 
+BENCH_ORDER_SEED = 12345   # bench.py: queries in np.random.default_rng(12345).permutation order
 
-@pytest.fixture(scope="module")
-def c3():
+
+def _gpu():
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
+
+
+@pytest.fixture(scope="module")
+def c3():
+    _gpu()
     w = synth.make_workload("C3")
     G = kgs.kgs_load_graph(w.graph)
-    order = np.random.default_rng(12345).permutation(len(w.queries))
+    order = np.random.default_rng(BENCH_ORDER_SEED).permutation(len(w.queries))
     yield w, G, [w.queries[i] for i in order]
     G.close()
 
 
-def _check(w, r, o, full=True):
+def _check(r, o, full=True, ctx=""):
     if full:
-        assert np.array_equal(r.a, o.a)
+        assert np.array_equal(r.a, o.a), ctx
         bad = np.argwhere(r.M != o.M)
-        assert bad.size == 0, f"M differs at {bad[:5].tolist()}"
-        assert r.centrals.tolist() == o.centrals.tolist()
-        assert r.central_depth.tolist() == o.central_depth.tolist()
-        assert r.central_key.tolist() == o.central_key.tolist()
-    assert r.stats["stop_reason"] == o.stop_reason and r.stats["levels"] == o.levels
-    assert [a.central for a in r.answers] == [a.central for a in o.answers]
+        assert bad.size == 0, f"{ctx} M differs at {bad[:5].tolist()}"
+        assert r.centrals.tolist() == o.centrals.tolist(), ctx
+        assert r.central_depth.tolist() == o.central_depth.tolist(), ctx
+        assert r.central_key.tolist() == o.central_key.tolist(), ctx
+    assert r.stats["stop_reason"] == o.stop_reason and r.stats["levels"] == o.levels, ctx
+    assert r.stats["n_centrals"] == len(o.centrals), ctx
+    assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
     for ra, oa in zip(r.answers, o.answers):
-        assert ra.depth == oa.depth and ra.score_key == oa.key and ra.score == oa.score
-        assert ra.nodes.tolist() == oa.nodes.tolist() and ra.arcs.tolist() == oa.arcs.tolist()
+        assert ra.depth == oa.depth and ra.score_key == oa.key and ra.score == oa.score, ctx
+        assert ra.nodes.tolist() == oa.nodes.tolist() and ra.arcs.tolist() == oa.arcs.tolist(), ctx
 
 
-def test_c3_bench_launch_configuration(c3):
-    """The first timed bench queries, device-resident path (kgs_query_device + fetch)."""
+def _batch_device(G, qs, k, groups, params=None):
+    """The bench's launch: keyword rows and lengths in HBM, one kgs_query_batch_device, then fetch."""
+    import torch
+    kwp = torch.full((len(qs), 8), -1, dtype=torch.int32)
+    for i, q in enumerate(qs):
+        kwp[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
+    kwd = kwp.cuda()
+    qld = torch.tensor([len(q) for q in qs], dtype=torch.int32, device="cuda")
+    s = torch.cuda.current_stream().cuda_stream
+    p = params if params is not None else kgs.kgs_params_default()
+    kgs.kgs_query_batch_device(G, len(qs), kwd.data_ptr(), qld.data_ptr(), k, p, groups, s)
+    return kgs.kgs_query_batch_fetch(G, [len(q) for q in qs], s)
+
+
+def test_c3_bench_timed_launch(c3):
+    """bench.py's timed step exactly: 350 queries, G = 8, default params, one launch.  The first four
+    queries of every size q = 2..8 in bench order (28 answers sets) against the oracle."""
+    w, G, qs = c3
+    res = _batch_device(G, qs, w.k, 8)
+    assert len(res) == len(qs)
+    picked, per_q = [], {}
+    for j, kw in enumerate(qs):
+        if per_q.get(len(kw), 0) < 4:
+            per_q[len(kw)] = per_q.get(len(kw), 0) + 1
+            picked.append(j)
+    assert sorted(per_q) == list(range(2, 9))
+    for j in picked:
+        _check(res[j], oracle.query(w.graph, qs[j], w.k), full=False, ctx=f"bench query {j} kw={qs[j]}")
+    assert any(res[j].stats["n_centrals"] > 512 for j in picked)   # pruning (prune = 1) actually cut
+
+
+def test_c3_latency_mode_full_state(c3):
+    """bench.py's latency mode (kgs_query_device + fetch, G = 1, recorded DAG), with the parity view
+    (want_levels = 1: every M entry, every central node's depth and key)."""
     import torch
     w, G, qs = c3
     s = torch.cuda.current_stream().cuda_stream
@@ -54,35 +100,19 @@ def test_c3_bench_launch_configuration(c3):
         t = torch.tensor(kw, dtype=torch.int32, device="cuda")
         kgs.kgs_query_device(G, t.data_ptr(), len(kw), w.k, p, s)
         r = kgs.kgs_query_fetch(G, len(kw), 1, s)
-        _check(w, r, oracle.query(w.graph, kw, w.k))
+        _check(r, oracle.query(w.graph, kw, w.k), ctx=f"kw={kw}")
 
 
 def test_c3_every_query_size(c3):
-    """One query of every size q = 2..8 through the host API (kgs_query)."""
+    """One query of every size q = 2..8 through the host API (kgs_query), default params."""
     w, G, _ = c3
     seen = set()
     for kw in w.queries:
         if len(kw) in seen:
             continue
         seen.add(len(kw))
-        r = kgs.kgs_query(G, kw, w.k, kgs.make_params(want_levels=1))
-        _check(w, r, oracle.query(w.graph, kw, w.k))
+        _check(kgs.kgs_query(G, kw, w.k), oracle.query(w.graph, kw, w.k), full=False, ctx=f"kw={kw}")
     assert seen == set(range(2, 9))
-
-
-def test_c5_stress_hubs():
-    """C5 (configs[4]): C3 + 16 planted hubs of 2^21 arcs, 8 high-frequency keywords, top-100:
-    exercises the big-node (grid-wide tile) expansion and the large candidate sets."""
-    import torch
-    if not torch.cuda.is_available():
-        pytest.skip("no CUDA device")
-    w = synth.make_workload("C5")
-    assert w.graph.meta["max_degree"] > (1 << 20)
-    G = kgs.kgs_load_graph(w.graph)
-    for kw in w.queries[:3]:
-        r = kgs.kgs_query(G, kw, w.k, kgs.make_params(want_levels=1))
-        _check(w, r, oracle.query(w.graph, kw, w.k))
-    G.close()
 
 
 def test_c3_pull_direction(c3):
@@ -92,4 +122,78 @@ def test_c3_pull_direction(c3):
     for kw in qs[5:7]:
         r = kgs.kgs_query(G, kw, w.k, kgs.make_params(want_levels=1, direction=kgs.KGS_DIR_PULL))
         assert r.stats["pull_level"] == 0
-        _check(w, r, oracle.query(w.graph, kw, w.k))
+        _check(r, oracle.query(w.graph, kw, w.k), ctx=f"kw={kw}")
+
+
+# C4 queries that only find k central nodes at level 5 (tools/workload_scan.py, search-only scan of all
+# 4096 queries on the B200): ~10^6 central nodes each.
+C4_LEVEL5 = (2683, 2906)
+
+
+def test_c4_sample_with_level5_queries(c3):
+    """configs[3]: 64 C4 queries (the first 62 of the set and two level-5 queries) in ONE launch, G = 8,
+    default params, on the C3 graph.  Ordinary queries: full oracle.  Level-5 queries: the oracle
+    scores the engine's answers plus the central nodes among 20000 seeded random ids (eval_ids); its
+    top-k over that set must equal the engine's answers (a sampled check that nothing beats them)."""
+    w3, G, _ = c3
+    c4 = synth.config_queries("C4", w3.graph)
+    qs = list(c4[:62]) + [c4[i] for i in C4_LEVEL5]
+    res = _batch_device(G, qs, w3.k, 8)
+    rng = np.random.default_rng(4096)
+    deep = 0
+    for j, (kw, r) in enumerate(zip(qs, res)):
+        ctx = f"C4 sample {j} kw={kw}"
+        if r.stats["levels"] < 5:
+            _check(r, oracle.query(w3.graph, kw, w3.k), full=False, ctx=ctx)
+            continue
+        deep += 1
+        assert r.stats["stop_reason"] == kgs.KGS_STOP_K and r.stats["n_centrals"] > 100_000, ctx
+        ids = np.concatenate([[a.central for a in r.answers], rng.integers(0, w3.graph.n, 20000)]).astype(np.int32)
+        o = oracle.query(w3.graph, kw, w3.k, eval_ids=ids)
+        sampled = int(np.isin(o.centrals, ids).sum())
+        assert sampled > len(r.answers) + 200, ctx      # the sample holds central nodes besides the answers
+        _check(r, o, full=False, ctx=ctx)
+    assert deep == len(C4_LEVEL5)
+
+
+def test_c5_ten_queries():
+    """configs[4]: C3 + 16 planted hubs of 2^21 arcs, 8 high-frequency keywords, top-100: 10 queries in
+    one batch launch (G = 8, default params) and the first 2 with the full state view."""
+    _gpu()
+    w = synth.make_workload("C5")
+    assert w.graph.meta["max_degree"] > (1 << 20) and len(w.queries) >= 10
+    G = kgs.kgs_load_graph(w.graph)
+    qs = w.queries[:10]
+    res = _batch_device(G, qs, w.k, 8)
+    exp = [oracle.query(w.graph, kw, w.k) for kw in qs]
+    for j, (r, o) in enumerate(zip(res, exp)):
+        _check(r, o, full=False, ctx=f"C5 batch {j}")
+    for kw, o in zip(qs[:2], exp[:2]):
+        _check(kgs.kgs_query(G, kw, w.k, kgs.make_params(want_levels=1)), o, ctx=f"C5 kw={kw}")
+    G.close()
+
+
+def test_tier4_extraction():
+    """A Central Graph of 1.1 M nodes: a hub c joined to 1.1 M nodes holding keyword 0 and to one node
+    holding keyword 1.  It overflows tiers 1-3b (the per-CTA arenas hold at most 2^20 nodes), so both its
+    extraction (the Eq. 6 key) and its emit run in the per-group tier-4 arena: latency mode (recorded DAG)
+    and a batch of query groups (pre-pass)."""
+    _gpu()
+    n0 = 1_100_000
+    a, c = n0, n0 + 1
+    edges = [(v, c) for v in range(n0)] + [(a, c)]
+    wts = (np.arange(n0 + 2) % 7 / 8.0).astype(np.float32)
+    g = synth.from_edges(n0 + 2, edges, wts, [list(range(n0)), [a]], 2.0)
+    o = oracle.query(g, [0, 1], 1)
+    assert len(o.answers) == 1 and len(o.answers[0].nodes) == n0 + 2
+    G = kgs.kgs_load_graph(g)
+    r = kgs.kgs_query(G, [0, 1], 1)
+    assert r.stats["n_tier4"] >= 1
+    _check(r, o, full=False, ctx="latency")
+    res = kgs.kgs_query_batch(G, [[0, 1], [1, 0], [0, 1]], 1, None, 3)
+    for rr in res:
+        assert rr.stats["n_tier4"] >= 1
+        assert rr.answers[0].central == c and rr.answers[0].score_key == o.answers[0].key
+        assert rr.answers[0].nodes.tolist() == o.answers[0].nodes.tolist()
+        assert rr.answers[0].arcs.tolist() == o.answers[0].arcs.tolist()
+    G.close()

@@ -221,18 +221,17 @@ def test_huge_central_graph_tier4():
     G.close()
 
 
-def test_batch_capacity_overflow_is_per_query(monkeypatch):
+def test_batch_capacity_overflow_is_per_query():
     """A query that exceeds an internal capacity (here the predecessor-arc regions, shrunk to 64 K arcs
-    with KGS_PCAP_ARCS, against a Central Graph of 150 000 predecessor arcs) is reported per query in a
+    with kgs_graph_desc.pred_arc_cap, against a Central Graph of 150 000 predecessor arcs) is reported per query in a
     batch (KGS_STOP_CAPACITY, no answers); the other queries of the batch keep their exact answers.
     A single kgs_query reports KGS_EINTERNAL."""
     _gpu()
-    monkeypatch.setenv("KGS_PCAP_ARCS", str(1 << 16))
     n0 = 150_000
     a, c = n0, n0 + 1
     g = synth.from_edges(n0 + 2, [(v, c) for v in range(n0)] + [(a, c)], [0.0] * (n0 + 2),
                          [list(range(n0)), [a]], 2.0)
-    G = kgs.kgs_load_graph(g)
+    G = kgs.kgs_load_graph(g, pred_arc_cap=1 << 16)
     qs = [[0, 1], [1], [1, 0], [1]]
     res = kgs.kgs_query_batch(G, qs, 1, None, 2)
     assert [r.stats["stop_reason"] for r in res] == [kgs.KGS_STOP_CAPACITY, kgs.KGS_STOP_K] * 2

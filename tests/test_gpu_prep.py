@@ -140,3 +140,20 @@ def test_device_pointer_inputs():
                                                  stream=st.cuda_stream)
     assert np.allclose(wr, wr_o, rtol=1e-13, atol=0) and np.abs(wn - wn_o).max() <= 1e-6
     assert (dev[1].cpu().numpy() == ci).all()          # borrowed inputs are not modified
+
+
+def test_summary_weights_reproduce_generator_c2():
+    """NEXT-2 against the dataset recipe: kgs_prep_summary_weights on the C2 generator's own edge labels
+    (R-MAT scale 20, 1024 Zipf labels) gives the weights the generator wrote, bit for bit (Eq. 2 terms in
+    label order, R6 for the 0.5 M nodes without in-arcs, R27 grid), and kgs_load_graph keeps them."""
+    _gpu()
+    gp = dict(synth.CONFIG_PARAMS["C2"]["graph"])
+    g = synth.rmat_graph(**gp, labels=True)
+    lab = g.meta["arc_labels"]
+    wn, wr = kgs.kgs_prep_summary_weights(g.row_ptr, lab)
+    iso = np.diff(g.row_ptr) == 0
+    assert iso.sum() > 0 and (wn[iso] == 0).all() and (wr[iso] == 0).all()
+    bad = np.flatnonzero(wn != g.weight)
+    assert bad.size == 0, f"{bad.size} weights differ, first {bad[:5].tolist()}"
+    wn_o, wr_o = oracle.summary_weights(g.row_ptr, lab)
+    assert np.array_equal(wn, wn_o) and np.array_equal(wr, wr_o)

@@ -131,18 +131,17 @@ def _outcome(exp, nc, mcap):
     return "none" if nc <= mcap else ("round1" if exp == mcap else "round2")
 
 
-def test_pruned_answers_and_evaluated_counts(monkeypatch):
+def test_pruned_answers_and_evaluated_counts():
     _gpu()
     outcomes = set()
     for seed, kwargs, k, lam, pmin, ext, mode in CASES:
-        monkeypatch.setenv("KGS_PRUNE_MIN", str(pmin))
         g = medium_graph(seed, **kwargs)
         G = kgs.kgs_load_graph(g)
         kw = list(range(len(g.kw_ptr) - 1))
         o = oracle.query(g, kw, k, lam=lam, extract_mode=ext)
         ctx = f"seed={seed} k={k} lam={lam} pmin={pmin} ext={ext} mode={mode} |C|={len(o.centrals)}"
         for prune in (mode, 0):
-            r = kgs.kgs_query(G, kw, k, kgs.make_params(lam=lam, prune=prune, extract_mode=ext))
+            r = kgs.kgs_query(G, kw, k, kgs.make_params(lam=lam, prune=prune, extract_mode=ext, prune_min=pmin))
             assert r.stats["n_centrals"] == len(o.centrals), ctx
             assert [a.central for a in r.answers] == [a.central for a in o.answers], (ctx, prune)
             for ra, oa in zip(r.answers, o.answers):
@@ -180,12 +179,11 @@ def test_batch_pruned_matches_oracle():
     G.close()
 
 
-def test_key_cutoff_in_round_two(monkeypatch):
+def test_key_cutoff_in_round_two():
     """Round 2 stops a candidate's extraction once its closure weight times d^lambda exceeds the k-th
     exact key (kgs_stats.n_cut).  Valid when level-cover must keep every source: no node holds two query
     keywords (disjoint keyword sets here), or level_cover = 0.  Answers must be the oracle's."""
     _gpu()
-    monkeypatch.setenv("KGS_PRUNE_MIN", "40")
     cuts = 0
     for seed, deg, k in ((0, 16, 5), (0, 16, 20), (1, 16, 5), (1, 16, 20), (0, 8, 50)):
         rng = np.random.default_rng(500 + seed)
@@ -199,7 +197,7 @@ def test_key_cutoff_in_round_two(monkeypatch):
         kw = list(range(q))
         for lc in (1, 0):
             o = oracle.query(g, kw, k, level_cover=lc)
-            r = kgs.kgs_query(G, kw, k, kgs.make_params(prune=1, level_cover=lc))
+            r = kgs.kgs_query(G, kw, k, kgs.make_params(prune=1, level_cover=lc, prune_min=40))
             ctx = f"seed={seed} deg={deg} k={k} lc={lc} |C|={len(o.centrals)}"
             assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
             for ra, oa in zip(r.answers, o.answers):

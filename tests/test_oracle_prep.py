@@ -7,6 +7,7 @@ is pinned to values worked by hand and to the bounds 1 <= w <= log2(1 + deg) (eq
 iff every in-edge has the same label; on the left iff all labels differ).
 """
 import math
+from fractions import Fraction
 
 import numpy as np
 import pytest
@@ -99,7 +100,17 @@ def test_eq2_worked_values():
     lab = np.array([x for r in rows for x in r], np.int32)
     wn, wr = oracle.summary_weights(rp, lab)
     assert wr.tolist() == [1.75, 1.0, 3.0, 0.0, 2.0, 61 / 16]
-    assert wn.tolist() == [np.float32(x / (61 / 16)) for x in wr.tolist()]
+    # R6: node 3 (no in-edges) is left out of the min / max and gets w' = 0, so min = 1 (node 1), max =
+    # 61/16; R27: w' is the grid point nearest (w - 1) / (45/16), ties up -- exact rationals here
+    want = []
+    for v, x in enumerate(wr.tolist()):
+        if v == 3:
+            want.append(0.0)
+            continue
+        t = (Fraction(x) - 1) / (Fraction(61, 16) - 1) * (1 << 24)
+        want.append(float(Fraction((t + Fraction(1, 2)).__floor__(), 1 << 24)))
+    assert wn.astype(np.float64).tolist() == want
+    assert want[1] == 0.0 and want[5] == 1.0 and want[0] == 4473924 / (1 << 24)   # (3/4) / (45/16) = 4/15
 
 
 def test_eq2_bounds_and_label_order_invariance():
@@ -119,6 +130,34 @@ def test_eq2_bounds_and_label_order_invariance():
     distinct = np.arange(int(rp[-1]), dtype=np.int32)
     assert (oracle.summary_weights(rp, distinct)[1] == 1.0).all()
     assert wn.min() == 0.0 and wn.max() == 1.0
+
+
+def test_eq2_isolated_nodes_leave_min_max_alone():
+    """R6: adding nodes without in-edges changes no other weight (a rule that put their w = 0 into the
+    min would rescale every w' to w / max)."""
+    rows = [[1, 1, 2], [3], [4, 4, 4, 4], [5, 6]]
+    rp = np.cumsum([0] + [len(r) for r in rows]).astype(np.int64)
+    lab = np.array([x for r in rows for x in r], np.int32)
+    wn, _ = oracle.summary_weights(rp, lab)
+    rows2 = [[], rows[0], [], rows[1], rows[2], [], rows[3], []]
+    rp2 = np.cumsum([0] + [len(r) for r in rows2]).astype(np.int64)
+    wn2, wr2 = oracle.summary_weights(rp2, np.array([x for r in rows2 for x in r], np.int32))
+    assert wn2[[1, 3, 4, 6]].tolist() == wn.tolist()
+    assert wn2[[0, 2, 5, 7]].tolist() == [0.0] * 4 and wr2[[0, 2, 5, 7]].tolist() == [0.0] * 4
+    assert wn.min() == 0.0 and wn.max() == 1.0
+
+
+def test_eq2_reproduces_the_generator():
+    """The Eq. 2 weights the input generator wrote (synth, R-MAT scale 14 with Zipf edge labels and two
+    planted hubs; an independent implementation of the dataset recipe) are what P2 computes from the
+    generator's labels, bit for bit (same label order, R6, R27)."""
+    import synth
+    g = synth.rmat_graph(14, 8, 21, n_hubs=2, hub_arcs=3000, n_labels=256, a_sources=1,
+                         a_pairs_per_source=1, labels=True)
+    lab = g.meta["arc_labels"]
+    assert (np.diff(g.row_ptr) == 0).any()                    # isolated nodes exist (R6 matters)
+    wn, _ = oracle.summary_weights(g.row_ptr, lab)
+    assert np.array_equal(wn, g.weight)
 
 
 def test_eq2_constant_weights_normalise_to_zero():

@@ -123,3 +123,22 @@ def test_degenerate_queries():
     assert r.answers[0].nodes.tolist() == [2] and r.answers[0].key == 0.0
     r = oracle.query(g, [0, 2], k=1)
     assert r.status == 0 and r.stop_reason == oracle.STOP_EMPTY_KEYWORD and r.answers == []
+
+
+def test_eval_ids_sampling_is_consistent():
+    """oracle.query(eval_ids=...) scores only the listed central nodes: their keys equal the full run's,
+    the others are NaN, and the answers are the full ranking restricted to the list."""
+    import synth
+    w = synth.make_workload("C1")
+    for kw in w.queries[:10]:
+        full = oracle.query(w.graph, kw, 5)
+        if len(full.centrals) < 4:
+            continue
+        sub = full.centrals[::3]
+        part = oracle.query(w.graph, kw, 5, eval_ids=sub)
+        assert part.M.tolist() == full.M.tolist() and part.centrals.tolist() == full.centrals.tolist()
+        keep = np.isin(full.centrals, sub)
+        assert part.central_key[keep].tolist() == full.central_key[keep].tolist()
+        assert np.isnan(part.central_key[~keep]).all()
+        ranked = sorted(zip(full.central_key[keep].tolist(), full.centrals[keep].tolist()))[:5]
+        assert [(a.key, a.central) for a in part.answers] == ranked

@@ -12,9 +12,8 @@ G = kgs.kgs_load_graph(w.graph)
 for i in (int(x) for x in sys.argv[1:]):
     kw = w.queries[i]
     for rec in os.environ.get("RECS", "1,0").split(","):
-        os.environ["KGS_DAG_RECORD"] = rec
         try:
-            r = kgs.kgs_query(G, kw, w.k, kgs.make_params(prune=int(os.environ.get("PRUNE", "1"))))
+            r = kgs.kgs_query(G, kw, w.k, kgs.make_params(prune=int(os.environ.get("PRUNE", "1")), dag_record=int(rec)))
             s = r.stats
             print(i, "rec", rec, "q", len(kw), {k: s[k] for k in ("levels", "n_centrals", "arcs_scanned", "td_arcs",
                                                                   "td_pred_arcs", "dag_arcs", "overflow", "ms_search",
