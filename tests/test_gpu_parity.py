@@ -245,3 +245,26 @@ def test_batch_capacity_overflow_is_per_query():
     with pytest.raises(kgs.KgsError):
         kgs.kgs_query(G, [0, 1], 1)
     G.close()
+
+
+def test_level_ring_resizing_across_alpha_and_groups():
+    """The level-slot ring has R = amax + 2 slots and amax depends on alpha when the largest weight is
+    below 1: a G = 1 query at alpha 0.05 (R = 7), then a G = 8 batch at alpha 0.4 (R = 5, new group
+    workspaces), then both again.  Every workspace must hold the largest ring (an undersized one would be
+    written out of bounds); every answer must equal the oracle's."""
+    _gpu()
+    w = synth.make_workload("C1")
+    g = w.graph
+    g.weight = (np.asarray(g.weight, np.float64) * 0.3).astype(np.float32)
+    G = kgs.kgs_load_graph(g)
+    qs = w.queries[:24]
+    for rnd in range(2):
+        for alpha, groups in ((0.05, 1), (0.4, 8), (0.05, 8), (0.4, 1)):
+            exp = [oracle.query(g, kw, w.k, alpha=alpha) for kw in qs]
+            p = kgs.make_params(alpha=alpha)
+            res = kgs.kgs_query_batch(G, qs, w.k, p, groups) if groups > 1 else [kgs.kgs_query(G, kw, w.k, p) for kw in qs]
+            for kw, r, o in zip(qs, res, exp):
+                ctx = (rnd, alpha, groups, kw)
+                assert r.stats["levels"] == o.levels and r.stats["stop_reason"] == o.stop_reason, ctx
+                assert [(a.central, a.score_key) for a in r.answers] == [(a.central, a.key) for a in o.answers], ctx
+    G.close()
