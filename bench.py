@@ -5,20 +5,19 @@ queries/s and GTEPS on the Wikidata-scale synthetic graph).
   python bench.py [--gpus N --steps K --warmup W]          CUDA path (libkgs), one rank per GPU
   python bench.py --impl reference [...]                   the CPU oracle on this box's host cores
 
-Workload: C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 2-8 keyword queries, top-20) at every N.
+Workload (--workload): C3 (BASELINE.json configs[2]: 2^25 nodes / 2^28 edges, 350 queries with q = 2..8,
+top-20; the default) or C4 (configs[3]: the same graph, 4096 queries with q ~ U{2..8}).  A step = the
+workload's whole batch through the whole hot path (activation gate, search, central detection, extraction
++ level-cover + Eq. 6 of the candidate central graphs, top-k, answer emit) in ONE engine launch per rank.
 N > 1 (torchrun): every rank holds a replica of the graph (rank 0 generates it and broadcasts it over
-NCCL) and answers the 350 C3 queries per step, starting at a rank-dependent offset; one NCCL all-gather of
-the top-k headers per step (inside the timed region).  The per-rank step is the same for every N (weak
-scaling).  C4's own query set (configs[3], 4096 queries with q ~ U{2..8}) is not used for the bench line:
-7 of its queries (0.17%) only find k central nodes at level 5, where ~1 M nodes become central at once and
-the exact top-down takes 40-50 s each (tools/workload_scan.py).
+NCCL), the step's batch is dealt round-robin over the ranks (dist.shard: total work fixed, strong
+scaling), and the top-k headers and answer subgraphs are all-gathered over NCCL inside the timed region.
 
-A step = one batch of queries through the whole hot path in ONE engine launch (activation gate, search,
-central detection, extraction + level-cover + Eq. 6 of every central graph, top-k, answer emit):
-the 350-query C3 set (each query once per step).  `value` = queries/s of device time over K steps (CUDA events on the launching stream, L2 flushed
-with a 512 MiB write between steps, outside the events; max over ranks).  The single-query latency
-mode (one launch per query, the whole GPU on it) gives `p50_ms` / `p95_ms`.  `e2e` = the same batches
-through kgs_query_batch from host keyword ids to host answers (wall clock, H2D + D2H inside).
+`value` = queries/s of device time over K steps (CUDA events on the launching stream, L2 flushed with a
+512 MiB write between steps, outside the events; max over ranks).  The single-query latency mode (one
+launch per query, the whole GPU on it) gives `p50_ms` / `p95_ms` and the expansion-phase roofline.
+`e2e` = the same batches through kgs_query_batch from host keyword ids to host answers (wall clock,
+H2D + D2H inside).  `cpu_baseline` = the oracle on ~15 s of the step's queries, pinned to one core.
 """
 from __future__ import annotations
 
@@ -38,7 +37,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "p50 query latency (ms) & queries/s, Wikidata-scale graph; GTEPS"
-BATCH = 350          # queries per step (the C3 latency set)
+WORKLOAD = "C3"      # the step's batch: C3's 350 queries (configs[2]) or C4's 4096 (configs[3], --workload C4)
 GROUPS = 8           # engine groups in batch mode (queries answered at the same time)
 RELABEL = os.environ.get("KGS_RELABEL", "1") != "0"   # ablation: 0 keeps the input node order internally
 
@@ -108,18 +107,71 @@ def load_peaks():
         return 6650.0, "fallback"
 
 
-def load_traffic():
-    """DRAM bytes per query of the engine from the newest committed ncu capture (profiles/): a capture of
-    the bench's own launch shape (r*_batch_traffic.json: one 350-query launch, G = 8) when there is one,
-    else the latency-mode per-query captures (r*_engine_traffic.json)."""
-    for pat, key in (("r*_batch_traffic.json", "dram_bytes_per_query"),
-                     ("r*_engine_traffic.json", "mean_dram_bytes_per_query")):
-        files = sorted(glob.glob(os.path.join(ROOT, "profiles", pat)))
-        if files:
-            with open(files[-1]) as f:
-                d = json.load(f)
-            return d[key], os.path.basename(files[-1])
-    return None, None
+ENGINE_SOURCES = ("paper_conf_icde_yangajtw19_b200/csrc/*.cu", "paper_conf_icde_yangajtw19_b200/csrc/*.h",
+                  "include/kgs.h")
+
+
+def source_hash() -> str:
+    """sha256 over the engine's sources (csrc/*.cu, *.h, include/kgs.h): identifies the build an ncu
+    capture was taken of (tools/make_batch_profile.py stores it next to the DRAM bytes)."""
+    import hashlib
+    h = hashlib.sha256()
+    for pat in ENGINE_SOURCES:
+        for f in sorted(glob.glob(os.path.join(ROOT, pat))):
+            h.update(os.path.basename(f).encode())
+            with open(f, "rb") as fh:
+                h.update(fh.read())
+    return h.hexdigest()
+
+
+def load_traffic(workload: str):
+    """DRAM bytes per query of the engine from the newest committed ncu capture of the bench's own launch
+    shape (profiles/r*_batch_traffic.json for this workload), with the git sha / source hash it was
+    taken at.  Returns (bytes per query or None, info dict)."""
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_batch_traffic.json")))
+    for f in reversed(files):
+        with open(f) as fh:
+            d = json.load(fh)
+        if d.get("workload", "C3") != workload:
+            continue
+        return d["dram_bytes_per_query"], {"traffic_source": os.path.basename(f), "traffic_sha": d.get("git_sha"),
+                                           "traffic_matches_source": d.get("src_sha256") == source_hash(),
+                                           "traffic_l2_hit_pct": d.get("l2_hit_pct")}
+    return None, {"traffic_source": None}
+
+
+def cpu_info() -> dict:
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count()}
+
+
+class pinned_core:
+    """Run the oracle on ONE host core (the `taskset -c <cpu>` of the CPU-baseline protocol)."""
+
+    def __enter__(self):
+        self.old = os.sched_getaffinity(0)
+        self.cpu = min(self.old)
+        os.sched_setaffinity(0, {self.cpu})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.old)
+        return False
+
+
+def expansion_bytes(st: dict) -> float:
+    """SURVEY.md §8(d) B_bfs: the bytes the expansion must move for one query — per frontier entry 16 B
+    row_ptr + 2 B own status + 1 B activation + 4 B queue slot, per inspected out-arc 4 B col_idx + 2 B
+    neighbour status, per new (node, keyword) hit 1 B M + 1 B new-hit mask + 4 B next frontier."""
+    return st["frontier_total"] * 23.0 + st["arcs_scanned"] * 6.0 + st.get("hits", 0) * 6.0
 
 
 def algorithmic_bytes(st: dict) -> float:
@@ -134,10 +186,23 @@ def algorithmic_bytes(st: dict) -> float:
 
 # ------------------------------------------------------------------------------------------ workloads
 def build_workload(name: str):
+    """C3 (configs[2]) or C4 (configs[3]: the C3 graph with its own 4096-query set)."""
     import synth
     t0 = time.time()
-    w = synth.make_workload(name)
+    if name == "C4":
+        w = synth.make_workload("C3")
+        w = synth.Workload("C4", w.graph, synth.config_queries("C4", w.graph), synth.CONFIG_PARAMS["C4"]["k"])
+    else:
+        w = synth.make_workload(name)
     return w, time.time() - t0
+
+
+def step_queries(name: str, queries):
+    """The queries of one step in their order: C3's 350 in the bench permutation, C4's 4096 as generated."""
+    if name == "C3":
+        order = np.random.default_rng(12345).permutation(len(queries))
+        return [queries[i] for i in order], [int(i) for i in order]
+    return list(queries), list(range(len(queries)))
 
 
 class _RemoteGraph:
@@ -194,35 +259,40 @@ def load_replicated(name, rank, world, dev, kgs):
     return SimpleNamespace(queries=queries, k=k), _RemoteGraph(n, m), G, gen_s, load_s
 
 
+def graph_desc(name, g):
+    return f"R-MAT scale 25, edge factor 8: {g.n} nodes, {g.n_arcs} arcs" + (" (the C3 graph)" if name == "C4" else "")
+
+
 def run_reference(args):
-    """The oracle, as it stands, on host cores (bench.py --impl reference): rank 0 only."""
+    """The oracle, as it stands, on ONE pinned host core (bench.py --impl reference): rank 0 only.  A step
+    is one query of the workload (the oracle is single-threaded); K steps after W warm-up queries."""
     rank, world = _env_int("RANK", 0), _env_int("WORLD_SIZE", 1)
     if rank != 0:
         return 0
     import oracle
-    name = "C3"   # the GPU arm's workload at every N
+    name = args.workload
     w, gen_s = build_workload(name)
-    order = np.random.default_rng(12345).permutation(len(w.queries))
-    qs = [w.queries[i] for i in order]
-    for i in range(args.warmup):
-        oracle.query(w.graph, qs[i % len(qs)], w.k)
+    qs, _ = step_queries(name, w.queries)
     lat = []
-    t_all = time.perf_counter()
-    for i in range(args.steps):
-        kw = qs[(args.warmup + i) % len(qs)]
-        t0 = time.perf_counter()
-        oracle.query(w.graph, kw, w.k)
-        lat.append((time.perf_counter() - t0) * 1e3)
-    tot = time.perf_counter() - t_all
+    with pinned_core() as pc:
+        for i in range(args.warmup):
+            oracle.query(w.graph, qs[i % len(qs)], w.k)
+        t_all = time.perf_counter()
+        for i in range(args.steps):
+            kw = qs[(args.warmup + i) % len(qs)]
+            t0 = time.perf_counter()
+            oracle.query(w.graph, kw, w.k)
+            lat.append((time.perf_counter() - t0) * 1e3)
+        tot = time.perf_counter() - t_all
     qps = args.steps / tot
     line = {"impl": "reference", "metric": METRIC, "value": qps, "unit": "queries/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot * 1e3 / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {w.graph.n} nodes, "
-                                                   f"{w.graph.n_arcs} arcs", "k": w.k, "queries": len(qs),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "config": {"workload": name, "graph": graph_desc(name, w.graph), "k": w.k, "queries": len(qs),
                        "step": "one query (the oracle is single-threaded; a step of the GPU arm is a batch)"},
             "p50_ms": statistics.median(lat),
-            "cpu_baseline": {"value": qps, "unit": "queries/s", "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": qps, "unit": "queries/s", "cores": 1, "kind": "oracle", "pinned_cpu": pc.cpu,
+                             **cpu_info(),
                              "sample": f"{args.steps} consecutive {name} queries after {args.warmup} warm-up"},
             "e2e": {"value": qps, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -235,8 +305,8 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="kgs", choices=["kgs", "reference"])
+    ap.add_argument("--workload", default=WORKLOAD, choices=["C3", "C4"])
     ap.add_argument("--groups", type=int, default=GROUPS)
-    ap.add_argument("--batch", type=int, default=BATCH)
     ap.add_argument("--latency-steps", type=int, default=200)
     ap.add_argument("--cpu-sample-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -263,8 +333,9 @@ def main():
     torch.cuda.set_device(dev)
     cuda = f"cuda:{dev}"
     import paper_conf_icde_yangajtw19_b200 as kgs
+    from paper_conf_icde_yangajtw19_b200 import dist as kd
 
-    name = "C3"
+    name = args.workload
     if world == 1:
         w, gen_s = build_workload(name)
         g = w.graph
@@ -273,33 +344,27 @@ def main():
         load_s = time.time() - t0
     else:
         w, g, G, gen_s, load_s = load_replicated(name, rank, world, dev, kgs)
-    order = np.random.default_rng(12345).permutation(len(w.queries))
-    allq = [w.queries[i] for i in order]
-    qids_all = [int(i) for i in order]
-    off = (rank * len(allq)) // world   # N > 1: the same set, rotated per rank
-    mine = [(off + i) % len(allq) for i in range(len(allq))]
+    allq, qids_all = step_queries(name, w.queries)
+    # one step = the workload's whole batch, dealt round-robin over the ranks (dist.shard): strong scaling
+    mine = kd.shard(len(allq), rank, world).tolist()
     queries = [allq[i] for i in mine]
     qids = [qids_all[i] for i in mine]
-    B = args.batch
+    B = len(queries)
     stream = torch.cuda.current_stream(dev)
     sh = stream.cuda_stream
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=cuda)
-
-    def batch_rows(step):
-        idx = [((step * B) + j) % len(queries) for j in range(B)]
-        kwp = torch.full((B, 8), -1, dtype=torch.int32)
-        for r, i in enumerate(idx):
-            kwp[r, :len(queries[i])] = torch.tensor(queries[i], dtype=torch.int32)
-        return idx, kwp.to(cuda), torch.tensor([len(queries[i]) for i in idx], dtype=torch.int32, device=cuda)
-
-    steps_in = [batch_rows(s) for s in range(args.warmup + args.steps)]
+    kwp = torch.full((B, 8), -1, dtype=torch.int32)
+    for r, q in enumerate(queries):
+        kwp[r, :len(q)] = torch.tensor(q, dtype=torch.int32)
+    kwd = kwp.to(cuda)
+    qld = torch.tensor([len(q) for q in queries], dtype=torch.int32, device=cuda)
+    qlens = [len(q) for q in queries]
     p = kgs.kgs_params_default()
 
-    # ---- batch mode (value): one engine launch per step, GROUPS queries at a time
-    for s in range(args.warmup):
-        _, kwd, qld = steps_in[s]
+    # ---- batch mode (value): one engine launch per step
+    for s_ in range(args.warmup):
         kgs.kgs_query_batch_device(G, B, kwd.data_ptr(), qld.data_ptr(), w.k, p, args.groups, sh)
-        kgs.kgs_query_batch_fetch(G, qld.tolist(), sh)
+        kgs.kgs_query_batch_fetch(G, qlens, sh)
     torch.cuda.synchronize(dev)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     stats, answers, subgraphs = [], [], []
@@ -309,27 +374,25 @@ def main():
         dist.barrier()
     torch.cuda.synchronize(dev)
     for i in range(args.steps):
-        idx, kwd, qld = steps_in[args.warmup + i]
         flush.fill_(i & 0xFF)                       # L2 flush between timed steps (outside the events)
         ev[i][0].record(stream)
         kgs.kgs_query_batch_device(G, B, kwd.data_ptr(), qld.data_ptr(), w.k, p, args.groups, sh)
         ev[i][1].record(stream)
-        res = kgs.kgs_query_batch_fetch(G, qld.tolist(), sh)   # after the end event: not timed
+        res = kgs.kgs_query_batch_fetch(G, qlens, sh)   # after the end event: not timed
         stats += [r.stats for r in res]
         if i == args.steps - 1:
-            answers = [(qids[j], [(a.central, a.depth, a.score_key) for a in r.answers]) for j, r in zip(idx, res)]
-            subgraphs = [(qids[j], [(a.nodes, a.arcs) for a in r.answers]) for j, r in zip(idx, res)]
+            answers = [(qids[j], [(a.central, a.depth, a.score_key) for a in r.answers]) for j, r in enumerate(res)]
+            subgraphs = [(qids[j], [(a.nodes, a.arcs) for a in r.answers]) for j, r in enumerate(res)]
     gather_ms = 0.0
     if dist:
         # NCCL all-gather of every rank's top-k headers (central, depth, key) and answer subgraphs
         # (sizes, then a padded gather of the variable payloads) of the last step
-        from paper_conf_icde_yangajtw19_b200 import dist as kd
         hdr = kd.pack_headers([q for q, _ in answers], [a for _, a in answers], w.k).to(cuda)
         pidx, pdat = kd.pack_payloads([q for q, _ in subgraphs], [s_ for _, s_ in subgraphs])
         pidx, pdat = pidx.to(cuda), pdat.to(cuda)
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        kd.gather_headers(hdr, len(answers) * world, world)
+        kd.gather_headers(hdr, len(allq), world)
         kd.gather_payloads(pidx, pdat)
         e1.record(stream)
     torch.cuda.synchronize(dev)
@@ -343,14 +406,16 @@ def main():
         t = torch.tensor([dev_ms], dtype=torch.float64, device=cuda)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dev_ms = float(t.item())
-    total_queries = args.steps * B * world
+    total_queries = args.steps * len(allq)
     value = total_queries / (dev_ms / 1e3)
-    arcs = sum(s["arcs_scanned"] for s in stats)   # GTEPS: arcs the search expanded
-    alg = sum(algorithmic_bytes(s) for s in stats)
+    arcs = sum(s_["arcs_scanned"] for s_ in stats)   # GTEPS: arcs the search expanded
+    alg = sum(algorithmic_bytes(s_) for s_ in stats)
+    exp_b = sum(expansion_bytes(s_) for s_ in stats)
+    exp_us = sum(s_["phases_us"].get("expand", 0.0) for s_ in stats)   # group time, G groups at once
+    n_groups = max(1, min(args.groups, B))
 
     # ---- single-query latency mode: the whole GPU on one query, one launch per query
-    lat = []
-    lat_stats = []
+    lat, lat_stats = [], []
     if rank == 0:
         nlat = min(args.latency_steps, len(queries))
         qdev = [torch.tensor(list(q), dtype=torch.int32, device=cuda) for q in queries[:nlat + args.warmup]]
@@ -371,14 +436,19 @@ def main():
     # ---- e2e: host keyword ids -> kgs_query_batch -> answers on the host (wall clock)
     e2e_ms, d2h = [], 0
     for i in range(min(args.steps, 3)):
-        idx = [((i * B) + j) % len(queries) for j in range(B)]
-        hq = [queries[j] for j in idx]
         torch.cuda.synchronize(dev)
+        if dist:
+            dist.barrier()
         t0 = time.perf_counter()
-        res = kgs.kgs_query_batch(G, hq, w.k, p, args.groups, sh)
-        e2e_ms.append((time.perf_counter() - t0) * 1e3)
+        res = kgs.kgs_query_batch(G, queries, w.k, p, args.groups, sh)
+        el = (time.perf_counter() - t0) * 1e3
+        if dist:
+            t = torch.tensor([el], dtype=torch.float64, device=cuda)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            el = float(t.item())
+        e2e_ms.append(el)
         d2h += sum(32 + a.nodes.nbytes + a.arcs.nbytes + 24 for r in res for a in r.answers)
-    e2e_qps = len(e2e_ms) * B / (sum(e2e_ms) / 1e3)
+    e2e_qps = len(e2e_ms) * len(allq) / (sum(e2e_ms) / 1e3)
     h2d = B * (4 * 8 + 4)
 
     if rank != 0:
@@ -386,18 +456,22 @@ def main():
             dist.destroy_process_group()
         return 0
     peak, peak_kind = load_peaks()
-    tr, tr_src = load_traffic()
+    tr, tr_info = load_traffic(name)
     achieved = alg / (sum(step_ms) / 1e3) / 1e9
-    lat_alg = sum(algorithmic_bytes(s) for s in lat_stats)
+    lat_alg = sum(algorithmic_bytes(s_) for s_ in lat_stats)
+    lat_exp_b = sum(expansion_bytes(s_) for s_ in lat_stats)
+    lat_exp_us = sum(s_["phases_us"].get("expand", 0.0) for s_ in lat_stats)
+    exp_lat = lat_exp_b / (lat_exp_us * 1e-6) / 1e9 if lat_exp_us else None
+    exp_bat = exp_b / (exp_us * 1e-6 / n_groups) / 1e9 if exp_us else None
     line = {
         "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": dev_ms / args.steps, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": name, "graph": f"R-MAT scale 25, edge factor 8: {g.n} nodes, {g.n_arcs} arcs",
-                   "k": w.k, "queries_per_step": B * world, "engine_groups": args.groups, "alpha": 0.1,
-                   "lambda": 0.2, "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
+        "config": {"workload": name, "graph": graph_desc(name, g), "k": w.k, "queries_per_step": len(allq),
+                   "queries_per_rank": B, "engine_groups": args.groups, "alpha": 0.1, "lambda": 0.2,
+                   "l2": "flushed between timed steps (512 MiB write)", "gen_s": round(gen_s, 1),
                    "load_s": round(load_s, 1), "node_order": "degree (internal relabel)" if RELABEL else "input",
-                   "parallelism": f"query-sharded x{world}" if world > 1 else "single GPU"},
+                   "parallelism": f"query-sharded x{world} (dist.shard, replicated graph)" if world > 1 else "single GPU"},
         "p50_ms": statistics.median(lat) if lat else None,
         "p95_ms": float(np.percentile(lat, 95)) if lat else None,
         "latency_mode": {"queries": len(lat), "qps": len(lat) / (sum(lat) / 1e3) if lat else None,
@@ -405,26 +479,35 @@ def main():
         "gteps": arcs / (dev_ms / 1e3) / 1e9 * world,
         "roofline": {"kernel": "k_engine", "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "peak_kind": peak_kind,
-                     "traffic": (tr * B) if tr else None, "traffic_source": tr_src,
+                     "traffic": (tr * len(allq)) if tr else None, **tr_info,
                      "algorithmic_bytes_per_launch": alg / args.steps,
-                     "latency_mode_achieved": (lat_alg / (sum(lat) / 1e3) / 1e9) if lat else None},
+                     "latency_mode_achieved": (lat_alg / (sum(lat) / 1e3) / 1e9) if lat else None,
+                     # the BFS expansion phase alone (north_star's target): B_bfs / expansion time from the
+                     # in-kernel %globaltimer stamps; latency mode = the whole GPU on one query's levels,
+                     # batch = summed group expansion time / G (groups expand concurrently)
+                     "expansion_achieved": exp_lat, "expansion_frac": (exp_lat / peak) if exp_lat else None,
+                     "expansion_frac_batch_est": (exp_bat / peak) if exp_bat else None,
+                     "expansion_bytes_per_query": (lat_exp_b / len(lat_stats)) if lat_stats else None},
         "e2e": {"value": e2e_qps, "unit": "queries/s", "ms_per_step": statistics.median(e2e_ms),
-                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h / len(e2e_ms)},
-        "gpu_launches": args.steps,   # one k_engine launch per step
+                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world / len(e2e_ms)},
+        "gpu_launches": args.steps,   # one k_engine launch per step (per rank)
         "clocks": clocks,
-        "stats_mean": {k: float(np.mean([s[k] for s in stats])) for k in
+        "stats_mean": {k: float(np.mean([s_[k] for s_ in stats])) for k in
                        ("levels", "n_centrals", "frontier_total", "arcs_scanned", "td_arcs", "overflow")},
     }
     if not args.no_cpu_baseline and world == 1:
         import oracle
-        t0 = time.perf_counter()
         done = 0
-        while time.perf_counter() - t0 < args.cpu_sample_s and done < len(queries):
-            oracle.query(g, queries[done], w.k)
-            done += 1
-        el = time.perf_counter() - t0
+        with pinned_core() as pc:
+            t0 = time.perf_counter()
+            while time.perf_counter() - t0 < args.cpu_sample_s and done < len(queries):
+                oracle.query(g, queries[done], w.k)
+                done += 1
+            el = time.perf_counter() - t0
         line["cpu_baseline"] = {"value": done / el, "unit": "queries/s", "cores": 1, "kind": "oracle",
-                                "sample": f"the first {done} {name} queries of a step ({el:.1f} s, single-threaded oracle)"}
+                                "pinned_cpu": pc.cpu, **cpu_info(),
+                                "sample": f"the first {done} {name} queries of a step ({el:.1f} s, single-threaded "
+                                          f"oracle pinned to one core)"}
     print(json.dumps(line), flush=True)
     if dist:
         dist.destroy_process_group()

@@ -43,7 +43,7 @@ def _load():
         vp, i64, i32, dbl = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_double
         L.oracle_query.restype = vp
         L.oracle_query.argtypes = [i64, vp, vp, vp, i64, vp, vp, dbl, i32, vp, i32, i64, dbl, dbl, i32, i32, i32, i32, i32,
-                                   vp, i64]
+                                   vp, i64, i32]
         L.oracle_activation.argtypes = [i64, vp, dbl, dbl, vp]
         L.oracle_snap_weights.argtypes = [i64, vp, vp]
         for f in ("oracle_a", "oracle_M", "oracle_centrals", "oracle_central_depth", "oracle_central_key"):
@@ -108,11 +108,13 @@ class Result:
 
 def query(g, kw_ids, k: int, *, alpha: float = 0.1, lam: float = 0.2, max_depth: int = 254,
           block_central: int = 1, extract_mode: int = EXTRACT_EXACT, bfs_form: int = BFS_LITERAL,
-          level_cover: int = 1, eval_ids=None) -> Result:
+          level_cover: int = 1, eval_ids=None, containment: int = 0) -> Result:
     """One query through the oracle.  ``g`` is a synth.Graph-like object (row_ptr, col_idx, weight,
     kw_ptr, kw_nodes, A, symmetric).  ``eval_ids`` (test sampling at sizes where scoring every central
     node is out of reach): only these central nodes are extracted and scored (the others' keys are NaN)
-    and the answers rank them alone."""
+    and the answers rank them alone.  ``level_cover``: 0 off, 1 the "contribute" reading (R13, default), 2
+    the "contains" reading (R13b, NEXT-3).  ``containment`` = 1: drop every Central Graph that strictly
+    contains another one's node set (R16, NEXT-3)."""
     L = _load()
     kw = np.ascontiguousarray(np.asarray(kw_ids, dtype=np.int32))
     q = int(kw.shape[0])
@@ -127,7 +129,7 @@ def query(g, kw_ids, k: int, *, alpha: float = 0.1, lam: float = 0.2, max_depth:
                        kn.ctypes.data, float(g.A), 1 if g.symmetric else 0, kw.ctypes.data, q, int(k),
                        float(alpha), float(lam), int(max_depth), int(block_central), int(extract_mode),
                        int(bfs_form), int(level_cover), None if ev is None else ev.ctypes.data,
-                       0 if ev is None else int(ev.shape[0]))
+                       0 if ev is None else int(ev.shape[0]), int(containment))
     try:
         st = L.oracle_status(h)
         if st != 0:

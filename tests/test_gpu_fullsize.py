@@ -126,7 +126,8 @@ def test_c3_pull_direction(c3):
 
 
 # C4 queries that only find k central nodes at level 5 (tools/workload_scan.py, search-only scan of all
-# 4096 queries on the B200): ~10^6 central nodes each.
+# 4096 queries on the B200, profiles/r02b_c4_scan.txt; query 11, also level 5, is in the first 62): ~10^6
+# central nodes each.
 C4_LEVEL5 = (2683, 2906)
 
 
@@ -153,7 +154,7 @@ def test_c4_sample_with_level5_queries(c3):
         sampled = int(np.isin(o.centrals, ids).sum())
         assert sampled > len(r.answers) + 200, ctx      # the sample holds central nodes besides the answers
         _check(r, o, full=False, ctx=ctx)
-    assert deep == len(C4_LEVEL5)
+    assert deep >= len(C4_LEVEL5) and all(r.stats["levels"] == 5 for r in res[-len(C4_LEVEL5):])
 
 
 def test_c5_ten_queries():
