@@ -103,7 +103,12 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *   max_depth      1..254, default 254 (255 encodes infinity in M).
  *   block_central  1 (default): a node identified as central no longer expands (Alg. 2 ln 2).
  *   extract_mode   KGS_EXTRACT_EXACT (default) or KGS_EXTRACT_LITERAL.
- *   level_cover    1 (default): apply level-cover pruning; 0 returns unpruned Central Graphs.
+ *   level_cover    level-cover pruning: 1 (default) a keyword node's level counts the keywords it
+ *                  contributes (it is a source of a hitting path of this Central Graph, reading R13);
+ *                  2 the keywords it contains (NEXT-3, reading R13b); 0 returns unpruned Central Graphs.
+ *   containment    1: drop every Central Graph whose pruned node set strictly contains the pruned node
+ *                  set of another Central Graph of C (NEXT-3, reading R16), answers = the k best of
+ *                  the rest among the best min(|C|, KGS_MAX_K); forces prune = 0.  0 (default): off.
  *   want_levels    1: also copy M and the central list back (for parity checks); default 0.
  *   prune          exact lower-bound pruning of the top-down phase (Eq. 6 keys are computed only for the
  *                  candidates whose (bound, id) can still beat the k-th exact (key, id); the answers are
@@ -141,6 +146,7 @@ typedef struct {
     int32_t pull_ratio;
     int64_t pull_min;
     int32_t prune_min, tile_light, dag_record, search_only;
+    int32_t containment;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 

@@ -434,6 +434,8 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.extract_mode != KGS_EXTRACT_EXACT && p.extract_mode != KGS_EXTRACT_LITERAL)
         return fail(KGS_EINVAL, "extract_mode");
     if (p.prune < 0 || p.prune > 2) return fail(KGS_EINVAL, "prune must be 0, 1 or 2");
+    if (p.level_cover < 0 || p.level_cover > 2) return fail(KGS_EINVAL, "level_cover must be 0, 1 or 2");
+    if (p.containment != 0 && p.containment != 1) return fail(KGS_EINVAL, "containment must be 0 or 1");
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
         p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1))
@@ -554,11 +556,12 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.nq = nq; a.kw = g->d_kw; a.qlen = g->d_qlen; a.qconst = qconst;
     a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
     a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
-    a.level_cover = p.level_cover ? 1 : 0;
+    a.level_cover = p.level_cover;
+    a.containment = p.containment;
     if (td) { a.td_only = 1; a.td_levels = td->levels; a.td_stop = td->stop; a.td_ncentral = td->n_central; }
     // the parity view wants every central's key.  The path bound needs the Thm. V.4 DAG to be made of
     // arcs the search traversed: exact extraction, or no central blocking.
-    a.prune = p.want_levels ? 0 : p.prune;
+    a.prune = (p.want_levels || p.containment) ? 0 : p.prune;
     if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
     a.prune_min = p.prune_min;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central

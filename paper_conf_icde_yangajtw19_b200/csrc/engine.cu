@@ -1447,8 +1447,11 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     if (S.scal[SC_OVF]) return CG_OVERFLOW;
     const int nn = S.scal[SC_NODES];
     const int na = S.scal[SC_ARCS] < S.acap ? S.scal[SC_ARCS] : S.acap;
-    // ---- level-cover
+    // ---- level-cover: a keyword node's level counts the keywords it contributes (R13: a source
+    // of a hitting path in DAG_i(c), inmask & zb) or, with level_cover = 2, the keywords it contains (R13b:
+    // zb, its m = 0 keywords)
     if (c.a.level_cover) {
+        const uint32_t lmask = c.a.level_cover == 2 ? 0xFFu : 0u;
         const uint32_t cov0 = S.zb[0];
         int sstar = c.qq.q + 1;
         if (cov0 != full) {
@@ -1456,7 +1459,7 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
             T.sync();
             for (int s = c.qq.q; s >= 1; --s) {
                 for (int j = 1 + r; j < nn; j += ts) {
-                    const uint32_t con = S.inmask[j] & S.zb[j];
+                    const uint32_t con = (S.inmask[j] | lmask) & S.zb[j];
                     if (__popc(con) == s) atomicOr(reinterpret_cast<unsigned *>(S.scal + SC_COV), con);
                 }
                 T.sync();
@@ -1465,8 +1468,9 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
             }
         }
         for (int j = r; j < nn; j += ts) {
-            const uint32_t con = S.inmask[j] & S.zb[j];
-            S.keep[j] = (j == 0 || __popc(con) >= sstar) ? con : 0u;
+            const uint32_t src = S.inmask[j] & S.zb[j];                 // the DAGs j is a kept source of
+            const uint32_t lvl = (S.inmask[j] | lmask) & S.zb[j];       // its level-cover level
+            S.keep[j] = (j == 0 || __popc(lvl) >= sstar) ? src : 0u;
         }
         T.sync();
         for (;;) {   // forward reachability from the kept sources inside each DAG_i
@@ -1731,6 +1735,108 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem, uint32_t k
     rank_list(c, dsmem, c.w.elist, kk, kk);
 }
 
+// ------------------------------------------------------------------------------------------ containment
+// NEXT-3, containment removal ("we remove the Central Graph that completely contains smaller ones",
+// reading R16): the answers are the k best (key, id) among the candidates whose pruned node set does not
+// strictly contain the pruned node set of another Central Graph of C, looked for among the best
+// W = min(|C|, KGS_MAX_K).  G(c) can only contain G(c') if it holds c' (c' is always in its own graph), so
+// a candidate is checked against the central nodes inside it (st hit mask = all keywords, Lemma V.1).
+// One CTA per ranked candidate: its graph in the CTA's large arena (membership by hash lookup), each inner
+// central's graph in the CTA's big arena.  Ranked positions are checked a chunk at a time until kk
+// survivors are known.  Every key is exact here (the host forces prune = 0).
+
+// index of node u in an arena after central_graph (-1: not in it)
+__device__ __forceinline__ int arena_find(const Arena &S, int32_t u) {
+    uint32_t h = hash32((uint32_t)u) & (uint32_t)(S.hcap - 1);
+    for (int probe = 0; probe < S.hcap; ++probe) {
+        const int32_t k = S.hkey[h];
+        if (k == u) return S.hval[h];
+        if (k == -1) return -1;
+        h = (h + 1) & (uint32_t)(S.hcap - 1);
+    }
+    return -1;
+}
+
+// kept nodes of an arena after central_graph (whole CTA)
+__device__ __forceinline__ int arena_kept(const Arena &S, long long *sh) {
+    const int nn = S.scal[SC_NODES];
+    int cnt = 0;
+    for (int j = threadIdx.x; j < nn; j += blockDim.x) cnt += S.keep[j] != 0u;
+    long long tot;
+    block_excl_scan64(cnt, &tot, sh);
+    return (int)tot;
+}
+
+__device__ void containment_select(const Ctx &c, long long *sh, char *dsmem, uint32_t kk) {
+    const Grp &G = c.G;
+    const EngineArgs &a = c.a;
+    Ctl *ctl = c.ctl;
+    const uint32_t nc = __ldcg(&ctl->n_central);
+    const uint32_t W = nc < (uint32_t)KGS_MAX_K ? nc : (uint32_t)KGS_MAX_K;
+    select_topk(c, sh, dsmem, W);                 // sel[0..W): ranked by (key, id); ends with a barrier
+    int32_t *removed = c.w.overflow;              // per ranked position (the extraction lists are done)
+    BlockTeam BT{sh};
+    Arena SL = carve(a.large_arenas + a.large_arena_bytes * blockIdx.x, a.large_hash, a.large_nodes, a.large_arcs,
+                     blockDim.x, false, true);
+    Arena S3 = carve(a.cta_arenas + a.cta_arena_bytes * blockIdx.x, a.big_hash, a.big_nodes, a.big_arcs, blockDim.x,
+                     true, true);
+    __shared__ int s_flag;
+    __shared__ uint32_t s_pos;
+    const uint32_t chunk = max((uint32_t)G.gcount, 2u * kk);
+    for (uint32_t p0 = 0; p0 < W; p0 += chunk) {
+        const uint32_t p1 = min(W, p0 + chunk);
+        for (uint32_t t = p0 + G.grank; t < p1; t += G.gcount) {
+            const int32_t idx = __ldcg(c.w.sel + t);
+            const int32_t cn = __ldcg(c.w.centrals + idx);
+            double key;
+            int rem = 0;
+            if (central_graph(BT, SL, c, cn, __ldcg(c.w.cdepth + idx), &key) != CG_OK) {
+                if (threadIdx.x == 0) atomicExch(&ctl->fatal, 6);
+            } else {
+                const int nn = SL.scal[SC_NODES];
+                const int nkc = arena_kept(SL, sh);
+                for (int j = 0; j < nn && !rem; ++j) {
+                    const int32_t x = SL.id[j];
+                    if (!SL.keep[j] || x == cn || (__ldcg(c.w.st + x) & 0xFFu) != c.qq.full) continue;
+                    if (central_graph(BT, S3, c, x, 0, &key) != CG_OK) {
+                        if (threadIdx.x == 0) atomicExch(&ctl->fatal, 6);
+                        break;
+                    }
+                    if (arena_kept(S3, sh) >= nkc) continue;
+                    if (threadIdx.x == 0) s_flag = 1;
+                    __syncthreads();
+                    const int nx = S3.scal[SC_NODES];
+                    for (int i = threadIdx.x; i < nx; i += blockDim.x) {
+                        if (!S3.keep[i]) continue;
+                        const int f = arena_find(SL, S3.id[i]);
+                        if (f < 0 || !SL.keep[f]) s_flag = 0;
+                    }
+                    __syncthreads();
+                    rem = s_flag;
+                    __syncthreads();
+                }
+            }
+            if (threadIdx.x == 0) removed[t] = rem;
+            __syncthreads();
+        }
+        G.sync();
+        if (threadIdx.x == 0) {   // survivors so far (every CTA computes the same count)
+            uint32_t kept = 0;
+            for (uint32_t t = 0; t < p1; ++t) kept += __ldcg(removed + t) == 0;
+            s_pos = kept;
+        }
+        __syncthreads();
+        if (s_pos >= kk) break;
+    }
+    if (G.grank == 0 && threadIdx.x == 0) {   // the first kk survivors in rank order
+        uint32_t kept = 0;
+        for (uint32_t t = 0; t < W && kept < kk; ++t)
+            if (__ldcg(removed + t) == 0) c.w.sel[kept++] = __ldcg(c.w.sel + t);
+        ctl->sel_count = kept;
+    }
+    G.sync();
+}
+
 // ------------------------------------------------------------------------------------------ top-down driver
 // Seeds of the predecessor pre-pass: every candidate list[0..cnt) (nullptr: all centrals), for every
 // keyword it does not contain itself (those have m = 0 and no predecessors).
@@ -1963,7 +2069,8 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
         }
         extract_list(c, sh, dsmem, nullptr, nc, qo);
         if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }   // emit counters (read after the select)
-        select_topk(c, sh, dsmem, kk);
+        if (a.containment) containment_select(c, sh, dsmem, kk);
+        else select_topk(c, sh, dsmem, kk);
     } else {
         const uint32_t m = mcap;
         for (int64_t i = G.gtid; i < nc; i += G.gsz) {   // lower bounds; cflag 2 = not extracted

@@ -188,7 +188,8 @@ struct EngineArgs {
     int qconst;                 // > 0: every query has this many keywords (qlen unused)
     uint32_t *next_query;       // global query counter
     // parameters (shared by the batch)
-    int k, max_depth, block_central, extract_mode, level_cover;
+    int k, max_depth, block_central, extract_mode, level_cover;   // level_cover: 0 off, 1 R13, 2 R13b
+    int containment;            // NEXT-3 R16: drop Central Graphs that strictly contain another one
     int tile_light;             // light frontiers up to this many nodes are expanded by group-wide tiles
     int td_only;                // 1: skip the search, the state comes from the vertex-partitioned search (vpart.cu)
     int td_levels, td_stop;     //    its stop level / reason
