@@ -183,7 +183,7 @@ def test_tier4_extraction():
     n0 = 1_100_000
     a, c = n0, n0 + 1
     edges = [(v, c) for v in range(n0)] + [(a, c)]
-    wts = (np.arange(n0 + 2) % 7 / 8.0).astype(np.float32)
+    wts = (np.arange(n0 + 2) % 7 * 0.003).astype(np.float32)   # < alpha / 4: every activation level is 0
     g = synth.from_edges(n0 + 2, edges, wts, [list(range(n0)), [a]], 2.0)
     o = oracle.query(g, [0, 1], 1)
     assert len(o.answers) == 1 and len(o.answers[0].nodes) == n0 + 2

@@ -33,7 +33,7 @@ def test_random_graphs_offgrid_weights():
     _gpu()
     rng = np.random.default_rng(77)
     for case in range(80):
-        n = int(rng.integers(4, 60))
+        n = int(rng.integers(6, 60))
         q = int(rng.integers(1, 6))
         g = R.random_graph(rng, n, float(rng.uniform(0.05, 0.3)), bool(rng.random() < 0.4), q, kw_size=(1, 5))
         g.weight = (rng.random(n) * rng.choice([1.0, 0.2, 1e-5])).astype(np.float32)

@@ -1,6 +1,6 @@
 """Driver for an ncu capture of ONE batch launch of the engine (the bench's launch shape): load a
 config's graph, run a warm batch (launch 1), then the captured batch (launch 2, `-s 1 -c 1`).
-Usage: profile_batch.py [config] [batch] [groups]"""
+Usage: profile_batch.py [config] [batch] [groups] [param=value ...]   (kgs_params fields, e.g. search_only=1)"""
 import os
 import sys
 
@@ -14,6 +14,8 @@ import synth  # noqa: E402
 name = sys.argv[1] if len(sys.argv) > 1 else "C3"
 batch = int(sys.argv[2]) if len(sys.argv) > 2 else 128
 groups = int(sys.argv[3]) if len(sys.argv) > 3 else 8
+over = dict(a.split("=") for a in sys.argv[4:])
+params = kgs.make_params(**{k: int(v) for k, v in over.items()})
 w = synth.make_workload(name)
 order = np.random.default_rng(12345).permutation(len(w.queries))
 qs = [w.queries[i] for i in order]
@@ -26,9 +28,11 @@ for rep in range(2):
         kwp[i, :len(q)] = torch.tensor(q, dtype=torch.int32)
     kwd = kwp.cuda()
     qld = torch.tensor([len(q) for q in sub], dtype=torch.int32, device="cuda")
-    kgs.kgs_query_batch_device(G, batch, kwd.data_ptr(), qld.data_ptr(), w.k, None, groups, s.cuda_stream)
+    kgs.kgs_query_batch_device(G, batch, kwd.data_ptr(), qld.data_ptr(), w.k, params, groups, s.cuda_stream)
     res = kgs.kgs_query_batch_fetch(G, [len(q) for q in sub], s.cuda_stream)
     st = [r.stats for r in res]
     print(f"launch {rep}: {batch} queries, G={groups}, ms_launch {st[0]['ms_launch']:.2f}, "
           f"arcs {sum(x['arcs_scanned'] for x in st)}, td_arcs {sum(x['td_arcs'] for x in st)}, "
-          f"centrals {sum(x['n_centrals'] for x in st)}", flush=True)
+          f"centrals {sum(x['n_centrals'] for x in st)}, dag_arcs {sum(x['dag_arcs'] for x in st)}, "
+          f"hits {sum(x['hits'] for x in st)}, frontier {sum(x['frontier_total'] for x in st)}, "
+          f"pred_arcs {sum(x['td_pred_arcs'] for x in st)}", flush=True)
