@@ -163,7 +163,7 @@ struct kgs_result {
 namespace {
 
 void free_work(DevWork &w) {
-    void *p[] = {w.st, w.nm, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
+    void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
                  w.gstate, w.huge};
@@ -177,7 +177,6 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     const int64_t n = g->n;
     w = DevWork{};
     CUDA_TRY(dmalloc(&w.st, n));
-    CUDA_TRY(dmalloc(&w.nm, (n + 3) / 4));
     CUDA_TRY(dmalloc(&w.M, n * 8));
     CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max({g->R_alloc, g->R, 2}) * (size_t)g->W));
     CUDA_TRY(dmalloc(&w.qlight, n));
@@ -530,7 +529,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        const size_t per = (size_t)g->n * 104 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
+        const size_t per = (size_t)g->n * 105 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
                            (size_t)pcap_of(g) * 20 +
                            g->huge_arena_bytes;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
@@ -953,7 +952,7 @@ kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centra
     if (st != KGS_OK) return st;
     const DevWork &w = g->works[0];
     // the replicated final state in the engine's layout (DevWork::st, M, centrals)
-    CUDA_TRY(launch_vp_pack_st(g->vp.hm, g->vp_gate, g->n, w.st, s));
+    CUDA_TRY(launch_vp_pack_st(g->vp.hm, g->vp_gate, g->act, g->n, w.st, s));
     CUDA_TRY(cudaMemcpyAsync(w.M, g->vp.M, (size_t)g->n * 8, cudaMemcpyDeviceToDevice, s));
     if (n_central) {
         CUDA_TRY(cudaMemcpyAsync(w.centrals, centrals_dev, sizeof(int32_t) * n_central, cudaMemcpyDeviceToDevice, s));

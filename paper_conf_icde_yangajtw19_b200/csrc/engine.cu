@@ -20,9 +20,11 @@
 // (the batch of BASELINE.json configs[3]).
 //
 // Data layout:
-//   st[v]   uint16: low byte = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of the level),
-//           high byte = gate (0 if v contains a query keyword, else a_v).  One 2-byte load per inspected arc.
-//   nm[v]   uint8 (packed in 32-bit words for atomicOr): bits newly hit during the current level.
+//   st[v]   uint32 status word: byte 0 = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of
+//           the level), byte 1 = gate (0 if v contains a query keyword, else a_v), byte 2 = nm, the bits
+//           newly hit during the current level (atomicOr), byte 3 = a_v.  One 4-byte load per inspected arc
+//           gives the target's mask and gate, and the hit that follows is an atomic on the same word
+//           (an L2 hit); a frontier node's merge and activation test read one word, not three arrays.
 //   M[v*8+i] uint8 hitting level, written once per (v, i) by the thread that set the bit; never reset.
 //   fbits   one frontier bitmap per level slot (R = amax+2 slots): "FIdentifier[v] <- 1 for level L" is one
 //           bit set on a bitmap word, so pushes never contend on a queue counter.  A node is re-queued
@@ -128,6 +130,13 @@ __device__ __forceinline__ int block_excl_scan(int x, int *total, long long *sh)
 __device__ __forceinline__ uint64_t ldrow(const uint8_t *M, int32_t v) {
     return __ldcg(reinterpret_cast<const unsigned long long *>(M) + v);
 }
+
+// fields of the status word st[v] (hm | gate << 8 | nm << 16 | a << 24)
+__device__ __forceinline__ uint32_t st_gate(uint32_t s) { return (s >> 8) & 0xFFu; }
+__device__ __forceinline__ uint32_t st_nm(uint32_t s) { return (s >> 16) & 0xFFu; }
+__device__ __forceinline__ uint32_t st_act(uint32_t s) { return s >> 24; }
+// the status word of a node nobody has hit yet: gate = a (not a keyword node), a
+__device__ __forceinline__ uint32_t st_fresh(uint32_t a) { return (a << 8) | (a << 24); }
 
 struct Q {   // the query a group is answering
     int32_t qi;
@@ -330,7 +339,7 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                                           uint32_t sx, unsigned &hits, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
-    const uint32_t gate = sx >> 8;
+    const uint32_t gate = st_gate(sx);
     if (gate <= (uint32_t)(l + 1)) {                     // ln 16-18: keyword node or a_x <= l+1
         ++dag;                                            // a Thm. V.4 arc (v -> x for these keywords)
         if (c.a.dag_record) {   // recorded predecessor arc
@@ -352,9 +361,7 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                 atomicMin(c.w.mw + (int64_t)x * 8 + i, __ldcg(c.w.mw + (int64_t)v * 8 + i));
             }
         }
-        const uint32_t sh = (uint32_t)(x & 3) << 3;
-        uint32_t *nw = c.w.nm + (x >> 2);
-        const uint32_t old = (atomicOr(nw, bits << sh) >> sh) & 0xFFu;
+        const uint32_t old = st_nm(atomicOr(c.w.st + x, bits << 16));
         const uint32_t nb = bits & ~old;
         if (nb) {
             hits += __popc(nb);
@@ -372,9 +379,10 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
 
 // Alg. 2 ln 2-7 for node v at level l: returns its expansion mask (0 = does not expand now).
 __device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool leader) {
-    const uint32_t hm = __ldcg(c.w.st + v) & 0xFFu;
+    const uint32_t sv = __ldcg(c.w.st + v);
+    const uint32_t hm = sv & 0xFFu;
     if (c.a.block_central && hm == c.qq.full) return 0;   // ln 2-3: central nodes do not expand
-    const int av = c.a.act[v];
+    const int av = (int)st_act(sv);
     if (av > l) {                                          // ln 5-7: not yet active
         if (leader) push(c, v, av);
         return 0;
@@ -419,7 +427,7 @@ struct BigTile {
 // index and status gathers issued before any of them is processed.
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint32_t cb, const int64_t *ptr,
-                                           const int32_t *idx, const uint16_t *st, BigTile &S, long long *sh,
+                                           const int32_t *idx, const uint32_t *st, BigTile &S, long long *sh,
                                            Prep prep, Visit visit, unsigned long long &arcs) {
     NodeT *node = reinterpret_cast<NodeT *>(S.node);
     for (uint32_t t0 = 0; t0 < cb; t0 += blockDim.x) {
@@ -459,7 +467,7 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
             }
             uint32_t sx[kBigUnroll];
 #pragma unroll
-            for (int k = 0; k < kBigUnroll; ++k) sx[k] = own[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+            for (int k = 0; k < kBigUnroll; ++k) sx[k] = own[k] >= 0 ? __ldcg(st + x[k]) : 0u;
 #pragma unroll
             for (int k = 0; k < kBigUnroll; ++k)
                 if (own[k] >= 0) visit(node[own[k]], x[k], sx[k]);
@@ -476,7 +484,7 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 // degrees and cost about the same.  ql = nullptr sweeps the nodes 0..c0-1 in contiguous batches (pull).
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
-                                             const int32_t *idx, const uint16_t *st, Prep prep, Visit visit,
+                                             const int32_t *idx, const uint32_t *st, Prep prep, Visit visit,
                                              unsigned long long &arcs) {
     const uint32_t warps = (uint32_t)(G.gsz >> 5);
     uint32_t B = (c0 + 2 * warps - 1) / (2 * warps);
@@ -523,7 +531,7 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
             }
             uint32_t sx[kLightUnroll];
 #pragma unroll
-            for (int k = 0; k < kLightUnroll; ++k) sx[k] = x[k] >= 0 ? (uint32_t)__ldcg(st + x[k]) : 0u;
+            for (int k = 0; k < kLightUnroll; ++k) sx[k] = x[k] >= 0 ? __ldcg(st + x[k]) : 0u;
 #pragma unroll
             for (int k = 0; k < kLightUnroll; ++k)
                 if (x[k] >= 0) visit(no[k], x[k], sx[k]);
@@ -540,7 +548,7 @@ __device__ __forceinline__ uint32_t pred_test(const Ctx &c, bool exact_block, ui
     const uint32_t hmu = su & 0xFFu;
     const uint32_t cand = P & hmu;
     if (!cand) return 0;
-    const int au = c.a.act[u];
+    const int au = (int)st_act(su);
     const uint64_t Mu = ldrow(c.w.M, u);
     uint32_t pb = 0, zb = 0;
     int maxrow = 0;
@@ -593,7 +601,7 @@ __device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const P
 __device__ __forceinline__ bool pd_prepare(const Ctx &c, int32_t x, PdNode &nd) {
     nd.P = __ldcg(c.w.pd_state + x) & 0xFFu;
     nd.hx = ldrow(c.w.M, x);
-    nd.gx = (int)(__ldcg(c.w.st + x) >> 8) - 1;
+    nd.gx = (int)st_gate(__ldcg(c.w.st + x)) - 1;
     nd.cidx = __ldcg(c.w.pd_cid + x);
     return nd.P != 0;
 }
@@ -787,7 +795,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
         const uint32_t sx = __ldcg(w.st + x);
         nd.x = x;
         nd.sx = sx;
-        return (full & ~sx & 0xFFu) != 0u && (sx >> 8) <= (uint32_t)(l + 1);
+        return (full & ~sx & 0xFFu) != 0u && st_gate(sx) <= (uint32_t)(l + 1);
     };
     auto plight = [&](int32_t x, bool leader, PullNode &nd) {
         if (!pprep(x, leader, nd)) return false;
@@ -801,7 +809,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
         const uint32_t hmu = su & 0xFFu;
         if (!(hmu & ~nd.sx & 0xFFu)) return;                 // u has none of the keywords x lacks
         if (a.block_central && hmu == full) return;           // ln 2-3
-        if ((int)__ldg(a.act + u) > l) return;               // ln 4-7
+        if ((int)st_act(su) > l) return;                     // ln 4-7
         uint32_t zb = 0;
         if (a.dag_record) {
             const uint64_t row = ldrow(w.M, u);
@@ -834,9 +842,10 @@ __device__ __forceinline__ void pull_waiting(const Ctx &c, int l, BigTile &S, lo
     volatile uint32_t *flag = &ctl->pull_wait[l & 1];
     unsigned long long arcs = 0;
     auto wprep = [&](int32_t v, bool, PullNode &nd) {
-        const uint32_t hm = __ldcg(w.st + v) & 0xFFu;
+        const uint32_t sv = __ldcg(w.st + v);
+        const uint32_t hm = sv & 0xFFu;
         if (!hm || (a.block_central && hm == full) || *flag) return false;
-        if ((int)__ldg(a.act + v) > l) { *flag = 1u; return false; }
+        if ((int)st_act(sv) > l) { *flag = 1u; return false; }
         nd.x = v;
         nd.sx = hm;
         return true;
@@ -847,13 +856,28 @@ __device__ __forceinline__ void pull_waiting(const Ctx &c, int l, BigTile &S, lo
         return true;
     };
     auto wvisit = [&](const PullNode &nd, int32_t x, uint32_t sx) {
-        if ((nd.sx & ~sx & 0xFFu) && (sx >> 8) > (uint32_t)(l + 1) && !*flag) *flag = 1u;
+        if ((nd.sx & ~sx & 0xFFu) && st_gate(sx) > (uint32_t)(l + 1) && !*flag) *flag = 1u;
     };
     expand_light<PullNode>(G, nullptr, (uint32_t)a.g.n, a.g.row_ptr, a.g.col_idx, w.st, wlight, wvisit, arcs);
     G.sync();
     expand_big<PullNode>(G, w.qbig, __ldcg(&ctl->pull_wbig[l & 1]), a.g.row_ptr, a.g.col_idx, w.st, S, sh,
                          wprep, wvisit, arcs);
     G.sync();
+}
+
+// Every node's status word to "not hit yet" (hm = nm = 0, gate = a, a), 4 nodes per 16-byte store.
+__device__ void reset_status_dense(const Ctx &c) {
+    const int64_t n = c.a.g.n, n4 = n / 4;
+    for (int64_t j = c.G.gtid; j < n4; j += c.G.gsz) {
+        const uint32_t a4 = *reinterpret_cast<const uint32_t *>(c.a.act + j * 4);
+        uint4 o;
+        o.x = st_fresh(a4 & 0xFFu);
+        o.y = st_fresh((a4 >> 8) & 0xFFu);
+        o.z = st_fresh((a4 >> 16) & 0xFFu);
+        o.w = st_fresh(a4 >> 24);
+        reinterpret_cast<uint4 *>(c.w.st)[j] = o;
+    }
+    for (int64_t v = n4 * 4 + c.G.gtid; v < n; v += c.G.gsz) c.w.st[v] = st_fresh(c.a.act[v]);
 }
 
 __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
@@ -864,8 +888,6 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const int64_t n = a.g.n, W = a.W;
     const int R = a.R, amax = R - 2;
     const uint32_t full = c.qq.full;
-    uint8_t *st8 = reinterpret_cast<uint8_t *>(w.st);
-    uint8_t *nm8 = reinterpret_cast<uint8_t *>(w.nm);
     const int64_t gtid = G.gtid, gsz = G.gsz;
 
     // ---- reset the state the previous query of this group left behind
@@ -873,18 +895,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const uint32_t done = __ldcg(w.gstate + 1);
     reset_mw_prev(c);
     if (!valid || (int)lastR != R || done == 0) {
-        const int64_t n8 = n / 8;
-        for (int64_t j = gtid; j < n8; j += gsz) {
-            const uint2 av = *reinterpret_cast<const uint2 *>(a.act + j * 8);
-            uint4 o;
-            o.x = ((av.x & 0xFFu) << 8) | ((av.x & 0xFF00u) << 16);
-            o.y = ((av.x >> 8) & 0xFF00u) | ((av.x >> 24) << 24);
-            o.z = ((av.y & 0xFFu) << 8) | ((av.y & 0xFF00u) << 16);
-            o.w = ((av.y >> 8) & 0xFF00u) | ((av.y >> 24) << 24);
-            *reinterpret_cast<uint4 *>(w.st + j * 8) = o;
-        }
-        for (int64_t v = n8 * 8 + gtid; v < n; v += gsz) w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
-        for (int64_t v = gtid; v < (n + 3) / 4; v += gsz) w.nm[v] = 0u;
+        reset_status_dense(c);
         for (int64_t j = gtid; j < (int64_t)R * W; j += gsz) w.fbits[j] = 0u;
         for (int64_t j = gtid; j < 2 * W; j += gsz) w.pd_bits[j] = 0u;
         for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
@@ -901,21 +912,11 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (prev_rec && pt > n / 16)
             for (int64_t j = gtid; j < pt; j += gsz) { w.pd_cid[w.touched[j]] = -1; w.pcnt[j] = 0; }
         if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
-            const int64_t n8 = n / 8;
-            for (int64_t j = gtid; j < n8; j += gsz) {
-                const uint2 av = *reinterpret_cast<const uint2 *>(a.act + j * 8);
-                uint4 o;
-                o.x = ((av.x & 0xFFu) << 8) | ((av.x & 0xFF00u) << 16);
-                o.y = ((av.x >> 8) & 0xFF00u) | ((av.x >> 24) << 24);
-                o.z = ((av.y & 0xFFu) << 8) | ((av.y & 0xFF00u) << 16);
-                o.w = ((av.y >> 8) & 0xFF00u) | ((av.y >> 24) << 24);
-                *reinterpret_cast<uint4 *>(w.st + j * 8) = o;
-            }
-            for (int64_t v = n8 * 8 + gtid; v < n; v += gsz) w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+            reset_status_dense(c);
         } else {
             for (int64_t j = gtid; j < pt; j += gsz) {
                 const int32_t v = w.touched[j];
-                w.st[v] = (uint16_t)((uint16_t)a.act[v] << 8);
+                w.st[v] = st_fresh(a.act[v]);
                 if (prev_rec) { w.pd_cid[v] = -1; w.pcnt[j] = 0; }
             }
         }
@@ -946,8 +947,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             const int32_t v = a.g.kw_nodes[kb[i] + (j - ko[i])];
             w.M[(int64_t)v * 8 + i] = 0;
             if (a.prune == 2) w.mw[(int64_t)v * 8 + i] = 0u;              // the path {v}: w_v added at merge
-            st8[2 * (int64_t)v + 1] = 0;                                  // keyword node: no gate (L210)
-            atomicOr(w.nm + (v >> 2), (1u << i) << ((v & 3) * 8));        // hit in B_i at level 0
+            // keyword node: no gate (L210); hit in B_i at level 0 (new-hit bit i)
+            atomicAnd(w.st + v, ~0xFF00u);
+            atomicOr(w.st + v, (1u << i) << 16);
             push(c, v, 0);
         }
     }
@@ -993,15 +995,15 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         auto merge_node = [&](int32_t v) {
                     // auto direction: out-arcs of the frontier nodes that can expand (a_v <= l, ln 4-7),
                     // bounded by the power of two of the class byte (no row_ptr load)
-                    if (count_lvl && !pulling && (int)a.act[v] <= l)
+                    const uint32_t sv = __ldcg(w.st + v);
+                    if (count_lvl && !pulling && (int)st_act(sv) <= l)
                         my_mf += cls_deg_bound(a.g.cls[v]);
-                    const uint32_t b = nm8[v];
+                    const uint32_t b = st_nm(sv);
                     if (!b) return false;
                     if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
-                    nm8[v] = 0;
-                    const uint32_t old = st8[2 * (int64_t)v];
+                    const uint32_t old = sv & 0xFFu;
                     const uint32_t nw = old | b;
-                    st8[2 * (int64_t)v] = (uint8_t)nw;
+                    w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
                     if (a.prune == 2) {   // lightest path to v for keyword i = min over predecessors + w_v
                         const uint32_t wv = weight_fx(__ldg(a.g.weight + v));
                         for (uint32_t bb = b; bb; bb &= bb - 1) {

@@ -126,8 +126,7 @@ struct DevGraph {
 
 // Per-group query workspace (all sized for n at load time).  One group answers one query at a time.
 struct DevWork {
-    uint16_t *st;       // [n] low byte: hit mask hm (bit i <=> M[v][i] finite); high byte: gate (0 for K, else a)
-    uint32_t *nm;       // [ceil(n/4)] new hits of the current level, one byte per node
+    uint32_t *st;       // [n] status word: hm | gate << 8 | nm << 16 | a << 24 (engine.cu "Data layout")
     uint8_t *M;         // [n*8] hitting levels, node-major, valid where the hm bit is set
     uint32_t *fbits;    // [R][W] frontier bitmaps, slot = level % R (FIdentifier)
     int32_t *qlight;    // [n] compacted frontier of the current level (big nodes replaced by -1)
@@ -249,7 +248,7 @@ cudaError_t launch_activation(const float *w, int64_t n, double A, double alpha,
 cudaError_t launch_degree_class(const int64_t *row_ptr, int64_t n, uint8_t *cls, cudaStream_t s);
 cudaError_t launch_snap_weights(float *w, int64_t n, cudaStream_t s);
 cudaError_t launch_validate(const DevGraph &g, int32_t *err, cudaStream_t s);
-cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
+cudaError_t launch_levels_out(const uint32_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
                               uint8_t *out, cudaStream_t s);
 cudaError_t launch_gather_u8(const uint8_t *src, const int32_t *perm, int64_t n, uint8_t *out, cudaStream_t s);
 cudaError_t launch_to_input_ids(const int32_t *ids, const int32_t *orig, int64_t cnt, int32_t *out, cudaStream_t s);
@@ -267,6 +266,7 @@ cudaError_t launch_vp_level(const DevGraph &g, const VpQuery &qd, const uint8_t 
                             cudaStream_t s);
 cudaError_t launch_vp_waiting(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
                               const uint8_t *gate, int l, int block_central, cudaStream_t s);
-cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, int64_t n, uint16_t *st, cudaStream_t s);
+cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, const uint8_t *act, int64_t n, uint32_t *st,
+                              cudaStream_t s);
 
 }  // namespace kgs

@@ -146,7 +146,7 @@ cudaError_t relabel_by_degree(int64_t n, int64_t m, int64_t P, int64_t **row_ptr
 }
 
 // ---- the parity view in input ids
-__global__ void k_levels_out_perm(const uint16_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
+__global__ void k_levels_out_perm(const uint32_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
                                   uint8_t *out) {
     const int64_t gt = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, gs = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v = gt; v < n; v += gs) {
@@ -164,7 +164,7 @@ __global__ void k_gather_i32(const int32_t *ids, const int32_t *orig, int64_t cn
         out[j] = orig ? orig[ids[j]] : ids[j];
 }
 
-cudaError_t launch_levels_out(const uint16_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
+cudaError_t launch_levels_out(const uint32_t *st, const uint8_t *M, const int32_t *perm, int64_t n, int q,
                               uint8_t *out, cudaStream_t s) {
     k_levels_out_perm<<<device_sm_count() * 8, 256, 0, s>>>(st, M, perm, n, q, out);
     return cudaGetLastError();

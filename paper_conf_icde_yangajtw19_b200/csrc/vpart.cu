@@ -192,11 +192,11 @@ __global__ void k_vp_biglist(const int64_t *__restrict__ in_ptr, int64_t lo, int
         if (in_ptr[x + 1] - in_ptr[x] > kVpBig) big[atomicAdd(nbig, 1)] = (int32_t)x;
 }
 
-// engine status word of the replicated final state: low byte hm, high byte gate (DevWork::st)
-__global__ void k_vp_pack_st(const uint8_t *__restrict__ hm, const uint8_t *__restrict__ gate, int64_t n,
-                             uint16_t *__restrict__ st) {
+// engine status word of the replicated final state: hm | gate << 8 | (nm = 0) | a << 24 (DevWork::st)
+__global__ void k_vp_pack_st(const uint8_t *__restrict__ hm, const uint8_t *__restrict__ gate,
+                             const uint8_t *__restrict__ act, int64_t n, uint32_t *__restrict__ st) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        st[v] = (uint16_t)(hm[v] | ((uint16_t)gate[v] << 8));
+        st[v] = (uint32_t)hm[v] | ((uint32_t)gate[v] << 8) | ((uint32_t)act[v] << 24);
 }
 
 static int vp_grid(int64_t items, int per_block) {
@@ -250,8 +250,9 @@ cudaError_t launch_vp_waiting(const DevGraph &g, const VpQuery &qd, const uint8_
     return cudaGetLastError();
 }
 
-cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, int64_t n, uint16_t *st, cudaStream_t s) {
-    if (n > 0) k_vp_pack_st<<<vp_grid(n, kVpBlock), kVpBlock, 0, s>>>(hm, gate, n, st);
+cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, const uint8_t *act, int64_t n, uint32_t *st,
+                              cudaStream_t s) {
+    if (n > 0) k_vp_pack_st<<<vp_grid(n, kVpBlock), kVpBlock, 0, s>>>(hm, gate, act, n, st);
     return cudaGetLastError();
 }
 

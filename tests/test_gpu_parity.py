@@ -268,3 +268,27 @@ def test_level_ring_resizing_across_alpha_and_groups():
                 assert r.stats["levels"] == o.levels and r.stats["stop_reason"] == o.stop_reason, ctx
                 assert [(a.central, a.score_key) for a in r.answers] == [(a.central, a.key) for a in o.answers], ctx
     G.close()
+
+
+def test_batch_modes_across_launches():
+    """The non-default top-down sources in query groups — the recorded DAG (dag_record = 1) and the
+    search-only analysis mode — over consecutive launches on the same workspaces: every launch's stop
+    level, |C| and (with answers) the answers must equal the oracle's."""
+    _gpu()
+    w = synth.make_workload("C2")
+    G = kgs.kgs_load_graph(w.graph)
+    qs = w.queries[::15][:20]
+    exp = [oracle.query(w.graph, kw, w.k) for kw in qs]
+    for params in (dict(dag_record=1), dict(search_only=1), dict(dag_record=0), dict(dag_record=1, prune=0)):
+        p = kgs.make_params(**params)
+        for launch in range(3):
+            res = kgs.kgs_query_batch(G, qs, w.k, p, 8)
+            for kw, r, o in zip(qs, res, exp):
+                ctx = (params, launch, kw)
+                assert r.stats["levels"] == o.levels and r.stats["stop_reason"] == o.stop_reason, ctx
+                assert r.stats["n_centrals"] == len(o.centrals), ctx
+                if not params.get("search_only"):
+                    assert [(a.central, a.score_key) for a in r.answers] == [(a.central, a.key) for a in o.answers], ctx
+                    for ra, oa in zip(r.answers, o.answers):
+                        assert ra.nodes.tolist() == oa.nodes.tolist() and ra.arcs.tolist() == oa.arcs.tolist(), ctx
+    G.close()
