@@ -1,6 +1,8 @@
 """profiles/<tag>_batch_ncu.md + <tag>_batch_traffic.json from one `ncu --set full` capture of a batch
 launch of the engine (tools/profile_batch.py: the bench's 350 C3 queries, G = 8, one launch).
-Usage: make_batch_profile.py tag details.csv raw.csv hot_lines.txt [queries]"""
+Usage: make_batch_profile.py tag details.csv raw.csv hot_lines.txt [queries] [git_sha] [workload]
+The traffic json records the git sha the capture was taken at and the sha256 of the engine sources
+(bench.source_hash) so that bench.py can tell whether its roofline.traffic describes the running build."""
 import csv
 import json
 import os
@@ -9,6 +11,10 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 tag, f_det, f_raw, f_hot = sys.argv[1:5]
 nq = int(sys.argv[5]) if len(sys.argv) > 5 else 350
+git_sha = sys.argv[6] if len(sys.argv) > 6 else None
+workload = sys.argv[7] if len(sys.argv) > 7 else "C3"
+sys.path.insert(0, ROOT)
+from bench import source_hash  # noqa: E402
 rows = list(csv.reader(open(f_det)))
 hdr = rows[0]
 want = {"GPU Speed Of Light Throughput": None, "Memory Workload Analysis": None, "Scheduler Statistics": None,
@@ -35,8 +41,8 @@ def num(name, scale=None):
 
 dur = num("Duration")
 bw = num("Memory Throughput") if vals.get("Memory Throughput", ("", ""))[1].endswith("/s") else None
-res = {"kernel": "k_engine", "launch": f"{nq} C3 queries, G = 8 (bench shape), one launch",
-       "duration_s_under_ncu": dur}
+res = {"kernel": "k_engine", "launch": f"{nq} {workload} queries, G = 8 (bench shape), one launch",
+       "workload": workload, "git_sha": git_sha, "src_sha256": source_hash(), "duration_s_under_ncu": dur}
 # DRAM bytes of the launch: dram__bytes_read.sum + dram__bytes_write.sum from the raw page
 raw = list(csv.reader(open(f_raw)))
 rh, ru = raw[0], raw[1]
