@@ -336,7 +336,7 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, uint32_t zbv, int32_t x,
-                                          uint32_t sx, unsigned &hits, unsigned &dag) {
+                                          uint32_t sx, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = st_gate(sx);
@@ -361,17 +361,17 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                 atomicMin(c.w.mw + (int64_t)x * 8 + i, __ldcg(c.w.mw + (int64_t)v * 8 + i));
             }
         }
-        const uint32_t old = st_nm(atomicOr(c.w.st + x, bits << 16));
-        const uint32_t nb = bits & ~old;
-        if (nb) {
-            hits += __popc(nb);
-            uint8_t *row = c.w.M + (int64_t)x * 8;
-            const uint8_t lv = (uint8_t)(l + 1);
+        // fire and forget (no returned value to wait for): every writer of this level sets the same bits and
+        // writes the same level l+1 into entries whose hit bit was clear at the level's start, and the
+        // frontier push is a bit set, so repeating them for arcs that lost a race changes nothing (Thm. V.2).
+        // The new (node, keyword) pairs are counted when the next merge folds nm into hm.
+        asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(c.w.st + x), "r"(bits << 16) : "memory");
+        uint8_t *row = c.w.M + (int64_t)x * 8;
+        const uint8_t lv = (uint8_t)(l + 1);
 #pragma unroll
-            for (int i = 0; i < kMaxQ; ++i)
-                if (nb & (1u << i)) row[i] = lv;          // ln 21: m_xi <- l+1
-            if (old == 0) push(c, x, l + 1);              // ln 22: FIdentifier[x] <- 1 (first new bit)
-        }
+        for (int i = 0; i < kMaxQ; ++i)
+            if (bits & (1u << i)) row[i] = lv;            // ln 21: m_xi <- l+1
+        push(c, x, l + 1);                                // ln 22: FIdentifier[x] <- 1
     } else {
         push(c, v, (int)gate - 1, true);                  // ln 19: v must retry when x opens
     }
@@ -783,7 +783,7 @@ __device__ void td_only_prepare(const Ctx &c, QOut *qo) {
 // One pulled level l (kgs_params.direction; called by search()): light candidates by a contiguous sweep of
 // all nodes, the ones with more than kBigDeg in-arcs afterwards in group-wide tiles.  (Inlined: out of line, the
 // call spilled the push path's level-loop state, p50 0.35 -> 0.43 ms; tools/ab_perf.py.)
-__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh, unsigned &my_hits,
+__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh,
                                          unsigned &my_dag, unsigned long long &my_arcs) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -818,7 +818,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
                 if (((row >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
             }
         }
-        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_hits, my_dag);
+        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_dag);
     };
     expand_light<PullNode>(G, nullptr, (uint32_t)n, a.g.in_ptr, a.g.in_idx, w.st, plight, pvisit, my_arcs);
     G.sync();
@@ -1001,6 +1001,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                     const uint32_t b = st_nm(sv);
                     if (!b) return false;
                     if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
+                    if (l > 0) my_hits += __popc(b);   // new (node, keyword) pairs of level l - 1's expansion
                     const uint32_t old = sv & 0xFFu;
                     const uint32_t nw = old | b;
                     w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
@@ -1071,9 +1072,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             // visit_arc as the push, so the hits, the recorded Thm. V.4 arcs and the lightest-path rows
             // are the same; no node is re-queued (ln 19): a pulling search has no work list (a level
             // without hits asks pull_waiting whether the list would still be non-empty).
-            const unsigned hits0 = my_hits;
-            pull_expand(c, l, S, sh, my_hits, my_dag, my_arcs);
-            cta_add((unsigned long long)(my_hits - hits0), &ctl->pull_marks[l & 1]);
+            const unsigned dag0 = my_dag;   // hitting arcs of this level: some (node, keyword) was marked
+            pull_expand(c, l, S, sh, my_dag, my_arcs);
+            cta_add((unsigned long long)(my_dag - dag0), &ctl->pull_marks[l & 1]);
             publish_flags(ctl);
             G.sync();
             stamp(G, qo, TS_EXPAND);
@@ -1105,7 +1106,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             return nd.hm != 0;
         };
         auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) {
-            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_hits, my_dag);
+            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_dag);
         };
         expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group

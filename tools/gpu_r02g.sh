@@ -5,8 +5,8 @@
 mkdir -p gpurun_out
 CS=/usr/local/cuda/bin/compute-sanitizer
 for tool in memcheck racecheck synccheck initcheck; do
-  n2=3; [ $tool = racecheck ] && n2=2
-  timeout 2400 $CS --tool $tool --kernel-name regex:k_engine --print-limit 50 python tools/sanitize_run.py 100 $n2 > gpurun_out/r02g_cs_$tool.log 2>&1
+  n2=3; [ $tool = racecheck ] && n2=1
+  timeout 2400 $CS --tool $tool --print-limit 50 python tools/sanitize_run.py 100 $n2 > gpurun_out/r02g_cs_$tool.log 2>&1
   echo "rc=$?" >> gpurun_out/r02g_cs_$tool.log
 done
-tail -4 gpurun_out/r02g_cs_*.log
+for f in gpurun_out/r02g_cs_*.log; do tail -n 4 $f; done
