@@ -163,7 +163,7 @@ struct kgs_result {
 namespace {
 
 void free_work(DevWork &w) {
-    void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
+    void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.qrec, w.qbrec, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
                  w.gstate, w.huge};
@@ -181,6 +181,8 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max({g->R_alloc, g->R, 2}) * (size_t)g->W));
     CUDA_TRY(dmalloc(&w.qlight, n));
     CUDA_TRY(dmalloc(&w.qbig, g->n_big));
+    CUDA_TRY(dmalloc(&w.qrec, n));
+    CUDA_TRY(dmalloc(&w.qbrec, std::max(g->n_big, g->n_big_in)));   // also the pre-pass's (in-arc classes)
     CUDA_TRY(dmalloc(&w.touched, n));
     CUDA_TRY(dmalloc(&w.qdef, n));
     CUDA_TRY(dmalloc(&w.centrals, n));
@@ -294,8 +296,10 @@ kgs_status kgs_load_graph(const kgs_graph_desc *d, kgs_graph **out) {
     if (on_dev) CUDA_TRY(cudaMemcpy(kp.data(), d->kw_ptr, sizeof(int64_t) * (V + 1), cudaMemcpyDeviceToHost));
     else std::memcpy(kp.data(), d->kw_ptr, sizeof(int64_t) * (V + 1));
     if (rp[0] != 0 || rp[n] != m) return fail(KGS_EINVAL, "row_ptr[0] must be 0 and row_ptr[n] == n_arcs");
-    for (int64_t v = 0; v < n; ++v)
+    for (int64_t v = 0; v < n; ++v) {
         if (rp[v + 1] < rp[v]) return fail(KGS_EINVAL, "row_ptr not non-decreasing");
+        if (rp[v + 1] - rp[v] >= (int64_t(1) << 31)) return fail(KGS_EINVAL, "a node has 2^31 or more arcs");
+    }
     if (kp[0] != 0) return fail(KGS_EINVAL, "kw_ptr[0] must be 0");
     for (int64_t t = 0; t < V; ++t)
         if (kp[t + 1] < kp[t]) return fail(KGS_EINVAL, "kw_ptr not non-decreasing");
@@ -529,7 +533,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        const size_t per = (size_t)g->n * 105 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
+        const size_t per = (size_t)g->n * 121 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
                            (size_t)pcap_of(g) * 20 +
                            g->huge_arena_bytes;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);

@@ -1,0 +1,57 @@
+"""Parity at the NEXT-4 sweep values (the paper's Exp-1/2/3): Knum 2..8, Topk 5..100 and alpha
+0.1..0.9 on the C2 graph (every point, several queries) and on the full-size C3 graph (one query per alpha
+and Topk point) — the GPU's answers against the oracle's, latency mode and query groups."""
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+kgs = pytest.importorskip("paper_conf_icde_yangajtw19_b200")
+SPEC = dict(band=(550, 1900), rare=None)
+
+
+def _gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+def _same(r, o, ctx):
+    assert r.stats["levels"] == o.levels and r.stats["stop_reason"] == o.stop_reason, ctx
+    assert [(a.central, a.score_key) for a in r.answers] == [(a.central, a.key) for a in o.answers], ctx
+    for ra, oa in zip(r.answers, o.answers):
+        assert ra.nodes.tolist() == oa.nodes.tolist() and ra.arcs.tolist() == oa.arcs.tolist(), ctx
+
+
+def test_c2_sweep_points():
+    _gpu()
+    w = synth.make_workload("C2")
+    g = w.graph
+    G = kgs.kgs_load_graph(g)
+    points = [(q, 20, 0.1) for q in range(2, 9)] + [(6, k, 0.1) for k in (5, 10, 50, 100)] + \
+             [(6, 20, a) for a in (0.3, 0.5, 0.7, 0.9)]
+    for q, k, alpha in points:
+        qs = synth.make_queries(g, 5000 + q, sizes={q: 4}, **SPEC)
+        p = kgs.make_params(alpha=alpha)
+        exp = [oracle.query(g, kw, k, alpha=alpha) for kw in qs]
+        for kw, o in zip(qs, exp):
+            _same(kgs.kgs_query(G, kw, k, p), o, (q, k, alpha, kw))
+        for kw, r, o in zip(qs, kgs.kgs_query_batch(G, qs, k, p, 4), exp):
+            _same(r, o, (q, k, alpha, kw, "batch"))
+    G.close()
+
+
+@pytest.mark.slow
+def test_c3_sweep_points():
+    _gpu()
+    w = synth.make_workload("C3", n_queries=1)
+    g = w.graph
+    G = kgs.kgs_load_graph(g)
+    q6 = synth.make_queries(g, 4006, sizes={6: 3}, band=(17000, 57000), rare=(300, 600), rare_frac=0.1)
+    for k, alpha in [(5, 0.1), (100, 0.1), (20, 0.3), (20, 0.5), (20, 0.7), (20, 0.9)]:
+        kw = q6[(k + int(alpha * 10)) % len(q6)]
+        _same(kgs.kgs_query(G, kw, k, kgs.make_params(alpha=alpha)), oracle.query(g, kw, k, alpha=alpha),
+              (k, alpha, kw))
+    G.close()
