@@ -6,7 +6,8 @@ NVFLAGS := -O3 -std=c++17 $(ARCH) -lineinfo -Xcompiler -fPIC \
 PKG := paper_conf_icde_yangajtw19_b200
 CSRC := $(PKG)/csrc
 LIB := $(PKG)/libkgs.so
-OBJS := $(CSRC)/api.o $(CSRC)/prep.o $(CSRC)/engine.o $(CSRC)/vpart.o $(CSRC)/relabel.o $(CSRC)/load.o
+OBJS := $(CSRC)/api.o $(CSRC)/prep.o $(CSRC)/engine.o $(CSRC)/vpart.o $(CSRC)/relabel.o $(CSRC)/load.o \
+        $(CSRC)/vpquery.o
 
 all: $(LIB) oracle/liboracle.so synth/libkgs_synth.so
 
@@ -14,7 +15,7 @@ $(CSRC)/%.o: $(CSRC)/%.cu $(CSRC)/kgs_internal.h include/kgs.h
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $@.ptxas.log || (cat $@.ptxas.log; exit 1)
 
 $(LIB): $(OBJS)
-	$(NVCC) $(ARCH) -shared -o $@ $(OBJS)
+	$(NVCC) $(ARCH) -shared -o $@ $(OBJS) -ldl
 
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fPIC -shared -ffp-contract=off -fno-fast-math -o $@ $< -lm

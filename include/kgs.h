@@ -269,10 +269,13 @@ typedef struct {
     uint8_t *hm;        /* [n_pad]     replicated hit masks (bit i = hit by keyword i); all_gather output */
     uint8_t *hm_slice;  /* [slice]     this rank's hit masks after the level; all_gather input */
     uint8_t *M;         /* [n_pad * 8] node-major hitting levels; this rank writes rows [lo, hi) */
-    int64_t *counts;    /* [3]         marks, new central nodes, waiting work-list nodes (all_reduce sum) */
+    int64_t *counts;    /* [4]         marks, new central nodes, waiting work-list nodes, changed owned nodes
+                                       (all_reduce sum) */
     int32_t *cent;      /* [slice]     this rank's central nodes (identification order) */
     uint8_t *cdep;      /* [slice]     their depths */
     int32_t *cent_n;    /* [1]         their count */
+    int64_t *chg;       /* [slice] or NULL: the level's changed owned nodes, id << 8 | new hit mask, for a
+                                       sparse exchange (kgs_vp_query uses it when few nodes change) */
 } kgs_vp_buffers;
 /* ceil(n / world) rounded up to a multiple of 16 (0 for bad arguments). */
 int64_t kgs_vp_slice(int64_t n_nodes, int32_t world);
@@ -290,6 +293,32 @@ kgs_status kgs_vp_waiting(kgs_graph *g, int32_t level, void *cuda_stream);
  * all-gathered central list (device, n_central entries), levels / stop_reason from the host loop. */
 kgs_status kgs_vp_topdown(kgs_graph *g, int64_t n_central, const int32_t *centrals_dev, const uint8_t *depth_dev,
                           int32_t levels, int32_t stop_reason, void *cuda_stream, kgs_result **out);
+
+/* ---- The whole vertex-partitioned query in the library ----
+ * kgs_vp_query runs the level loop above on every rank: the level calls, the exchanges (dense all_gather
+ * of the owned hit-mask slices, or a sparse all_gather of (id << 8 | mask) change lists when fewer than n/16
+ * nodes changed in the level), the counter all_reduces, the stop rules of kgs_query (Def. 4, Thm. V.3,
+ * R9, R22), the final gathers of M and of the central lists, and the top-down — and returns the same result
+ * as kgs_query on every rank.  The ranks' collectives go through a transport:
+ *   all_gather(ctx, send, recv, bytes, stream)   recv[r * bytes ..] = rank r's send (device buffers)
+ *   all_reduce_sum_i64(ctx, buf, count, stream)  in place, int64 sum over the ranks (device buffer)
+ * each returning 0 on success, enqueued on (or completed with respect to) the given CUDA stream.
+ * kgs_vp_nccl_transport gives the library's own NCCL communicator over NVLink / NVSwitch (rank 0 calls
+ * kgs_vp_nccl_unique_id and the caller broadcasts the 128 bytes); callers may supply their own (the
+ * CPU tests stage through gloo).  Every rank must call kgs_vp_query with the same query and parameters. */
+typedef struct {
+    void *ctx;
+    int32_t (*all_gather)(void *ctx, const void *send, void *recv, int64_t bytes, void *cuda_stream);
+    int32_t (*all_reduce_sum_i64)(void *ctx, int64_t *buf, int64_t count, void *cuda_stream);
+    int32_t owned;       /* 1: created by kgs_vp_nccl_transport, release with kgs_vp_transport_free */
+    int32_t host_staged; /* 1: the callbacks take HOST buffers (the library copies around them) */
+} kgs_vp_transport;
+kgs_status kgs_vp_nccl_unique_id(uint8_t *id /* [128] */);
+kgs_status kgs_vp_nccl_transport(const uint8_t *id /* [128] */, int32_t rank, int32_t world, int32_t device,
+                                 kgs_vp_transport *out);
+void kgs_vp_transport_free(kgs_vp_transport *t);
+kgs_status kgs_vp_query(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t k, const kgs_params *p, int32_t rank,
+                        int32_t world, const kgs_vp_transport *t, void *cuda_stream, kgs_result **out);
 
 /* ---- Load-time preprocessing: the steps that produce kgs_load_graph's inputs.
  * Both run on the raw CSR before kgs_load_graph, on `device`, on `cuda_stream` (NULL = default),

@@ -70,7 +70,19 @@ class kgs_stats(ctypes.Structure):
 class kgs_vp_buffers(ctypes.Structure):
     _fields_ = [("hm", ctypes.c_void_p), ("hm_slice", ctypes.c_void_p), ("M", ctypes.c_void_p),
                 ("counts", ctypes.c_void_p), ("cent", ctypes.c_void_p), ("cdep", ctypes.c_void_p),
-                ("cent_n", ctypes.c_void_p)]
+                ("cent_n", ctypes.c_void_p), ("chg", ctypes.c_void_p)]
+
+
+# collectives of the vertex partition's transport (kgs_vp_transport): all_gather(ctx, send, recv, bytes,
+# stream) and all_reduce_sum_i64(ctx, buf, count, stream), 0 = success
+VP_ALL_GATHER = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
+                                 ctypes.c_void_p)
+VP_ALL_REDUCE = ctypes.CFUNCTYPE(ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p)
+
+
+class kgs_vp_transport(ctypes.Structure):
+    _fields_ = [("ctx", ctypes.c_void_p), ("all_gather", VP_ALL_GATHER), ("all_reduce_sum_i64", VP_ALL_REDUCE),
+                ("owned", ctypes.c_int32), ("host_staged", ctypes.c_int32)]
 
 
 EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query", "kgs_query_device",
@@ -78,7 +90,8 @@ EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query
             "kgs_result_centrals", "kgs_result_activation", "kgs_result_stats", "kgs_result_phases",
             "kgs_result_free", "kgs_last_error", "kgs_version", "kgs_query_batch", "kgs_query_batch_device",
             "kgs_query_batch_fetch", "kgs_vp_slice", "kgs_vp_begin", "kgs_vp_level", "kgs_vp_waiting",
-            "kgs_vp_topdown", "kgs_prep_pair_distances", "kgs_prep_summary_weights"]
+            "kgs_vp_topdown", "kgs_prep_pair_distances", "kgs_prep_summary_weights", "kgs_vp_nccl_unique_id",
+            "kgs_vp_nccl_transport", "kgs_vp_transport_free", "kgs_vp_query"]
 
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
                "search_end", "extract", "extract_big", "select", "emit"]
@@ -143,6 +156,15 @@ def lib():
         L.kgs_vp_waiting.restype = i32
         L.kgs_vp_topdown.argtypes = [vp, i64, vp, vp, i32, i32, vp, ctypes.POINTER(vp)]
         L.kgs_vp_topdown.restype = i32
+        L.kgs_vp_nccl_unique_id.argtypes = [vp]
+        L.kgs_vp_nccl_unique_id.restype = i32
+        L.kgs_vp_nccl_transport.argtypes = [vp, i32, i32, i32, ctypes.POINTER(kgs_vp_transport)]
+        L.kgs_vp_nccl_transport.restype = i32
+        L.kgs_vp_transport_free.argtypes = [ctypes.POINTER(kgs_vp_transport)]
+        L.kgs_vp_transport_free.restype = None
+        L.kgs_vp_query.argtypes = [vp, vp, i32, i32, ctypes.POINTER(kgs_params), i32, i32,
+                                   ctypes.POINTER(kgs_vp_transport), vp, ctypes.POINTER(vp)]
+        L.kgs_vp_query.restype = i32
         L.kgs_prep_pair_distances.argtypes = [i64, i64, vp, vp, i32, vp, vp, i32, i32, i32, vp, vp, vp]
         L.kgs_prep_pair_distances.restype = i32
         L.kgs_prep_summary_weights.argtypes = [i64, i64, vp, vp, i32, i32, vp, vp, vp]
@@ -387,6 +409,36 @@ def kgs_vp_topdown(graph: Graph, n_central: int, cent_ptr: int, dep_ptr: int, le
     _check(lib().kgs_vp_topdown(graph.handle, int(n_central), ctypes.c_void_p(cent_ptr), ctypes.c_void_p(dep_ptr),
                                 int(levels), int(stop_reason), ctypes.c_void_p(stream), ctypes.byref(h)))
     return _read_result(h, graph.n, int(q), want_levels)
+
+
+def kgs_vp_nccl_unique_id() -> bytes:
+    """128-byte NCCL unique id (rank 0; broadcast it to the other ranks)."""
+    buf = (ctypes.c_uint8 * 128)()
+    _check(lib().kgs_vp_nccl_unique_id(buf))
+    return bytes(buf)
+
+
+def kgs_vp_nccl_transport(uid: bytes, rank: int, world: int, device: int) -> kgs_vp_transport:
+    """The library's own NCCL communicator for kgs_vp_query (free with kgs_vp_transport_free)."""
+    t = kgs_vp_transport()
+    buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+    _check(lib().kgs_vp_nccl_transport(buf, int(rank), int(world), int(device), ctypes.byref(t)))
+    return t
+
+
+def kgs_vp_transport_free(t: kgs_vp_transport) -> None:
+    lib().kgs_vp_transport_free(ctypes.byref(t))
+
+
+def kgs_vp_query(graph: Graph, kw_ids, k: int, params: kgs_params | None, rank: int, world: int,
+                 transport: kgs_vp_transport, stream: int = 0) -> Result:
+    """The whole vertex-partitioned query in the library (level loop, exchanges, stop rules, top-down)."""
+    kw = np.ascontiguousarray(np.asarray(kw_ids, dtype=np.int32))
+    p = params if params is not None else kgs_params_default()
+    h = ctypes.c_void_p()
+    _check(lib().kgs_vp_query(graph.handle, kw.ctypes.data, int(kw.shape[0]), int(k), ctypes.byref(p), int(rank),
+                              int(world), ctypes.byref(transport), ctypes.c_void_p(stream), ctypes.byref(h)))
+    return _read_result(h, graph.n, int(kw.shape[0]), p.want_levels)
 
 
 # ---- load-time preprocessing (SURVEY §8(f) NEXT-2): the inputs kgs_load_graph takes ----

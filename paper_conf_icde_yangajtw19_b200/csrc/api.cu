@@ -178,6 +178,9 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     w = DevWork{};
     CUDA_TRY(dmalloc(&w.st, n));
     CUDA_TRY(dmalloc(&w.M, n * 8));
+    // M is never reset between queries (a row entry is valid where hm has its bit), but every byte is
+    // written once here so that no read of a whole 8-byte row touches uninitialised memory
+    CUDA_TRY(cudaMemset(w.M, 0xFF, (size_t)n * 8));
     CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max({g->R_alloc, g->R, 2}) * (size_t)g->W));
     CUDA_TRY(dmalloc(&w.qlight, n));
     CUDA_TRY(dmalloc(&w.qbig, g->n_big));
@@ -225,6 +228,8 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
 
 namespace kgs {
 kgs_status set_error(kgs_status s, const std::string &msg) { return fail(s, msg); }
+int64_t graph_nodes(const kgs_graph *g) { return g->n; }
+int graph_device(const kgs_graph *g) { return g->device; }
 }  // namespace kgs
 
 extern "C" {
@@ -895,6 +900,7 @@ kgs_status kgs_vp_begin(kgs_graph *g, const int32_t *kw_ids, int32_t q, int32_t 
     VpBufs vb{};
     vb.hm = b->hm; vb.hm_slice = b->hm_slice; vb.M = b->M;
     vb.counts = reinterpret_cast<unsigned long long *>(b->counts);
+    vb.chg = reinterpret_cast<long long *>(b->chg);
     vb.cent = b->cent; vb.cdep = b->cdep; vb.cent_n = b->cent_n;
     vb.n_pad = n_pad; vb.lo = lo; vb.hi = hi;
     // an empty T_i: nothing can be central (reading R17)

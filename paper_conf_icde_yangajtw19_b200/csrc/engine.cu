@@ -185,8 +185,7 @@ __device__ __forceinline__ void set_bit(uint32_t *bits, int fi, int32_t v, bool 
     const uint32_t bit = 1u << (v & 31);
     if (check && (__ldcg(word) & bit)) return;
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
-    uint32_t *f = cta_flags() + fi;
-    if (!*f) *f = 1u;
+    atomicOr(cta_flags() + fi, 1u);   // the CTA's "slot non-empty" flag (shared; every writer sets the same bit)
 }
 
 // All threads of the CTA: publish the CTA's flags (then the caller's group barrier makes them visible).
@@ -1389,6 +1388,7 @@ __device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu, b
         if (k == u) {
             int v;
             while ((v = atomicAdd(S.hval + h, 0)) == -1) { }
+            __threadfence_block();   // acquire: the inserter's id / zb stores precede its publication of hval
             return v >= 0 ? v : -1;
         }
         h = (h + 1) & (uint32_t)(S.hcap - 1);

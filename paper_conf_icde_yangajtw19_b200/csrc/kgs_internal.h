@@ -234,7 +234,8 @@ struct VpBufs {                    // exchange buffers (caller-owned device memo
     uint8_t *hm;                   // [n_pad] replicated hit masks (all-gather output)
     uint8_t *hm_slice;             // [slice] this rank's hit masks after the level (all-gather input)
     uint8_t *M;                    // [n_pad * 8] node-major hitting levels; rows [lo, hi) are this rank's
-    unsigned long long *counts;    // [3] marks, new centrals, waiting work-list nodes (all-reduce sum)
+    unsigned long long *counts;    // [4] marks, new centrals, waiting work-list nodes, changed nodes (all-reduce sum)
+    long long *chg;                // [slice] or null: changed owned nodes of the level, id << 8 | new mask
     int32_t *cent;                 // [slice] this rank's central nodes
     uint8_t *cdep;                 // [slice] their depths
     int32_t *cent_n;               // [1] their count
@@ -268,6 +269,7 @@ cudaError_t launch_vp_level(const DevGraph &g, const VpQuery &qd, const uint8_t 
                             cudaStream_t s);
 cudaError_t launch_vp_waiting(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
                               const uint8_t *gate, int l, int block_central, cudaStream_t s);
+cudaError_t launch_vp_apply(const long long *list, int64_t cnt, uint8_t *hm, cudaStream_t s);
 cudaError_t launch_vp_pack_st(const uint8_t *hm, const uint8_t *gate, const uint8_t *act, int64_t n, uint32_t *st,
                               cudaStream_t s);
 

@@ -68,9 +68,13 @@ __global__ void k_vp_expmask(const uint8_t *__restrict__ hm, const uint8_t *__re
 
 __device__ __forceinline__ void vp_finish_node(int64_t x, int64_t lo, uint32_t h, uint32_t nb, int l, uint32_t full,
                                                uint8_t *hm_slice, uint8_t *M, int32_t *cent, uint8_t *cdep,
-                                               int32_t *cent_n, unsigned &marks, unsigned &newc) {
+                                               int32_t *cent_n, unsigned &marks, unsigned &newc,
+                                               unsigned long long *counts, long long *chg) {
     hm_slice[x - lo] = (uint8_t)(h | nb);
     if (!nb) return;
+    // a changed owned node: counted (counts[3]) and listed (id << 8 | new mask) for the sparse exchange
+    const unsigned long long p = atomicAdd(counts + 3, 1ull);
+    if (chg) chg[p] = ((long long)x << 8) | (long long)(h | nb);
     for (int i = 0; i < kMaxQ; ++i)
         if ((nb >> i) & 1u) M[x * 8 + i] = (uint8_t)(l + 1);   // m_xi <- l+1 (Alg. 2 ln 21)
     marks += __popc(nb);
@@ -99,7 +103,8 @@ __global__ void __launch_bounds__(kVpBlock) k_vp_pull(const int64_t *__restrict_
                                                       const uint8_t *__restrict__ gate, const uint8_t *__restrict__ act,
                                                       int block_central, int64_t lo, int64_t hi, int l,
                                                       uint32_t full, uint8_t *hm_slice, uint8_t *M, int32_t *cent,
-                                                      uint8_t *cdep, int32_t *cent_n, unsigned long long *counts) {
+                                                      uint8_t *cdep, int32_t *cent_n, unsigned long long *counts,
+                                                      long long *chg) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
     unsigned marks = 0, newc = 0, wait = 0;
@@ -117,7 +122,8 @@ __global__ void __launch_bounds__(kVpBlock) k_vp_pull(const int64_t *__restrict_
                 acc = __reduce_or_sync(0xffffffffu, acc);
                 if ((acc & need) == need) break;
             }
-        if (lane == 0) vp_finish_node(x, lo, h, acc & need, l, full, hm_slice, M, cent, cdep, cent_n, marks, newc);
+        if (lane == 0)
+            vp_finish_node(x, lo, h, acc & need, l, full, hm_slice, M, cent, cdep, cent_n, marks, newc, counts, chg);
     }
     vp_count(marks, newc, wait, counts);
 }
@@ -128,7 +134,7 @@ __global__ void __launch_bounds__(kVpBlock) k_vp_pull_big(const int64_t *__restr
                                                           const uint8_t *__restrict__ gate, const int32_t *__restrict__ big,
                                                           int nbig, int64_t lo, int l, uint32_t full, uint8_t *hm_slice,
                                                           uint8_t *M, int32_t *cent, uint8_t *cdep, int32_t *cent_n,
-                                                          unsigned long long *counts) {
+                                                          unsigned long long *counts, long long *chg) {
     __shared__ uint32_t s_acc;
     unsigned marks = 0, newc = 0;
     for (int b = blockIdx.x; b < nbig; b += gridDim.x) {
@@ -154,7 +160,7 @@ __global__ void __launch_bounds__(kVpBlock) k_vp_pull_big(const int64_t *__restr
             acc = all;
         }
         if (threadIdx.x == 0)
-            vp_finish_node(x, lo, h, s_acc & need, l, full, hm_slice, M, cent, cdep, cent_n, marks, newc);
+            vp_finish_node(x, lo, h, s_acc & need, l, full, hm_slice, M, cent, cdep, cent_n, marks, newc, counts, chg);
         __syncthreads();
     }
     vp_count(marks, newc, 0u, counts);
@@ -199,6 +205,14 @@ __global__ void k_vp_pack_st(const uint8_t *__restrict__ hm, const uint8_t *__re
         st[v] = (uint32_t)hm[v] | ((uint32_t)gate[v] << 8) | ((uint32_t)act[v] << 24);
 }
 
+// sparse exchange: the gathered (id << 8 | mask) lists of every rank into the replicated hit masks
+__global__ void k_vp_apply(const long long *__restrict__ list, int64_t cnt, uint8_t *__restrict__ hm) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < cnt; j += (int64_t)gridDim.x * blockDim.x) {
+        const long long e = list[j];
+        if (e >= 0) hm[e >> 8] = (uint8_t)(e & 0xFF);
+    }
+}
+
 static int vp_grid(int64_t items, int per_block) {
     int64_t g = (items + per_block - 1) / per_block;
     if (g > device_sm_count() * 16) g = device_sm_count() * 16;
@@ -209,7 +223,7 @@ cudaError_t launch_vp_begin(const DevGraph &g, const VpQuery &qd, const uint8_t 
                             cudaStream_t s) {
     cudaMemsetAsync(b.hm, 0, (size_t)b.n_pad, s);
     cudaMemcpyAsync(gate, act, (size_t)g.n, cudaMemcpyDeviceToDevice, s);
-    cudaMemsetAsync(b.counts, 0, 3 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(b.counts, 0, 4 * sizeof(unsigned long long), s);
     cudaMemsetAsync(b.cent_n, 0, sizeof(int32_t), s);
     k_vp_init<<<device_sm_count() * 4, kVpBlock, 0, s>>>(g.kw_ptr, g.kw_nodes, qd, b.hm, gate, b.M);
     k_vp_ident0<<<vp_grid(b.hi - b.lo, kVpBlock), kVpBlock, 0, s>>>(b.hm, b.lo, b.hi, qd.full, b.cent, b.cdep,
@@ -226,27 +240,32 @@ cudaError_t launch_vp_biglist(const DevGraph &g, int64_t lo, int64_t hi, int32_t
 cudaError_t launch_vp_level(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
                             const uint8_t *gate, uint8_t *X, const int32_t *big, int nbig, int l, int block_central,
                             cudaStream_t s) {
-    cudaMemsetAsync(b.counts, 0, 3 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(b.counts, 0, 4 * sizeof(unsigned long long), s);
     k_vp_expmask<<<vp_grid(b.n_pad / 16, kVpBlock), kVpBlock, 0, s>>>(b.hm, act, b.n_pad, g.n, l, qd.full,
                                                                         block_central, X);
     if (b.hi > b.lo)
         k_vp_pull<<<vp_grid(b.hi - b.lo, kVpBlock / 32), kVpBlock, 0, s>>>(
             g.in_ptr, g.in_idx, b.hm, X, gate, act, block_central, b.lo, b.hi, l, qd.full, b.hm_slice, b.M, b.cent,
-            b.cdep, b.cent_n, b.counts);
+            b.cdep, b.cent_n, b.counts, b.chg);
     if (nbig)
         k_vp_pull_big<<<nbig < device_sm_count() * 4 ? nbig : device_sm_count() * 4, kVpBlock, 0, s>>>(
             g.in_ptr, g.in_idx, b.hm, X, gate, big, nbig, b.lo, l, qd.full, b.hm_slice, b.M, b.cent, b.cdep, b.cent_n,
-            b.counts);
+            b.counts, b.chg);
     return cudaGetLastError();
 }
 
 cudaError_t launch_vp_waiting(const DevGraph &g, const VpQuery &qd, const uint8_t *act, const VpBufs &b,
                               const uint8_t *gate, int l, int block_central, cudaStream_t s) {
-    cudaMemsetAsync(b.counts, 0, 3 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(b.counts, 0, 4 * sizeof(unsigned long long), s);
     if (b.hi > b.lo)
         k_vp_waiting<<<vp_grid(b.hi - b.lo, kVpBlock / 32), kVpBlock, 0, s>>>(g.row_ptr, g.col_idx, b.hm, gate, act,
                                                                              block_central, b.lo, b.hi, l, qd.full,
                                                                              b.counts);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_vp_apply(const long long *list, int64_t cnt, uint8_t *hm, cudaStream_t s) {
+    if (cnt > 0) k_vp_apply<<<vp_grid(cnt, kVpBlock), kVpBlock, 0, s>>>(list, cnt, hm);
     return cudaGetLastError();
 }
 

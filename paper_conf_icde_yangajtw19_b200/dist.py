@@ -129,12 +129,10 @@ def run_sharded(graph, queries, k: int, rank: int, world: int, params=None, grou
 
 
 # --------------------------------------------------------------------------- vertex partition (one query)
-# SURVEY §8(e) "a single query": 1-D vertex partition, CSR replicated, one exchange per level.  The
-# level kernels are libkgs's (kgs_vp_*); this driver only moves their buffers between ranks and applies
-# the stop rules of Def. 4 / Thm. V.3 to the reduced counters.  NCCL collectives run on the device
-# buffers directly; with gloo (tests) they are staged through host memory.
-
-STOP_K, STOP_EXHAUSTED, STOP_MAX_DEPTH, STOP_EMPTY_KEYWORD = 0, 1, 2, 3
+# SURVEY §8(e) "a single query": 1-D vertex partition, CSR replicated, one exchange per level.  The level
+# loop, the exchanges (dense or sparse) and the stop rules run in the library (kgs_vp_query, vpquery.cu);
+# this module only provides the transport: the library's own NCCL communicator when the group is NCCL, or
+# host-staged callbacks over the group's collectives (gloo, the CPU / one-GPU tests).
 
 
 def _is_nccl(group=None) -> bool:
@@ -142,136 +140,78 @@ def _is_nccl(group=None) -> bool:
     return dist.get_backend(group) == "nccl"
 
 
-def all_gather_into(out: torch.Tensor, inp: torch.Tensor, group=None) -> None:
-    """out = concat over ranks of inp (equal sizes)."""
+class GroupTransport:
+    """kgs_vp_transport whose callbacks run torch.distributed collectives of `group` on HOST buffers (the
+    library copies its device buffers around them: host_staged = 1).  For gloo groups."""
+
+    def __init__(self, group=None):
+        import ctypes
+
+        import torch.distributed as dist
+
+        from . import VP_ALL_GATHER, VP_ALL_REDUCE, kgs_vp_transport
+        self.dist, self.ctypes, self.group = dist, ctypes, group
+        self.world = dist.get_world_size(group)
+        self._ag = VP_ALL_GATHER(self._all_gather)
+        self._ar = VP_ALL_REDUCE(self._all_reduce)
+        self.t = kgs_vp_transport(None, self._ag, self._ar, 0, 1)
+
+    def _all_gather(self, ctx, send, recv, nbytes, stream):
+        try:
+            c = self.ctypes
+            x = torch.frombuffer(bytearray(c.string_at(send, nbytes)), dtype=torch.uint8) if nbytes else \
+                torch.zeros(0, dtype=torch.uint8)
+            parts = [torch.empty(nbytes, dtype=torch.uint8) for _ in range(self.world)]
+            self.dist.all_gather(parts, x, group=self.group)
+            out = torch.cat(parts).contiguous()
+            if out.numel():
+                c.memmove(recv, out.data_ptr(), out.numel())
+            return 0
+        except Exception:   # noqa: BLE001 — reported to the library as a failed collective
+            return -1
+
+    def _all_reduce(self, ctx, buf, count, stream):
+        try:
+            c = self.ctypes
+            x = torch.frombuffer(bytearray(c.string_at(buf, 8 * count)), dtype=torch.int64)
+            self.dist.all_reduce(x, group=self.group)
+            c.memmove(buf, x.data_ptr(), 8 * count)
+            return 0
+        except Exception:   # noqa: BLE001
+            return -1
+
+
+_nccl_transports = {}
+
+
+def nccl_transport(group=None):
+    """The library's NCCL communicator for `group` (rank 0 makes the id, the group broadcasts it), cached."""
     import torch.distributed as dist
-    if _is_nccl(group):
-        dist.all_gather_into_tensor(out, inp, group=group)
-        return
-    world = dist.get_world_size(group)
-    parts = [torch.empty(inp.shape, dtype=inp.dtype) for _ in range(world)]
-    dist.all_gather(parts, inp.cpu(), group=group)
-    out.copy_(torch.cat(parts).to(out.device))
 
-
-def all_reduce_sum(t: torch.Tensor, group=None) -> None:
-    import torch.distributed as dist
-    if _is_nccl(group):
-        dist.all_reduce(t, group=group)
-        return
-    h = t.cpu()
-    dist.all_reduce(h, group=group)
-    t.copy_(h.to(t.device))
-
-
-def vp_alloc(n: int, slice_: int, world: int, device) -> dict:
-    """The exchange buffers of kgs_vp_buffers (torch owns the device memory)."""
-    n_pad = slice_ * world
-    return dict(hm=torch.zeros(n_pad, dtype=torch.uint8, device=device),
-                hm_slice=torch.zeros(slice_, dtype=torch.uint8, device=device),
-                M=torch.full((n_pad * 8,), 255, dtype=torch.uint8, device=device),
-                counts=torch.zeros(3, dtype=torch.int64, device=device),
-                cent=torch.zeros(max(slice_, 1), dtype=torch.int32, device=device),
-                cdep=torch.zeros(max(slice_, 1), dtype=torch.uint8, device=device),
-                cent_n=torch.zeros(1, dtype=torch.int32, device=device))
-
-
-def vp_search(ops, kw, k: int, max_depth: int, rank: int, world: int, group=None) -> dict:
-    """The level loop over `ops` (begin / level on this rank's rows; see LibVpOps).  Returns the stop
-    level and reason, |C| and the all-gathered state (hm, M, central list)."""
-    b = ops.bufs
-    slice_ = b["hm_slice"].shape[0]
-    amax, empty = ops.begin(kw, k, rank, world)
-    if empty:   # reading R17: some T_i is empty, nothing can be central
-        return dict(levels=0, stop=STOP_EMPTY_KEYWORD, n_central=0, cent=b["cent"][:0], cdep=b["cdep"][:0])
-    all_reduce_sum(b["counts"], group)
-    n_central = int(b["counts"][1].item())
-    level = 0
-    while True:
-        if n_central >= k:
-            stop = STOP_K
-            break
-        if level == max_depth:
-            stop = STOP_MAX_DEPTH
-            break
-        ops.level(level)
-        all_gather_into(b["hm"], b["hm_slice"], group)
-        all_reduce_sum(b["counts"], group)
-        marks, new_c, waiting = (int(x) for x in b["counts"].tolist())
-        n_central += new_c
-        if marks == 0 and waiting == 0 and level + 1 < amax:   # gated neighbours are possible
-            ops.waiting(level)
-            all_reduce_sum(b["counts"], group)
-            waiting = int(b["counts"][2].item())
-        if marks == 0 and waiting == 0:   # the work-list of Alg. 2 is empty at level + 1
-            level += 1
-            stop = STOP_EXHAUSTED
-            break
-        level += 1
-    # owned M rows and central lists to every rank
-    mine = b["M"][rank * slice_ * 8:(rank + 1) * slice_ * 8].clone()
-    all_gather_into(b["M"], mine, group)
-    cnt = b["cent_n"].to(torch.int64)
-    counts = torch.zeros(world, dtype=torch.int64, device=cnt.device)
-    all_gather_into(counts, cnt, group)
-    counts = counts.tolist()
-    width = max(max(counts), 1)
-    cpad = torch.full((width,), -1, dtype=torch.int32, device=b["cent"].device)
-    dpad = torch.zeros(width, dtype=torch.uint8, device=b["cent"].device)
-    cpad[:counts[rank]] = b["cent"][:counts[rank]]
-    dpad[:counts[rank]] = b["cdep"][:counts[rank]]
-    call = torch.empty(width * world, dtype=torch.int32, device=cpad.device)
-    dall = torch.empty(width * world, dtype=torch.uint8, device=cpad.device)
-    all_gather_into(call, cpad, group)
-    all_gather_into(dall, dpad, group)
-    keep = torch.cat([torch.arange(r * width, r * width + counts[r], device=cpad.device) for r in range(world)])
-    cent, cdep = call[keep].contiguous(), dall[keep].contiguous()
-    assert cent.shape[0] == n_central, (cent.shape[0], n_central)
-    return dict(levels=level, stop=stop, n_central=n_central, cent=cent, cdep=cdep)
-
-
-class LibVpOps:
-    """The level kernels of libkgs (kgs_vp_begin / kgs_vp_level / kgs_vp_topdown) over torch buffers."""
-
-    def __init__(self, graph, params=None, device=None):
-        import paper_conf_icde_yangajtw19_b200 as kgs
-        self.kgs = kgs
-        self.graph = graph
-        self.params = params if params is not None else kgs.kgs_params_default()
-        self.device = device if device is not None else torch.device("cuda", torch.cuda.current_device())
-        self.stream = torch.cuda.current_stream(self.device).cuda_stream
-        self.bufs = None
-        self.k = 0
-
-    def alloc(self, world: int):
-        slice_ = self.kgs.kgs_vp_slice(self.graph.n, world)
-        self.bufs = vp_alloc(self.graph.n, slice_, world, self.device)
-        b = self.bufs
-        self.cbufs = self.kgs.kgs_vp_buffers(b["hm"].data_ptr(), b["hm_slice"].data_ptr(), b["M"].data_ptr(),
-                                             b["counts"].data_ptr(), b["cent"].data_ptr(), b["cdep"].data_ptr(),
-                                             b["cent_n"].data_ptr())
-
-    def begin(self, kw, k, rank, world):
-        self.kw, self.k = list(kw), int(k)
-        return self.kgs.kgs_vp_begin(self.graph, kw, k, self.params, rank, world, self.cbufs, self.stream)
-
-    def level(self, level):
-        self.kgs.kgs_vp_level(self.graph, level, self.stream)
-
-    def waiting(self, level):
-        self.kgs.kgs_vp_waiting(self.graph, level, self.stream)
-
-    def topdown(self, s):
-        return self.kgs.kgs_vp_topdown(self.graph, s["n_central"], s["cent"].data_ptr(), s["cdep"].data_ptr(),
-                                       s["levels"], s["stop"], len(self.kw), self.params.want_levels, self.stream)
+    import paper_conf_icde_yangajtw19_b200 as kgs
+    key = id(group)
+    if key not in _nccl_transports:
+        rank, world = dist.get_rank(group), dist.get_world_size(group)
+        dev = torch.cuda.current_device()
+        uid = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev}")
+        if rank == 0:
+            uid.copy_(torch.frombuffer(bytearray(kgs.kgs_vp_nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(uid, 0, group=group)
+        _nccl_transports[key] = kgs.kgs_vp_nccl_transport(bytes(uid.cpu().numpy()), rank, world, dev)
+    return _nccl_transports[key]
 
 
 def vp_query(graph, kw, k: int, params=None, group=None):
-    """One query answered by all ranks of `group` with the vertex-partitioned search (every rank holds
-    the graph).  Every rank returns the same Result (= kgs_query's)."""
+    """One query answered by all ranks of `group` with the vertex-partitioned search (every rank holds the
+    graph): kgs_vp_query over the group's transport.  Every rank returns the same Result (= kgs_query's)."""
     import torch.distributed as dist
+
+    import paper_conf_icde_yangajtw19_b200 as kgs
     rank, world = dist.get_rank(group), dist.get_world_size(group)
-    ops = LibVpOps(graph, params)
-    ops.alloc(world)
-    s = vp_search(ops, kw, k, ops.params.max_depth, rank, world, group)
-    return ops.topdown(s)
+    p = params if params is not None else kgs.kgs_params_default()
+    stream = torch.cuda.current_stream().cuda_stream
+    if _is_nccl(group):
+        t = nccl_transport(group)
+        return kgs.kgs_vp_query(graph, kw, k, p, rank, world, t, stream)
+    gt = GroupTransport(group)
+    return kgs.kgs_vp_query(graph, kw, k, p, rank, world, gt.t, stream)

@@ -1,9 +1,10 @@
-"""Vertex-partitioned search of one query (dist.vp_search) over gloo on CPU, world sizes
-2 and 3: the per-level exchanges (all-gather of the hit masks, all-reduce of the counters), the stop
-rules and the final all-gathers of M and of the central lists.  The level kernels are the test-only numpy
-stand-in (vp_numpy_ops) so this runs without a GPU; the state every rank ends with must equal the
-oracle's search (M, central set with depths, stop level and reason).  The C-ABI slice rule is checked
-against the library (a host-only call)."""
+"""Vertex-partitioned search of one query over gloo on CPU, world sizes 2 and 3: the
+protocol of kgs_vp_query (csrc/vpquery.cu) — per-level exchanges (dense all-gather of the hit masks, or
+sparse change lists), all-reduce of the counters, the stop rules, the final all-gathers of M and of the
+central lists — as the test-side model vp_numpy_ops.vp_search over numpy stand-ins of the level kernels, so
+this runs without a GPU; the state every rank ends with must equal the oracle's search.  The transport the
+product uses with gloo (dist.GroupTransport, host-staged callbacks) is checked on its own, and the C-ABI
+slice rule against the library (a host-only call)."""
 import os
 import socket
 
@@ -49,8 +50,7 @@ def _worker(rank, world, port, out_q):
     sys.path.insert(0, os.path.join(root, "tests"))
     import torch.distributed as dist
 
-    from paper_conf_icde_yangajtw19_b200 import dist as kd
-    from vp_numpy_ops import NumpyVpOps
+    from vp_numpy_ops import NumpyVpOps, vp_search
 
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
@@ -59,10 +59,10 @@ def _worker(rank, world, port, out_q):
     for g, kw, k, par in _cases():
         ops = NumpyVpOps(g, alpha=par.get("alpha", 0.1), block_central=par.get("block_central", 1))
         ops.alloc(world)
-        s = kd.vp_search(ops, kw, k, par.get("max_depth", 254), rank, world)
+        s = vp_search(ops, kw, k, par.get("max_depth", 254), rank, world)
         M = ops.bufs["M"].numpy().reshape(-1, 8)[:g.n, :len(kw)].copy()
         order = np.argsort(s["cent"].numpy(), kind="stable")
-        res.append(dict(levels=s["levels"], stop=s["stop"], n_central=s["n_central"], M=M,
+        res.append(dict(levels=s["levels"], stop=s["stop"], n_central=s["n_central"], M=M, sparse=s["sparse"],
                         cent=s["cent"].numpy()[order].tolist(), cdep=s["cdep"].numpy()[order].tolist()))
     out_q.put((rank, res))
     dist.barrier()
@@ -92,6 +92,7 @@ def test_vp_search_equals_oracle(world):
             assert s["levels"] == o.levels or o.stop_reason == oracle.STOP_EMPTY_KEYWORD, ctx_
             assert s["cent"] == o.centrals.tolist() and s["cdep"] == o.central_depth.tolist(), ctx_
             assert (s["M"] == o.M).all(), ctx_
+    assert any(got[0][ci]["sparse"] for ci in range(len(_cases())))   # the sparse exchange was exercised
 
 
 def test_vp_slice_rule_matches_library():
@@ -101,3 +102,47 @@ def test_vp_slice_rule_matches_library():
         s = kgs.kgs_vp_slice(n, w)
         assert s == slice_size(n, w) and s % 16 == 0 and s * w >= n
     assert kgs.kgs_vp_slice(5, 0) == 0
+
+
+def _transport_worker(rank, world, port, out_q):
+    import ctypes
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icde_yangajtw19_b200 import dist as kd
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    gt = kd.GroupTransport()
+    send = (ctypes.c_uint8 * 5)(*[rank * 10 + i for i in range(5)])
+    recv = (ctypes.c_uint8 * (5 * world))()
+    rc1 = gt.t.all_gather(None, ctypes.addressof(send), ctypes.addressof(recv), 5, None)
+    buf = (ctypes.c_int64 * 4)(rank, 1, -rank, 1 << 40)
+    rc2 = gt.t.all_reduce_sum_i64(None, ctypes.addressof(buf), 4, None)
+    out_q.put((rank, rc1, rc2, list(recv), list(buf), gt.t.host_staged))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_group_transport_callbacks(world):
+    """dist.GroupTransport (the gloo transport of kgs_vp_query): all_gather / all_reduce callbacks on host
+    buffers give every rank the concatenation / the sum."""
+    pytest.importorskip("paper_conf_icde_yangajtw19_b200")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_transport_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, rc1, rc2, recv, buf, staged in got:
+        assert rc1 == 0 and rc2 == 0 and staged == 1
+        assert recv == [r * 10 + i for r in range(world) for i in range(5)]
+        assert buf == [sum(range(world)), world, -sum(range(world)), world << 40]
