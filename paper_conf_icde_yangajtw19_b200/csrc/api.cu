@@ -163,7 +163,7 @@ struct kgs_result {
 namespace {
 
 void free_work(DevWork &w) {
-    void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.qrec, w.qbrec, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
+    void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
                  w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
                  w.gstate, w.huge};
@@ -184,8 +184,6 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.fbits, (size_t)std::max({g->R_alloc, g->R, 2}) * (size_t)g->W));
     CUDA_TRY(dmalloc(&w.qlight, n));
     CUDA_TRY(dmalloc(&w.qbig, g->n_big));
-    CUDA_TRY(dmalloc(&w.qrec, n));
-    CUDA_TRY(dmalloc(&w.qbrec, std::max(g->n_big, g->n_big_in)));   // also the pre-pass's (in-arc classes)
     CUDA_TRY(dmalloc(&w.touched, n));
     CUDA_TRY(dmalloc(&w.qdef, n));
     CUDA_TRY(dmalloc(&w.centrals, n));
@@ -538,7 +536,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if ((int)g->works.size() < G) {   // each group needs its own workspace: keep them within free memory
         size_t free_b = 0, total_b = 0;
         cudaMemGetInfo(&free_b, &total_b);
-        const size_t per = (size_t)g->n * 121 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
+        const size_t per = (size_t)g->n * 105 + (size_t)std::max(g->R, 2) * g->W * 4 + (size_t)(16ll << 20) * 18 +
                            (size_t)pcap_of(g) * 20 +
                            g->huge_arena_bytes;
         const int more = (int)std::min<size_t>((size_t)(G - (int)g->works.size()), (size_t)(0.8 * free_b) / per);
@@ -554,6 +552,12 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     CUDA_TRY(grow_dev(&g->d_nodes, &g->d_nodes_cap, (size_t)nq * k * 64 + (16u << 20)));
     CUDA_TRY(grow_dev(&g->d_arcs, &g->d_arcs_cap, 2 * ((size_t)nq * k * 64 + (32u << 20))));
     CUDA_TRY(cudaMemsetAsync(g->d_ctr, 0, 4 * sizeof(unsigned long long), s));
+    // the result headers are copied back whole: clear them so that no byte the engine leaves unwritten
+    // (phase stamps beyond n_stamp, answer slots beyond count) is uninitialised memory
+    CUDA_TRY(cudaMemsetAsync(g->d_qout, 0, sizeof(QOut) * (size_t)nq, s));
+    CUDA_TRY(cudaMemsetAsync(g->d_hdr, 0, sizeof(int32_t) * (size_t)nq * k * 4, s));
+    CUDA_TRY(cudaMemsetAsync(g->d_key, 0, sizeof(double) * (size_t)nq * k, s));
+    CUDA_TRY(cudaMemsetAsync(g->d_off, 0, sizeof(long long) * (size_t)nq * k * 2, s));
     EngineArgs a{};
     a.g.n = g->n; a.g.m = g->m; a.g.row_ptr = g->row_ptr; a.g.col_idx = g->col_idx; a.g.in_ptr = g->in_ptr;
     a.g.in_idx = g->in_idx; a.g.weight = g->weight; a.g.cls = g->cls; a.g.cls_in = g->cls_in; a.g.n_kw = g->n_kw;

@@ -233,78 +233,41 @@ constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16
 // compact_deferred spreads the deferred nodes over every thread of the group.
 constexpr int kLocalNodes = kBlock;
 
-// The per-node work is split in two so that several nodes' loads are in flight at once: pre(v) issues
-// the node's loads and returns them (NodePre), on_node(v, pre) applies the merge and returns flags: bit 0
-// = v goes to the aux list, bit 1 = v expands at this level.  With expansion records (rec / brec non-null,
-// the search) the compaction also writes, next to every queue entry, the node's arc range (pre.b, pre.e:
-// its row_ptr pair, loaded with the state), or degree 0 when it does not expand: the expansion then reads
-// the range with the queue instead of a dependent state -> row_ptr chain.
-struct NodePre {
-    uint64_t s;
-    int64_t b, e;
-};
-__device__ __forceinline__ int4 exp_rec(bool expands, const NodePre &p) {
-    return make_int4(expands ? (int)(p.e - p.b) : 0, 0, (int)(uint32_t)(p.b & 0xFFFFFFFFll), (int)(p.b >> 32));
-}
-
 template <class OnNode, class OnAux>
-__device__ __forceinline__ void compact_apply(int32_t *ql, int64_t pos, int32_t v, const NodePre &pv, uint8_t cl,
-                                              int32_t *qb, uint32_t *nb, int4 *rec, int4 *brec, int32_t *aux,
-                                              uint32_t *naux, OnNode &on_node, OnAux &on_aux) {
-    const int f = on_node(v, pv);
-    if (cls_big(cl)) {
-        const uint32_t bi = atomicAdd(nb, 1u);
-        qb[bi] = v;
-        ql[pos] = -1;
-        if (brec) { brec[bi] = exp_rec(f & 2, pv); rec[pos] = make_int4(0, 0, 0, 0); }
-    } else if (rec) {
-        rec[pos] = exp_rec(f & 2, pv);
-    }
-    if (f & 1) {
+__device__ __forceinline__ void compact_node(int32_t *ql, int64_t pos, const uint8_t *cls, int32_t *qb, uint32_t *nb,
+                                             int32_t *aux, uint32_t *naux, OnNode &on_node, OnAux &on_aux) {
+    const int32_t v = ql[pos];
+    const bool flag = on_node(v);
+    if (cls_big(cls[v])) { qb[atomicAdd(nb, 1u)] = v; ql[pos] = -1; }
+    if (flag) {
         const uint32_t p = agg_slot(naux, 0x5u);
         aux[p] = v;
         on_aux(v, p);
     }
 }
 
-// The deferred nodes of compact(), strided over the group, kDefUnroll per thread with their queue, state
-// and class loads issued before any of them is applied.  Call after a group barrier; returns whether
+// The deferred nodes of compact(), strided over the group.  Call after a group barrier; returns whether
 // there were any (then the caller needs another barrier before reading the queues).
-constexpr int kDefUnroll = 4;
-template <class Pre, class OnNode, class OnAux>
+template <class OnNode, class OnAux>
 __device__ __forceinline__ bool compact_deferred(const Grp &G, const int32_t *qdef, uint32_t nd, int32_t *ql,
-                                                 const uint8_t *cls, int32_t *qb, uint32_t *nb, int4 *rec,
-                                                 int4 *brec, int32_t *aux, uint32_t *naux, Pre pre, OnNode on_node,
-                                                 OnAux on_aux) {
-    for (int64_t j0 = G.gtid; j0 < nd; j0 += kDefUnroll * G.gsz) {
-        int64_t pos[kDefUnroll];
-        int32_t v[kDefUnroll];
-        NodePre pv[kDefUnroll];
-        uint8_t cl[kDefUnroll];
+                                                 const uint8_t *cls, int32_t *qb, uint32_t *nb, int32_t *aux,
+                                                 uint32_t *naux, OnNode on_node, OnAux on_aux) {
+    constexpr int U = 4;   // the queue-position loads of U deferred nodes are in flight together
+    for (int64_t j0 = G.gtid; j0 < nd; j0 += U * G.gsz) {
+        int64_t pos[U];
 #pragma unroll
-        for (int k = 0; k < kDefUnroll; ++k) {
-            const int64_t j = j0 + k * G.gsz;
-            pos[k] = j < nd ? (int64_t)__ldcg(qdef + j) : -1;
-        }
+        for (int k = 0; k < U; ++k) pos[k] = j0 + k * G.gsz < nd ? (int64_t)__ldcg(qdef + j0 + k * G.gsz) : -1;
 #pragma unroll
-        for (int k = 0; k < kDefUnroll; ++k) v[k] = pos[k] >= 0 ? __ldcg(ql + pos[k]) : -1;
-#pragma unroll
-        for (int k = 0; k < kDefUnroll; ++k) {
-            pv[k] = v[k] >= 0 ? pre(v[k]) : NodePre{0ull, 0, 0};
-            cl[k] = v[k] >= 0 ? __ldg(cls + v[k]) : (uint8_t)0;
-        }
-#pragma unroll
-        for (int k = 0; k < kDefUnroll; ++k)
-            if (v[k] >= 0) compact_apply(ql, pos[k], v[k], pv[k], cl[k], qb, nb, rec, brec, aux, naux, on_node, on_aux);
+        for (int k = 0; k < U; ++k)
+            if (pos[k] >= 0) compact_node(ql, pos[k], cls, qb, nb, aux, naux, on_node, on_aux);
     }
     return nd != 0;
 }
 
-template <class Pre, class OnNode, class OnAux>
+template <class OnNode, class OnAux>
 __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W, const uint8_t *cls, int32_t *ql,
-                                        uint32_t *nl, int32_t *qb, uint32_t *nb, int4 *rec, int4 *brec,
-                                        int32_t *aux, uint32_t *naux, int32_t *qdef, uint32_t *ndef, long long *sh,
-                                        Pre pre, OnNode on_node, OnAux on_aux) {
+                                        uint32_t *nl, int32_t *qb, uint32_t *nb, int32_t *aux, uint32_t *naux,
+                                        int32_t *qdef, uint32_t *ndef, long long *sh, OnNode on_node, OnAux on_aux) {
     const int64_t step = (int64_t)blockDim.x * kWpt;
     const int64_t cw = ((W + G.gcount - 1) / G.gcount + kWpt - 1) / kWpt * kWpt;
     const int64_t w0 = (int64_t)G.grank * cw, w1 = w0 + cw < W ? w0 + cw : W;
@@ -352,18 +315,8 @@ __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W,
             int flag = 0;
             if (j < tot) {
                 v = ql[seg0 + j];
-                const NodePre pv = pre(v);
-                const uint8_t cl = __ldg(cls + v);
-                const int f = on_node(v, pv);
-                flag = f & 1;
-                if (cls_big(cl)) {
-                    const uint32_t bi = atomicAdd(nb, 1u);
-                    qb[bi] = v;
-                    ql[seg0 + j] = -1;
-                    if (brec) { brec[bi] = exp_rec(f & 2, pv); rec[seg0 + j] = make_int4(0, 0, 0, 0); }
-                } else if (rec) {
-                    rec[seg0 + j] = exp_rec(f & 2, pv);
-                }
+                flag = on_node(v) ? 1 : 0;
+                if (cls_big(cls[v])) { qb[atomicAdd(nb, 1u)] = v; ql[seg0 + j] = -1; }
             }
             long long atot;
             const long long aex = block_excl_scan64(flag, &atot, sh);
@@ -390,7 +343,7 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, uint32_t zbv, int32_t x,
-                                          uint32_t sx, unsigned &dag) {
+                                          uint32_t sx, unsigned &hits, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = st_gate(sx);
@@ -415,20 +368,33 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                 atomicMin(c.w.mw + (int64_t)x * 8 + i, __ldcg(c.w.mw + (int64_t)v * 8 + i));
             }
         }
-        // fire and forget (no returned value to wait for): every writer of this level sets the same bits and
-        // writes the same level l+1 into entries whose hit bit was clear at the level's start, and the
-        // frontier push is a bit set, so repeating them for arcs that lost a race changes nothing (Thm. V.2).
-        // The new (node, keyword) pairs are counted when the next merge folds nm into hm.
-        asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(c.w.st + x), "r"(bits << 16) : "memory");
-        uint8_t *row = c.w.M + (int64_t)x * 8;
-        const uint8_t lv = (uint8_t)(l + 1);
+        const uint32_t old = st_nm(atomicOr(c.w.st + x, bits << 16));
+        const uint32_t nb = bits & ~old;
+        if (nb) {
+            hits += __popc(nb);
+            uint8_t *row = c.w.M + (int64_t)x * 8;
+            const uint8_t lv = (uint8_t)(l + 1);
 #pragma unroll
-        for (int i = 0; i < kMaxQ; ++i)
-            if (bits & (1u << i)) row[i] = lv;            // ln 21: m_xi <- l+1
-        push(c, x, l + 1);                                // ln 22: FIdentifier[x] <- 1
+            for (int i = 0; i < kMaxQ; ++i)
+                if (nb & (1u << i)) row[i] = lv;          // ln 21: m_xi <- l+1
+            if (old == 0) push(c, x, l + 1);              // ln 22: FIdentifier[x] <- 1 (first new bit)
+        }
     } else {
         push(c, v, (int)gate - 1, true);                  // ln 19: v must retry when x opens
     }
+}
+
+// Alg. 2 ln 2-7 for node v at level l: returns its expansion mask (0 = does not expand now).
+__device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool leader) {
+    const uint32_t sv = __ldcg(c.w.st + v);
+    const uint32_t hm = sv & 0xFFu;
+    if (c.a.block_central && hm == c.qq.full) return 0;   // ln 2-3: central nodes do not expand
+    const int av = (int)st_act(sv);
+    if (av > l) {                                          // ln 5-7: not yet active
+        if (leader) push(c, v, av);
+        return 0;
+    }
+    return hm;                                             // ln 8-11: every hit instance has m <= l
 }
 
 constexpr int kTileMax = kBlock;
@@ -469,8 +435,7 @@ struct BigTile {
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint32_t cb, const int64_t *ptr,
                                            const int32_t *idx, const uint32_t *st, BigTile &S, long long *sh,
-                                           Prep prep, Visit visit, unsigned long long &arcs,
-                                           const int4 *rec = nullptr) {
+                                           Prep prep, Visit visit, unsigned long long &arcs) {
     NodeT *node = reinterpret_cast<NodeT *>(S.node);
     for (uint32_t t0 = 0; t0 < cb; t0 += blockDim.x) {
         const int nt = (int)min((uint32_t)blockDim.x, cb - t0);
@@ -479,10 +444,7 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
         if (j < nt) {
             const int32_t v = __ldcg(qb + t0 + j);   // -1: a big node listed in the light queue
             NodeT nd{};
-            if (rec) {   // expansion record of the merge: the arc range, degree 0 = does not expand
-                const int4 r = __ldcg(rec + t0 + j);
-                if (v >= 0 && r.x > 0) { deg = r.x; s0 = (long long)(uint32_t)r.z | ((long long)r.w << 32); prep(v, G.grank == 0, nd); }
-            } else if (v >= 0 && prep(v, G.grank == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
+            if (v >= 0 && prep(v, G.grank == 0, nd)) { s0 = ptr[v]; deg = ptr[v + 1] - s0; }
             node[j] = nd;
             S.start[j] = s0;
         }
@@ -530,7 +492,7 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
                                              const int32_t *idx, const uint32_t *st, Prep prep, Visit visit,
-                                             unsigned long long &arcs, const int4 *rec = nullptr) {
+                                             unsigned long long &arcs) {
     const uint32_t warps = (uint32_t)(G.gsz >> 5);
     uint32_t B = (c0 + 2 * warps - 1) / (2 * warps);
     B = B < 1 ? 1u : (B > 32 ? 32u : B);
@@ -543,10 +505,7 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
         int deg = 0;
         if (lane < B && i < c0) {
             const int32_t v = ql ? __ldcg(ql + i) : (int32_t)i;   // -1: a big node, expanded by expand_big
-            if (rec) {   // expansion record of the merge: the arc range, degree 0 = does not expand
-                const int4 r = __ldcg(rec + i);
-                if (v >= 0 && r.x > 0) { deg = r.x; start = (int64_t)(uint32_t)r.z | ((int64_t)r.w << 32); prep(v, true, nd); }
-            } else if (v >= 0 && prep(v, true, nd)) { start = ptr[v]; deg = (int)(ptr[v + 1] - start); }
+            if (v >= 0 && prep(v, true, nd)) { start = ptr[v]; deg = (int)(ptr[v + 1] - start); }
         }
         int incl = deg;
 #pragma unroll
@@ -700,26 +659,20 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (!__ldcg(&ctl->pd_flag[slot])) break;
         uint32_t *qn = ctl->pd_qn[slot];
         if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; }
-        auto pd_pre = [&](int32_t u) {
-            return NodePre{(uint64_t)__ldcg(c.w.pd_state + u) | ((uint64_t)(uint32_t)__ldcg(c.w.pd_cid + u) << 32),
-                           __ldg(c.a.g.in_ptr + u), __ldg(c.a.g.in_ptr + u + 1)};
-        };
-        auto pd_node = [&](int32_t u, const NodePre &pre) {
-            const uint64_t pv = pre.s;
-            const uint32_t s = (uint32_t)pv;
+        auto pd_node = [&](int32_t u) {
+            const uint32_t s = __ldcg(c.w.pd_state + u);
             const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
             const uint32_t bits = nx & ~dn;
             c.w.pd_state[u] = bits | ((dn | bits) << 16);
-            return ((bits != 0 && (int32_t)(pv >> 32) < 0) ? 1 : 0) | (bits != 0 ? 2 : 0);   // expands: bits to do
+            return bits != 0 && __ldcg(c.w.pd_cid + u) < 0;
         };
         auto pd_aux = [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; };
         if (G.gtid == 0) ctl->pd_ndef[slot ^ 1] = 0u;
         compact(G, c.w.pd_bits + (int64_t)slot * W, W, c.a.g.cls_in, c.w.pd_qlight, &qn[0], c.w.pd_qbig, &qn[1],
-                c.w.qrec, c.w.qbrec, c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, pd_pre, pd_node,
-                pd_aux);
+                c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, pd_node, pd_aux);
         G.sync();
         if (compact_deferred(G, c.w.qdef, __ldcg(&ctl->pd_ndef[slot]), c.w.pd_qlight, c.a.g.cls_in, c.w.pd_qbig,
-                             &qn[1], c.w.qrec, c.w.qbrec, c.w.pd_touched, &ctl->n_cid, pd_pre, pd_node, pd_aux))
+                             &qn[1], c.w.pd_touched, &ctl->n_cid, pd_node, pd_aux))
             G.sync();
         stamp(G, qo, TS_PD_MERGE);
         const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
@@ -728,13 +681,11 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int nflag = kFlagPd + (slot ^ 1);
         auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
         auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) { pd_visit(c, exact_block, nd, u, su, nbits, nflag); };
-        // the expansion records of the compaction (the search's qrec / qbrec arrays, idle now) give the in-arc
-        // ranges: a node whose bits are all done has degree 0
-        expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs, c.w.qbrec);
+        expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)c.a.tile_light)   // small frontier: tiles over the whole group
-            expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs, c.w.qrec);
+            expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         else
-            expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs, c.w.qrec);
+            expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
@@ -839,7 +790,7 @@ __device__ void td_only_prepare(const Ctx &c, QOut *qo) {
 // One pulled level l (kgs_params.direction; called by search()): light candidates by a contiguous sweep of
 // all nodes, the ones with more than kBigDeg in-arcs afterwards in group-wide tiles.  (Inlined: out of line, the
 // call spilled the push path's level-loop state, p50 0.35 -> 0.43 ms; tools/ab_perf.py.)
-__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh,
+__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh, unsigned &my_hits,
                                          unsigned &my_dag, unsigned long long &my_arcs) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -874,7 +825,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
                 if (((row >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
             }
         }
-        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_dag);
+        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_hits, my_dag);
     };
     expand_light<PullNode>(G, nullptr, (uint32_t)n, a.g.in_ptr, a.g.in_idx, w.st, plight, pvisit, my_arcs);
     G.sync();
@@ -1048,55 +999,41 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             ctl->mf[(l + 1) & 1] = 0ull; ctl->pull_nbig[(l + 1) & 1] = 0u;
         }
         // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
-        // one load of the status word and the row_ptr pair per frontier node (NodePre)
-        auto merge_pre = [&](int32_t v) {
-            return NodePre{(uint64_t)__ldcg(w.st + v), __ldg(a.g.row_ptr + v), __ldg(a.g.row_ptr + v + 1)};
-        };
-        auto merge_node = [&](int32_t v, const NodePre &p) {
-                    const uint32_t sv = (uint32_t)p.s;
+        auto merge_node = [&](int32_t v) {
+                    // auto direction: out-arcs of the frontier nodes that can expand (a_v <= l, ln 4-7),
+                    // bounded by the power of two of the class byte (no row_ptr load)
+                    const uint32_t sv = __ldcg(w.st + v);
+                    if (count_lvl && !pulling && (int)st_act(sv) <= l)
+                        my_mf += cls_deg_bound(a.g.cls[v]);
                     const uint32_t b = st_nm(sv);
+                    if (!b) return false;
+                    if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
                     const uint32_t old = sv & 0xFFu;
                     const uint32_t nw = old | b;
-                    const int av = (int)st_act(sv);
-                    int f = 0;
-                    // auto direction: out-arcs of the frontier nodes that can expand (a_v <= l, ln 4-7)
-                    if (count_lvl && !pulling && av <= l) my_mf += (unsigned long long)(p.e - p.b);
-                    if (b) {
-                        if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
-                        if (l > 0) my_hits += __popc(b);   // new (node, keyword) pairs of level l - 1's expansion
-                        w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
-                        if (a.prune == 2) {   // lightest path to v for keyword i = min over predecessors + w_v
-                            const uint32_t wv = weight_fx(__ldg(a.g.weight + v));
-                            for (uint32_t bb = b; bb; bb &= bb - 1) {
-                                uint32_t *q = w.mw + (int64_t)v * 8 + (__ffs(bb) - 1);
-                                *q = *q + wv;
-                            }
+                    w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
+                    if (a.prune == 2) {   // lightest path to v for keyword i = min over predecessors + w_v
+                        const uint32_t wv = weight_fx(__ldg(a.g.weight + v));
+                        for (uint32_t bb = b; bb; bb &= bb - 1) {
+                            uint32_t *p = w.mw + (int64_t)v * 8 + (__ffs(bb) - 1);
+                            *p = *p + wv;
                         }
-                        if (nw == full && old != full) {                        // Lemma V.1: depth = l
-                            const uint32_t ci = agg_slot(&ctl->n_central, 1u);
-                            w.centrals[ci] = v;
-                            w.cdepth[ci] = (uint8_t)l;
-                        }
-                        if (old == 0) f |= 1;
                     }
-                    // Alg. 2 ln 2-7 for v at level l, decided here (hm is final for the level): a central node
-                    // does not expand (ln 2-3), an inactive one is re-queued at a_v (ln 5-7), the others expand
-                    // with their whole mask (ln 8-11); the expansion reads the decision as the arc range
-                    if (!(a.block_central && nw == full) && nw) {
-                        if (av > l) push(c, v, av);
-                        else f |= 2;
+                    if (nw == full && old != full) {                        // Lemma V.1: depth = l
+                        const uint32_t ci = agg_slot(&ctl->n_central, 1u);
+                        w.centrals[ci] = v;
+                        w.cdepth[ci] = (uint8_t)l;
                     }
-                    return f;
+                    return old == 0;
                 };
         auto merge_aux = [&](int32_t v, uint32_t pos) {   // recorded DAG: compact id = touched position
             if (a.dag_record) { w.pd_touched[pos] = v; w.pd_cid[v] = (int32_t)pos; }
         };
-        compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.qrec, w.qbrec, w.touched,
-                &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_pre, merge_node, merge_aux);
+        compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
+                &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
         if (count_lvl && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
         G.sync();
-        if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.qrec, w.qbrec,
-                             w.touched, &ctl->n_touched, merge_pre, merge_node, merge_aux)) {
+        if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.touched,
+                             &ctl->n_touched, merge_node, merge_aux)) {
             if (count_lvl && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
             G.sync();
         }
@@ -1141,9 +1078,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             // visit_arc as the push, so the hits, the recorded Thm. V.4 arcs and the lightest-path rows
             // are the same; no node is re-queued (ln 19): a pulling search has no work list (a level
             // without hits asks pull_waiting whether the list would still be non-empty).
-            const unsigned dag0 = my_dag;   // hitting arcs of this level: some (node, keyword) was marked
-            pull_expand(c, l, S, sh, my_dag, my_arcs);
-            cta_add((unsigned long long)(my_dag - dag0), &ctl->pull_marks[l & 1]);
+            const unsigned hits0 = my_hits;
+            pull_expand(c, l, S, sh, my_hits, my_dag, my_arcs);
+            cta_add((unsigned long long)(my_hits - hits0), &ctl->pull_marks[l & 1]);
             publish_flags(ctl);
             G.sync();
             stamp(G, qo, TS_EXPAND);
@@ -1161,10 +1098,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             }
             continue;
         }
-        // the merge decided who expands (expansion records): fill the node's mask (and sources)
-        auto prep = [&](int32_t v, bool, FwdNode &nd) {
+        auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
             nd.v = v;
-            nd.hm = __ldcg(w.st + v) & 0xFFu;
+            nd.hm = prepare(c, l, v, leader);
             nd.zb = 0;
             if (a.dag_record && nd.hm) {
                 const uint64_t row = ldrow(w.M, v);
@@ -1176,13 +1112,13 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             return nd.hm != 0;
         };
         auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) {
-            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_dag);
+            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_hits, my_dag);
         };
-        expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs, w.qbrec);
+        expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
-            expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs, w.qrec);
+            expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         else
-            expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs, w.qrec);
+            expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_EXPAND);
@@ -1388,7 +1324,7 @@ __device__ __forceinline__ int arena_insert(Arena &S, int32_t u, uint32_t zbu, b
         if (k == u) {
             int v;
             while ((v = atomicAdd(S.hval + h, 0)) == -1) { }
-            __threadfence_block();   // acquire: the inserter's id / zb stores precede its publication of hval
+            __threadfence_block();   // acquire: the inserter's id stores precede its publication of hval
             return v >= 0 ? v : -1;
         }
         h = (h + 1) & (uint32_t)(S.hcap - 1);
@@ -1501,7 +1437,7 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
                 if (j < 0) continue;
                 if (fresh && cut_on) atomicAdd(S.wsum, (unsigned long long)weight_fx(__ldg(c.a.g.weight + u)));
                 const uint32_t old = atomicOr(S.inmask + j, pb);
-                const uint32_t nbits = pb & ~old & ~S.zb[j];
+                const uint32_t nbits = pb & ~old & ~zbu;   // zb(u) is a property of u: the inserter stored this value
                 if (nbits) {
                     const uint32_t oldp = atomicOr(S.pending + j, nbits);
                     if (oldp == 0) fifo_push(S, j);

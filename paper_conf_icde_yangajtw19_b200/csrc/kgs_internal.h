@@ -131,8 +131,6 @@ struct DevWork {
     uint32_t *fbits;    // [R][W] frontier bitmaps, slot = level % R (FIdentifier)
     int32_t *qlight;    // [n] compacted frontier of the current level (big nodes replaced by -1)
     int32_t *qbig;      // [n_big] compacted frontier, big nodes
-    int4 *qrec;         // [n] expansion record per qlight entry: {degree (0 = does not expand), -, row start}
-    int4 *qbrec;        // [n_big] the same per qbig entry
     int32_t *touched;   // [n] nodes whose hm became non-zero (sparse reset of the next query)
     int32_t *qdef;      // [n] compaction: queue positions deferred to the group-wide pass (dense tiles)
     int32_t *centrals;  // [n] central ids in identification order
