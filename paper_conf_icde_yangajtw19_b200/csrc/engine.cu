@@ -343,7 +343,7 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
 // sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, uint32_t zbv, int32_t x,
-                                          uint32_t sx, unsigned &hits, unsigned &dag) {
+                                          uint32_t sx, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
     if (!bits) return;
     const uint32_t gate = st_gate(sx);
@@ -368,17 +368,17 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                 atomicMin(c.w.mw + (int64_t)x * 8 + i, __ldcg(c.w.mw + (int64_t)v * 8 + i));
             }
         }
-        const uint32_t old = st_nm(atomicOr(c.w.st + x, bits << 16));
-        const uint32_t nb = bits & ~old;
-        if (nb) {
-            hits += __popc(nb);
-            uint8_t *row = c.w.M + (int64_t)x * 8;
-            const uint8_t lv = (uint8_t)(l + 1);
+        // fire and forget (no returned value to wait for): every writer of this level sets the same bits and
+        // writes the same level l+1 into entries whose hit bit was clear at the level's start, and the
+        // frontier push is a bit set, so repeating them for arcs that lost a race changes nothing (Thm. V.2).
+        // The new (node, keyword) pairs are counted when the next merge folds nm into hm.
+        asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(c.w.st + x), "r"(bits << 16) : "memory");
+        uint8_t *row = c.w.M + (int64_t)x * 8;
+        const uint8_t lv = (uint8_t)(l + 1);
 #pragma unroll
-            for (int i = 0; i < kMaxQ; ++i)
-                if (nb & (1u << i)) row[i] = lv;          // ln 21: m_xi <- l+1
-            if (old == 0) push(c, x, l + 1);              // ln 22: FIdentifier[x] <- 1 (first new bit)
-        }
+        for (int i = 0; i < kMaxQ; ++i)
+            if (bits & (1u << i)) row[i] = lv;            // ln 21: m_xi <- l+1
+        push(c, x, l + 1);                                // ln 22: FIdentifier[x] <- 1
     } else {
         push(c, v, (int)gate - 1, true);                  // ln 19: v must retry when x opens
     }
@@ -621,15 +621,25 @@ __device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cn
     const int64_t rcap = c.rec_cap;
     __shared__ uint32_t s_pre[kRecStripes + 1];
     static_assert(kRecStripes <= kBlock, "one thread per region");
+    static_assert(kRecStripes == 4 * kWarp, "four warps scan the region counts");
+    __shared__ uint32_t s_wsum[4];
     __syncthreads();
-    if (threadIdx.x < kRecStripes) {
-        int64_t k = threadIdx.x < ns ? (int64_t)__ldcg(&cnt[threadIdx.x * kRecStride]) : 0;
-        s_pre[threadIdx.x + 1] = (uint32_t)(k < rcap ? k : rcap);
+    uint32_t incl = 0;
+    if (threadIdx.x < kRecStripes) {   // inclusive scan of the region counts: warp scans + 4 warp totals
+        const int64_t k = threadIdx.x < ns ? (int64_t)__ldcg(&cnt[threadIdx.x * kRecStride]) : 0;
+        incl = (uint32_t)(k < rcap ? k : rcap);
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+            if ((int)lane_id() >= o) incl += t;
+        }
+        if (lane_id() == 31) s_wsum[threadIdx.x >> 5] = incl;
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        s_pre[0] = 0;
-        for (int r = 0; r < kRecStripes; ++r) s_pre[r + 1] += s_pre[r];
+    if (threadIdx.x < kRecStripes) {
+        for (int w = 0; w < (int)(threadIdx.x >> 5); ++w) incl += s_wsum[w];
+        s_pre[threadIdx.x + 1] = incl;
+        if (threadIdx.x == 0) s_pre[0] = 0;
     }
     __syncthreads();
     const int64_t T = s_pre[kRecStripes];
@@ -691,11 +701,15 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         stamp(G, qo, TS_PD_EXPAND);
     }
     if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
-    if (G.gtid == 0) {
-        ctl->pd_rounds = r;
-        uint32_t np = 0;
-        for (int k = 0; k < rec_stripes(G); ++k) np += __ldcg(&ctl->pd_cnt[k * kRecStride]);
-        ctl->n_parcs = np;
+    if (G.grank == 0) {   // the append regions' counts, one per thread, then a warp sum (not 128 serial loads)
+        __shared__ uint32_t s_np;
+        if (threadIdx.x == 0) s_np = 0;
+        __syncthreads();
+        uint32_t k = threadIdx.x < (unsigned)rec_stripes(G) ? __ldcg(&ctl->pd_cnt[threadIdx.x * kRecStride]) : 0u;
+        k = __reduce_add_sync(0xffffffffu, k);
+        if ((threadIdx.x & 31) == 0 && k) atomicAdd(&s_np, k);
+        __syncthreads();
+        if (threadIdx.x == 0) { ctl->pd_rounds = r; ctl->n_parcs = s_np; }
     }
     build_pred_csr(c, sh, qo);
 }
@@ -790,7 +804,7 @@ __device__ void td_only_prepare(const Ctx &c, QOut *qo) {
 // One pulled level l (kgs_params.direction; called by search()): light candidates by a contiguous sweep of
 // all nodes, the ones with more than kBigDeg in-arcs afterwards in group-wide tiles.  (Inlined: out of line, the
 // call spilled the push path's level-loop state, p50 0.35 -> 0.43 ms; tools/ab_perf.py.)
-__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh, unsigned &my_hits,
+__device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, long long *sh,
                                          unsigned &my_dag, unsigned long long &my_arcs) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -825,7 +839,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
                 if (((row >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
             }
         }
-        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_hits, my_dag);
+        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_dag);
     };
     expand_light<PullNode>(G, nullptr, (uint32_t)n, a.g.in_ptr, a.g.in_idx, w.st, plight, pvisit, my_arcs);
     G.sync();
@@ -908,23 +922,31 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
     } else {
         const Ctl *pv = w.ctl[(done + 1) & 1];   // the previous query's block
-        // a recorded DAG gave compact ids to exactly the touched nodes (pd_state unused): one loop below
-        const bool prev_rec = pv->rec_used != 0;
-        if (!prev_rec)
-            for (int64_t j = gtid; j < (int64_t)pv->n_cid; j += gsz) {
+        // Predecessor-list state (pd_cid compact ids, pd_state).  A recorded-DAG query gives compact ids to
+        // all of its touched nodes and reads pd_cid / pd_state of no other node (closures and recorded arcs
+        // only hold hit nodes), so it resets neither — it only leaves the workspace "dirty" (gstate[2] bit
+        // 1).  A pre-pass query reads pd_cid / pd_state of its closure nodes, which may have been touched by
+        // any earlier query: after dirty queries it resets both densely (sequential writes), otherwise the
+        // previous pre-pass's list.  pcnt is indexed by compact id: its prefix is reset in every case.
+        const bool dirty = (valid & 2u) != 0;
+        const int64_t pn = (int64_t)pv->n_cid;
+        if (a.dag_record) {
+            for (int64_t j = gtid; j < pn; j += gsz) w.pcnt[j] = 0;
+        } else if (dirty) {
+            for (int64_t v = gtid; v < n; v += gsz) { w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[v] = 0; }
+        } else {
+            for (int64_t j = gtid; j < pn; j += gsz) {
                 const int32_t v = w.pd_touched[j];
                 w.pd_state[v] = 0u; w.pd_cid[v] = -1; w.pcnt[j] = 0;
             }
+        }
         const int64_t pt = (int64_t)pv->n_touched;
-        if (prev_rec && pt > n / 16)
-            for (int64_t j = gtid; j < pt; j += gsz) { w.pd_cid[w.touched[j]] = -1; w.pcnt[j] = 0; }
         if (pt > n / 16) {   // many touched rows: a dense sweep beats scattered 2-byte writes
             reset_status_dense(c);
         } else {
             for (int64_t j = gtid; j < pt; j += gsz) {
                 const int32_t v = w.touched[j];
                 w.st[v] = st_fresh(a.act[v]);
-                if (prev_rec) { w.pd_cid[v] = -1; w.pcnt[j] = 0; }
             }
         }
         for (int s = 0; s < R; ++s)   // level slots still pending when the previous query stopped
@@ -978,17 +1000,14 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     unsigned long long my_mf = 0;
     for (int l = 0;; ++l) {
         // ---- enqueue frontiers: anything pending at this or a later level?
-        __shared__ int s_pend;
-        if (pulling) {
-            if (threadIdx.x == 0) s_pend = 1;
-        } else if (threadIdx.x == 0) {
-            bool pend = false;
+        int any_pend = 1;
+        if (!pulling) {   // the slot flags of levels l..max(l, amax), one per thread (R <= 256 slots)
             const int top = l > amax ? l : amax;
-            for (int L = l; L <= top; ++L) pend |= __ldcg(&ctl->slot_flag[L % R]) != 0u;
-            s_pend = pend;
+            const int L = l + (int)threadIdx.x;
+            const bool pend = L <= top && __ldcg(&ctl->slot_flag[L < R ? L : L % R]) != 0u;
+            any_pend = __syncthreads_or(pend);
         }
-        __syncthreads();
-        if (!s_pend) {
+        if (!any_pend) {
             if (gtid == 0) { ctl->stop_reason = empty ? KGS_STOP_EMPTY_KEYWORD : KGS_STOP_EXHAUSTED; ctl->levels = l; }
             break;
         }
@@ -1008,6 +1027,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                     const uint32_t b = st_nm(sv);
                     if (!b) return false;
                     if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
+                    if (l > 0) my_hits += __popc(b);   // new (node, keyword) pairs of level l - 1's expansion
                     const uint32_t old = sv & 0xFFu;
                     const uint32_t nw = old | b;
                     w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
@@ -1078,9 +1098,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             // visit_arc as the push, so the hits, the recorded Thm. V.4 arcs and the lightest-path rows
             // are the same; no node is re-queued (ln 19): a pulling search has no work list (a level
             // without hits asks pull_waiting whether the list would still be non-empty).
-            const unsigned hits0 = my_hits;
-            pull_expand(c, l, S, sh, my_hits, my_dag, my_arcs);
-            cta_add((unsigned long long)(my_hits - hits0), &ctl->pull_marks[l & 1]);
+            const unsigned dag0 = my_dag;   // hitting arcs of this level: some (node, keyword) was marked
+            pull_expand(c, l, S, sh, my_dag, my_arcs);
+            cta_add((unsigned long long)(my_dag - dag0), &ctl->pull_marks[l & 1]);
             publish_flags(ctl);
             G.sync();
             stamp(G, qo, TS_EXPAND);
@@ -1112,7 +1132,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             return nd.hm != 0;
         };
         auto visit = [&](const FwdNode &nd, int32_t x, uint32_t sx) {
-            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_hits, my_dag);
+            visit_arc(c, l, nd.v, nd.hm, nd.zb, x, sx, my_dag);
         };
         expand_big<FwdNode>(G, w.qbig, c1, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
@@ -1157,19 +1177,25 @@ __device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
     const DevWork &w = c.w;
     const uint32_t nt = __ldcg(&ctl->n_touched);
     __shared__ unsigned long long s_rec[2];
-    if (threadIdx.x == 0) {
-        unsigned long long tot = 0, over = 0;
+    if (threadIdx.x == 0) { s_rec[0] = 0ull; s_rec[1] = 0ull; }
+    __syncthreads();
+    {   // the append regions' counts, one per thread (not 128 serial loads by one thread)
         const int ns = rec_stripes(G);
-        for (int r = 0; r < ns; ++r) {
-            const int64_t k = (int64_t)__ldcg(&ctl->rec_cnt[r * kRecStride]);
-            tot += (unsigned long long)k;
-            over |= k > w.pcap / ns;
+        const int64_t k = threadIdx.x < (unsigned)ns ? (int64_t)__ldcg(&ctl->rec_cnt[threadIdx.x * kRecStride]) : 0;
+        const unsigned long long tot = __reduce_add_sync(0xffffffffu, (unsigned)k);   // < 2^32 per warp (pcap)
+        const unsigned over = __any_sync(0xffffffffu, k > w.pcap / ns);
+        if ((threadIdx.x & 31) == 0) {
+            if (tot) atomicAdd(&s_rec[0], tot);
+            if (over) s_rec[1] = 1ull;
         }
-        s_rec[0] = tot; s_rec[1] = over;
     }
     __syncthreads();
     if (s_rec[1]) {   // a region overflowed: forget the compact ids, use the pre-pass
-        for (int64_t j = G.gtid; j < nt; j += G.gsz) w.pd_cid[__ldcg(w.pd_touched + j)] = -1;
+        for (int64_t j = G.gtid; j < nt; j += G.gsz) {   // the pre-pass reads both for its (touched) nodes
+            const int32_t v = __ldcg(w.pd_touched + j);
+            w.pd_cid[v] = -1;
+            w.pd_state[v] = 0u;
+        }
         G.sync();
         if (G.gtid == 0) { ctl->n_parcs = 0; ctl->n_cid = 0; ctl->rec_overflow = 1; }
         G.sync();
@@ -2241,7 +2267,9 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->td_arcs = ctl->td_arcs;
             qo->t_end = globaltimer_ns();
             w.gstate[1] = done + 1;
-            w.gstate[2] = a.td_only ? 0u : 1u;   // after a top-down-only query the next one resets densely
+            // after a top-down-only query the next one resets densely; bit 1: a recorded-DAG query left its
+            // compact ids (search() "Predecessor-list state")
+            w.gstate[2] = a.td_only ? 0u : (1u | (ctl->rec_used || a.dag_record ? 2u : 0u));
             w.gstate[3] = (uint32_t)a.R;
         }
         G.sync();
