@@ -178,12 +178,10 @@ __device__ __forceinline__ uint32_t *cta_flags() {
 }
 
 // Set v's bit in bitmap `bits` and mark CTA flag `fi`.  The bit is set with a reduction (no return
-// value).  check: read the word first and skip the reduction when the bit is set (pushes that repeat:
-// Alg. 2 ln 19 re-queues v once per gated neighbour); the others are already unique per node.
-__device__ __forceinline__ void set_bit(uint32_t *bits, int fi, int32_t v, bool check) {
+// value, nothing to wait for).
+__device__ __forceinline__ void set_bit(uint32_t *bits, int fi, int32_t v) {
     uint32_t *word = bits + (v >> 5);
     const uint32_t bit = 1u << (v & 31);
-    if (check && (__ldcg(word) & bit)) return;
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(word), "r"(bit) : "memory");
     atomicOr(cta_flags() + fi, 1u);   // the CTA's "slot non-empty" flag (shared; every writer sets the same bit)
 }
@@ -217,9 +215,9 @@ struct Ctx {        // everything a group needs while answering one query
 __device__ __forceinline__ int32_t in_id(const EngineArgs &a, int32_t v) { return a.g.orig ? __ldg(a.g.orig + v) : v; }
 
 // Schedule node v for the joint frontier of level L (FIdentifier[v] <- 1).
-__device__ __forceinline__ void push(const Ctx &c, int32_t v, int L, bool check = false) {
+__device__ __forceinline__ void push(const Ctx &c, int32_t v, int L) {
     const int s = L < c.a.R ? L : L % c.a.R;   // L < R except for new hits past level R - 1 (no division)
-    set_bit(c.w.fbits + (int64_t)s * c.a.W, s, v, check);
+    set_bit(c.w.fbits + (int64_t)s * c.a.W, s, v);
 }
 
 constexpr int kWpt = 8;   // bitmap words per thread per compaction step (two 16-byte loads)
@@ -380,7 +378,12 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
             if (bits & (1u << i)) row[i] = lv;            // ln 21: m_xi <- l+1
         push(c, x, l + 1);                                // ln 22: FIdentifier[x] <- 1
     } else {
-        push(c, v, (int)gate - 1, true);                  // ln 19: v must retry when x opens
+        // ln 19: v must retry when x opens.  A node re-queues once per gated neighbour, often many times
+        // at once (the arcs of one node are spread over lanes and warps): the lanes of a warp with the same
+        // (node, level) push once, and the push is a fire-and-forget reduction (no read of the word first)
+        const uint64_t key = ((uint64_t)(uint32_t)v << 8) | (uint64_t)(gate - 1);
+        const unsigned peers = __match_any_sync(__activemask(), key);
+        if ((int)lane_id() == __ffs(peers) - 1) push(c, v, (int)gate - 1);
     }
 }
 
@@ -601,7 +604,7 @@ __device__ __forceinline__ void pd_visit(const Ctx &c, bool exact_block, const P
     const uint32_t nb = pb & ~zbu;        // sources (m = 0) have no predecessors
     if (nb) {
         const uint32_t old = atomicOr(c.w.pd_state + u, nb << 8);
-        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u, false);
+        if (((old >> 8) & 0xFFu) == 0) set_bit(nbits, nflag, u);
     }
 }
 
@@ -1886,7 +1889,7 @@ __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
         uint32_t zb = 0;
         for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
         const uint32_t bits = c.qq.full & ~zb;
-        if (bits) { atomicOr(c.w.pd_state + cn, bits << 8); set_bit(c.w.pd_bits, kFlagPd, cn, false); }
+        if (bits) { atomicOr(c.w.pd_state + cn, bits << 8); set_bit(c.w.pd_bits, kFlagPd, cn); }
     }
     publish_flags(c.ctl);
     G.sync();
