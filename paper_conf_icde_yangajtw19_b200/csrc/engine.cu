@@ -725,7 +725,26 @@ __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
     const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
     const int64_t chunk = (ncid + G.gcount - 1) / G.gcount;
     const int64_t lo = (int64_t)G.grank * chunk, hi = lo + chunk < ncid ? lo + chunk : ncid;
-    int run = 0;
+    // pass 1: the CTA's total over its chunk of compact ids
+    int part = 0;
+    for (int64_t j = lo + threadIdx.x; j < hi; j += blockDim.x) part += __ldcg(c.w.pcnt + j);
+    {
+        int tot;
+        block_excl_scan(part, &tot, sh);
+        if (threadIdx.x == 0) c.w.scan_tmp[G.grank] = tot;
+    }
+    G.sync();
+    // pass 2: every CTA sums the totals before it itself (no serial scan on one CTA, no extra barrier),
+    // then scans its chunk again writing the offsets
+    int off = 0;
+    {
+        int p = 0;
+        for (int b = threadIdx.x; b < G.grank; b += blockDim.x) p += __ldcg(c.w.scan_tmp + b);
+        int tot;
+        block_excl_scan(p, &tot, sh);
+        off = tot;
+    }
+    int run = off;
     for (int64_t t0 = lo; t0 < lo + chunk; t0 += blockDim.x) {
         const int64_t j = t0 + threadIdx.x;
         const int v = j < hi ? __ldcg(c.w.pcnt + j) : 0;
@@ -734,23 +753,7 @@ __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
         if (j < hi) c.w.pred_ptr[j] = run + ex;
         run += tot;
     }
-    if (threadIdx.x == 0) c.w.scan_tmp[G.grank] = run;
-    G.sync();
-    if (G.grank == 0) {   // exclusive scan of the per-CTA sums
-        int carry = 0;
-        for (int b0 = 0; b0 < G.gcount; b0 += blockDim.x) {
-            const int b = b0 + threadIdx.x;
-            const int v = b < G.gcount ? __ldcg(c.w.scan_tmp + b) : 0;
-            int tot;
-            const int ex = block_excl_scan(v, &tot, sh);
-            if (b < G.gcount) c.w.scan_tmp[b] = carry + ex;
-            carry += tot;
-        }
-        if (threadIdx.x == 0) c.w.pred_ptr[ncid] = carry;
-    }
-    G.sync();
-    const int off = __ldcg(c.w.scan_tmp + G.grank);
-    for (int64_t j = lo + threadIdx.x; j < hi; j += blockDim.x) c.w.pred_ptr[j] += off;
+    if (G.grank == G.gcount - 1 && threadIdx.x == 0) c.w.pred_ptr[ncid] = run;
     G.sync();
     auto scatter = [&](int64_t ai) {
         const int64_t pos = (int64_t)__ldcg(c.w.pred_ptr + c.w.pa_x[ai]) + c.w.pa_slot[ai];
