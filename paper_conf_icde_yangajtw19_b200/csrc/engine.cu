@@ -265,11 +265,18 @@ __device__ __forceinline__ bool compact_deferred(const Grp &G, const int32_t *qd
 template <class OnNode, class OnAux>
 __device__ __forceinline__ void compact(const Grp &G, uint32_t *bits, int64_t W, const uint8_t *cls, int32_t *ql,
                                         uint32_t *nl, int32_t *qb, uint32_t *nb, int32_t *aux, uint32_t *naux,
-                                        int32_t *qdef, uint32_t *ndef, long long *sh, OnNode on_node, OnAux on_aux) {
+                                        int32_t *qdef, uint32_t *ndef, long long *sh, uint32_t *tile_ctr, OnNode on_node,
+                                        OnAux on_aux) {
+    // tiles of blockDim * kWpt words taken from a counter (zero on entry): a CTA whose tiles hold many set
+    // bits (the hub regions of the degree order) does not hold the whole group at the next barrier
     const int64_t step = (int64_t)blockDim.x * kWpt;
-    const int64_t cw = ((W + G.gcount - 1) / G.gcount + kWpt - 1) / kWpt * kWpt;
-    const int64_t w0 = (int64_t)G.grank * cw, w1 = w0 + cw < W ? w0 + cw : W;
-    for (int64_t base = w0; base < w1; base += step) {
+    for (;;) {
+        __syncthreads();
+        if (threadIdx.x == 0) sh[37] = (long long)atomicAdd(tile_ctr, 1u);
+        __syncthreads();
+        const int64_t base = sh[37] * step;
+        if (base >= W) break;
+        const int64_t w1 = base + step < W ? base + step : W;
         const int64_t wi = base + (int64_t)threadIdx.x * kWpt;
         uint32_t word[kWpt];
         if (wi + kWpt <= w1) {
@@ -671,7 +678,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int slot = r & 1;
         if (!__ldcg(&ctl->pd_flag[slot])) break;
         uint32_t *qn = ctl->pd_qn[slot];
-        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; }
+        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u; }
         auto pd_node = [&](int32_t u) {
             const uint32_t s = __ldcg(c.w.pd_state + u);
             const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
@@ -682,7 +689,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         auto pd_aux = [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; };
         if (G.gtid == 0) ctl->pd_ndef[slot ^ 1] = 0u;
         compact(G, c.w.pd_bits + (int64_t)slot * W, W, c.a.g.cls_in, c.w.pd_qlight, &qn[0], c.w.pd_qbig, &qn[1],
-                c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, pd_node, pd_aux);
+                c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, &ctl->pd_ctile[slot], pd_node, pd_aux);
         G.sync();
         if (compact_deferred(G, c.w.qdef, __ldcg(&ctl->pd_ndef[slot]), c.w.pd_qlight, c.a.g.cls_in, c.w.pd_qbig,
                              &qn[1], c.w.pd_touched, &ctl->n_cid, pd_node, pd_aux))
@@ -1021,6 +1028,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         uint32_t *qn = ctl->qn[l & 1];
         if (gtid == 0) {
             ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; ctl->ndef[(l + 1) & 1] = 0u;
+            ctl->ctile[(l + 1) & 1] = 0u;
             ctl->mf[(l + 1) & 1] = 0ull; ctl->pull_nbig[(l + 1) & 1] = 0u;
         }
         // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
@@ -1055,7 +1063,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             if (a.dag_record) { w.pd_touched[pos] = v; w.pd_cid[v] = (int32_t)pos; }
         };
         compact(G, w.fbits + (int64_t)s * W, W, a.g.cls, w.qlight, &qn[0], w.qbig, &qn[1], w.touched,
-                &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, merge_node, merge_aux);
+                &ctl->n_touched, w.qdef, &ctl->ndef[l & 1], sh, &ctl->ctile[l & 1], merge_node, merge_aux);
         if (count_lvl && !pulling) { cta_add(my_mf, &ctl->mf[l & 1]); my_mf = 0; }
         G.sync();
         if (compact_deferred(G, w.qdef, __ldcg(&ctl->ndef[l & 1]), w.qlight, a.g.cls, w.qbig, &qn[1], w.touched,
@@ -1884,7 +1892,9 @@ __device__ void containment_select(const Ctx &c, long long *sh, char *dsmem, uin
 // keyword it does not contain itself (those have m = 0 and no predecessors).
 __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
     const Grp &G = c.G;
-    if (G.gtid == 0) { c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; }   // round 0 of this call
+    if (G.gtid == 0) {   // round 0 of this call
+        c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; c.ctl->pd_ctile[0] = 0u;
+    }
     for (int64_t j = G.gtid; j < cnt; j += G.gsz) {
         const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;
         const int32_t cn = __ldcg(c.w.centrals + idx);

@@ -85,6 +85,8 @@ struct Ctl {
     uint32_t n_cut;                // candidates stopped by the exact key cut-off (pruning round 2)
     uint32_t work_huge2;           // ... beyond the per-CTA large arenas too (tier 4, one CTA of the group)
     uint32_t n_tier4;              // Central Graphs this query extracted in the tier-4 arena (all passes)
+    uint32_t ctile[2];             // [level parity] compaction: next bitmap tile to take
+    uint32_t pd_ctile[2];          // [round parity] the same for the predecessor pre-pass
 };
 
 // Per-query summary written by the engine (device), read back by the host.
