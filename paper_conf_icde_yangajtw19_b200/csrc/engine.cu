@@ -499,16 +499,24 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 // Batch bi holds the queue entries bi, bi + nbatch, bi + 2 nbatch, ...: the queue is in node-id order,
 // and in the degree order (relabel.cu) neighbouring ids have similar degrees, so strided batches mix
 // degrees and cost about the same.  ql = nullptr sweeps the nodes 0..c0-1 in contiguous batches (pull).
+// bctr (zero on entry, or null for the static assignment): warps take their batches from this counter, so a
+// warp that drew heavy batches does not hold the group at the next barrier.
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
                                              const int32_t *idx, const uint32_t *st, Prep prep, Visit visit,
-                                             unsigned long long &arcs) {
+                                             unsigned long long &arcs, uint32_t *bctr = nullptr) {
     const uint32_t warps = (uint32_t)(G.gsz >> 5);
     uint32_t B = (c0 + 2 * warps - 1) / (2 * warps);
     B = B < 1 ? 1u : (B > 32 ? 32u : B);
     const uint32_t nbatch = (c0 + B - 1) / B;
     const unsigned lane = lane_id();
-    for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi += warps) {
+    auto next_batch = [&](uint32_t cur) -> uint32_t {
+        if (!bctr) return cur + warps;
+        uint32_t b = 0;
+        if (lane == 0) b = atomicAdd(bctr, 1u) + warps;   // the first `warps` batches are taken statically
+        return __shfl_sync(0xffffffffu, b, 0);
+    };
+    for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi = next_batch(bi)) {
         const uint32_t i = ql ? bi + lane * nbatch : bi * B + lane;   // no queue: nodes 0..c0-1, contiguous
         NodeT nd{};
         int64_t start = 0;
@@ -678,7 +686,8 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int slot = r & 1;
         if (!__ldcg(&ctl->pd_flag[slot])) break;
         uint32_t *qn = ctl->pd_qn[slot];
-        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u; }
+        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u;
+                           ctl->pd_xbatch[slot ^ 1] = 0u; }
         auto pd_node = [&](int32_t u) {
             const uint32_t s = __ldcg(c.w.pd_state + u);
             const uint32_t nx = (s >> 8) & 0xFFu, dn = (s >> 16) & 0xFFu;
@@ -705,7 +714,8 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (c0 <= (uint32_t)c.a.tile_light)   // small frontier: tiles over the whole group
             expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         else
-            expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs);
+            expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs,
+                                 &ctl->pd_xbatch[slot]);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
@@ -1028,7 +1038,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         uint32_t *qn = ctl->qn[l & 1];
         if (gtid == 0) {
             ctl->qn[(l + 1) & 1][0] = 0u; ctl->qn[(l + 1) & 1][1] = 0u; ctl->ndef[(l + 1) & 1] = 0u;
-            ctl->ctile[(l + 1) & 1] = 0u;
+            ctl->ctile[(l + 1) & 1] = 0u; ctl->xbatch[(l + 1) & 1] = 0u;
             ctl->mf[(l + 1) & 1] = 0ull; ctl->pull_nbig[(l + 1) & 1] = 0u;
         }
         // compact the level's bitmap; merge new hits into hm and identify central nodes (L262-266)
@@ -1152,7 +1162,8 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (c0 <= (uint32_t)a.tile_light)   // small frontier: tiles over the whole group
             expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         else
-            expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs);
+            expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs,
+                                  &ctl->xbatch[l & 1]);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_EXPAND);
@@ -1894,6 +1905,7 @@ __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
     const Grp &G = c.G;
     if (G.gtid == 0) {   // round 0 of this call
         c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; c.ctl->pd_ctile[0] = 0u;
+        c.ctl->pd_xbatch[0] = 0u;
     }
     for (int64_t j = G.gtid; j < cnt; j += G.gsz) {
         const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;

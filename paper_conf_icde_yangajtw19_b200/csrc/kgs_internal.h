@@ -87,6 +87,8 @@ struct Ctl {
     uint32_t n_tier4;              // Central Graphs this query extracted in the tier-4 arena (all passes)
     uint32_t ctile[2];             // [level parity] compaction: next bitmap tile to take
     uint32_t pd_ctile[2];          // [round parity] the same for the predecessor pre-pass
+    uint32_t xbatch[2];            // [level parity] expansion: next warp batch beyond the first round
+    uint32_t pd_xbatch[2];         // [round parity] the same for the pre-pass
 };
 
 // Per-query summary written by the engine (device), read back by the host.
