@@ -500,7 +500,10 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
 // and in the degree order (relabel.cu) neighbouring ids have similar degrees, so strided batches mix
 // degrees and cost about the same.  ql = nullptr sweeps the nodes 0..c0-1 in contiguous batches (pull).
 // bctr (zero on entry, or null for the static assignment): warps take their batches from this counter, so a
-// warp that drew heavy batches does not hold the group at the next barrier.
+// warp that drew heavy batches does not hold the group at the next barrier.  Used by query groups of at
+// most kDynBatchCtas CTAs (batch mode); with the whole grid on one query (latency mode) the thousands of
+// warps contending for one counter cost more than the imbalance (p50 0.252 -> 0.278 ms).
+constexpr int kDynBatchCtas = 64;
 template <class NodeT, class Prep, class Visit>
 __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, uint32_t c0, const int64_t *ptr,
                                              const int32_t *idx, const uint32_t *st, Prep prep, Visit visit,
@@ -715,7 +718,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         else
             expand_light<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, prep, visit, my_arcs,
-                                 &ctl->pd_xbatch[slot]);
+                                 G.gcount <= kDynBatchCtas ? &ctl->pd_xbatch[slot] : nullptr);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
@@ -1163,7 +1166,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             expand_big<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, S, sh, prep, visit, my_arcs);
         else
             expand_light<FwdNode>(G, w.qlight, c0, a.g.row_ptr, a.g.col_idx, w.st, prep, visit, my_arcs,
-                                  &ctl->xbatch[l & 1]);
+                                  G.gcount <= kDynBatchCtas ? &ctl->xbatch[l & 1] : nullptr);
         publish_flags(ctl);
         G.sync();
         stamp(G, qo, TS_EXPAND);
@@ -1581,6 +1584,54 @@ __device__ void team_sort(const Team &T, unsigned long long *buf, int len) {
         }
 }
 
+// Warp bitonic sort in registers (E elements per lane, element i = e * 32 + lane): the tier-1 emit sorts
+// at most 256 nodes or arcs, and sorting them through memory with a warp barrier per step cost a
+// single-query launch ~20 us.
+template <int E>
+__device__ __forceinline__ void warp_sort_regs(unsigned long long *buf, int len) {
+    const int lane = (int)(threadIdx.x & 31u);
+    unsigned long long x[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) x[e] = e * 32 + lane < len ? buf[e * 32 + lane] : ~0ull;
+#pragma unroll
+    for (int k = 2; k <= 32 * E; k <<= 1)
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            if (j >= 32) {
+                const int d = j >> 5;
+#pragma unroll
+                for (int e = 0; e < E; ++e)
+                    if ((e & d) == 0) {
+                        const bool up = ((e * 32 + lane) & k) == 0;
+                        const unsigned long long a = x[e], b = x[e | d];
+                        const unsigned long long lo = a < b ? a : b, hi = a < b ? b : a;
+                        x[e] = up ? lo : hi;
+                        x[e | d] = up ? hi : lo;
+                    }
+            } else {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    const unsigned long long y = __shfl_xor_sync(0xffffffffu, x[e], j);
+                    const int i = e * 32 + lane;
+                    const bool keep_min = ((i & j) == 0) == ((i & k) == 0);
+                    x[e] = keep_min ? (x[e] < y ? x[e] : y) : (x[e] < y ? y : x[e]);
+                }
+            }
+        }
+    __syncwarp();
+#pragma unroll
+    for (int e = 0; e < E; ++e)
+        if (e * 32 + lane < len) buf[e * 32 + lane] = x[e];
+    __syncwarp();
+}
+__device__ void team_sort(const WarpTeam &T, unsigned long long *buf, int len) {
+    if (len <= 32) warp_sort_regs<1>(buf, len);
+    else if (len <= 64) warp_sort_regs<2>(buf, len);
+    else if (len <= 128) warp_sort_regs<4>(buf, len);
+    else if (len <= 256) warp_sort_regs<8>(buf, len);
+    else team_sort<WarpTeam>(T, buf, len);
+}
+
 // Reserve cnt entries of an answer arena without ever moving its counter past cap: a reservation that
 // does not fit fails (-1) and leaves the counter as it was, so later (smaller) answers still fit and only
 // the overflowing query is marked (KGS_STOP_CAPACITY).
@@ -1686,6 +1737,31 @@ __device__ __forceinline__ bool prefix_match(uint64_t hi, uint32_t lo, uint64_t 
 // Ends with a group barrier.
 __device__ void rank_list(const Ctx &c, char *dsmem, const int32_t *list, uint32_t cnt, uint32_t kk) {
     const Grp &G = c.G;
+    if (cnt <= 32) {   // one warp sorts in registers: (key bits, input id) with the candidate index riding along
+        if (G.grank == 0 && threadIdx.x < 32) {
+            const int lane = (int)threadIdx.x;
+            uint64_t a = ~0ull, b = ~0ull;   // a = key bits, b = input id << 32 | candidate index
+            if (lane < (int)cnt) {
+                const int32_t idx = list ? __ldcg(list + lane) : lane;
+                uint32_t lo;
+                comp_key(c, (uint32_t)idx, a, lo);
+                b = ((uint64_t)lo << 32) | (uint32_t)idx;
+            }
+#pragma unroll
+            for (int k = 2; k <= 32; k <<= 1)
+#pragma unroll
+                for (int j = k >> 1; j > 0; j >>= 1) {
+                    const uint64_t oa = __shfl_xor_sync(0xffffffffu, a, j), ob = __shfl_xor_sync(0xffffffffu, b, j);
+                    const bool mine_less = a < oa || (a == oa && b < ob);
+                    const bool keep_min = ((lane & j) == 0) == ((lane & k) == 0);
+                    if (keep_min != mine_less) { a = oa; b = ob; }
+                }
+            if (lane < (int)kk) c.w.sel[lane] = (int32_t)(uint32_t)b;
+            if (lane == 0) c.ctl->sel_count = kk;
+        }
+        G.sync();
+        return;
+    }
     if (G.grank == 0) {
         unsigned long long *khi = reinterpret_cast<unsigned long long *>(dsmem);
         uint32_t *klo = reinterpret_cast<uint32_t *>(khi + KGS_MAX_K);
