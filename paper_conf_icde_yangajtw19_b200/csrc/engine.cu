@@ -21,7 +21,7 @@
 //
 // Data layout:
 //   st[v]   uint32 status word: byte 0 = hit mask hm (bit i <=> M[v][i] finite, snapshot at the start of
-//           the level), byte 1 = gate (0 if v contains a query keyword, else a_v), byte 2 = nm, the bits
+//           the level), byte 1 = K flag (v contains a query keyword: gate 0, else the gate is a_v), byte 2 = nm, the bits
 //           newly hit during the current level (atomicOr), byte 3 = a_v.  One 4-byte load per inspected arc
 //           gives the target's mask and gate, and the hit that follows is an atomic on the same word
 //           (an L2 hit); a frontier node's merge and activation test read one word, not three arrays.
@@ -131,12 +131,13 @@ __device__ __forceinline__ uint64_t ldrow(const uint8_t *M, int32_t v) {
     return __ldcg(reinterpret_cast<const unsigned long long *>(M) + v);
 }
 
-// fields of the status word st[v] (hm | gate << 8 | nm << 16 | a << 24)
-__device__ __forceinline__ uint32_t st_gate(uint32_t s) { return (s >> 8) & 0xFFu; }
+// fields of the status word st[v] (hm | K << 8 | nm << 16 | a << 24; K = 1: v holds a query keyword)
+// gate (L210): 0 for a keyword node, else a_v
+__device__ __forceinline__ uint32_t st_gate(uint32_t s) { return (s & 0x100u) ? 0u : (s >> 24); }
 __device__ __forceinline__ uint32_t st_nm(uint32_t s) { return (s >> 16) & 0xFFu; }
 __device__ __forceinline__ uint32_t st_act(uint32_t s) { return s >> 24; }
-// the status word of a node nobody has hit yet: gate = a (not a keyword node), a
-__device__ __forceinline__ uint32_t st_fresh(uint32_t a) { return (a << 8) | (a << 24); }
+// the status word of a node nobody has hit yet: not a keyword node, a
+__device__ __forceinline__ uint32_t st_fresh(uint32_t a) { return a << 24; }
 
 struct Q {   // the query a group is answering
     int32_t qi;
@@ -420,7 +421,7 @@ struct FwdNode {
     uint32_t zb;     // keywords for which v is a source (m = 0), recorded with its arcs
 };
 
-struct PullNode {   // a node x pulling at level l: its status word (hit mask | gate << 8)
+struct PullNode {   // a node x pulling at level l: its status word
     int32_t x;
     uint32_t sx;
 };
@@ -972,7 +973,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         } else {
             for (int64_t j = gtid; j < pt; j += gsz) {
                 const int32_t v = w.touched[j];
-                w.st[v] = st_fresh(a.act[v]);
+                w.st[v] = st_fresh(st_act(__ldcg(w.st + v)));   // a_v is byte 3 of the word itself
             }
         }
         for (int s = 0; s < R; ++s)   // level slots still pending when the previous query stopped
@@ -1002,9 +1003,8 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             const int32_t v = a.g.kw_nodes[kb[i] + (j - ko[i])];
             w.M[(int64_t)v * 8 + i] = 0;
             if (a.prune == 2) w.mw[(int64_t)v * 8 + i] = 0u;              // the path {v}: w_v added at merge
-            // keyword node: no gate (L210); hit in B_i at level 0 (new-hit bit i)
-            atomicAnd(w.st + v, ~0xFF00u);
-            atomicOr(w.st + v, (1u << i) << 16);
+            // keyword node (no gate, L210) and hit in B_i at level 0 (new-hit bit i): one atomic
+            atomicOr(w.st + v, 0x100u | ((1u << i) << 16));
             push(c, v, 0);
         }
     }
@@ -1632,10 +1632,16 @@ __device__ void team_sort(const WarpTeam &T, unsigned long long *buf, int len) {
     else team_sort<WarpTeam>(T, buf, len);
 }
 
-// Reserve cnt entries of an answer arena without ever moving its counter past cap: a reservation that
-// does not fit fails (-1) and leaves the counter as it was, so later (smaller) answers still fit and only
-// the overflowing query is marked (KGS_STOP_CAPACITY).
+// Reserve cnt entries of an answer arena; -1 if they do not fit, leaving the counter as it was, so later
+// (smaller) answers still fit and only the overflowing query is marked (KGS_STOP_CAPACITY).  The common
+// case is one atomicAdd (a CAS loop serialised the k concurrent winners of a query on one address: ~15 us
+// of a single-query launch); a reservation that lands past cap is undone and retried exactly with CAS (a
+// concurrent reservation can then see the counter briefly high and fail too — only when the arena is
+// within one answer of full).
 __device__ __forceinline__ long long arena_reserve(unsigned long long *ctr, unsigned long long cnt, long long cap) {
+    const unsigned long long old = atomicAdd(ctr, cnt);
+    if (old + cnt <= (unsigned long long)cap) return (long long)old;
+    atomicAdd(ctr, (unsigned long long)(-(long long)cnt));   // undo
     unsigned long long cur = atomicAdd(ctr, 0ull);
     for (;;) {
         if (cur + cnt > (unsigned long long)cap) return -1;

@@ -130,7 +130,7 @@ struct DevGraph {
 
 // Per-group query workspace (all sized for n at load time).  One group answers one query at a time.
 struct DevWork {
-    uint32_t *st;       // [n] status word: hm | gate << 8 | nm << 16 | a << 24 (engine.cu "Data layout")
+    uint32_t *st;       // [n] status word: hm | K << 8 | nm << 16 | a << 24 (engine.cu "Data layout")
     uint8_t *M;         // [n*8] hitting levels, node-major, valid where the hm bit is set
     uint32_t *fbits;    // [R][W] frontier bitmaps, slot = level % R (FIdentifier)
     int32_t *qlight;    // [n] compacted frontier of the current level (big nodes replaced by -1)

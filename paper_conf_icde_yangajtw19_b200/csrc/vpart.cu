@@ -198,11 +198,12 @@ __global__ void k_vp_biglist(const int64_t *__restrict__ in_ptr, int64_t lo, int
         if (in_ptr[x + 1] - in_ptr[x] > kVpBig) big[atomicAdd(nbig, 1)] = (int32_t)x;
 }
 
-// engine status word of the replicated final state: hm | gate << 8 | (nm = 0) | a << 24 (DevWork::st)
+// engine status word of the replicated final state: hm | K << 8 | (nm = 0) | a << 24 (DevWork::st); the
+// engine's gate is 0 when K is set, else a: K = (gate == 0) gives the same gate for every node
 __global__ void k_vp_pack_st(const uint8_t *__restrict__ hm, const uint8_t *__restrict__ gate,
                              const uint8_t *__restrict__ act, int64_t n, uint32_t *__restrict__ st) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        st[v] = (uint32_t)hm[v] | ((uint32_t)gate[v] << 8) | ((uint32_t)act[v] << 24);
+        st[v] = (uint32_t)hm[v] | (gate[v] == 0 ? 0x100u : 0u) | ((uint32_t)act[v] << 24);
 }
 
 // sparse exchange: the gathered (id << 8 | mask) lists of every rank into the replicated hit masks
