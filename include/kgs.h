@@ -182,6 +182,7 @@ typedef struct {
     int32_t pull_level;    /* first level expanded by pull (kgs_params.direction), -1: push throughout */
     int32_t n_cut;         /* candidates whose extraction stopped at the exact key cut-off (prune round 2) */
     int32_t n_tier4;       /* Central Graphs extracted in the per-group tier-4 arena (beyond the per-CTA arenas) */
+    int64_t td_arcs_big;   /* td_arcs of predecessor-list nodes with more than 2048 in-arcs (the hubs) */
 } kgs_stats;
 
 /* Load a graph onto params-independent device state.  Validates the CSR and the index

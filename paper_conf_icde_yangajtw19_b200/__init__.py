@@ -64,7 +64,7 @@ class kgs_stats(ctypes.Structure):
                 ("td_pred_arcs", ctypes.c_int64), ("ms_search", ctypes.c_float), ("ms_topdown", ctypes.c_float),
                 ("ms_total", ctypes.c_float), ("ms_launch", ctypes.c_float), ("group", ctypes.c_int32),
                 ("n_evaluated", ctypes.c_int32), ("dag_arcs", ctypes.c_int64), ("pull_level", ctypes.c_int32),
-                ("n_cut", ctypes.c_int32), ("n_tier4", ctypes.c_int32)]
+                ("n_cut", ctypes.c_int32), ("n_tier4", ctypes.c_int32), ("td_arcs_big", ctypes.c_int64)]
 
 
 class kgs_vp_buffers(ctypes.Structure):

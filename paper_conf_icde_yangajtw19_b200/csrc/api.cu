@@ -674,6 +674,7 @@ kgs_status fetch(kgs_graph *g, cudaStream_t s, kgs_result **results) {
         st.hits = (int64_t)o.hits;
         st.dag_arcs = (int64_t)o.dag_arcs;
         st.td_arcs = (int64_t)o.td_arcs;
+        st.td_arcs_big = (int64_t)o.td_arcs_big;
         st.td_pred_arcs = o.n_parcs;
         st.n_evaluated = (int32_t)o.n_eval;
         st.n_tier4 = (int32_t)o.n_tier4;

@@ -684,7 +684,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const int64_t W = c.a.W;
     // seeds (the candidates to extract, for every keyword they do not contain) were set by seed_pd: round 0
     // starts from them.  A second call continues the same DAG: done bits persist, the CSR is rebuilt.
-    unsigned long long my_arcs = 0;
+    unsigned long long my_arcs = 0, my_arcs_big = 0;   // in-arcs of light / big (> kBigDeg in-arcs) nodes
     int r = 0;
     for (;; ++r) {
         const int slot = r & 1;
@@ -714,7 +714,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int nflag = kFlagPd + (slot ^ 1);
         auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
         auto visit = [&](const PdNode &nd, int32_t u, uint32_t su) { pd_visit(c, exact_block, nd, u, su, nbits, nflag); };
-        expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
+        expand_big<PdNode>(G, c.w.pd_qbig, c1, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs_big);
         if (c0 <= (uint32_t)c.a.tile_light)   // small frontier: tiles over the whole group
             expand_big<PdNode>(G, c.w.pd_qlight, c0, c.a.g.in_ptr, c.a.g.in_idx, c.w.st, S, sh, prep, visit, my_arcs);
         else
@@ -724,7 +724,8 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         G.sync();
         stamp(G, qo, TS_PD_EXPAND);
     }
-    if (my_arcs) atomicAdd(&ctl->td_arcs, my_arcs);
+    if (my_arcs + my_arcs_big) atomicAdd(&ctl->td_arcs, my_arcs + my_arcs_big);
+    if (my_arcs_big) atomicAdd(&ctl->td_arcs_big, my_arcs_big);
     if (G.grank == 0) {   // the append regions' counts, one per thread, then a warp sum (not 128 serial loads)
         __shared__ uint32_t s_np;
         if (threadIdx.x == 0) s_np = 0;
@@ -2375,6 +2376,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
             qo->hits = ctl->hits;
             qo->dag_arcs = ctl->dag_arcs;
             qo->td_arcs = ctl->td_arcs;
+            qo->td_arcs_big = ctl->td_arcs_big;
             qo->t_end = globaltimer_ns();
             w.gstate[1] = done + 1;
             // after a top-down-only query the next one resets densely; bit 1: a recorded-DAG query left its

@@ -62,6 +62,7 @@ struct Ctl {
     uint32_t n_cid;                // nodes of the union of closures that have predecessor lists
     uint32_t n_parcs;              // predecessor arcs found
     unsigned long long td_arcs;    // in-arcs inspected by the pre-pass
+    unsigned long long td_arcs_big;   // ... of them, in-arcs of nodes with more than kBigDeg in-arcs
     int32_t pd_rounds;
     uint32_t n_eval;               // candidates whose exact key was computed (all of C without pruning)
     uint32_t n_elist2;             // second pruning round: candidates whose bound still beats the threshold
@@ -96,7 +97,7 @@ constexpr int kMaxStamps = 48;
 struct QOut {
     int32_t levels, stop_reason, count, fatal;
     uint32_t n_central, n_overflow, n_cid, n_parcs, n_eval, n_tier4;
-    unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs;
+    unsigned long long frontier_total, arcs_scanned, hits, td_arcs, dag_arcs, td_arcs_big;
     unsigned long long t_start, t_search_end, t_end;   // %globaltimer ns
     int32_t group, n_stamp;
     int32_t pull_level, n_cut;     // first pulled level (-1: push throughout); key cut-offs

@@ -35,4 +35,5 @@ for rep in range(2):
           f"arcs {sum(x['arcs_scanned'] for x in st)}, td_arcs {sum(x['td_arcs'] for x in st)}, "
           f"centrals {sum(x['n_centrals'] for x in st)}, dag_arcs {sum(x['dag_arcs'] for x in st)}, "
           f"hits {sum(x['hits'] for x in st)}, frontier {sum(x['frontier_total'] for x in st)}, "
-          f"pred_arcs {sum(x['td_pred_arcs'] for x in st)}", flush=True)
+          f"pred_arcs {sum(x['td_pred_arcs'] for x in st)}, td_arcs_big {sum(x['td_arcs_big'] for x in st)}",
+          flush=True)
