@@ -575,9 +575,19 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
 __device__ __forceinline__ uint32_t pred_test(const Ctx &c, bool exact_block, uint32_t P, uint64_t hx, int gx,
                                               int32_t u, uint32_t su, uint32_t &zbu) {
     const uint32_t hmu = su & 0xFFu;
-    const uint32_t cand = P & hmu;
+    uint32_t cand = P & hmu;
     if (!cand) return 0;
     const int au = (int)st_act(su);
+    // m_xi = 1 + max{a_u, m_ui, g_x} needs a_u <= m_xi - 1: a test on the status word alone, before the
+    // M row of u is loaded (most in-arcs of the pre-pass are not predecessor arcs)
+    {
+        const uint32_t rep = (uint32_t)au * 0x01010101u;   // per byte: m_xi > a_u
+        const uint32_t g0 = __vcmpgtu4((uint32_t)hx, rep), g1 = __vcmpgtu4((uint32_t)(hx >> 32), rep);
+        const uint32_t b0 = ((g0 >> 7) & 1u) | ((g0 >> 14) & 2u) | ((g0 >> 21) & 4u) | ((g0 >> 28) & 8u);
+        const uint32_t b1 = ((g1 >> 7) & 1u) | ((g1 >> 14) & 2u) | ((g1 >> 21) & 4u) | ((g1 >> 28) & 8u);
+        cand &= b0 | (b1 << 4);
+    }
+    if (!cand) return 0;
     const uint64_t Mu = ldrow(c.w.M, u);
     uint32_t pb = 0, zb = 0;
     int maxrow = 0;
