@@ -60,11 +60,14 @@ __device__ __forceinline__ void group_sync(GroupBar *b, int gcount, unsigned &ep
     __syncthreads();
 }
 
+// The CTA's group (uniform over the CTA: it lives in shared memory, so that neither it nor the running
+// query's keywords occupy registers or a stack frame in the whole kernel).
 struct Grp {
     int g, grank, gcount;
-    int64_t gtid, gsz;
+    int64_t gsz;
     GroupBar *bar;
     mutable unsigned episode;   // barriers passed by this CTA in this launch (thread 0)
+    __device__ __forceinline__ int64_t gtid() const { return (int64_t)grank * blockDim.x + threadIdx.x; }
     __device__ __forceinline__ void sync() const { group_sync(bar, gcount, episode); }
 };
 
@@ -148,7 +151,7 @@ struct Q {   // the query a group is answering
 
 // phase timestamp of the current query (group leader only)
 __device__ __forceinline__ void stamp(const Grp &G, QOut *o, int tag) {
-    if (G.gtid == 0) {
+    if (G.gtid() == 0) {
         const int i = o->n_stamp;
         if (i < kMaxStamps) { o->stamp[i] = globaltimer_ns(); o->stamp_tag[i] = tag; o->n_stamp = i + 1; }
     }
@@ -252,7 +255,7 @@ __device__ __forceinline__ bool compact_deferred(const Grp &G, const int32_t *qd
                                                  const uint8_t *cls, int32_t *qb, uint32_t *nb, int32_t *aux,
                                                  uint32_t *naux, OnNode on_node, OnAux on_aux) {
     constexpr int U = 4;   // the queue-position loads of U deferred nodes are in flight together
-    for (int64_t j0 = G.gtid; j0 < nd; j0 += U * G.gsz) {
+    for (int64_t j0 = G.gtid(); j0 < nd; j0 += U * G.gsz) {
         int64_t pos[U];
 #pragma unroll
         for (int k = 0; k < U; ++k) pos[k] = j0 + k * G.gsz < nd ? (int64_t)__ldcg(qdef + j0 + k * G.gsz) : -1;
@@ -463,8 +466,8 @@ __device__ __forceinline__ void expand_big(const Grp &G, const int32_t *qb, uint
         const long long ex = block_excl_scan64(deg, &T, sh);
         S.incl[j] = ex + deg;
         __syncthreads();
-        if (G.gtid == 0) arcs += (unsigned long long)T;
-        for (long long e = G.gtid; e < T; e += kBigUnroll * G.gsz) {
+        if (G.gtid() == 0) arcs += (unsigned long long)T;
+        for (long long e = G.gtid(); e < T; e += kBigUnroll * G.gsz) {
             int own[kBigUnroll];
             int32_t x[kBigUnroll];
 #pragma unroll
@@ -520,7 +523,7 @@ __device__ __forceinline__ void expand_light(const Grp &G, const int32_t *ql, ui
         if (lane == 0) b = atomicAdd(bctr, 1u) + warps;   // the first `warps` batches are taken statically
         return __shfl_sync(0xffffffffu, b, 0);
     };
-    for (uint32_t bi = (uint32_t)(G.gtid >> 5); bi < nbatch; bi = next_batch(bi)) {
+    for (uint32_t bi = (uint32_t)(G.gtid() >> 5); bi < nbatch; bi = next_batch(bi)) {
         const uint32_t i = ql ? bi + lane * nbatch : bi * B + lane;   // no queue: nodes 0..c0-1, contiguous
         NodeT nd{};
         int64_t start = 0;
@@ -675,7 +678,7 @@ __device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cn
     }
     __syncthreads();
     const int64_t T = s_pre[kRecStripes];
-    for (int64_t j = c.G.gtid; j < T; j += c.G.gsz) {
+    for (int64_t j = c.G.gtid(); j < T; j += c.G.gsz) {
         int lo = 0, hi = kRecStripes - 1;   // region r with s_pre[r] <= j < s_pre[r + 1]
         while (lo < hi) {
             const int mid = (lo + hi + 1) >> 1;
@@ -700,7 +703,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         const int slot = r & 1;
         if (!__ldcg(&ctl->pd_flag[slot])) break;
         uint32_t *qn = ctl->pd_qn[slot];
-        if (G.gtid == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u;
+        if (G.gtid() == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u;
                            ctl->pd_xbatch[slot ^ 1] = 0u; }
         auto pd_node = [&](int32_t u) {
             const uint32_t s = __ldcg(c.w.pd_state + u);
@@ -710,7 +713,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             return bits != 0 && __ldcg(c.w.pd_cid + u) < 0;
         };
         auto pd_aux = [&](int32_t u, uint32_t pos) { c.w.pd_cid[u] = (int32_t)pos; };
-        if (G.gtid == 0) ctl->pd_ndef[slot ^ 1] = 0u;
+        if (G.gtid() == 0) ctl->pd_ndef[slot ^ 1] = 0u;
         compact(G, c.w.pd_bits + (int64_t)slot * W, W, c.a.g.cls_in, c.w.pd_qlight, &qn[0], c.w.pd_qbig, &qn[1],
                 c.w.pd_touched, &ctl->n_cid, c.w.qdef, &ctl->pd_ndef[slot], sh, &ctl->pd_ctile[slot], pd_node, pd_aux);
         G.sync();
@@ -719,7 +722,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
             G.sync();
         stamp(G, qo, TS_PD_MERGE);
         const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
-        if (G.gtid == 0) ctl->pd_flag[slot] = 0u;
+        if (G.gtid() == 0) ctl->pd_flag[slot] = 0u;
         uint32_t *nbits = c.w.pd_bits + (int64_t)(slot ^ 1) * W;
         const int nflag = kFlagPd + (slot ^ 1);
         auto prep = [&](int32_t x, bool, PdNode &nd) { return pd_prepare(c, x, nd); };
@@ -806,7 +809,7 @@ __device__ void reset_mw_prev(const Ctx &c) {
     const Ctl *pv = w.ctl[(done + 1) & 1];
     const int64_t pt = (int64_t)pv->n_touched;
     const uint4 ones = make_uint4(~0u, ~0u, ~0u, ~0u);
-    for (int64_t j = c.G.gtid; j < 2 * pt; j += c.G.gsz) {
+    for (int64_t j = c.G.gtid(); j < 2 * pt; j += c.G.gsz) {
         const int32_t v = w.touched[j >> 1];
         reinterpret_cast<uint4 *>(w.mw + (int64_t)v * 8)[j & 1] = ones;
     }
@@ -816,7 +819,7 @@ __device__ void reset_mw_prev(const Ctx &c) {
 // left in the predecessor pre-pass state, then take |C|, the stop level and reason from the host.
 __device__ void td_only_prepare(const Ctx &c, QOut *qo) {
     const DevWork &w = c.w;
-    const int64_t gtid = c.G.gtid, gsz = c.G.gsz, n = c.a.g.n;
+    const int64_t gtid = c.G.gtid(), gsz = c.G.gsz, n = c.a.g.n;
     reset_mw_prev(c);
     const uint32_t valid = __ldcg(w.gstate + 2), done = __ldcg(w.gstate + 1);
     if (!valid || done == 0) {
@@ -927,7 +930,7 @@ __device__ __forceinline__ void pull_waiting(const Ctx &c, int l, BigTile &S, lo
 // Every node's status word to "not hit yet" (hm = nm = 0, gate = a, a), 4 nodes per 16-byte store.
 __device__ void reset_status_dense(const Ctx &c) {
     const int64_t n = c.a.g.n, n4 = n / 4;
-    for (int64_t j = c.G.gtid; j < n4; j += c.G.gsz) {
+    for (int64_t j = c.G.gtid(); j < n4; j += c.G.gsz) {
         const uint32_t a4 = *reinterpret_cast<const uint32_t *>(c.a.act + j * 4);
         uint4 o;
         o.x = st_fresh(a4 & 0xFFu);
@@ -936,7 +939,7 @@ __device__ void reset_status_dense(const Ctx &c) {
         o.w = st_fresh(a4 >> 24);
         reinterpret_cast<uint4 *>(c.w.st)[j] = o;
     }
-    for (int64_t v = n4 * 4 + c.G.gtid; v < n; v += c.G.gsz) c.w.st[v] = st_fresh(c.a.act[v]);
+    for (int64_t v = n4 * 4 + c.G.gtid(); v < n; v += c.G.gsz) c.w.st[v] = st_fresh(c.a.act[v]);
 }
 
 __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
@@ -947,7 +950,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     const int64_t n = a.g.n, W = a.W;
     const int R = a.R, amax = R - 2;
     const uint32_t full = c.qq.full;
-    const int64_t gtid = G.gtid, gsz = G.gsz;
+    const int64_t gtid = G.gtid(), gsz = G.gsz;
 
     // ---- reset the state the previous query of this group left behind
     const uint32_t valid = __ldcg(w.gstate + 2), lastR = __ldcg(w.gstate + 3);
@@ -1001,13 +1004,16 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
     stamp(G, qo, TS_RESET);
     // ---- initialisation: M = 0 on T_i, keyword nodes ungated, F_0 = K
     {
-        int64_t kb[kMaxQ], ko[kMaxQ + 1];
-        ko[0] = 0;
-        for (int i = 0; i < c.qq.q; ++i) {
-            const int32_t t = c.qq.kw[i];
-            kb[i] = a.g.kw_ptr[t];
-            ko[i + 1] = ko[i] + (a.g.kw_ptr[t + 1] - kb[i]);
+        __shared__ int64_t kb[kMaxQ], ko[kMaxQ + 1];   // the keywords' postings, concatenated (shared: no stack)
+        if (threadIdx.x == 0) {
+            ko[0] = 0;
+            for (int i = 0; i < c.qq.q; ++i) {
+                const int32_t t = c.qq.kw[i];
+                kb[i] = a.g.kw_ptr[t];
+                ko[i + 1] = ko[i] + (a.g.kw_ptr[t + 1] - kb[i]);
+            }
         }
+        __syncthreads();
         for (int64_t j = gtid; j < ko[c.qq.q]; j += gsz) {
             int i = 0;
             while (j >= ko[i + 1]) ++i;
@@ -1230,13 +1236,13 @@ __device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
     }
     __syncthreads();
     if (s_rec[1]) {   // a region overflowed: forget the compact ids, use the pre-pass
-        for (int64_t j = G.gtid; j < nt; j += G.gsz) {   // the pre-pass reads both for its (touched) nodes
+        for (int64_t j = G.gtid(); j < nt; j += G.gsz) {   // the pre-pass reads both for its (touched) nodes
             const int32_t v = __ldcg(w.pd_touched + j);
             w.pd_cid[v] = -1;
             w.pd_state[v] = 0u;
         }
         G.sync();
-        if (G.gtid == 0) { ctl->n_parcs = 0; ctl->n_cid = 0; ctl->rec_overflow = 1; }
+        if (G.gtid() == 0) { ctl->n_parcs = 0; ctl->n_cid = 0; ctl->rec_overflow = 1; }
         G.sync();
         return false;
     }
@@ -1245,7 +1251,7 @@ __device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
         w.pa_x[r] = cid;
         w.pa_slot[r] = atomicAdd(w.pcnt + cid, 1);
     });
-    if (G.gtid == 0) { ctl->n_cid = nt; ctl->rec_used = 1; ctl->n_parcs = (uint32_t)s_rec[0]; }
+    if (G.gtid() == 0) { ctl->n_cid = nt; ctl->rec_used = 1; ctl->n_parcs = (uint32_t)s_rec[0]; }
     G.sync();
     stamp(G, qo, TS_PD_MERGE);
     build_pred_csr(c, sh, qo);
@@ -1830,13 +1836,13 @@ __device__ void select_topk(const Ctx &c, long long *sh, char *dsmem, uint32_t k
     __shared__ uint32_t hsh[256];
     __shared__ uint32_t s_bucket, s_before, s_exact;
     const bool group_wide = nc > kCtaSelectMax;
-    if (G.gtid == 0) ctl->sel_count = 0;
+    if (G.gtid() == 0) ctl->sel_count = 0;
     if (group_wide) {
-        for (int64_t j = G.gtid; j < 12 * 256; j += G.gsz) (&ctl->hist[0][0])[j] = 0u;
+        for (int64_t j = G.gtid(); j < 12 * 256; j += G.gsz) (&ctl->hist[0][0])[j] = 0u;
         G.sync();
     }
     if (group_wide || G.grank == 0) {
-        const int64_t t0 = group_wide ? G.gtid : (int64_t)threadIdx.x;
+        const int64_t t0 = group_wide ? G.gtid() : (int64_t)threadIdx.x;
         const int64_t ts = group_wide ? G.gsz : (int64_t)blockDim.x;
         uint64_t phi = 0;
         uint32_t plo = 0, want = kk;
@@ -1996,11 +2002,11 @@ __device__ void containment_select(const Ctx &c, long long *sh, char *dsmem, uin
 // keyword it does not contain itself (those have m = 0 and no predecessors).
 __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
     const Grp &G = c.G;
-    if (G.gtid == 0) {   // round 0 of this call
+    if (G.gtid() == 0) {   // round 0 of this call
         c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; c.ctl->pd_ctile[0] = 0u;
         c.ctl->pd_xbatch[0] = 0u;
     }
-    for (int64_t j = G.gtid; j < cnt; j += G.gsz) {
+    for (int64_t j = G.gtid(); j < cnt; j += G.gsz) {
         const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;
         const int32_t cn = __ldcg(c.w.centrals + idx);
         const uint64_t Mc = ldrow(c.w.M, cn);
@@ -2024,7 +2030,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
     Ctl *ctl = c.ctl;
     const uint32_t multi = __ldcg(&ctl->multi_kw);
     const double kInf = __longlong_as_double(0x7FF0000000000000ll);
-    if (G.gtid == 0) {
+    if (G.gtid() == 0) {
         ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->work_huge = 0; ctl->work_huge2 = 0;
         ctl->n_eval += cnt;
     }
@@ -2225,12 +2231,12 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             pred_dag(c, S, sh, qo);
         }
         extract_list(c, sh, dsmem, nullptr, nc, qo);
-        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }   // emit counters (read after the select)
+        if (G.gtid() == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }   // emit counters (read after the select)
         if (a.containment) containment_select(c, sh, dsmem, kk);
         else select_topk(c, sh, dsmem, kk);
     } else {
         const uint32_t m = mcap;
-        for (int64_t i = G.gtid; i < nc; i += G.gsz) {   // lower bounds; cflag 2 = not extracted
+        for (int64_t i = G.gtid(); i < nc; i += G.gsz) {   // lower bounds; cflag 2 = not extracted
             const int32_t cn = __ldcg(c.w.centrals + i);
             double lb;
             if (a.prune == 2) {   // the kept graph holds a lightest-or-heavier path from T_i to c, every i
@@ -2247,7 +2253,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
         select_topk(c, sh, dsmem, m);                          // sel[0..m): the m smallest (LB, id)
         uint64_t bhi; uint32_t blo;
         comp_key(c, (uint32_t)__ldcg(c.w.sel + m - 1), bhi, blo);
-        for (int64_t j = G.gtid; j < m; j += G.gsz) c.w.elist[j] = __ldcg(c.w.sel + j);
+        for (int64_t j = G.gtid(); j < m; j += G.gsz) c.w.elist[j] = __ldcg(c.w.sel + j);
         G.sync();
         if (!rec) {
             seed_pd(c, c.w.elist, m);
@@ -2261,7 +2267,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
         uint32_t n2 = 0;
         if (bhi < thi || (bhi == thi && blo < tlo)) {
             // round 2: every candidate not extracted yet whose (LB, id) still ranks before T
-            for (int64_t i = G.gtid; i < nc; i += G.gsz) {
+            for (int64_t i = G.gtid(); i < nc; i += G.gsz) {
                 if (__ldcg(c.w.cflag + i) != 2) continue;
                 uint64_t hi; uint32_t lo;
                 comp_key(c, (uint32_t)i, hi, lo);
@@ -2277,11 +2283,11 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
             extract_list(c, sh, dsmem, c.w.elist + m, n2, qo, cut);
         }
-        if (G.gtid == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }
+        if (G.gtid() == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }
         if (m + n2 <= (uint32_t)KGS_MAX_K) {
             rank_list(c, dsmem, c.w.elist, m + n2, kk);
         } else {   // the candidates never extracted rank after every extracted one
-            for (int64_t i = G.gtid; i < nc; i += G.gsz)
+            for (int64_t i = G.gtid(); i < nc; i += G.gsz)
                 if (__ldcg(c.w.cflag + i) == 2) c.w.ckey[i] = __longlong_as_double(0x7FF0000000000000ll);
             G.sync();
             select_topk(c, sh, dsmem, kk);
@@ -2303,23 +2309,25 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
     __shared__ long long sh[40];
     __shared__ int32_t s_q[2 + kMaxQ];
     // group of this CTA: contiguous ranges, sizes differ by at most one
-    Grp G;
-    {
+    __shared__ Grp s_grp;
+    if (threadIdx.x == 0) {
+        Grp &G = s_grp;
         const int nb = gridDim.x, gsz_b = nb / a.G, extra = nb % a.G;
         const int b = blockIdx.x;
         const int cut = extra * (gsz_b + 1);
         if (b < cut) { G.g = b / (gsz_b + 1); G.grank = b % (gsz_b + 1); G.gcount = gsz_b + 1; }
         else { G.g = extra + (b - cut) / gsz_b; G.grank = (b - cut) % gsz_b; G.gcount = gsz_b; }
-        G.gtid = (int64_t)G.grank * blockDim.x + threadIdx.x;
         G.gsz = (int64_t)G.gcount * blockDim.x;
         G.bar = a.bars + G.g;
         G.episode = 0;
     }
+    __syncthreads();
+    const Grp &G = s_grp;
     for (int t = threadIdx.x; t < kFlagSlots; t += blockDim.x) cta_flags()[t] = 0u;   // (synced below)
     const DevWork &w = a.works[G.g];
     for (;;) {
         // the group leader takes the next query of the batch
-        if (G.gtid == 0) {
+        if (G.gtid() == 0) {
             const uint32_t qi = atomicAdd(a.next_query, 1u);
             w.gstate[0] = qi;
         }
@@ -2334,18 +2342,22 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         }
         __syncthreads();
         if (s_q[0] >= a.nq) break;
-        Q qq;
-        qq.qi = s_q[0];
-        qq.q = s_q[1];
-        qq.full = (1u << qq.q) - 1u;
-        for (int i = 0; i < kMaxQ; ++i) qq.kw[i] = s_q[2 + i];
+        __shared__ Q s_query;   // written by thread 0 after the previous query's last group barrier
+        if (threadIdx.x == 0) {
+            s_query.qi = s_q[0];
+            s_query.q = s_q[1];
+            s_query.full = (1u << s_query.q) - 1u;
+            for (int i = 0; i < kMaxQ; ++i) s_query.kw[i] = s_q[2 + i];
+        }
+        __syncthreads();
+        const Q &qq = s_query;
         bool bad = qq.q < 1 || qq.q > kMaxQ;   // device-side validation (kgs_query_batch_device)
         for (int i = 0; !bad && i < qq.q; ++i) {
             if (qq.kw[i] < 0 || qq.kw[i] >= a.g.n_kw) bad = true;
             for (int j = 0; j < i; ++j) if (qq.kw[j] == qq.kw[i]) bad = true;
         }
         if (bad) {
-            if (G.gtid == 0) {
+            if (G.gtid() == 0) {
                 QOut *qo = a.qout + qq.qi;
                 qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
                 qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1; qo->n_cut = 0;
@@ -2357,10 +2369,10 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         Ctl *ctl = w.ctl[done & 1];
         {   // zero this query's control block
             uint32_t *cw = reinterpret_cast<uint32_t *>(ctl);
-            for (int64_t j = G.gtid; j < (int64_t)(sizeof(Ctl) / 4); j += G.gsz) cw[j] = 0u;
+            for (int64_t j = G.gtid(); j < (int64_t)(sizeof(Ctl) / 4); j += G.gsz) cw[j] = 0u;
         }
         QOut *qo = a.qout + qq.qi;
-        if (G.gtid == 0) { qo->n_stamp = 0; qo->t_start = globaltimer_ns(); qo->group = G.g; }
+        if (G.gtid() == 0) { qo->n_stamp = 0; qo->t_start = globaltimer_ns(); qo->group = G.g; }
         G.sync();
         stamp(G, qo, TS_START);
         const int rns = rec_stripes(G);
@@ -2368,7 +2380,7 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         if (a.td_only) td_only_prepare(c, qo);
         else search(c, s_big, sh, qo);
         if (!a.search_only) topdown(c, s_big, sh, dsmem, qo);   // search_only: workload analysis (no answers)
-        if (G.gtid == 0) {
+        if (G.gtid() == 0) {
             qo->levels = ctl->levels;
             qo->stop_reason = ctl->stop_reason;
             qo->count = (int32_t)ctl->sel_count;
