@@ -242,6 +242,14 @@ kgs_status kgs_result_centrals(const kgs_result *r, int32_t *ids, uint8_t *depth
 /* Activation levels a (n bytes, Eqs. 3-5 at the query's alpha) — only if want_levels was 1. */
 kgs_status kgs_result_activation(const kgs_result *r, uint8_t *a, int64_t cap);
 kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s);
+/* Every answer of a result in flat host arrays with one call (kgs_result_answer takes one call per answer):
+ * kgs_result_sizes gives count, the total number of answer nodes and of answer arcs; kgs_result_export
+ * fills central / depth / score_key [count], node_off / arc_off [count + 1] (answer i's nodes are
+ * nodes[node_off[i] .. node_off[i + 1]), its arcs arcs[2 * arc_off[i] .. 2 * arc_off[i + 1])), nodes
+ * [total_nodes] and arcs [2 * total_arcs], in rank order.  Caller-owned buffers. */
+kgs_status kgs_result_sizes(const kgs_result *r, int32_t *count, int64_t *total_nodes, int64_t *total_arcs);
+kgs_status kgs_result_export(const kgs_result *r, int32_t *central, int32_t *depth, double *score_key,
+                             int64_t *node_off, int32_t *nodes, int64_t *arc_off, int32_t *arcs);
 /* Phase trace of the search kernel (the paper's per-phase profile): *n stamps, each a
  * tag (0 start, 1 reset, 2 sources, 3 merge+identify, 4 expansion, 5..8 top-down pre-pass: seeds,
  * merge, expansion, CSR, 9 end of search) and a %globaltimer time in ns, in execution order. */

@@ -91,7 +91,8 @@ EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query
             "kgs_result_free", "kgs_last_error", "kgs_version", "kgs_query_batch", "kgs_query_batch_device",
             "kgs_query_batch_fetch", "kgs_vp_slice", "kgs_vp_begin", "kgs_vp_level", "kgs_vp_waiting",
             "kgs_vp_topdown", "kgs_prep_pair_distances", "kgs_prep_summary_weights", "kgs_vp_nccl_unique_id",
-            "kgs_vp_nccl_transport", "kgs_vp_transport_free", "kgs_vp_query"]
+            "kgs_vp_nccl_transport", "kgs_vp_transport_free", "kgs_vp_query", "kgs_result_sizes",
+            "kgs_result_export"]
 
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
                "search_end", "extract", "extract_big", "select", "emit"]
@@ -133,6 +134,10 @@ def lib():
         L.kgs_result_centrals.restype = i32
         L.kgs_result_stats.argtypes = [vp, ctypes.POINTER(kgs_stats)]
         L.kgs_result_stats.restype = i32
+        L.kgs_result_sizes.argtypes = [vp, vp, vp, vp]
+        L.kgs_result_sizes.restype = i32
+        L.kgs_result_export.argtypes = [vp] * 8
+        L.kgs_result_export.restype = i32
         L.kgs_query_batch.argtypes = [vp, i32, vp, vp, i32, ctypes.POINTER(kgs_params), i32, vp, vp]
         L.kgs_query_batch.restype = i32
         L.kgs_query_batch_device.argtypes = [vp, i32, vp, vp, i32, ctypes.POINTER(kgs_params), i32, vp]
@@ -279,15 +284,23 @@ class Result:
 def _read_result(h, n, q, want_levels) -> Result:
     L = lib()
     try:
-        cnt = L.kgs_result_count(h)
-        answers = []
-        a = kgs_answer()
-        for i in range(cnt):
-            _check(L.kgs_result_answer(h, i, ctypes.byref(a)))
-            nodes = np.ctypeslib.as_array(a.nodes, shape=(a.n_nodes,)).copy() if a.n_nodes else np.zeros(0, np.int32)
-            arcs = (np.ctypeslib.as_array(a.arcs, shape=(2 * a.n_arcs,)).copy().reshape(-1, 2) if a.n_arcs
-                    else np.zeros((0, 2), np.int32))
-            answers.append(Answer(a.central, a.depth, a.score, a.score_key, nodes, arcs))
+        # every answer in flat arrays with one call (kgs_result_export); answers hold views into them
+        cnt, tn, ta = ctypes.c_int32(), ctypes.c_int64(), ctypes.c_int64()
+        _check(L.kgs_result_sizes(h, ctypes.byref(cnt), ctypes.byref(tn), ctypes.byref(ta)))
+        cnt = cnt.value
+        cen = np.empty(cnt, np.int32)
+        dep = np.empty(cnt, np.int32)
+        key = np.empty(cnt, np.float64)
+        noff = np.empty(cnt + 1, np.int64)
+        aoff = np.empty(cnt + 1, np.int64)
+        nodes = np.empty(max(tn.value, 1), np.int32)
+        arcs = np.empty(max(2 * ta.value, 2), np.int32)
+        _check(L.kgs_result_export(h, cen.ctypes.data, dep.ctypes.data, key.ctypes.data, noff.ctypes.data,
+                                   nodes.ctypes.data, aoff.ctypes.data, arcs.ctypes.data))
+        arcs2 = arcs.reshape(-1, 2)
+        score = key.astype(np.float32)
+        answers = [Answer(int(cen[i]), int(dep[i]), float(score[i]), float(key[i]), nodes[noff[i]:noff[i + 1]],
+                          arcs2[aoff[i]:aoff[i + 1]]) for i in range(cnt)]
         st = kgs_stats()
         _check(L.kgs_result_stats(h, ctypes.byref(st)))
         stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
@@ -298,9 +311,11 @@ def _read_result(h, n, q, want_levels) -> Result:
         m = min(nph.value, 64)
         # per-phase durations (us): time from the previous stamp to this one, summed by phase name
         ph = {}
-        for i in range(1, m):
-            nm = PHASE_NAMES[tags[i]] if 0 <= tags[i] < len(PHASE_NAMES) else str(tags[i])
-            ph[nm] = ph.get(nm, 0.0) + (int(tns[i]) - int(tns[i - 1])) / 1e3
+        if m > 1:
+            dur = np.diff(tns[:m].astype(np.int64)) / 1e3
+            sums = np.bincount(tags[1:m], weights=dur)
+            for t in np.flatnonzero(np.bincount(tags[1:m])):
+                ph[PHASE_NAMES[t] if t < len(PHASE_NAMES) else str(t)] = float(sums[t])
         stats["phases_us"] = ph
         res = Result(answers, stats)
         if want_levels:

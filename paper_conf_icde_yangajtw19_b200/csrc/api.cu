@@ -1019,6 +1019,43 @@ kgs_status kgs_result_centrals(const kgs_result *r, int32_t *ids, uint8_t *depth
     return KGS_OK;
 }
 
+kgs_status kgs_result_sizes(const kgs_result *r, int32_t *count, int64_t *total_nodes, int64_t *total_arcs) {
+    if (!r || !count || !total_nodes || !total_arcs) return fail(KGS_EINVAL, "null argument");
+    *count = (int32_t)r->ans.size();
+    int64_t tn = 0, ta = 0;
+    for (const auto &a : r->ans) { tn += a.n_nodes; ta += a.n_arcs; }
+    *total_nodes = tn;
+    *total_arcs = ta;
+    return KGS_OK;
+}
+
+kgs_status kgs_result_export(const kgs_result *r, int32_t *central, int32_t *depth, double *score_key,
+                             int64_t *node_off, int32_t *nodes, int64_t *arc_off, int32_t *arcs) {
+    if (!r || !central || !depth || !score_key || !node_off || !arc_off) return fail(KGS_EINVAL, "null argument");
+    int64_t tn = 0, ta = 0;
+    node_off[0] = 0;
+    arc_off[0] = 0;
+    for (size_t i = 0; i < r->ans.size(); ++i) {
+        const kgs_answer &a = r->ans[i];
+        central[i] = a.central;
+        depth[i] = a.depth;
+        score_key[i] = a.score_key;
+        if (a.n_nodes) {
+            if (!nodes) return fail(KGS_EINVAL, "null nodes buffer");
+            std::memcpy(nodes + tn, a.nodes, sizeof(int32_t) * (size_t)a.n_nodes);
+        }
+        if (a.n_arcs) {
+            if (!arcs) return fail(KGS_EINVAL, "null arcs buffer");
+            std::memcpy(arcs + 2 * ta, a.arcs, sizeof(int32_t) * 2 * (size_t)a.n_arcs);
+        }
+        tn += a.n_nodes;
+        ta += a.n_arcs;
+        node_off[i + 1] = tn;
+        arc_off[i + 1] = ta;
+    }
+    return KGS_OK;
+}
+
 kgs_status kgs_result_stats(const kgs_result *r, kgs_stats *s) {
     if (!r || !s) return fail(KGS_EINVAL, "null argument");
     *s = r->stats;
