@@ -138,7 +138,11 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *   dag_record     -1 [auto: on for single-query launches] / 0 / 1: the top-down's predecessor lists come
  *                  from the arcs the search recorded (1) or from the in-arc pre-pass (0); the recorded DAG
  *                  is used only where it is exact (extract_mode EXACT, or block_central 0)
- *   search_only    0 [0] / 1: workload analysis — stop after the search (no top-down, no answers) */
+ *   search_only    0 [0] / 1: workload analysis — stop after the search (no top-down, no answers)
+ *   mk_min         >= 0 [4096]: with level_cover = 1 and at least this many candidates in pruning round 2,
+ *                  decide per candidate whether level-cover can keep fewer than all of its sources (a pass
+ *                  over the predecessor DAG, engine.cu mk_reach) instead of once per query, so that the
+ *                  exact key cut-off applies to more candidates */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
@@ -147,6 +151,7 @@ typedef struct {
     int64_t pull_min;
     int32_t prune_min, tile_light, dag_record, search_only;
     int32_t containment;
+    int32_t mk_min;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 

@@ -253,6 +253,7 @@ void kgs_params_default(kgs_params *p) {
     p->tile_light = 8 * kBlock;
     p->dag_record = -1;
     p->search_only = 0;
+    p->mk_min = 4096;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -444,9 +445,9 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.containment != 0 && p.containment != 1) return fail(KGS_EINVAL, "containment must be 0 or 1");
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
-        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1))
+        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0)
         return fail(KGS_EINVAL, "tuning parameters out of range (pull_ratio >= 1, pull_min >= 0, prune_min >= 1, "
-                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1)");
+                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0)");
     return KGS_OK;
 }
 
@@ -576,6 +577,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.prune = (p.want_levels || p.containment) ? 0 : p.prune;
     if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
     a.prune_min = p.prune_min;
+    a.mk_min = p.mk_min;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
         // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass.
         // Auto: on for the single-query (latency) launch, where the pre-pass's rounds of group barriers

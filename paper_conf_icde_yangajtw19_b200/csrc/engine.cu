@@ -800,6 +800,57 @@ __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
     stamp(G, qo, TS_PD_CSR);
 }
 
+// Which keywords can a source holding two or more query keywords cover for c (the key cut-off's validity,
+// central_graph)?  reach(x) = the keywords i such that some node v holding i and at least one other query
+// keyword reaches x along predecessor arcs of keyword i (v in DAG_i(x)): over the shared DAG's arcs u -> x
+// with keyword bits b, reach(x) |= b & (zb(u) if |zb(u)| >= 2) | b & reach(u), to a fixpoint (a chain is
+// at most the search depth long).  Level-cover (R13) can only pick s* >= 2 for c if the keywords of the
+// nodes contributing two or more cover Q with zb(c), and each such node v contributes i only if v is a
+// source in DAG_i(c) — so s* >= 2 implies reach(c) | zb(c) = Q.  The DAG holds every closure arc of the
+// candidates seeded so far (a superset of one candidate's), so reach over-approximates: the test is safe.
+// Stored per compact id in pcnt (the CSR is built; pcnt's prefix is reset by the next query); the arc
+// records' pa_u becomes the predecessor's compact id (-1: a source without a list) on the first pass.
+__device__ void mk_reach(const Ctx &c) {
+    const Grp &G = c.G;
+    Ctl *ctl = c.ctl;
+    const uint32_t mk = __ldcg(&ctl->multi_kw) & c.qq.full;
+    const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
+    uint32_t *R = reinterpret_cast<uint32_t *>(c.w.pcnt);
+    for (int64_t j = G.gtid(); j < ncid; j += G.gsz) R[j] = 0u;
+    if (G.gtid() == 0) { ctl->mk_changed[0] = 0u; ctl->mk_changed[1] = 0u; }
+    G.sync();
+    const uint32_t *cnt = ctl->rec_used ? ctl->rec_cnt : ctl->pd_cnt;
+    for (int pass = 0;; ++pass) {
+        bool changed = false;
+        for_each_record(c, cnt, [&](int64_t ai) {
+            const uint32_t b = c.w.pa_b[ai];
+            const uint32_t pb = b & 0xFFu & mk;
+            int32_t cu;
+            if (pass == 0) {
+                const int32_t u = c.w.pa_u[ai];
+                cu = pb ? __ldcg(c.w.pd_cid + u) : -1;
+                c.w.pa_u[ai] = cu;
+            } else {
+                cu = __ldcg(c.w.pa_u + ai);
+            }
+            if (!pb) return;
+            const uint32_t zbu = b >> 8;
+            const uint32_t add = pb & ((__popc(zbu) >= 2 ? zbu : 0u) | (cu >= 0 ? __ldcg(R + cu) : 0u));
+            if (!add) return;
+            const int32_t xc = c.w.pa_x[ai];
+            if (add & ~__ldcg(R + xc)) { atomicOr(R + xc, add); changed = true; }
+        });
+        if (__syncthreads_or(changed) && threadIdx.x == 0) ctl->mk_changed[pass & 1] = 1u;
+        G.sync();
+        const bool more = __ldcg(&ctl->mk_changed[pass & 1]) != 0u;
+        if (G.gtid() == 0) ctl->mk_changed[(pass + 1) & 1] = 0u;   // read by every CTA before the next barrier
+        G.sync();
+        if (!more) break;
+    }
+    if (G.gtid() == 0) ctl->mk_reach = 1u;
+    G.sync();
+}
+
 // ------------------------------------------------------------------------------------------ search
 // The previous query's lightest-path rows (prune mode 2), through its touched list (always complete).
 __device__ void reset_mw_prev(const Ctx &c) {
@@ -1283,7 +1334,7 @@ struct BlockTeam {
     __device__ __forceinline__ int scan_excl(int x, int *total) const { return block_excl_scan(x, total, sh); }
 };
 
-enum { SC_NODES = 0, SC_ARCS, SC_HEAD, SC_TAIL, SC_OVF, SC_CHANGED, SC_COV, SC_SSTAR, SC_NOUT, SC_AOUT, SC_N };
+enum { SC_NODES = 0, SC_ARCS, SC_HEAD, SC_TAIL, SC_OVF, SC_CHANGED, SC_COV, SC_SSTAR, SC_NOUT, SC_AOUT, SC_CUT, SC_N };
 
 struct Arena {
     int32_t *hkey;      // [hcap] node id or -1
@@ -1447,8 +1498,16 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     const uint64_t Mc = ldrow(c.w.M, cn);
     uint32_t zbc = 0;
     for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
+    // s* >= 2 needs sources holding >= 2 query keywords that cover Q with zb(c): multi is the union of
+    // the keyword sets of such nodes (graph-wide), or per candidate the keywords i for which one of them
+    // reaches c inside DAG_i (the shared predecessor DAG's arcs, pd_state byte 3, mk_reach)
+    const uint32_t reach = c.a.level_cover == 1 && c.ctl->mk_reach ? (__ldcg(c.w.pd_state + cn) >> 24) : multi;
     const bool cut_on = cut < kNoCut &&
-                        (!c.a.level_cover || ((multi | zbc) & full) != full);
+                        (!c.a.level_cover || ((reach | zbc) & full) != full);
+    auto over_cut = [&]() {   // the closure weight so far, times d^lambda, already exceeds the cut
+        return __dmul_rn(c.a.dpow[depth], (double)*reinterpret_cast<volatile unsigned long long *>(S.wsum) *
+                                              (1.0 / 16777216.0)) > cut;
+    };
     if (r == 0) {
         bool fresh;
         const int j = arena_insert(S, cn, zbc, fresh);  // index 0
@@ -1461,9 +1520,8 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     // ---- backward closure, batch by batch (all pending nodes of a round in parallel)
     for (;;) {
         const int head = S.scal[SC_HEAD], tail = S.scal[SC_TAIL];
-        if (head == tail || S.scal[SC_OVF]) break;
-        if (cut_on && __dmul_rn(c.a.dpow[depth], (double)*reinterpret_cast<volatile unsigned long long *>(S.wsum) *
-                                                     (1.0 / 16777216.0)) > cut) {
+        if (head == tail || S.scal[SC_OVF] || S.scal[SC_CUT]) break;
+        if (cut_on && over_cut()) {
             T.sync();
             return CG_CUT;
         }
@@ -1489,7 +1547,12 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
             for (int e = r, it = 0; e < tot; e += ts, ++it) {
                 // the arena overflowed: the next tier redoes this graph, stop scanning (a hub's list of
                 // millions of predecessors kept a tier-1 warp busy for milliseconds, C5)
-                if ((it & 31) == 0 && *reinterpret_cast<volatile int32_t *>(S.scal + SC_OVF)) break;
+                if ((it & 31) == 0) {
+                    if (*reinterpret_cast<volatile int32_t *>(S.scal + SC_OVF) ||
+                        *reinterpret_cast<volatile int32_t *>(S.scal + SC_CUT)) break;
+                    // the cut can be decided inside a round (a hub's list of thousands of predecessors)
+                    if (cut_on && it && over_cut()) { S.scal[SC_CUT] = 1; break; }
+                }
                 int lo = 0, hi = nb - 1;       // owner = first o with incl[o] > e
                 while (lo < hi) {
                     const int mid = (lo + hi) >> 1;
@@ -1525,6 +1588,8 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
         T.sync();
     }
     T.sync();
+    // an overflowing arena still holds a partial closure: its weight is a lower bound of the key
+    if (S.scal[SC_CUT] || (S.scal[SC_OVF] && cut_on && over_cut())) { T.sync(); return CG_CUT; }
     if (S.scal[SC_OVF]) return CG_OVERFLOW;
     const int nn = S.scal[SC_NODES];
     const int na = S.scal[SC_ARCS] < S.acap ? S.scal[SC_ARCS] : S.acap;
@@ -2279,8 +2344,11 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
                 seed_pd(c, c.w.elist + m, n2);
                 pred_dag(c, S, sh, qo);
             }
-            // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union)
+            // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union);
+            // with many candidates, which of them can have s* >= 2 is decided per candidate (mk_reach)
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
+            if (!a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min && (__ldcg(&ctl->multi_kw) & c.qq.full))
+                mk_reach(c);
             extract_list(c, sh, dsmem, c.w.elist + m, n2, qo, cut);
         }
         if (G.gtid() == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }

@@ -90,6 +90,8 @@ struct Ctl {
     uint32_t pd_ctile[2];          // [round parity] the same for the predecessor pre-pass
     uint32_t xbatch[2];            // [level parity] expansion: next warp batch beyond the first round
     uint32_t pd_xbatch[2];         // [round parity] the same for the pre-pass
+    uint32_t mk_reach;             // pcnt holds, per compact id, the keywords a multi-keyword source reaches it in
+    uint32_t mk_changed[2];        // [pass parity] mk_reach fixpoint
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -200,6 +202,7 @@ struct EngineArgs {
     uint32_t td_ncentral;       //    and |C| (works[0].centrals / cdepth hold the list)
     int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
+    int mk_min;                 // round 2: per-candidate s* >= 2 test (mk_reach) from this many candidates
     int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
     int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
     int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio

@@ -206,3 +206,50 @@ def test_key_cutoff_in_round_two():
             cuts += r.stats["n_cut"]
         G.close()
     assert cuts > 0
+
+
+def test_key_cutoff_per_candidate_multi_keyword_sources():
+    """A few nodes hold two query keywords, so graph-wide level-cover could keep only some sources
+    (s* >= 2) and the query-wide test switches the cut-off off.  mk_reach decides it per candidate: the
+    keywords for which a two-keyword node reaches c inside DAG_i(c); where they cannot cover Q with zb(c),
+    every source is kept and the cut-off applies.  The candidates near the two-keyword nodes (small pruned
+    graphs, the likely winners) must still get their exact keys: answers equal the oracle's with the
+    per-candidate test on (mk_min = 0) and off, in latency mode (recorded DAG and pre-pass) and in a batch."""
+    _gpu()
+    cuts_on = cuts_off = 0
+    for seed, deg, k, n_multi in ((0, 16, 5, 3), (1, 16, 20, 10), (2, 8, 20, 30), (3, 16, 50, 6)):
+        rng = np.random.default_rng(900 + seed)
+        n, q = 6000, 3
+        g0 = medium_graph(900 + seed, n=n, deg=deg, q=q, kw_size=10, wpow=3.0)
+        perm = rng.permutation(n)
+        kws = [perm[i * 100:(i + 1) * 100].tolist() for i in range(q)]
+        for j in range(n_multi):   # node holding keywords i and i+1 (every pair, so they cover Q)
+            i = j % q
+            kws[(i + 1) % q].append(kws[i][j // q])
+        kws = [sorted(set(x)) for x in kws]
+        edges = [(u, int(v)) for u in range(n) for v in g0.col_idx[g0.row_ptr[u]:g0.row_ptr[u + 1]] if u < v]
+        g = synth.from_edges(n, edges, g0.weight, kws, 2.0)
+        G = kgs.kgs_load_graph(g)
+        kw = list(range(q))
+        o = oracle.query(g, kw, k)
+        ctx0 = f"seed={seed} deg={deg} k={k} multi={n_multi} |C|={len(o.centrals)}"
+        runs = []
+        for mk in (0, 1 << 30):
+            for rec in (1, 0):
+                p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, dag_record=rec)
+                runs.append((f"mk={mk} rec={rec}", kgs.kgs_query(G, kw, k, p), mk))
+            p = kgs.make_params(prune=1, prune_min=40, mk_min=mk)
+            for j, r in enumerate(kgs.kgs_query_batch(G, [kw, kw[::-1], kw], k, p, 3)):
+                runs.append((f"mk={mk} batch {j}", r, mk))
+        for tag, r, mk in runs:
+            ctx = f"{ctx0} {tag}"
+            assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
+            for ra, oa in zip(r.answers, o.answers):
+                assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist(), ctx
+                assert ra.arcs.tolist() == oa.arcs.tolist(), ctx
+            if mk == 0:
+                cuts_on += r.stats["n_cut"]
+            else:
+                cuts_off += r.stats["n_cut"]
+        G.close()
+    assert cuts_off == 0 and cuts_on > 0, (cuts_on, cuts_off)

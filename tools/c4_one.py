@@ -17,6 +17,6 @@ for i in (int(x) for x in sys.argv[1:]):
             s = r.stats
             print(i, "rec", rec, "q", len(kw), {k: s[k] for k in ("levels", "n_centrals", "arcs_scanned", "td_arcs",
                                                                   "td_pred_arcs", "dag_arcs", "overflow", "ms_search",
-                                                                  "ms_topdown", "n_evaluated")}, {k: round(v) for k, v in s["phases_us"].items()}, flush=True)
+                                                                  "ms_topdown", "n_evaluated", "n_cut")}, {k: round(v) for k, v in s["phases_us"].items()}, flush=True)
         except Exception as e:
             print(i, "rec", rec, "failed:", e, flush=True)

@@ -20,6 +20,14 @@ w = synth.make_workload(name)
 order = np.random.default_rng(12345).permutation(len(w.queries))
 qs = [w.queries[i] for i in order]
 G = kgs.kgs_load_graph(w.graph)
+if os.environ.get("L2GRAN"):   # experiment: cudaLimitMaxL2FetchGranularity (0x05) on the primary context
+    import ctypes
+    torch.cuda.init()
+    rt = ctypes.CDLL("libcudart.so.12")
+    rc = rt.cudaDeviceSetLimit(0x05, ctypes.c_size_t(int(os.environ["L2GRAN"]))) if os.environ["L2GRAN"] != "0" else -1
+    got = ctypes.c_size_t(0)
+    rt.cudaDeviceGetLimit(ctypes.byref(got), 0x05)
+    print("L2 fetch granularity", os.environ["L2GRAN"], "rc", rc, "now", got.value, flush=True)
 s = torch.cuda.current_stream()
 for rep in range(2):
     sub = [qs[(rep * batch + j) % len(qs)] for j in range(batch)]

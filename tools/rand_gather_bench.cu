@@ -5,6 +5,7 @@
 // Build: nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o /tmp/rgb tools/rand_gather_bench.cu
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 __device__ __forceinline__ uint32_t mix(uint32_t x) {
@@ -46,7 +47,19 @@ __global__ void k_stream(const uint4 *__restrict__ a, int64_t n, uint32_t *out) 
     if (acc == 0x12345678u) out[0] = acc;
 }
 
-int main() {
+int main(int argc, char **argv) {
+    // optional argument: cudaLimitMaxL2FetchGranularity in bytes (0 = leave the driver default)
+    const int gran = argc > 1 ? atoi(argv[1]) : 0;
+    if (gran > 0) {
+        cudaError_t e = cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)gran);
+        size_t got = 0;
+        cudaDeviceGetLimit(&got, cudaLimitMaxL2FetchGranularity);
+        printf("cudaLimitMaxL2FetchGranularity set %d -> %s, now %zu\n", gran, cudaGetErrorString(e), got);
+    } else {
+        size_t got = 0;
+        cudaDeviceGetLimit(&got, cudaLimitMaxL2FetchGranularity);
+        printf("cudaLimitMaxL2FetchGranularity default %zu\n", got);
+    }
     const uint64_t words = 1ull << 30;   // 4 GiB
     uint32_t *a, *out;
     cudaMalloc(&a, words * 4);
