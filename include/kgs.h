@@ -142,7 +142,10 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *   mk_min         >= 0 [4096]: with level_cover = 1 and at least this many candidates in pruning round 2,
  *                  decide per candidate whether level-cover can keep fewer than all of its sources (a pass
  *                  over the predecessor DAG, engine.cu mk_reach) instead of once per query, so that the
- *                  exact key cut-off applies to more candidates */
+ *                  exact key cut-off applies to more candidates
+ *   defer_min      >= 0 [65536]: in a launch of several query groups, a query that identifies more central
+ *                  nodes than this is answered at the end of the launch by all CTAs together (its top-down
+ *                  parallelises over the whole GPU instead of holding one group); 0 = never */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
@@ -152,6 +155,7 @@ typedef struct {
     int32_t prune_min, tile_light, dag_record, search_only;
     int32_t containment;
     int32_t mk_min;
+    int32_t defer_min;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 
@@ -181,7 +185,8 @@ typedef struct {
     int64_t td_pred_arcs;  /* predecessor arcs (Thm. V.4) in the union of all Central Graphs */
     float ms_search, ms_topdown, ms_total;   /* this query: bottom-up search, top-down, total (device clock) */
     float ms_launch;       /* the whole engine launch that answered it (all queries of the batch) */
-    int32_t group;         /* engine group (set of CTAs) that answered the query */
+    int32_t group;         /* engine group (set of CTAs) that answered the query; n_groups: the whole grid
+                              at the end of the launch (a deferred query, kgs_params.defer_min) */
     int32_t n_evaluated;   /* Central Graphs whose exact key was computed (|C| unless prune skipped some) */
     int64_t dag_arcs;      /* arcs the search traversed that hit their target: the Thm. V.4 arcs of all hit nodes */
     int32_t pull_level;    /* first level expanded by pull (kgs_params.direction), -1: push throughout */

@@ -109,7 +109,9 @@ struct kgs_graph {
     size_t d_off_cap = 0;
     int32_t *d_nodes = nullptr, *d_arcs = nullptr;
     size_t d_nodes_cap = 0, d_arcs_cap = 0;
-    unsigned long long *d_ctr = nullptr;   // [0] next query, [1..2] arena counters
+    unsigned long long *d_ctr = nullptr;   // [0] next query, [1..2] arena counters, [3] deferred queries
+    int32_t *d_defer = nullptr;            // [nq] deferred queries (engine.cu run_query)
+    size_t d_defer_cap = 0;
     // pinned host staging
     int32_t *h_kw = nullptr, *h_qlen = nullptr;
     size_t h_kw_cap = 0, h_qlen_cap = 0;
@@ -254,6 +256,7 @@ void kgs_params_default(kgs_params *p) {
     p->dag_record = -1;
     p->search_only = 0;
     p->mk_min = 4096;
+    p->defer_min = 1 << 16;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -263,7 +266,7 @@ void kgs_free_graph(kgs_graph *g) {
     for (auto &w : g->works) free_work(w);
     void *ptrs[] = {g->row_ptr, g->col_idx, g->kw_ptr, g->kw_nodes, g->weight, g->cls, g->act, g->amax_dev, g->dpow,
                     g->works_dev, g->bars, g->warp_arenas, g->cta_arenas, g->large_arenas, g->d_kw, g->d_qlen, g->d_qout, g->d_hdr,
-                    g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr, g->vp_gate, g->vp_X, g->vp_big,
+                    g->d_key, g->d_off, g->d_nodes, g->d_arcs, g->d_ctr, g->d_defer, g->vp_gate, g->vp_X, g->vp_big,
                     g->vp_nbig_dev, g->orig, g->perm};
     for (void *p : ptrs) if (p) cudaFree(p);
     if (!g->symmetric) { cudaFree(g->in_ptr); cudaFree(g->in_idx); cudaFree(g->cls_in); }
@@ -445,9 +448,9 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.containment != 0 && p.containment != 1) return fail(KGS_EINVAL, "containment must be 0 or 1");
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
-        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0)
+        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0 || p.defer_min < 0)
         return fail(KGS_EINVAL, "tuning parameters out of range (pull_ratio >= 1, pull_min >= 0, prune_min >= 1, "
-                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0)");
+                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0, defer_min >= 0)");
     return KGS_OK;
 }
 
@@ -504,8 +507,8 @@ kgs_status prepare(kgs_graph *g, const kgs_params &p, int G, cudaStream_t s) {
         if (g->works_dev) cudaFree(g->works_dev);
         if (g->bars) cudaFree(g->bars);
         CUDA_TRY(dmalloc(&g->works_dev, g->works.size()));
-        CUDA_TRY(dmalloc(&g->bars, g->works.size()));
-        CUDA_TRY(cudaMemset(g->bars, 0, sizeof(GroupBar) * g->works.size()));
+        CUDA_TRY(dmalloc(&g->bars, g->works.size() + 1));   // + the whole grid's (deferred queries)
+        CUDA_TRY(cudaMemset(g->bars, 0, sizeof(GroupBar) * (g->works.size() + 1)));
         g->works_dev_n = 0;
     }
     if (g->works_dev_n != (int)g->works.size() || invalidate) {
@@ -546,6 +549,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     kgs_status st = prepare(g, p, G, s);
     if (st != KGS_OK) return st;
     CUDA_TRY(grow_dev(&g->d_qout, &g->d_qout_cap, (size_t)nq));
+    CUDA_TRY(grow_dev(&g->d_defer, &g->d_defer_cap, (size_t)nq));
     CUDA_TRY(grow_dev(&g->d_hdr, &g->d_hdr_cap, (size_t)nq * k * 4));
     CUDA_TRY(grow_dev(&g->d_key, &g->d_key_cap, (size_t)nq * k));
     CUDA_TRY(grow_dev(&g->d_off, &g->d_off_cap, (size_t)nq * k * 2));
@@ -568,6 +572,9 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.works = g->works_dev; a.bars = g->bars; a.G = G;
     a.nq = nq; a.kw = g->d_kw; a.qlen = g->d_qlen; a.qconst = qconst;
     a.next_query = reinterpret_cast<uint32_t *>(g->d_ctr);
+    a.defer_min = td ? 0 : p.defer_min;
+    a.defer_cnt = reinterpret_cast<uint32_t *>(g->d_ctr + 3);
+    a.defer_list = g->d_defer;
     a.k = k; a.max_depth = p.max_depth; a.block_central = p.block_central ? 1 : 0; a.extract_mode = p.extract_mode;
     a.level_cover = p.level_cover;
     a.containment = p.containment;
@@ -601,7 +608,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.large_hash = g->large_hash; a.large_nodes = g->large_nodes; a.large_arcs = g->large_arcs;
     a.big_hash = g->big_hash; a.big_nodes = g->big_nodes; a.big_arcs = g->big_arcs;
     a.huge_hash = g->huge_hash; a.huge_nodes = g->huge_nodes; a.huge_arcs = g->huge_arcs;
-    CUDA_TRY(cudaMemsetAsync(g->bars, 0, sizeof(GroupBar) * (size_t)G, s));   // monotonic group barriers
+    CUDA_TRY(cudaMemsetAsync(g->bars, 0, sizeof(GroupBar) * (size_t)(G + 1), s));   // monotonic group barriers
     CUDA_TRY(cudaEventRecord(g->ev[0], s));
     CUDA_TRY(launch_engine(a, g->grid, s));
     CUDA_TRY(cudaEventRecord(g->ev[1], s));

@@ -2369,6 +2369,98 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
 #ifndef KGS_MINB
 #define KGS_MINB 2   // CTAs per SM the register budget is sized for
 #endif
+// One query of the batch, end to end, by the CTAs of group G (s_q: the query index and its keywords,
+// staged in shared memory by the caller).
+__device__ __forceinline__ void run_query(const EngineArgs &a, const Grp &G, const DevWork &w, BigTile &s_big,
+                                       long long *sh, char *dsmem, const int32_t *s_q) {
+    __shared__ Q s_query;   // written by thread 0 after the previous query's last group barrier
+    if (threadIdx.x == 0) {
+        s_query.qi = s_q[0];
+        s_query.q = s_q[1];
+        s_query.full = (1u << s_query.q) - 1u;
+        for (int i = 0; i < kMaxQ; ++i) s_query.kw[i] = s_q[2 + i];
+    }
+    __syncthreads();
+    const Q &qq = s_query;
+    bool bad = qq.q < 1 || qq.q > kMaxQ;   // device-side validation (kgs_query_batch_device)
+    for (int i = 0; !bad && i < qq.q; ++i) {
+        if (qq.kw[i] < 0 || qq.kw[i] >= a.g.n_kw) bad = true;
+        for (int j = 0; j < i; ++j) if (qq.kw[j] == qq.kw[i]) bad = true;
+    }
+    if (bad) {
+        if (G.gtid() == 0) {
+            QOut *qo = a.qout + qq.qi;
+            qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
+            qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1; qo->n_cut = 0;
+        }
+        G.sync();
+        return;
+    }
+    const uint32_t done = __ldcg(w.gstate + 1);
+    Ctl *ctl = w.ctl[done & 1];
+    {   // zero this query's control block
+        uint32_t *cw = reinterpret_cast<uint32_t *>(ctl);
+        for (int64_t j = G.gtid(); j < (int64_t)(sizeof(Ctl) / 4); j += G.gsz) cw[j] = 0u;
+    }
+    QOut *qo = a.qout + qq.qi;
+    if (G.gtid() == 0) {
+        qo->n_stamp = 0; qo->t_start = globaltimer_ns();
+        qo->group = a.G > 1 && G.gcount == (int)gridDim.x ? a.G : G.g;   // a.G: the whole grid (deferred)
+    }
+    G.sync();
+    stamp(G, qo, TS_START);
+    const int rns = rec_stripes(G);
+    const Ctx c{a, w, ctl, G, qq, rns, G.grank % rns, w.pcap / rns};
+    if (a.td_only) td_only_prepare(c, qo);
+    else search(c, s_big, sh, qo);
+    // a query group that finds more than defer_min central nodes leaves the query to the whole grid at the
+    // end of the launch (its top-down parallelises over every CTA; on 1/G of the GPU it held the batch)
+    const bool defer = a.defer_min > 0 && G.gcount < (int)gridDim.x && !a.search_only &&
+                       __ldcg(&ctl->n_central) > (uint32_t)a.defer_min;
+    if (defer) {
+        if (G.gtid() == 0) a.defer_list[atomicAdd(a.defer_cnt, 1u)] = qq.qi;
+    } else if (!a.search_only) {
+        topdown(c, s_big, sh, dsmem, qo);   // search_only: workload analysis (no answers)
+    }
+    if (G.gtid() == 0) {
+        if (!defer) {
+            qo->levels = ctl->levels;
+            qo->stop_reason = ctl->stop_reason;
+            qo->count = (int32_t)ctl->sel_count;
+            qo->fatal = ctl->fatal;
+            qo->n_central = ctl->n_central;
+            qo->n_overflow = ctl->n_overflow;
+            qo->n_cid = ctl->n_cid;
+            qo->n_parcs = ctl->n_parcs;
+            qo->n_eval = ctl->n_eval;
+            qo->n_tier4 = ctl->n_tier4;
+            qo->pull_level = ctl->pull_at - 1;
+            qo->n_cut = (int32_t)ctl->n_cut;
+            qo->frontier_total = ctl->frontier_total;
+            qo->arcs_scanned = ctl->arcs_scanned;
+            qo->hits = ctl->hits;
+            qo->dag_arcs = ctl->dag_arcs;
+            qo->td_arcs = ctl->td_arcs;
+            qo->td_arcs_big = ctl->td_arcs_big;
+            qo->t_end = globaltimer_ns();
+        }
+        w.gstate[1] = done + 1;
+        // after a top-down-only query the next one resets densely; bit 1: a recorded-DAG query left its
+        // compact ids (search() "Predecessor-list state")
+        w.gstate[2] = a.td_only ? 0u : (1u | (ctl->rec_used || a.dag_record ? 2u : 0u));
+        w.gstate[3] = (uint32_t)a.R;
+    }
+    G.sync();
+}
+
+__device__ __forceinline__ void stage_query(const EngineArgs &a, int32_t *s_q, uint32_t qi) {
+    s_q[0] = (int32_t)qi;
+    if (qi < (uint32_t)a.nq) {
+        s_q[1] = a.qconst > 0 ? a.qconst : a.qlen[qi];
+        for (int i = 0; i < kMaxQ; ++i) s_q[2 + i] = a.kw[(int64_t)qi * kMaxQ + i];
+    }
+}
+
 __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
     // one dynamic shared region, reused phase by phase: expansion tiles (search, pre-pass), the per-warp
     // tier-1 extraction arenas (top-down), the rank sort of the selection
@@ -2390,91 +2482,41 @@ __global__ void __launch_bounds__(kBlock, KGS_MINB) k_engine(EngineArgs a) {
         G.episode = 0;
     }
     __syncthreads();
-    const Grp &G = s_grp;
     for (int t = threadIdx.x; t < kFlagSlots; t += blockDim.x) cta_flags()[t] = 0u;   // (synced below)
-    const DevWork &w = a.works[G.g];
+    // phase 1: each group takes the batch's queries one by one; phase 2 (query groups only): the deferred
+    // queries, every CTA of the grid as one group (group 0's workspace, barrier a.bars[G])
+    bool fin = false;
+    uint32_t t_def = 0, n_def = 0;
     for (;;) {
-        // the group leader takes the next query of the batch
-        if (G.gtid() == 0) {
-            const uint32_t qi = atomicAdd(a.next_query, 1u);
-            w.gstate[0] = qi;
-        }
-        G.sync();
-        if (threadIdx.x == 0) {
-            const uint32_t qi = __ldcg(w.gstate);
-            s_q[0] = (int32_t)qi;
-            if (qi < (uint32_t)a.nq) {
-                s_q[1] = a.qconst > 0 ? a.qconst : a.qlen[qi];
-                for (int i = 0; i < kMaxQ; ++i) s_q[2 + i] = a.kw[(int64_t)qi * kMaxQ + i];
-            }
-        }
-        __syncthreads();
-        if (s_q[0] >= a.nq) break;
-        __shared__ Q s_query;   // written by thread 0 after the previous query's last group barrier
-        if (threadIdx.x == 0) {
-            s_query.qi = s_q[0];
-            s_query.q = s_q[1];
-            s_query.full = (1u << s_query.q) - 1u;
-            for (int i = 0; i < kMaxQ; ++i) s_query.kw[i] = s_q[2 + i];
-        }
-        __syncthreads();
-        const Q &qq = s_query;
-        bool bad = qq.q < 1 || qq.q > kMaxQ;   // device-side validation (kgs_query_batch_device)
-        for (int i = 0; !bad && i < qq.q; ++i) {
-            if (qq.kw[i] < 0 || qq.kw[i] >= a.g.n_kw) bad = true;
-            for (int j = 0; j < i; ++j) if (qq.kw[j] == qq.kw[i]) bad = true;
-        }
-        if (bad) {
-            if (G.gtid() == 0) {
-                QOut *qo = a.qout + qq.qi;
-                qo->stop_reason = KGS_STOP_INVALID_QUERY; qo->count = 0; qo->levels = 0; qo->fatal = 0;
-                qo->n_central = 0; qo->n_stamp = 0; qo->group = G.g; qo->pull_level = -1; qo->n_cut = 0;
-            }
+        if (!fin) {
+            const Grp &G = s_grp;
+            const DevWork &w = a.works[G.g];
+            if (G.gtid() == 0) w.gstate[0] = atomicAdd(a.next_query, 1u);   // the group leader takes the next query
             G.sync();
-            continue;
+            if (threadIdx.x == 0) stage_query(a, s_q, __ldcg(w.gstate));
+            __syncthreads();
+            if (s_q[0] >= a.nq) {
+                if (a.G == 1 || a.defer_min <= 0) break;
+                if (threadIdx.x == 0) {
+                    Grp &Gf = s_grp;
+                    Gf.g = 0; Gf.grank = blockIdx.x; Gf.gcount = gridDim.x;
+                    Gf.gsz = (int64_t)Gf.gcount * blockDim.x;
+                    Gf.bar = a.bars + a.G;
+                    Gf.episode = 0;
+                }
+                __syncthreads();
+                s_grp.sync();   // every group is done: the deferred list is complete
+                n_def = __ldcg(a.defer_cnt);
+                fin = true;
+            }
         }
-        const uint32_t done = __ldcg(w.gstate + 1);
-        Ctl *ctl = w.ctl[done & 1];
-        {   // zero this query's control block
-            uint32_t *cw = reinterpret_cast<uint32_t *>(ctl);
-            for (int64_t j = G.gtid(); j < (int64_t)(sizeof(Ctl) / 4); j += G.gsz) cw[j] = 0u;
+        if (fin) {
+            if (t_def >= n_def) break;
+            if (threadIdx.x == 0) stage_query(a, s_q, (uint32_t)__ldcg(a.defer_list + t_def));
+            ++t_def;
+            __syncthreads();
         }
-        QOut *qo = a.qout + qq.qi;
-        if (G.gtid() == 0) { qo->n_stamp = 0; qo->t_start = globaltimer_ns(); qo->group = G.g; }
-        G.sync();
-        stamp(G, qo, TS_START);
-        const int rns = rec_stripes(G);
-        const Ctx c{a, w, ctl, G, qq, rns, G.grank % rns, w.pcap / rns};
-        if (a.td_only) td_only_prepare(c, qo);
-        else search(c, s_big, sh, qo);
-        if (!a.search_only) topdown(c, s_big, sh, dsmem, qo);   // search_only: workload analysis (no answers)
-        if (G.gtid() == 0) {
-            qo->levels = ctl->levels;
-            qo->stop_reason = ctl->stop_reason;
-            qo->count = (int32_t)ctl->sel_count;
-            qo->fatal = ctl->fatal;
-            qo->n_central = ctl->n_central;
-            qo->n_overflow = ctl->n_overflow;
-            qo->n_cid = ctl->n_cid;
-            qo->n_parcs = ctl->n_parcs;
-            qo->n_eval = ctl->n_eval;
-            qo->n_tier4 = ctl->n_tier4;
-            qo->pull_level = ctl->pull_at - 1;
-            qo->n_cut = (int32_t)ctl->n_cut;
-            qo->frontier_total = ctl->frontier_total;
-            qo->arcs_scanned = ctl->arcs_scanned;
-            qo->hits = ctl->hits;
-            qo->dag_arcs = ctl->dag_arcs;
-            qo->td_arcs = ctl->td_arcs;
-            qo->td_arcs_big = ctl->td_arcs_big;
-            qo->t_end = globaltimer_ns();
-            w.gstate[1] = done + 1;
-            // after a top-down-only query the next one resets densely; bit 1: a recorded-DAG query left its
-            // compact ids (search() "Predecessor-list state")
-            w.gstate[2] = a.td_only ? 0u : (1u | (ctl->rec_used || a.dag_record ? 2u : 0u));
-            w.gstate[3] = (uint32_t)a.R;
-        }
-        G.sync();
+        run_query(a, s_grp, a.works[s_grp.g], s_big, sh, dsmem, s_q);
     }
 }
 

@@ -193,6 +193,9 @@ struct EngineArgs {
     const int32_t *qlen;        // [nq]
     int qconst;                 // > 0: every query has this many keywords (qlen unused)
     uint32_t *next_query;       // global query counter
+    int defer_min;              // query groups: a query with more central nodes is left to the whole grid
+    uint32_t *defer_cnt;        // deferred queries so far
+    int32_t *defer_list;        // [nq] their indices
     // parameters (shared by the batch)
     int k, max_depth, block_central, extract_mode, level_cover;   // level_cover: 0 off, 1 R13, 2 R13b
     int containment;            // NEXT-3 R16: drop Central Graphs that strictly contain another one

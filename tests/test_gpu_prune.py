@@ -253,3 +253,37 @@ def test_key_cutoff_per_candidate_multi_keyword_sources():
                 cuts_off += r.stats["n_cut"]
         G.close()
     assert cuts_off == 0 and cuts_on > 0, (cuts_on, cuts_off)
+
+
+def test_deferred_queries_run_on_the_whole_grid():
+    """In a launch of query groups, a query with more than defer_min central nodes is left to the end of
+    the launch, where every CTA answers it as one group (kgs_stats.group == n_groups).  Answers equal the
+    oracle's with deferral on (several deferred queries, mixed with ordinary ones) and off, and a later
+    single-query launch on the same workspaces is unaffected."""
+    _gpu()
+    g = medium_graph(21, n=20000, deg=8, q=4, kw_size=150)
+    G = kgs.kgs_load_graph(g)
+    rng = np.random.default_rng(21)
+    qs = [sorted(rng.choice(4, size=int(rng.integers(2, 5)), replace=False).tolist()) for _ in range(24)]
+    exp = {tuple(kw): oracle.query(g, kw, 20) for kw in map(tuple, qs)}
+    ncs = sorted(len(o.centrals) for o in exp.values())
+    thr = ncs[len(ncs) // 2]   # about half of the queries are deferred
+    for dmin, groups in ((thr, 4), (thr, 8), (0, 4), (1, 3)):
+        res = kgs.kgs_query_batch(G, qs, 20, kgs.make_params(defer_min=dmin), groups)
+        deferred = 0
+        for kw, r in zip(qs, res):
+            o = exp[tuple(kw)]
+            ctx = f"defer_min={dmin} G={groups} kw={kw} |C|={len(o.centrals)}"
+            assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
+            for ra, oa in zip(r.answers, o.answers):
+                assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist(), ctx
+                assert ra.arcs.tolist() == oa.arcs.tolist(), ctx
+            assert r.stats["stop_reason"] == o.stop_reason and r.stats["levels"] == o.levels, ctx
+            should = dmin > 0 and len(o.centrals) > dmin
+            assert (r.stats["group"] == groups) == should, ctx
+            deferred += should
+        if dmin:
+            assert deferred > 0
+    r = kgs.kgs_query(G, qs[0], 20)
+    assert [a.central for a in r.answers] == [a.central for a in exp[tuple(qs[0])].answers]
+    G.close()
