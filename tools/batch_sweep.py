@@ -26,18 +26,22 @@ for i, q in enumerate(qs):
 kwd = kwp.cuda()
 qld = torch.tensor([len(q) for q in qs], dtype=torch.int32, device="cuda")
 s = torch.cuda.current_stream()
+# PARAMS="defer_min=0 mk_min=4096": kgs_params overrides
+params = kgs.make_params(**{k: int(v) for k, v in (x.split("=") for x in os.environ.get("PARAMS", "").split())})
 for g in groups:
     for rep in range(3):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         e0.record(s)
-        kgs.kgs_query_batch_device(G, len(qs), kwd.data_ptr(), qld.data_ptr(), w.k, None, g, s.cuda_stream)
+        kgs.kgs_query_batch_device(G, len(qs), kwd.data_ptr(), qld.data_ptr(), w.k, params, g, s.cuda_stream)
         e1.record(s)
         res = kgs.kgs_query_batch_fetch(G, [len(q) for q in qs], s.cuda_stream)
         ms = e0.elapsed_time(e1)
         lat = sorted(r.stats["ms_total"] for r in res)
     print(f"{name} G={g:3d} batch={len(qs)} launch {ms:8.2f} ms  {len(qs) / ms * 1e3:9.1f} q/s  "
-          f"query latency p50 {lat[len(lat) // 2]:.3f} ms p95 {lat[int(len(lat) * .95)]:.3f} ms", flush=True)
+          f"query latency p50 {lat[len(lat) // 2]:.3f} ms p95 {lat[int(len(lat) * .95)]:.3f} ms "
+          f"deferred {sum(r.stats['group'] == g for r in res) if g > 1 else 0} "
+          f"max {lat[-1]:.1f} ms  {os.environ.get('PARAMS', '')}", flush=True)
     ph = {}
     for r in res:
         for k, v in r.stats["phases_us"].items():

@@ -57,10 +57,15 @@ for r in raw[2:]:
     res["dram_bytes_per_launch"] = rd + wr
     res["dram_bytes_per_query"] = (rd + wr) / nq
     res["l2_hit_pct"] = float(d["lts__t_sector_hit_rate.pct"])
-json.dump(res, open(os.path.join(ROOT, "profiles", f"{tag}_batch_traffic.json"), "w"), indent=1)
+# (kernel replay: the DRAM bytes of the last pass; bench.py's roofline.traffic comes from the single-pass
+# capture of tools/make_traffic.py instead)
+json.dump(res, open(os.path.join(ROOT, "profiles", f"{tag}_batch_fullset.json"), "w"), indent=1)
 out = [f"# Batch-launch profile {tag} — k_engine, {res['launch']}", "",
        "`ncu --set full --import-source on --clock-control none` of one launch (tools/gpu_ncu_batch.sh).  "
-       "Times under ncu are not bench values.", ""]
+       "Times under ncu are not bench values.  Kernel replay restores memory before each of ~40 passes; the "
+       "work of the pass whose counters are shown can differ from the bench launch's (see the launch lines of "
+       "profile_batch.py) — the DRAM bytes per launch behind bench.py's roofline.traffic come from a "
+       "single-pass capture (tools/make_traffic.py, <tag>_batch_traffic.json).", ""]
 if "dram_bytes_per_launch" in res:
     out.append(f"* DRAM traffic per launch: {res['dram_bytes_per_launch'] / 1e9:.1f} GB "
                f"({res['dram_bytes_per_query'] / 1e6:.0f} MB per query)")
