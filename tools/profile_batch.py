@@ -17,8 +17,8 @@ groups = int(sys.argv[3]) if len(sys.argv) > 3 else 8
 over = dict(a.split("=") for a in sys.argv[4:])
 params = kgs.make_params(**{k: int(v) for k, v in over.items()})
 w = synth.make_workload(name)
-order = np.random.default_rng(12345).permutation(len(w.queries))
-qs = [w.queries[i] for i in order]
+from bench import step_queries  # noqa: E402  (the bench's query order: C3 permuted, C4 as generated)
+qs, _ = step_queries(name, w.queries)
 G = kgs.kgs_load_graph(w.graph)
 if os.environ.get("L2GRAN"):   # experiment: cudaLimitMaxL2FetchGranularity (0x05) on the primary context
     import ctypes
