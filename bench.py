@@ -45,6 +45,9 @@ WORKLOAD = "C4"      # the step's batch: C4's 4096 queries (configs[3]) or C3's 
 # sample (cpu_baseline, --impl reference) skips them and says so.
 ORACLE_SKIP = {"C4": (11, 1422, 1619, 2557, 2683, 2906, 3629)}
 GROUPS = 8           # engine groups in batch mode (queries answered at the same time)
+# DRAM bytes/s a stream of independent random 4-byte gathers moves on this B200 (37.7 G gathers/s, 124 B of
+# DRAM read per gather: tools/rand_gather_bench.cu, profiles/r02d_random_access.txt)
+RANDOM_GATHER_DRAM_GBS = 37.7 * 124
 RELABEL = os.environ.get("KGS_RELABEL", "1") != "0"   # ablation: 0 keeps the input node order internally
 
 
@@ -497,7 +500,17 @@ def main():
                      # batch = summed group expansion time / G (groups expand concurrently)
                      "expansion_achieved": exp_lat, "expansion_frac": (exp_lat / peak) if exp_lat else None,
                      "expansion_frac_batch_est": (exp_bat / peak) if exp_bat else None,
-                     "expansion_bytes_per_query": (lat_exp_b / len(lat_stats)) if lat_stats else None},
+                     "expansion_bytes_per_query": (lat_exp_b / len(lat_stats)) if lat_stats else None,
+                     # what the DRAM actually moved (the ncu capture's bytes per query x queries / the step
+                     # time) against what a pure random 4-byte gather stream moves on this part (37.7 G
+                     # gathers/s x 124 B of DRAM each, profiles/r02d_random_access.txt): the engine's
+                     # accesses are random lines, so this, not the algorithmic bytes, is how close the
+                     # launch runs to its memory system's ceiling for this access pattern
+                     "dram_achieved": (tr * len(allq) / (dev_ms / args.steps / 1e3) / 1e9) if tr else None,
+                     "dram_frac": (tr * len(allq) / (dev_ms / args.steps / 1e3) / 1e9 / peak) if tr else None,
+                     "random_gather_dram_ceiling": RANDOM_GATHER_DRAM_GBS,
+                     "random_gather_frac": (tr * len(allq) / (dev_ms / args.steps / 1e3) / 1e9 /
+                                            RANDOM_GATHER_DRAM_GBS) if tr else None},
         "e2e": {"value": e2e_qps, "unit": "queries/s", "ms_per_step": statistics.median(e2e_ms),
                 "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world / len(e2e_ms)},
         "gpu_launches": args.steps,   # one k_engine launch per step (per rank)

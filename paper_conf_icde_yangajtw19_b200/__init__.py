@@ -96,7 +96,8 @@ EXPORTED = ["kgs_load_graph", "kgs_free_graph", "kgs_params_default", "kgs_query
             "kgs_result_export"]
 
 PHASE_NAMES = ["start", "reset", "sources", "merge", "expand", "pd_seed", "pd_merge", "pd_expand", "pd_csr",
-               "search_end", "extract", "extract_big", "select", "emit"]
+               "search_end", "extract", "extract_big", "select", "emit", "pd_merge2", "pd_expand2", "extract2",
+               "mk_reach"]
 KGS_STOP_INVALID_QUERY = -1
 KGS_STOP_CAPACITY = -2
 

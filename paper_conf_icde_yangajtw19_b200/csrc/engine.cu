@@ -690,7 +690,7 @@ __device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cn
 
 __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo);
 
-__device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
+__device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo, bool round2 = false) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const bool exact_block = c.a.extract_mode == KGS_EXTRACT_EXACT && c.a.block_central;
@@ -720,7 +720,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         if (compact_deferred(G, c.w.qdef, __ldcg(&ctl->pd_ndef[slot]), c.w.pd_qlight, c.a.g.cls_in, c.w.pd_qbig,
                              &qn[1], c.w.pd_touched, &ctl->n_cid, pd_node, pd_aux))
             G.sync();
-        stamp(G, qo, TS_PD_MERGE);
+        stamp(G, qo, round2 ? TS_PD_MERGE2 : TS_PD_MERGE);
         const uint32_t c0 = __ldcg(&qn[0]), c1 = __ldcg(&qn[1]);
         if (G.gtid() == 0) ctl->pd_flag[slot] = 0u;
         uint32_t *nbits = c.w.pd_bits + (int64_t)(slot ^ 1) * W;
@@ -735,7 +735,7 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                                  G.gcount <= kDynBatchCtas ? &ctl->pd_xbatch[slot] : nullptr);
         publish_flags(ctl);
         G.sync();
-        stamp(G, qo, TS_PD_EXPAND);
+        stamp(G, qo, round2 ? TS_PD_EXPAND2 : TS_PD_EXPAND);
     }
     if (my_arcs + my_arcs_big) atomicAdd(&ctl->td_arcs, my_arcs + my_arcs_big);
     if (my_arcs_big) atomicAdd(&ctl->td_arcs_big, my_arcs_big);
@@ -2121,7 +2121,7 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         }
     }
     G.sync();
-    stamp(G, qo, TS_EXTRACT);
+    stamp(G, qo, cut < kNoCut ? TS_EXTRACT2 : TS_EXTRACT);
     const uint32_t no = __ldcg(&ctl->n_overflow);
     BlockTeam BT{sh};
     if (no) {
@@ -2342,13 +2342,16 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             n2 = __ldcg(&ctl->n_elist2);
             if (!rec) {
                 seed_pd(c, c.w.elist + m, n2);
-                pred_dag(c, S, sh, qo);
+                pred_dag(c, S, sh, qo, true);
             }
             // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union);
             // with many candidates, which of them can have s* >= 2 is decided per candidate (mk_reach)
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
             if (!a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min && (__ldcg(&ctl->multi_kw) & c.qq.full))
+            {
                 mk_reach(c);
+                stamp(G, qo, TS_MK);
+            }
             extract_list(c, sh, dsmem, c.w.elist + m, n2, qo, cut);
         }
         if (G.gtid() == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }

@@ -114,7 +114,8 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 }
 // tags of the phase stamps
 enum { TS_START = 0, TS_RESET, TS_SCATTER, TS_MERGE, TS_EXPAND, TS_PD_SEED, TS_PD_MERGE, TS_PD_EXPAND, TS_PD_CSR,
-       TS_END, TS_EXTRACT, TS_EXTRACT_BIG, TS_SELECT, TS_EMIT };
+       TS_END, TS_EXTRACT, TS_EXTRACT_BIG, TS_SELECT, TS_EMIT,
+       TS_PD_MERGE2, TS_PD_EXPAND2, TS_EXTRACT2, TS_MK };   // pruning round 2's pre-pass and extraction
 
 struct DevGraph {
     int64_t n, m;

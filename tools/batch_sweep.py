@@ -49,3 +49,14 @@ for g in groups:
     tot = sum(ph.values()) or 1.0
     print("   group-time share: " + " ".join(f"{k}={v / tot:.1%}" for k, v in sorted(ph.items(), key=lambda x: -x[1])),
           flush=True)
+    # the same split by query class: |C| <= 512 (no pruning: every central extracted) and > 512
+    for lo, hi in ((0, 512), (513, 10 ** 5), (10 ** 5 + 1, 10 ** 9)):
+        sub = [r for r in res if lo <= r.stats["n_centrals"] <= hi]
+        if not sub:
+            continue
+        ph = {}
+        for r in sub:
+            for k, v in r.stats["phases_us"].items():
+                ph[k] = ph.get(k, 0.0) + v
+        print(f"   |C| in [{lo}, {hi}]: {len(sub)} queries, group time {sum(ph.values()) / tot:.1%} of all: " +
+              " ".join(f"{k}={v / tot:.1%}" for k, v in sorted(ph.items(), key=lambda x: -x[1])[:6]), flush=True)

@@ -10,6 +10,10 @@ import oracle  # noqa: E402
 import paper_conf_icde_yangajtw19_b200 as kgs  # noqa: E402
 import synth  # noqa: E402
 
+# SAN_PARAMS="mk_min=0 prune_min=40 defer_min=20": kgs_params overrides for both launch kinds (drives the
+# per-candidate cut-off test and the deferred whole-grid queries on the small configs)
+P = os.environ.get("SAN_PARAMS", "")
+params = kgs.make_params(**{k: int(v) for k, v in (x.split("=") for x in P.split())}) if P else None
 n1 = int(sys.argv[1]) if len(sys.argv) > 1 else 100
 n2 = int(sys.argv[2]) if len(sys.argv) > 2 else 3
 bad = 0
@@ -20,8 +24,8 @@ for name, cnt in (("C1", n1), ("C2", n2)):
     qs = w.queries[:cnt] if name == "C1" else w.queries[::97][:cnt]
     exp = [oracle.query(w.graph, kw, w.k) for kw in qs]
     G = kgs.kgs_load_graph(w.graph)
-    single = [kgs.kgs_query(G, kw, w.k) for kw in qs]
-    batch = kgs.kgs_query_batch(G, qs, w.k, None, 4)
+    single = [kgs.kgs_query(G, kw, w.k, params) for kw in qs]
+    batch = kgs.kgs_query_batch(G, qs, w.k, params, 4)
     for kw, o, r1, r2 in zip(qs, exp, single, batch):
         want = [(a.central, a.key, a.nodes.tolist(), a.arcs.tolist()) for a in o.answers]
         for r in (r1, r2):
