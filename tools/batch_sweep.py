@@ -59,4 +59,4 @@ for g in groups:
             for k, v in r.stats["phases_us"].items():
                 ph[k] = ph.get(k, 0.0) + v
         print(f"   |C| in [{lo}, {hi}]: {len(sub)} queries, group time {sum(ph.values()) / tot:.1%} of all: " +
-              " ".join(f"{k}={v / tot:.1%}" for k, v in sorted(ph.items(), key=lambda x: -x[1])[:6]), flush=True)
+              " ".join(f"{k}={v / tot:.1%}" for k, v in sorted(ph.items(), key=lambda x: -x[1])[:12]), flush=True)
