@@ -585,6 +585,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
     a.prune_min = p.prune_min;
     a.mk_min = p.mk_min;
+    a.rm_ok = !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
         // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass.
         // Auto: on for the single-query (latency) launch, where the pre-pass's rounds of group barriers

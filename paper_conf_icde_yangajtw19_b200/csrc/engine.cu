@@ -138,6 +138,12 @@ __device__ __forceinline__ uint64_t ldrow(const uint8_t *M, int32_t v) {
 // gate (L210): 0 for a keyword node, else a_v
 __device__ __forceinline__ uint32_t st_gate(uint32_t s) { return (s & 0x100u) ? 0u : (s >> 24); }
 __device__ __forceinline__ uint32_t st_nm(uint32_t s) { return (s >> 16) & 0xFFu; }
+// byte 1 bits 1-7 (rm): keyword i < 7 is reached from a node holding i and another query keyword along
+// hitting arcs of keyword i (set at the level-0 merge for such sources, carried by visit_arc's reduction).
+// In the exact reading the hitting arcs are the Thm. V.4 predecessor arcs, so rm(c) is exactly the set of
+// keywords for which a two-keyword source lies in DAG_i(c) (central_graph's key cut-off validity).
+constexpr uint32_t kRmMask = 0x7Fu;
+__device__ __forceinline__ uint32_t st_rm(uint32_t s) { return (s >> 9) & kRmMask; }
 __device__ __forceinline__ uint32_t st_act(uint32_t s) { return s >> 24; }
 // the status word of a node nobody has hit yet: not a keyword node, a
 __device__ __forceinline__ uint32_t st_fresh(uint32_t a) { return a << 24; }
@@ -350,7 +356,7 @@ __device__ __forceinline__ uint32_t weight_fx(float wt) {
 }
 
 // One inspected arc v -> x of Alg. 2 ln 12-22, for all keywords of v at once (hmv = v's snapshot mask,
-// sx = st[x] gathered by the caller).
+// zbv = v's source bits (recorded DAG only) | rm(v) << 8, sx = st[x] gathered by the caller).
 __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32_t hmv, uint32_t zbv, int32_t x,
                                           uint32_t sx, unsigned &dag) {
     const uint32_t bits = hmv & ~sx & 0xFFu;            // ln 13-15: only instances where x is unhit
@@ -368,7 +374,7 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
                 const int64_t r = stripe * rcap + ai;
                 c.w.pa_u[r] = v;
                 c.w.pa_x[r] = x;
-                c.w.pa_b[r] = (uint16_t)(bits | (zbv << 8));
+                c.w.pa_b[r] = (uint16_t)(bits | ((zbv & 0xFFu) << 8));
             }
         }
         if (c.a.prune == 2) {   // x is hit at l+1 for these keywords: v is a Thm. V.4 predecessor of (x, i)
@@ -381,7 +387,9 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
         // writes the same level l+1 into entries whose hit bit was clear at the level's start, and the
         // frontier push is a bit set, so repeating them for arcs that lost a race changes nothing (Thm. V.2).
         // The new (node, keyword) pairs are counted when the next merge folds nm into hm.
-        asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(c.w.st + x), "r"(bits << 16) : "memory");
+        // with the new-hit bits, the keywords of these that a two-keyword source reaches v in (rm, byte 1)
+        const uint32_t red = (bits << 16) | ((bits & (zbv >> 8) & kRmMask) << 9);
+        asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(c.w.st + x), "r"(red) : "memory");
         uint8_t *row = c.w.M + (int64_t)x * 8;
         const uint8_t lv = (uint8_t)(l + 1);
 #pragma unroll
@@ -399,8 +407,9 @@ __device__ __forceinline__ void visit_arc(const Ctx &c, int l, int32_t v, uint32
 }
 
 // Alg. 2 ln 2-7 for node v at level l: returns its expansion mask (0 = does not expand now).
-__device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool leader) {
+__device__ __forceinline__ uint32_t prepare(const Ctx &c, int l, int32_t v, bool leader, uint32_t &rm) {
     const uint32_t sv = __ldcg(c.w.st + v);
+    rm = st_rm(sv);
     const uint32_t hm = sv & 0xFFu;
     if (c.a.block_central && hm == c.qq.full) return 0;   // ln 2-3: central nodes do not expand
     const int av = (int)st_act(sv);
@@ -931,7 +940,7 @@ __device__ __forceinline__ void pull_expand(const Ctx &c, int l, BigTile &S, lon
                 if (((row >> (8 * i)) & 0xFF) == 0) zb |= 1u << i;
             }
         }
-        visit_arc(c, l, u, hmu, zb, nd.x, nd.sx, my_dag);
+        visit_arc(c, l, u, hmu, zb | (st_rm(su) << 8), nd.x, nd.sx, my_dag);
     };
     expand_light<PullNode>(G, nullptr, (uint32_t)n, a.g.in_ptr, a.g.in_idx, w.st, plight, pvisit, my_arcs);
     G.sync();
@@ -1121,11 +1130,12 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
                         my_mf += cls_deg_bound(a.g.cls[v]);
                     const uint32_t b = st_nm(sv);
                     if (!b) return false;
-                    if (l == 0 && (b & (b - 1))) atomicOr(&ctl->multi_kw, b);   // v holds >= 2 query keywords
+                    uint32_t rself = 0;   // a source of two or more query keywords reaches itself (st_rm)
+                    if (l == 0 && (b & (b - 1))) { atomicOr(&ctl->multi_kw, b); rself = (b & kRmMask) << 9; }
                     if (l > 0) my_hits += __popc(b);   // new (node, keyword) pairs of level l - 1's expansion
                     const uint32_t old = sv & 0xFFu;
                     const uint32_t nw = old | b;
-                    w.st[v] = (sv & 0xFF00FF00u) | nw;     // hm |= nm, nm = 0 (no expansion runs during the merge)
+                    w.st[v] = (sv & 0xFF00FF00u) | nw | rself;   // hm |= nm, nm = 0 (no expansion runs during the merge)
                     if (a.prune == 2) {   // lightest path to v for keyword i = min over predecessors + w_v
                         const uint32_t wv = weight_fx(__ldg(a.g.weight + v));
                         for (uint32_t bb = b; bb; bb &= bb - 1) {
@@ -1215,8 +1225,9 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
         }
         auto prep = [&](int32_t v, bool leader, FwdNode &nd) {
             nd.v = v;
-            nd.hm = prepare(c, l, v, leader);
-            nd.zb = 0;
+            uint32_t rm;
+            nd.hm = prepare(c, l, v, leader, rm);
+            nd.zb = rm << 8;   // zb (recorded DAG) in bits 0-7, rm in bits 8-14
             if (a.dag_record && nd.hm) {
                 const uint64_t row = ldrow(w.M, v);
                 for (uint32_t b = nd.hm; b; b &= b - 1) {
@@ -1501,7 +1512,13 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     // s* >= 2 needs sources holding >= 2 query keywords that cover Q with zb(c): multi is the union of
     // the keyword sets of such nodes (graph-wide), or per candidate the keywords i for which one of them
     // reaches c inside DAG_i (the shared predecessor DAG's arcs, pd_state byte 3, mk_reach)
-    const uint32_t reach = c.a.level_cover == 1 && c.ctl->mk_reach ? (__ldcg(c.w.pd_state + cn) >> 24) : multi;
+    uint32_t reach = multi;
+    if (c.a.level_cover == 1 && c.a.rm_ok)   // rm: exact for keywords 0-6, keyword 7 assumed reached
+        reach &= st_rm(__ldcg(c.w.st + cn)) | (c.qq.q > 7 ? ~kRmMask : 0u);
+    if (c.a.level_cover == 1 && c.ctl->mk_reach) {   // mk_reach's fixpoint, per compact id (in pcnt)
+        const int32_t cid = __ldcg(c.w.pd_cid + cn);
+        if (cid >= 0) reach &= (uint32_t)__ldcg(c.w.pcnt + cid);
+    }
     const bool cut_on = cut < kNoCut &&
                         (!c.a.level_cover || ((reach | zbc) & full) != full);
     auto over_cut = [&]() {   // the closure weight so far, times d^lambda, already exceeds the cut
@@ -2347,7 +2364,8 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union);
             // with many candidates, which of them can have s* >= 2 is decided per candidate (mk_reach)
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
-            if (!a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min && (__ldcg(&ctl->multi_kw) & c.qq.full))
+            if (!a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min && (__ldcg(&ctl->multi_kw) & c.qq.full) &&
+                (!a.rm_ok || c.qq.q > 7))
             {
                 mk_reach(c);
                 stamp(G, qo, TS_MK);

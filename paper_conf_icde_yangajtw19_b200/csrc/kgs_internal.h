@@ -207,6 +207,7 @@ struct EngineArgs {
     int prune;                  // top-down pruning: 0 off, 1 bound w_c, 2 bound max_i lightest path_i
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
     int mk_min;                 // round 2: per-candidate s* >= 2 test (mk_reach) from this many candidates
+    int rm_ok;                  // the search's rm bits decide the s* >= 2 test (hitting arcs = Thm. V.4 arcs)
     int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
     int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
     int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio

@@ -287,3 +287,60 @@ def test_deferred_queries_run_on_the_whole_grid():
     r = kgs.kgs_query(G, qs[0], 20)
     assert [a.central for a in r.answers] == [a.central for a in exp[tuple(qs[0])].answers]
     G.close()
+
+
+def test_key_cutoff_never_drops_a_two_level_winner():
+    """Hand-built: the Central Graph that must win keeps only two-keyword sources (s* = 2), while its whole
+    closure is heavy.  Keywords A, B, C (q = 3), every activation level 0 (A = 0.1).  Candidate c (w 0.5)
+    is joined to m1 (holds A, B) and m2 (holds B, C), both of weight 0, and to 20 nodes of each keyword of
+    weight 0.9: level-cover keeps {c, m1, m2} (m1, m2 contribute two keywords each and cover Q), key 0.5;
+    its closure weighs 54.5.  60 filler centrals (w 0.01, one heavy A, B and C neighbour each, key 2.71)
+    fill pruning round 1 (prune_min 8: the 40 smallest bounds), so c is extracted in round 2 with the cut
+    at T = 2.71: an invalid cut would drop it.  Answers must be the oracle's (c first)."""
+    _gpu()
+    n_fill, n_side = 60, 20
+    nodes = {}
+
+    def nid(name):
+        return nodes.setdefault(name, len(nodes))
+
+    edges, kws, w = [], [[], [], []], {}
+    c, m1, m2 = nid("c"), nid("m1"), nid("m2")
+    w[c], w[m1], w[m2] = 0.5, 0.0, 0.0
+    kws[0].append(m1); kws[1].append(m1); kws[1].append(m2); kws[2].append(m2)
+    edges += [(c, m1), (c, m2)]
+    for i in range(3):
+        for j in range(n_side):
+            v = nid(f"s{i}_{j}")
+            w[v] = 0.9
+            kws[i].append(v)
+            edges.append((c, v))
+    for f in range(n_fill):
+        fv = nid(f"f{f}")
+        w[fv] = 0.01
+        for i in range(3):
+            v = nid(f"f{f}_{i}")
+            w[v] = 0.9
+            kws[i].append(v)
+            edges.append((fv, v))
+    n = len(nodes)
+    wt = np.array([w[i] for i in range(n)], dtype=np.float64)
+    wt = (np.floor(wt * (1 << 24) + 0.5) / (1 << 24)).astype(np.float32)
+    g = synth.from_edges(n, edges, wt, [sorted(x) for x in kws], 0.1)
+    o = oracle.query(g, [0, 1, 2], 5)
+    assert o.answers[0].central == c and o.answers[0].nodes.tolist() == sorted([c, m1, m2])
+    G = kgs.kgs_load_graph(g)
+    runs = []
+    for mk in (0, 1 << 30):
+        for rec in (1, 0):
+            runs.append((mk, rec, kgs.kgs_query(G, [0, 1, 2], 5,
+                                                kgs.make_params(prune_min=8, mk_min=mk, dag_record=rec))))
+        for r in kgs.kgs_query_batch(G, [[0, 1, 2], [2, 1, 0]], 5, kgs.make_params(prune_min=8, mk_min=mk), 2):
+            runs.append((mk, "batch", r))
+    for mk, rec, r in runs:
+        ctx = f"mk_min={mk} rec={rec}"
+        assert r.stats["n_evaluated"] < len(o.centrals) or r.stats["n_cut"] >= 0, ctx
+        assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
+        for ra, oa in zip(r.answers, o.answers):
+            assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist(), ctx
+    G.close()
