@@ -145,7 +145,10 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *                  exact key cut-off applies to more candidates
  *   defer_min      >= 0 [65536]: in a launch of several query groups, a query that identifies more central
  *                  nodes than this is answered at the end of the launch by all CTAs together (its top-down
- *                  parallelises over the whole GPU instead of holding one group); 0 = never */
+ *                  parallelises over the whole GPU instead of holding one group); 0 = never
+ *   lazy_dag       0 / 1 [1]: pruning round 2 extends the shared predecessor DAG only as far as the
+ *                  candidates' walks need before the exact key cut-off stops them (candidates whose cut is
+ *                  valid, decided from the search's rm bits); 0 builds every round-2 closure first */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
@@ -156,6 +159,7 @@ typedef struct {
     int32_t containment;
     int32_t mk_min;
     int32_t defer_min;
+    int32_t lazy_dag;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 

@@ -167,7 +167,7 @@ namespace {
 void free_work(DevWork &w) {
     void *p[] = {w.st, w.M, w.fbits, w.qlight, w.qbig, w.touched, w.qdef, w.centrals, w.cdepth, w.ckey, w.overflow,
                  w.cflag, w.sel, w.elist, w.mw, w.ctl[0], w.ctl[1], w.pd_state, w.pd_cid, w.pd_touched, w.pd_bits, w.pd_qlight,
-                 w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp,
+                 w.pd_qbig, w.pcnt, w.pred_ptr, w.pred_u, w.pred_b, w.pa_u, w.pa_x, w.pa_b, w.pa_slot, w.scan_tmp, w.lz,
                  w.gstate, w.huge};
     for (void *x : p) if (x) cudaFree(x);
     w = DevWork{};
@@ -219,6 +219,7 @@ kgs_status alloc_work(kgs_graph *g, DevWork &w, int64_t pcap) {
     CUDA_TRY(dmalloc(&w.pa_b, (size_t)pcap));
     CUDA_TRY(dmalloc(&w.pa_slot, (size_t)pcap));
     CUDA_TRY(dmalloc(&w.scan_tmp, 4096));
+    CUDA_TRY(dmalloc(&w.lz, n));
     CUDA_TRY(dmalloc(&w.gstate, 4));
     CUDA_TRY(cudaMemset(w.gstate, 0, 4 * sizeof(uint32_t)));   // not valid: the first query resets densely
     return KGS_OK;
@@ -257,6 +258,7 @@ void kgs_params_default(kgs_params *p) {
     p->search_only = 0;
     p->mk_min = 4096;
     p->defer_min = 1 << 16;
+    p->lazy_dag = 1;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -448,9 +450,10 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.containment != 0 && p.containment != 1) return fail(KGS_EINVAL, "containment must be 0 or 1");
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
-        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0 || p.defer_min < 0)
+        p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0 || p.defer_min < 0 ||
+        (p.lazy_dag != 0 && p.lazy_dag != 1))
         return fail(KGS_EINVAL, "tuning parameters out of range (pull_ratio >= 1, pull_min >= 0, prune_min >= 1, "
-                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0, defer_min >= 0)");
+                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0, defer_min >= 0, lazy_dag 0/1)");
     return KGS_OK;
 }
 
@@ -585,6 +588,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     if (a.prune == 2 && !(p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central)) a.prune = 1;
     a.prune_min = p.prune_min;
     a.mk_min = p.mk_min;
+    a.lazy_dag = p.lazy_dag;
     a.rm_ok = !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
         // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass.

@@ -699,7 +699,8 @@ __device__ __forceinline__ void for_each_record(const Ctx &c, const uint32_t *cn
 
 __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo);
 
-__device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo, bool round2 = false) {
+__device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo, bool round2 = false,
+                         int max_rounds = 1 << 30) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const bool exact_block = c.a.extract_mode == KGS_EXTRACT_EXACT && c.a.block_central;
@@ -711,6 +712,23 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo, bool
     for (;; ++r) {
         const int slot = r & 1;
         if (!__ldcg(&ctl->pd_flag[slot])) break;
+        if (r >= max_rounds) {
+            // lazy round 2: the predecessors just found are not expanded further unless a candidate's walk
+            // asks for them — drop the next round's frontier and its pending bits (pd_state byte 1)
+            uint32_t *bits = c.w.pd_bits + (int64_t)slot * W;
+            for (int64_t j = G.gtid(); j < W; j += G.gsz) {
+                uint32_t x = __ldcg(bits + j);
+                if (!x) continue;
+                bits[j] = 0u;
+                for (; x; x &= x - 1) {
+                    const int32_t v = (int32_t)(j * 32 + __ffs(x) - 1);
+                    c.w.pd_state[v] = __ldcg(c.w.pd_state + v) & ~0xFF00u;
+                }
+            }
+            if (G.gtid() == 0) ctl->pd_flag[slot] = 0u;
+            G.sync();
+            break;
+        }
         uint32_t *qn = ctl->pd_qn[slot];
         if (G.gtid() == 0) { ctl->pd_qn[slot ^ 1][0] = 0u; ctl->pd_qn[slot ^ 1][1] = 0u; ctl->pd_ctile[slot ^ 1] = 0u;
                            ctl->pd_xbatch[slot ^ 1] = 0u; }
@@ -1345,7 +1363,7 @@ struct BlockTeam {
     __device__ __forceinline__ int scan_excl(int x, int *total) const { return block_excl_scan(x, total, sh); }
 };
 
-enum { SC_NODES = 0, SC_ARCS, SC_HEAD, SC_TAIL, SC_OVF, SC_CHANGED, SC_COV, SC_SSTAR, SC_NOUT, SC_AOUT, SC_CUT, SC_N };
+enum { SC_NODES = 0, SC_ARCS, SC_HEAD, SC_TAIL, SC_OVF, SC_CHANGED, SC_COV, SC_SSTAR, SC_NOUT, SC_AOUT, SC_CUT, SC_INC, SC_N };
 
 struct Arena {
     int32_t *hkey;      // [hcap] node id or -1
@@ -1471,6 +1489,23 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
     S.fifo[pos % S.ncap] = j;
 }
 
+// Is the closure weight a lower bound of c's key (level-cover keeps every source: s* = 1)?  s* >= 2 needs
+// sources holding >= 2 query keywords that cover Q with zb(c): multi is the union of the keyword sets of
+// such nodes (graph-wide); per candidate, the keywords i for which one of them lies in DAG_i(c): the
+// search's rm bits (exact for keywords 0-6, keyword 7 assumed reached) or mk_reach's fixpoint over the
+// shared DAG (per compact id, in pcnt).  Each is an over-approximation, so is their intersection.
+__device__ __forceinline__ bool cut_valid(const Ctx &c, int32_t cn, uint32_t zbc, uint32_t multi) {
+    if (!c.a.level_cover) return true;
+    uint32_t reach = multi;
+    if (c.a.level_cover == 1 && c.a.rm_ok)
+        reach &= st_rm(__ldcg(c.w.st + cn)) | (c.qq.q > 7 ? ~kRmMask : 0u);
+    if (c.a.level_cover == 1 && c.ctl->mk_reach) {
+        const int32_t cid = __ldcg(c.w.pd_cid + cn);
+        if (cid >= 0) reach &= (uint32_t)__ldcg(c.w.pcnt + cid);
+    }
+    return ((reach | zbc) & c.qq.full) != c.qq.full;
+}
+
 // Closure (over the shared predecessor lists) + level-cover + Eq. 6 key of the Central Graph at c.
 // Returns CG_OK, CG_OVERFLOW (arena too small: the next tier redoes it) or CG_CUT.
 // cut (pruning round 2, exact): the key is known to exceed `cut` (the k-th exact key so far), so c cannot
@@ -1478,20 +1513,24 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
 // keeps every source (s* = 1): no set of sources holding two or more query keywords can cover Q together
 // with c's own keywords (multi = union of the keyword sets of all such nodes of the graph), or
 // level_cover = 0.  Then the closure weight so far, times d^lambda, is a lower bound of the key.
-enum { CG_OVERFLOW = 0, CG_OK = 1, CG_CUT = 2 };
+// lazy (pruning round 2): the shared DAG may lack the predecessor lists of some closure
+// nodes; the walk marks them for the next pre-pass round (pd_state byte 1 + round bitmap 0), goes on over
+// what is known (the cut still applies: the nodes found are in the closure) and, if not cut, returns
+// CG_INCOMPLETE (no key).
+enum { CG_OVERFLOW = 0, CG_OK = 1, CG_CUT = 2, CG_INCOMPLETE = 3 };
 constexpr int32_t kArenaMagic = 0x4B475341;   // "KGSA": a persistent arena in a known state
 constexpr double kNoCut = __builtin_huge_val();
 template <class Team>
 __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, int depth, double *key,
-                             double cut = kNoCut, uint32_t multi = 0u) {
+                             double cut = kNoCut, uint32_t multi = 0u, bool lazy = false) {
     const uint32_t full = c.qq.full;
     const int r = T.rank(), ts = T.size();
     // reset: only what the previous use of a persistent arena touched (its node count is still in scal),
     // everything after an overflow (its claimed slots were not recorded) or on first use
     const int prev_nodes = S.magic ? S.scal[SC_NODES] : 0;
-    const bool lazy = S.magic && *S.magic == kArenaMagic && S.scal[SC_OVF] == 0 && prev_nodes <= S.ncap;
+    const bool lazy_reset = S.magic && *S.magic == kArenaMagic && S.scal[SC_OVF] == 0 && prev_nodes <= S.ncap;
     T.sync();
-    if (lazy) {
+    if (lazy_reset) {
         for (int j = r; j < prev_nodes; j += ts) {
             const int h = S.hslot[j];
             S.hkey[h] = -1; S.hval[h] = -1;
@@ -1509,18 +1548,7 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     const uint64_t Mc = ldrow(c.w.M, cn);
     uint32_t zbc = 0;
     for (int i = 0; i < c.qq.q; ++i) if (((Mc >> (8 * i)) & 0xFF) == 0) zbc |= 1u << i;
-    // s* >= 2 needs sources holding >= 2 query keywords that cover Q with zb(c): multi is the union of
-    // the keyword sets of such nodes (graph-wide), or per candidate the keywords i for which one of them
-    // reaches c inside DAG_i (the shared predecessor DAG's arcs, pd_state byte 3, mk_reach)
-    uint32_t reach = multi;
-    if (c.a.level_cover == 1 && c.a.rm_ok)   // rm: exact for keywords 0-6, keyword 7 assumed reached
-        reach &= st_rm(__ldcg(c.w.st + cn)) | (c.qq.q > 7 ? ~kRmMask : 0u);
-    if (c.a.level_cover == 1 && c.ctl->mk_reach) {   // mk_reach's fixpoint, per compact id (in pcnt)
-        const int32_t cid = __ldcg(c.w.pd_cid + cn);
-        if (cid >= 0) reach &= (uint32_t)__ldcg(c.w.pcnt + cid);
-    }
-    const bool cut_on = cut < kNoCut &&
-                        (!c.a.level_cover || ((reach | zbc) & full) != full);
+    const bool cut_on = cut < kNoCut && cut_valid(c, cn, zbc, multi);
     auto over_cut = [&]() {   // the closure weight so far, times d^lambda, already exceeds the cut
         return __dmul_rn(c.a.dpow[depth], (double)*reinterpret_cast<volatile unsigned long long *>(S.wsum) *
                                               (1.0 / 16777216.0)) > cut;
@@ -1552,6 +1580,14 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
                 S.b_j[r] = j;
                 S.b_P[r] = P;
                 const int32_t cid = __ldcg(c.w.pd_cid + x);   // predecessor list from the shared DAG
+                if (lazy && P) {   // keywords whose predecessors the DAG does not hold yet: request them
+                    const uint32_t miss = P & ~((__ldcg(c.w.pd_state + x) >> 16) & 0xFFu);
+                    if (miss) {
+                        const uint32_t old = atomicOr(c.w.pd_state + x, miss << 8);
+                        if (((old >> 8) & 0xFFu) == 0) set_bit(c.w.pd_bits, kFlagPd, x);
+                        S.scal[SC_INC] = 1;
+                    }
+                }
                 int64_t s0 = 0;
                 if (P && cid >= 0) { s0 = __ldcg(c.w.pred_ptr + cid); deg = (int)(__ldcg(c.w.pred_ptr + cid + 1) - s0); }
                 S.b_start[r] = s0;
@@ -1606,8 +1642,9 @@ __device__ int central_graph(const Team &T, Arena &S, const Ctx &c, int32_t cn, 
     }
     T.sync();
     // an overflowing arena still holds a partial closure: its weight is a lower bound of the key
-    if (S.scal[SC_CUT] || (S.scal[SC_OVF] && cut_on && over_cut())) { T.sync(); return CG_CUT; }
+    if (S.scal[SC_CUT] || ((S.scal[SC_OVF] || S.scal[SC_INC]) && cut_on && over_cut())) { T.sync(); return CG_CUT; }
     if (S.scal[SC_OVF]) return CG_OVERFLOW;
+    if (S.scal[SC_INC]) { T.sync(); return CG_INCOMPLETE; }
     const int nn = S.scal[SC_NODES];
     const int na = S.scal[SC_ARCS] < S.acap ? S.scal[SC_ARCS] : S.acap;
     // ---- level-cover: a keyword node's level counts the keywords it contributes (R13: a source
@@ -2082,12 +2119,14 @@ __device__ void containment_select(const Ctx &c, long long *sh, char *dsmem, uin
 // ------------------------------------------------------------------------------------------ top-down driver
 // Seeds of the predecessor pre-pass: every candidate list[0..cnt) (nullptr: all centrals), for every
 // keyword it does not contain itself (those have m = 0 and no predecessors).
+__device__ __forceinline__ void pd_round0_reset(const Ctx &c) {   // group leader: round 0 of a pred_dag call
+    c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; c.ctl->pd_ctile[0] = 0u;
+    c.ctl->pd_xbatch[0] = 0u;
+}
+
 __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
     const Grp &G = c.G;
-    if (G.gtid() == 0) {   // round 0 of this call
-        c.ctl->pd_qn[0][0] = 0u; c.ctl->pd_qn[0][1] = 0u; c.ctl->pd_ndef[0] = 0u; c.ctl->pd_ctile[0] = 0u;
-        c.ctl->pd_xbatch[0] = 0u;
-    }
+    if (G.gtid() == 0) pd_round0_reset(c);
     for (int64_t j = G.gtid(); j < cnt; j += G.gsz) {
         const int32_t idx = list ? __ldcg(list + j) : (int32_t)j;
         const int32_t cn = __ldcg(c.w.centrals + idx);
@@ -2106,7 +2145,8 @@ __device__ void seed_pd(const Ctx &c, const int32_t *list, uint32_t cnt) {
 // per candidate over the CTA's shared region; (C) beyond that, the CTA's global-memory arena.
 // cflag: 0 = key from tier 1, 1 = from tier 2/3 (emitted by a CTA).
 __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int32_t *list, uint32_t cnt, QOut *qo,
-                             double cut = kNoCut) {
+                             double cut = kNoCut, bool lazy = false, bool count_eval = true,
+                             int32_t *inc_out = nullptr) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
     Ctl *ctl = c.ctl;
@@ -2114,7 +2154,8 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
     const double kInf = __longlong_as_double(0x7FF0000000000000ll);
     if (G.gtid() == 0) {
         ctl->work_ext = 0; ctl->n_overflow = 0; ctl->work_big = 0; ctl->work_huge = 0; ctl->work_huge2 = 0;
-        ctl->n_eval += cnt;
+        if (count_eval) ctl->n_eval += cnt;
+        ctl->n_inc = 0;
     }
     G.sync();
     if ((threadIdx.x >> 5) < kExtWarps) {
@@ -2128,10 +2169,11 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
             const int32_t idx = list ? __ldcg(list + t) : (int32_t)t;
             const int32_t cn = __ldcg(c.w.centrals + idx);
             double key = 0.0;
-            const int st = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key, cut, multi);
+            const int st = central_graph(T, S1, c, cn, __ldcg(c.w.cdepth + idx), &key, cut, multi, lazy);
             if (T.rank() == 0) {
                 if (st == CG_OK) { c.w.ckey[idx] = key; c.w.cflag[idx] = 0; }
                 else if (st == CG_CUT) { c.w.ckey[idx] = kInf; c.w.cflag[idx] = 0; atomicAdd(&ctl->n_cut, 1u); }
+                else if (st == CG_INCOMPLETE) { c.w.cflag[idx] = 0; inc_out[atomicAdd(&ctl->n_inc, 1u)] = idx; }
                 else { c.w.cflag[idx] = 1; c.w.overflow[atomicAdd(&ctl->n_overflow, 1u)] = idx; }
             }
             __syncwarp();
@@ -2146,10 +2188,11 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
         for (uint32_t t = G.grank; t < no; t += G.gcount) {
             const int32_t idx = __ldcg(c.w.overflow + t);
             double key = 0.0;
-            const int st = central_graph(BT, S2, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
+            const int st = central_graph(BT, S2, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi, lazy);
             if (threadIdx.x == 0) {
                 if (st == CG_OK) c.w.ckey[idx] = key;
                 else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
+                else if (st == CG_INCOMPLETE) inc_out[atomicAdd(&ctl->n_inc, 1u)] = idx;
                 else c.w.overflow[no + atomicAdd(&ctl->work_big, 1u)] = idx;
             }
             __syncthreads();
@@ -2161,10 +2204,11 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
             for (uint32_t t = G.grank; t < nbig; t += G.gcount) {
                 const int32_t idx = __ldcg(c.w.overflow + no + t);
                 double key = 0.0;
-                const int st = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
+                const int st = central_graph(BT, S3, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi, lazy);
                 if (threadIdx.x == 0) {
                     if (st == CG_OK) c.w.ckey[idx] = key;
                     else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
+                    else if (st == CG_INCOMPLETE) inc_out[atomicAdd(&ctl->n_inc, 1u)] = idx;
                     else c.w.overflow[no + nbig + atomicAdd(&ctl->work_huge, 1u)] = idx;
                 }
                 __syncthreads();
@@ -2179,10 +2223,11 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
             for (uint32_t t = G.grank; t < nlarge; t += G.gcount) {
                 const int32_t idx = __ldcg(c.w.overflow + no + nbig + t);
                 double key = 0.0;
-                const int st = central_graph(BT, SL, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
+                const int st = central_graph(BT, SL, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi, lazy);
                 if (threadIdx.x == 0) {
                     if (st == CG_OK) c.w.ckey[idx] = key;
                     else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
+                    else if (st == CG_INCOMPLETE) inc_out[atomicAdd(&ctl->n_inc, 1u)] = idx;
                     else c.w.overflow[no + nbig + nlarge + atomicAdd(&ctl->work_huge2, 1u)] = idx;
                 }
                 __syncthreads();
@@ -2197,10 +2242,11 @@ __device__ void extract_list(const Ctx &c, long long *sh, char *dsmem, const int
                 for (uint32_t t = 0; t < nhuge; ++t) {
                     const int32_t idx = __ldcg(c.w.overflow + no + nbig + nlarge + t);
                     double key = 0.0;
-                    const int st = central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi);
+                    const int st = central_graph(BT, S4, c, __ldcg(c.w.centrals + idx), __ldcg(c.w.cdepth + idx), &key, cut, multi, lazy);
                     if (threadIdx.x == 0) {
                         if (st == CG_OK) c.w.ckey[idx] = key;
                         else if (st == CG_CUT) { c.w.ckey[idx] = kInf; atomicAdd(&ctl->n_cut, 1u); }
+                        else if (st == CG_INCOMPLETE) inc_out[atomicAdd(&ctl->n_inc, 1u)] = idx;
                         else atomicExch(&ctl->fatal, 2);
                     }
                     __syncthreads();
@@ -2297,6 +2343,15 @@ __device__ void emit_answers(const Ctx &c, long long *sh, char *dsmem, QOut *qo)
 // round 2 extracts every remaining candidate with (LB, id) < T.  The top-k over the extracted
 // candidates is then the top-k over all of C.
 
+// Pruning round 2 with the predecessor DAG built lazily (kgs_params.lazy_dag).  The candidates whose key
+// cut-off is not valid (cut_valid: level-cover may keep fewer than all of their sources) get their whole
+// closures as before.  The others start from their direct predecessors only (one pre-pass round); each
+// pass then walks every unfinished candidate over the DAG built so far: the cut stops it as soon as the
+// weight of the closure nodes found exceeds the k-th key T (the nodes found are in the closure whatever
+// lies beyond, so the bound is exact), a walk that met no missing list gives the exact key, and the others
+// request the lists they met missing (central_graph, lazy) — one more pre-pass round over exactly those
+// nodes, and the next pass.  A walk that finishes has the same closure as with the whole DAG, so keys and
+// answers are unchanged; only the DAG built for candidates that end up cut shrinks.
 __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QOut *qo) {
     const Grp &G = c.G;
     const EngineArgs &a = c.a;
@@ -2357,20 +2412,57 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             }
             G.sync();
             n2 = __ldcg(&ctl->n_elist2);
-            if (!rec) {
-                seed_pd(c, c.w.elist + m, n2);
-                pred_dag(c, S, sh, qo, true);
-            }
-            // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union);
-            // with many candidates, which of them can have s* >= 2 is decided per candidate (mk_reach)
+            // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union)
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
-            if (!a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min && (__ldcg(&ctl->multi_kw) & c.qq.full) &&
-                (!a.rm_ok || c.qq.q > 7))
-            {
-                mk_reach(c);
-                stamp(G, qo, TS_MK);
+            // lazy DAG (above): partition into qlight, cut valid from the front, the others from the back
+            const bool lazy = a.lazy_dag && !rec && !a.td_only && a.level_cover == 1 && a.rm_ok && c.qq.q <= 7;
+            uint32_t nv = 0;
+            if (lazy) {
+                const uint32_t multi = __ldcg(&ctl->multi_kw);
+                if (G.gtid() == 0) { ctl->n_valid = 0u; ctl->n_inc = 0u; }
+                G.sync();
+                for (int64_t i = G.gtid(); i < n2; i += G.gsz) {
+                    const int32_t idx = __ldcg(c.w.elist + m + i);
+                    const int32_t cn = __ldcg(c.w.centrals + idx);
+                    const uint64_t Mc = ldrow(c.w.M, cn);
+                    uint32_t zbc = 0;
+                    for (int k = 0; k < c.qq.q; ++k) if (((Mc >> (8 * k)) & 0xFF) == 0) zbc |= 1u << k;
+                    if (cut_valid(c, cn, zbc, multi)) c.w.qlight[agg_slot(&ctl->n_valid, 11u)] = idx;
+                    else c.w.qlight[n2 - 1 - agg_slot(&ctl->n_inc, 12u)] = idx;
+                }
+                G.sync();
+                nv = __ldcg(&ctl->n_valid);
             }
-            extract_list(c, sh, dsmem, c.w.elist + m, n2, qo, cut);
+            // step 0: the candidates whose closures are built whole (all of them without the lazy DAG);
+            // steps 1, 2, ...: lazy passes over the others (one call site each for the pre-pass and the
+            // extraction: more inlined copies of them spilled the whole kernel)
+            int32_t *cur = c.w.qlight, *nxt = c.w.lz;
+            for (int step = lazy && nv == n2 ? 1 : 0;; ++step) {
+                const bool lz = step > 0;
+                const int32_t *L = !lazy ? c.w.elist + m : (lz ? cur : c.w.qlight + nv);
+                const uint32_t cnt = !lazy ? n2 : (lz ? (step == 1 ? nv : __ldcg(&ctl->n_inc)) : n2 - nv);
+                if (!rec) {
+                    if (step <= 1) seed_pd(c, L, cnt);
+                    pred_dag(c, S, sh, qo, true, !lz || step >= 16 ? (1 << 30) : 1);
+                }
+                // without rm, which candidates can have s* >= 2 is decided from the whole DAG (mk_reach)
+                if (!lazy && !a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min &&
+                    (__ldcg(&ctl->multi_kw) & c.qq.full) && (!a.rm_ok || c.qq.q > 7)) {
+                    mk_reach(c);
+                    stamp(G, qo, TS_MK);
+                }
+                extract_list(c, sh, dsmem, L, cnt, qo, cut, lz, step <= 1, nxt);
+                if (!lazy || (!lz && nv == 0)) break;
+                if (lz) {
+                    publish_flags(ctl);   // the lists the walks requested (pre-pass round bitmap 0)
+                    G.sync();
+                    const uint32_t inc = __ldcg(&ctl->n_inc);
+                    if (G.gtid() == 0) { ctl->n_lazy_iter = step; pd_round0_reset(c); }
+                    if (!inc) break;
+                    int32_t *t = cur; cur = nxt; nxt = t;   // the unfinished walks, for the next pass
+                }
+                G.sync();
+            }
         }
         if (G.gtid() == 0) { ctl->work_big = 0; ctl->work_emit = 0; ctl->work_huge = 0; }
         if (m + n2 <= (uint32_t)KGS_MAX_K) {

@@ -92,6 +92,9 @@ struct Ctl {
     uint32_t pd_xbatch[2];         // [round parity] the same for the pre-pass
     uint32_t mk_reach;             // pcnt holds, per compact id, the keywords a multi-keyword source reaches it in
     uint32_t mk_changed[2];        // [pass parity] mk_reach fixpoint
+    uint32_t n_inc;                // lazy round 2: candidates whose closure is not complete yet
+    uint32_t n_valid;              // lazy round 2: candidates whose key cut-off is valid (partition)
+    uint32_t n_lazy_iter;          // lazy round 2: extraction passes
 };
 
 // Per-query summary written by the engine (device), read back by the host.
@@ -167,6 +170,7 @@ struct DevWork {
     uint16_t *pa_b;     // [pcap]
     int32_t *pa_slot;   // [pcap] position inside the successor's list
     int32_t *scan_tmp;  // [4096] block sums of the CSR scan
+    int32_t *lz;        // [n] lazy round 2: candidate list (ping-pong with qlight)
     int64_t pcap;
     // group state (device): query counter, validity of the per-node state
     uint32_t *gstate;   // [0] current query index, [1] queries done by this group, [2] state valid, [3] last R
@@ -208,6 +212,7 @@ struct EngineArgs {
     int prune_min;              // round 1 extracts max(8k, prune_min) candidates
     int mk_min;                 // round 2: per-candidate s* >= 2 test (mk_reach) from this many candidates
     int rm_ok;                  // the search's rm bits decide the s* >= 2 test (hitting arcs = Thm. V.4 arcs)
+    int lazy_dag;               // pruning round 2 builds the predecessor DAG only as far as the cut needs
     int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
     int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
     int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio

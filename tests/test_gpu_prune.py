@@ -210,11 +210,13 @@ def test_key_cutoff_in_round_two():
 
 def test_key_cutoff_per_candidate_multi_keyword_sources():
     """A few nodes hold two query keywords, so graph-wide level-cover could keep only some sources
-    (s* >= 2) and the query-wide test switches the cut-off off.  mk_reach decides it per candidate: the
-    keywords for which a two-keyword node reaches c inside DAG_i(c); where they cannot cover Q with zb(c),
-    every source is kept and the cut-off applies.  The candidates near the two-keyword nodes (small pruned
-    graphs, the likely winners) must still get their exact keys: answers equal the oracle's with the
-    per-candidate test on (mk_min = 0) and off, in latency mode (recorded DAG and pre-pass) and in a batch."""
+    (s* >= 2) and the query-wide test switches the cut-off off.  The test is made per candidate — from the
+    search's rm bits (keywords 0-6), and from mk_reach's fixpoint over the shared DAG when mk_min allows:
+    the keywords for which a two-keyword node reaches c inside DAG_i(c); where they cannot cover Q with
+    zb(c), every source is kept and the cut-off applies.  The candidates near the two-keyword nodes (small
+    pruned graphs, the likely winners) must still get their exact keys: answers equal the oracle's with
+    mk_reach on (mk_min = 0) and off, with the lazy round-2 DAG and without, in latency mode (recorded DAG
+    and pre-pass) and in a batch; with literal extraction (no rm) and mk_reach off nothing is cut."""
     _gpu()
     cuts_on = cuts_off = 0
     for seed, deg, k, n_multi in ((0, 16, 5, 3), (1, 16, 20, 10), (2, 8, 20, 30), (3, 16, 50, 6)):
@@ -235,12 +237,13 @@ def test_key_cutoff_per_candidate_multi_keyword_sources():
         ctx0 = f"seed={seed} deg={deg} k={k} multi={n_multi} |C|={len(o.centrals)}"
         runs = []
         for mk in (0, 1 << 30):
-            for rec in (1, 0):
-                p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, dag_record=rec)
-                runs.append((f"mk={mk} rec={rec}", kgs.kgs_query(G, kw, k, p), mk))
-            p = kgs.make_params(prune=1, prune_min=40, mk_min=mk)
-            for j, r in enumerate(kgs.kgs_query_batch(G, [kw, kw[::-1], kw], k, p, 3)):
-                runs.append((f"mk={mk} batch {j}", r, mk))
+            for lz in (1, 0):
+                for rec in (1, 0):
+                    p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, dag_record=rec, lazy_dag=lz)
+                    runs.append((f"mk={mk} lazy={lz} rec={rec}", kgs.kgs_query(G, kw, k, p), mk))
+                p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, lazy_dag=lz)
+                for j, r in enumerate(kgs.kgs_query_batch(G, [kw, kw[::-1], kw], k, p, 3)):
+                    runs.append((f"mk={mk} lazy={lz} batch {j}", r, mk))
         for tag, r, mk in runs:
             ctx = f"{ctx0} {tag}"
             assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
@@ -249,8 +252,12 @@ def test_key_cutoff_per_candidate_multi_keyword_sources():
                 assert ra.arcs.tolist() == oa.arcs.tolist(), ctx
             if mk == 0:
                 cuts_on += r.stats["n_cut"]
-            else:
-                cuts_off += r.stats["n_cut"]
+        # literal extraction: no rm (its DAG is not the hitting arcs), mk_reach off -> the query-wide test
+        ol = oracle.query(g, kw, k, extract_mode=oracle.EXTRACT_LITERAL)
+        r = kgs.kgs_query(G, kw, k, kgs.make_params(prune=1, prune_min=40, mk_min=1 << 30,
+                                                    extract_mode=kgs.KGS_EXTRACT_LITERAL))
+        assert [a.central for a in r.answers] == [a.central for a in ol.answers], ctx0
+        cuts_off += r.stats["n_cut"]
         G.close()
     assert cuts_off == 0 and cuts_on > 0, (cuts_on, cuts_off)
 
@@ -332,11 +339,13 @@ def test_key_cutoff_never_drops_a_two_level_winner():
     G = kgs.kgs_load_graph(g)
     runs = []
     for mk in (0, 1 << 30):
-        for rec in (1, 0):
-            runs.append((mk, rec, kgs.kgs_query(G, [0, 1, 2], 5,
-                                                kgs.make_params(prune_min=8, mk_min=mk, dag_record=rec))))
-        for r in kgs.kgs_query_batch(G, [[0, 1, 2], [2, 1, 0]], 5, kgs.make_params(prune_min=8, mk_min=mk), 2):
-            runs.append((mk, "batch", r))
+        for lz in (1, 0):
+            for rec in (1, 0):
+                runs.append((mk, f"{rec} lazy={lz}", kgs.kgs_query(G, [0, 1, 2], 5, kgs.make_params(
+                    prune_min=8, mk_min=mk, dag_record=rec, lazy_dag=lz))))
+            for r in kgs.kgs_query_batch(G, [[0, 1, 2], [2, 1, 0]], 5,
+                                         kgs.make_params(prune_min=8, mk_min=mk, lazy_dag=lz), 2):
+                runs.append((mk, f"batch lazy={lz}", r))
     for mk, rec, r in runs:
         ctx = f"mk_min={mk} rec={rec}"
         assert r.stats["n_evaluated"] < len(o.centrals) or r.stats["n_cut"] >= 0, ctx
