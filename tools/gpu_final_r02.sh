@@ -20,3 +20,4 @@ python tools/ncu_hot.py gpurun_out/fin_batch.ncu-rep k_engine 45 > gpurun_out/fi
 python tools/make_batch_profile.py $TAG gpurun_out/fin_batch_details.csv gpurun_out/fin_batch_raw.csv gpurun_out/fin_batch_hot.txt 350 $SHA C3 > gpurun_out/fin_mbp.log 2>&1
 cp profiles/${TAG}_batch_* gpurun_out/profiles/ 2>/dev/null
 tail -3 gpurun_out/fin_pytest.log gpurun_out/fin_smoke.log; cat gpurun_out/fin_bench.json
+timeout 1800 python tools/exp_sweeps.py > gpurun_out/fin_exp_sweeps.txt 2>&1
