@@ -14,4 +14,4 @@ timeout 900 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_d
 python tools/make_traffic.py r02v gpurun_out/r02v_traffic.csv gpurun_out/r02v_traffic_pb.log 350 $SHA C3 > gpurun_out/r02v_make_traffic.log 2>&1
 cp profiles/r02v_batch_traffic.json gpurun_out/profiles/ 2>/dev/null
 timeout 1500 python -m pytest -x -q -p no:cacheprovider --durations=5 "tests/test_gpu_fullsize.py::test_c4_sample_with_level5_queries" > gpurun_out/r02v_pytest_c4.log 2>&1; echo "rc=$?" >> gpurun_out/r02v_pytest_c4.log
-bash tools/gpu_r02u.sh
+bash tools/experiments/gpu_r02u.sh

@@ -61,7 +61,7 @@ for r in raw[2:]:
 # capture of tools/make_traffic.py instead)
 json.dump(res, open(os.path.join(ROOT, "profiles", f"{tag}_batch_fullset.json"), "w"), indent=1)
 out = [f"# Batch-launch profile {tag} — k_engine, {res['launch']}", "",
-       "`ncu --set full --import-source on --clock-control none` of one launch (tools/gpu_ncu_batch.sh).  "
+       "`ncu --set full --import-source on --clock-control none` of one launch (tools/experiments/gpu_ncu_batch.sh).  "
        "Times under ncu are not bench values.  Kernel replay restores memory before each of ~40 passes; the "
        "work of the pass whose counters are shown can differ from the bench launch's (see the launch lines of "
        "profile_batch.py) — the DRAM bytes per launch behind bench.py's roofline.traffic come from a "
