@@ -137,16 +137,22 @@ def load_traffic(workload: str):
     """DRAM bytes per query of the engine from the newest committed ncu capture of the bench's own launch
     shape (profiles/r*_batch_traffic.json for this workload), with the git sha / source hash it was
     taken at.  Returns (bytes per query or None, info dict)."""
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_batch_traffic.json")))
-    for f in reversed(files):
+    # a capture of the running sources first (src_sha256), then the newest capture (captured_unix; older
+    # files without it by name)
+    cands = []
+    here = source_hash()
+    for f in glob.glob(os.path.join(ROOT, "profiles", "r*_batch_traffic.json")):
         with open(f) as fh:
             d = json.load(fh)
         if d.get("workload", "C3") != workload:
             continue
-        return d["dram_bytes_per_query"], {"traffic_source": os.path.basename(f), "traffic_sha": d.get("git_sha"),
-                                           "traffic_matches_source": d.get("src_sha256") == source_hash(),
-                                           "traffic_l2_hit_pct": d.get("l2_hit_pct")}
-    return None, {"traffic_source": None}
+        cands.append((d.get("src_sha256") == here, d.get("captured_unix", 0), os.path.basename(f), d))
+    if not cands:
+        return None, {"traffic_source": None}
+    match, _, name, d = max(cands, key=lambda t: (t[0], t[1], t[2]))
+    return d["dram_bytes_per_query"], {"traffic_source": name, "traffic_sha": d.get("git_sha"),
+                                       "traffic_matches_source": match, "traffic_l2_hit_pct": d.get("l2_hit_pct"),
+                                       "traffic_same_work": d.get("same_work")}
 
 
 def cpu_info() -> dict:

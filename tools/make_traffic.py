@@ -11,6 +11,7 @@ import json
 import os
 import re
 import sys
+import time
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 tag, f_csv, f_log, nq, sha = sys.argv[1:6]
@@ -35,7 +36,7 @@ rd, wr = m["dram__bytes_read.sum"], m["dram__bytes_write.sum"]
 res = {"kernel": "k_engine", "launch": f"{nq} {workload} queries, G = 8 (bench shape), one launch",
        "capture": "single pass (--metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,"
                   "lts__t_sector_hit_rate.pct), no kernel replay",
-       "workload": workload, "git_sha": sha, "src_sha256": source_hash(),
+       "workload": workload, "git_sha": sha, "src_sha256": source_hash(), "captured_unix": int(time.time()),
        "duration_s_under_ncu": m.get("gpu__time_duration.sum"),
        "arcs_captured_launch": arcs.get(1), "arcs_uncaptured_launch": arcs.get(0),
        "same_work": arcs.get(0) is not None and arcs.get(0) == arcs.get(1),
