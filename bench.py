@@ -343,6 +343,7 @@ def main():
         # gloo (NCCL refuses two ranks on one device); the collectives of dist.py stage through the host
         if os.environ.get("KGS_BENCH_ONE_GPU") == "1":
             local = 0
+            args.groups = max(1, args.groups // world)   # the ranks share one GPU's memory
             torch.cuda.set_device(0)
             dist.init_process_group("gloo")
         else:
