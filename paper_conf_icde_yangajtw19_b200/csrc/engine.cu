@@ -2415,7 +2415,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
             // exact cut-off: the k-th key so far (vertex-partitioned top-down has no multi-keyword union)
             const double cut = a.td_only ? kNoCut : __ldcg(c.w.ckey + __ldcg(c.w.sel + kk - 1));
             // lazy DAG (above): partition into qlight, cut valid from the front, the others from the back
-            const bool lazy = a.lazy_dag && !rec && !a.td_only && a.level_cover == 1 && a.rm_ok && c.qq.q <= 7;
+            const bool lazy = a.lazy_dag && !rec && !a.td_only && a.level_cover == 1 && a.rm_ok;
             uint32_t nv = 0;
             if (lazy) {
                 const uint32_t multi = __ldcg(&ctl->multi_kw);
@@ -2445,8 +2445,9 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
                     if (step <= 1) seed_pd(c, L, cnt);
                     pred_dag(c, S, sh, qo, true, !lz || step >= 16 ? (1 << 30) : 1);
                 }
-                // without rm, which candidates can have s* >= 2 is decided from the whole DAG (mk_reach)
-                if (!lazy && !a.td_only && a.level_cover == 1 && n2 >= (uint32_t)a.mk_min &&
+                // where rm cannot decide (no rm, or keyword 7 of a q = 8 query), which of the candidates
+                // whose closures are whole can have s* >= 2 is decided from the DAG (mk_reach)
+                if (!lz && !a.td_only && a.level_cover == 1 && cnt >= (uint32_t)a.mk_min &&
                     (__ldcg(&ctl->multi_kw) & c.qq.full) && (!a.rm_ok || c.qq.q > 7)) {
                     mk_reach(c);
                     stamp(G, qo, TS_MK);

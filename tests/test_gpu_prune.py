@@ -296,14 +296,16 @@ def test_deferred_queries_run_on_the_whole_grid():
     G.close()
 
 
-def test_key_cutoff_never_drops_a_two_level_winner():
+@pytest.mark.parametrize("q", [3, 8])
+def test_key_cutoff_never_drops_a_two_level_winner(q):
     """Hand-built: the Central Graph that must win keeps only two-keyword sources (s* = 2), while its whole
-    closure is heavy.  Keywords A, B, C (q = 3), every activation level 0 (A = 0.1).  Candidate c (w 0.5)
-    is joined to m1 (holds A, B) and m2 (holds B, C), both of weight 0, and to 20 nodes of each keyword of
-    weight 0.9: level-cover keeps {c, m1, m2} (m1, m2 contribute two keywords each and cover Q), key 0.5;
-    its closure weighs 54.5.  60 filler centrals (w 0.01, one heavy A, B and C neighbour each, key 2.71)
-    fill pruning round 1 (prune_min 8: the 40 smallest bounds), so c is extracted in round 2 with the cut
-    at T = 2.71: an invalid cut would drop it.  Answers must be the oracle's (c first)."""
+    closure is heavy.  Keywords 0..q-1, every activation level 0 (A = 0.1).  Candidate c (w 0.5) is joined
+    to two-keyword nodes of weight 0 that cover Q (q = 3: m1 holds 0, 1 and m2 holds 1, 2; q = 8: the pairs
+    (0, 1), (2, 3), (4, 5), (6, 7) — keyword 7 has no rm bit) and to 20 nodes of each keyword of weight
+    0.9: level-cover keeps c and the two-keyword nodes, key 0.5, while the closure weighs 0.5 + 18 q.  60
+    filler centrals (w 0.01, one heavy neighbour per keyword, key 0.01 + 0.9 q) fill pruning round 1
+    (prune_min 8: the 8k = 40 smallest bounds), so c is extracted in round 2 with the cut at T = the 5th
+    key: an invalid cut would drop it.  Answers must be the oracle's (c first), lazy DAG on and off."""
     _gpu()
     n_fill, n_side = 60, 20
     nodes = {}
@@ -311,12 +313,19 @@ def test_key_cutoff_never_drops_a_two_level_winner():
     def nid(name):
         return nodes.setdefault(name, len(nodes))
 
-    edges, kws, w = [], [[], [], []], {}
-    c, m1, m2 = nid("c"), nid("m1"), nid("m2")
-    w[c], w[m1], w[m2] = 0.5, 0.0, 0.0
-    kws[0].append(m1); kws[1].append(m1); kws[1].append(m2); kws[2].append(m2)
-    edges += [(c, m1), (c, m2)]
-    for i in range(3):
+    edges, kws, w = [], [[] for _ in range(q)], {}
+    c = nid("c")
+    w[c] = 0.5
+    pairs = [(0, 1), (1, 2)] if q == 3 else [(0, 1), (2, 3), (4, 5), (6, 7)]
+    multi = []
+    for j, (i1, i2) in enumerate(pairs):
+        m = nid(f"m{j}")
+        w[m] = 0.0
+        kws[i1].append(m)
+        kws[i2].append(m)
+        edges.append((c, m))
+        multi.append(m)
+    for i in range(q):
         for j in range(n_side):
             v = nid(f"s{i}_{j}")
             w[v] = 0.9
@@ -325,7 +334,7 @@ def test_key_cutoff_never_drops_a_two_level_winner():
     for f in range(n_fill):
         fv = nid(f"f{f}")
         w[fv] = 0.01
-        for i in range(3):
+        for i in range(q):
             v = nid(f"f{f}_{i}")
             w[v] = 0.9
             kws[i].append(v)
@@ -334,21 +343,21 @@ def test_key_cutoff_never_drops_a_two_level_winner():
     wt = np.array([w[i] for i in range(n)], dtype=np.float64)
     wt = (np.floor(wt * (1 << 24) + 0.5) / (1 << 24)).astype(np.float32)
     g = synth.from_edges(n, edges, wt, [sorted(x) for x in kws], 0.1)
-    o = oracle.query(g, [0, 1, 2], 5)
-    assert o.answers[0].central == c and o.answers[0].nodes.tolist() == sorted([c, m1, m2])
+    kw = list(range(q))
+    o = oracle.query(g, kw, 5)
+    assert o.answers[0].central == c and o.answers[0].nodes.tolist() == sorted([c] + multi)
     G = kgs.kgs_load_graph(g)
     runs = []
     for mk in (0, 1 << 30):
         for lz in (1, 0):
             for rec in (1, 0):
-                runs.append((mk, f"{rec} lazy={lz}", kgs.kgs_query(G, [0, 1, 2], 5, kgs.make_params(
+                runs.append((mk, f"{rec} lazy={lz}", kgs.kgs_query(G, kw, 5, kgs.make_params(
                     prune_min=8, mk_min=mk, dag_record=rec, lazy_dag=lz))))
-            for r in kgs.kgs_query_batch(G, [[0, 1, 2], [2, 1, 0]], 5,
+            for r in kgs.kgs_query_batch(G, [kw, kw[::-1]], 5,
                                          kgs.make_params(prune_min=8, mk_min=mk, lazy_dag=lz), 2):
                 runs.append((mk, f"batch lazy={lz}", r))
     for mk, rec, r in runs:
-        ctx = f"mk_min={mk} rec={rec}"
-        assert r.stats["n_evaluated"] < len(o.centrals) or r.stats["n_cut"] >= 0, ctx
+        ctx = f"q={q} mk_min={mk} rec={rec}"
         assert [a.central for a in r.answers] == [a.central for a in o.answers], ctx
         for ra, oa in zip(r.answers, o.answers):
             assert ra.score_key == oa.key and ra.nodes.tolist() == oa.nodes.tolist(), ctx
