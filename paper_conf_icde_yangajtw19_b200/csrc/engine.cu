@@ -835,14 +835,14 @@ __device__ void build_pred_csr(const Ctx &c, long long *sh, QOut *qo) {
 // nodes contributing two or more cover Q with zb(c), and each such node v contributes i only if v is a
 // source in DAG_i(c) — so s* >= 2 implies reach(c) | zb(c) = Q.  The DAG holds every closure arc of the
 // candidates seeded so far (a superset of one candidate's), so reach over-approximates: the test is safe.
-// Stored per compact id in pcnt (the CSR is built; pcnt's prefix is reset by the next query); the arc
-// records' pa_u becomes the predecessor's compact id (-1: a source without a list) on the first pass.
+// Stored per compact id in lz (free until the lazy passes start; pcnt must keep the list counts, which a
+// later lazy pre-pass round extends).
 __device__ void mk_reach(const Ctx &c) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const uint32_t mk = __ldcg(&ctl->multi_kw) & c.qq.full;
     const int64_t ncid = (int64_t)__ldcg(&ctl->n_cid);
-    uint32_t *R = reinterpret_cast<uint32_t *>(c.w.pcnt);
+    uint32_t *R = reinterpret_cast<uint32_t *>(c.w.lz);
     for (int64_t j = G.gtid(); j < ncid; j += G.gsz) R[j] = 0u;
     if (G.gtid() == 0) { ctl->mk_changed[0] = 0u; ctl->mk_changed[1] = 0u; }
     G.sync();
@@ -852,15 +852,9 @@ __device__ void mk_reach(const Ctx &c) {
         for_each_record(c, cnt, [&](int64_t ai) {
             const uint32_t b = c.w.pa_b[ai];
             const uint32_t pb = b & 0xFFu & mk;
-            int32_t cu;
-            if (pass == 0) {
-                const int32_t u = c.w.pa_u[ai];
-                cu = pb ? __ldcg(c.w.pd_cid + u) : -1;
-                c.w.pa_u[ai] = cu;
-            } else {
-                cu = __ldcg(c.w.pa_u + ai);
-            }
             if (!pb) return;
+            // (the records stay as they are: a lazy pre-pass round after this rebuilds the CSR from them)
+            const int32_t cu = __ldcg(c.w.pd_cid + __ldcg(c.w.pa_u + ai));
             const uint32_t zbu = b >> 8;
             const uint32_t add = pb & ((__popc(zbu) >= 2 ? zbu : 0u) | (cu >= 0 ? __ldcg(R + cu) : 0u));
             if (!add) return;
@@ -1493,7 +1487,7 @@ __device__ __forceinline__ void fifo_push(Arena &S, int j) {
 // sources holding >= 2 query keywords that cover Q with zb(c): multi is the union of the keyword sets of
 // such nodes (graph-wide); per candidate, the keywords i for which one of them lies in DAG_i(c): the
 // search's rm bits (exact for keywords 0-6, keyword 7 assumed reached) or mk_reach's fixpoint over the
-// shared DAG (per compact id, in pcnt).  Each is an over-approximation, so is their intersection.
+// shared DAG (per compact id, in lz).  Each is an over-approximation, so is their intersection.
 __device__ __forceinline__ bool cut_valid(const Ctx &c, int32_t cn, uint32_t zbc, uint32_t multi) {
     if (!c.a.level_cover) return true;
     uint32_t reach = multi;
@@ -1501,7 +1495,7 @@ __device__ __forceinline__ bool cut_valid(const Ctx &c, int32_t cn, uint32_t zbc
         reach &= st_rm(__ldcg(c.w.st + cn)) | (c.qq.q > 7 ? ~kRmMask : 0u);
     if (c.a.level_cover == 1 && c.ctl->mk_reach) {
         const int32_t cid = __ldcg(c.w.pd_cid + cn);
-        if (cid >= 0) reach &= (uint32_t)__ldcg(c.w.pcnt + cid);
+        if (cid >= 0) reach &= (uint32_t)__ldcg(c.w.lz + cid);
     }
     return ((reach | zbc) & c.qq.full) != c.qq.full;
 }
@@ -2454,6 +2448,7 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
                 }
                 extract_list(c, sh, dsmem, L, cnt, qo, cut, lz, step <= 1, nxt);
                 if (!lazy || (!lz && nv == 0)) break;
+                if (!lz && G.gtid() == 0) ctl->mk_reach = 0u;   // lz becomes a candidate list (next barrier)
                 if (lz) {
                     publish_flags(ctl);   // the lists the walks requested (pre-pass round bitmap 0)
                     G.sync();
