@@ -725,8 +725,11 @@ __device__ void pred_dag(const Ctx &c, BigTile &S, long long *sh, QOut *qo, bool
                     c.w.pd_state[v] = __ldcg(c.w.pd_state + v) & ~0xFF00u;
                 }
             }
-            if (G.gtid() == 0) ctl->pd_flag[slot] = 0u;
+            // every CTA has read pd_flag[slot] (and cleared its words) before the flag is reset: a CTA
+            // reaching the check above after the reset would skip this barrier and desynchronise the group's
+            // barriers (the one-GPU two-process runs hit it as illegal addresses / instructions, r02ag)
             G.sync();
+            if (G.gtid() == 0) ctl->pd_flag[slot] = 0u;   // next read: the next call, after build_pred_csr's barriers
             break;
         }
         uint32_t *qn = ctl->pd_qn[slot];
