@@ -148,7 +148,10 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *                  parallelises over the whole GPU instead of holding one group); 0 = never
  *   lazy_dag       0 / 1 [1]: pruning round 2 extends the shared predecessor DAG only as far as the
  *                  candidates' walks need before the exact key cut-off stops them (candidates whose cut is
- *                  valid, decided from the search's rm bits); 0 builds every round-2 closure first */
+ *                  valid, decided from the search's rm bits); 0 builds every round-2 closure first
+ *   rec_max        >= 0 [2^22]: a recorded DAG (dag_record) of more arcs is dropped for the pre-pass when
+ *                  pruning runs (more than max(8k, prune_min) central nodes): its lists cover every touched
+ *                  node, the pre-pass only the candidates' closures (with the lazy round 2) */
 typedef struct {
     double alpha, lambda;
     int32_t max_depth, block_central, extract_mode, level_cover, want_levels, prune;
@@ -160,6 +163,7 @@ typedef struct {
     int32_t mk_min;
     int32_t defer_min;
     int32_t lazy_dag;
+    int32_t rec_max;
 } kgs_params;
 enum { KGS_DIR_AUTO = 0, KGS_DIR_PUSH = 1, KGS_DIR_PULL = 2 };
 

@@ -48,7 +48,8 @@ class kgs_params(ctypes.Structure):
                 ("direction", ctypes.c_int32), ("pull_ratio", ctypes.c_int32), ("pull_min", ctypes.c_int64),
                 ("prune_min", ctypes.c_int32), ("tile_light", ctypes.c_int32), ("dag_record", ctypes.c_int32),
                 ("search_only", ctypes.c_int32), ("containment", ctypes.c_int32), ("mk_min", ctypes.c_int32),
-                ("defer_min", ctypes.c_int32), ("lazy_dag", ctypes.c_int32)]
+                ("defer_min", ctypes.c_int32), ("lazy_dag", ctypes.c_int32),
+                ("rec_max", ctypes.c_int32)]
 
 
 class kgs_answer(ctypes.Structure):
@@ -196,7 +197,7 @@ def kgs_params_default() -> kgs_params:
 def make_params(alpha=0.1, lam=0.2, max_depth=254, block_central=1, extract_mode=KGS_EXTRACT_EXACT,
                 level_cover=1, want_levels=0, prune=1, direction=0, **tuning) -> kgs_params:
     """kgs_params from the defaults; ``tuning`` sets other fields by name (containment, pull_ratio,
-    pull_min, prune_min, tile_light, dag_record, search_only, mk_min, defer_min, lazy_dag)."""
+    pull_min, prune_min, tile_light, dag_record, search_only, mk_min, defer_min, lazy_dag, rec_max)."""
     p = kgs_params_default()
     p.alpha, p.lambda_, p.max_depth = float(alpha), float(lam), int(max_depth)
     p.block_central, p.extract_mode = int(block_central), int(extract_mode)

@@ -259,6 +259,7 @@ void kgs_params_default(kgs_params *p) {
     p->mk_min = 4096;
     p->defer_min = 1 << 16;
     p->lazy_dag = 1;
+    p->rec_max = 1 << 22;
 }
 
 void kgs_free_graph(kgs_graph *g) {
@@ -451,9 +452,9 @@ kgs_status check_params(const kgs_params &p, int32_t k) {
     if (p.direction < KGS_DIR_AUTO || p.direction > KGS_DIR_PULL) return fail(KGS_EINVAL, "direction must be 0, 1 or 2");
     if (p.pull_ratio < 1 || p.pull_min < 0 || p.prune_min < 1 || p.tile_light < 0 || p.dag_record < -1 ||
         p.dag_record > 1 || (p.search_only != 0 && p.search_only != 1) || p.mk_min < 0 || p.defer_min < 0 ||
-        (p.lazy_dag != 0 && p.lazy_dag != 1))
+        (p.lazy_dag != 0 && p.lazy_dag != 1) || p.rec_max < 0)
         return fail(KGS_EINVAL, "tuning parameters out of range (pull_ratio >= 1, pull_min >= 0, prune_min >= 1, "
-                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0, defer_min >= 0, lazy_dag 0/1)");
+                                "tile_light >= 0, dag_record -1/0/1, search_only 0/1, mk_min >= 0, defer_min >= 0, lazy_dag 0/1, rec_max >= 0)");
     return KGS_OK;
 }
 
@@ -589,6 +590,7 @@ kgs_status launch(kgs_graph *g, int nq, int k, const kgs_params &p, int G, cudaS
     a.prune_min = p.prune_min;
     a.mk_min = p.mk_min;
     a.lazy_dag = p.lazy_dag;
+    a.rec_max = p.rec_max;
     a.rm_ok = !td && (p.extract_mode == KGS_EXTRACT_EXACT || !p.block_central) ? 1 : 0;
     {   // recorded predecessor DAG: valid for the exact reading (R12), and for any mode without central
         // blocking; the literal Thm. V.4 with blocking and the top-down-only launch use the pre-pass.

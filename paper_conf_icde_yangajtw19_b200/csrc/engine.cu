@@ -1293,7 +1293,7 @@ __device__ void search(const Ctx &c, BigTile &S, long long *sh, QOut *qo) {
 // that can expand keyword i into x at level m_xi - 1 is scanned at that level).  Turn them
 // into the predecessor CSR keyed by the compact ids the merge gave the touched nodes.  Returns false
 // (and leaves the pre-pass state clean) when the record buffer overflowed.
-__device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
+__device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo, unsigned long long max_arcs) {
     const Grp &G = c.G;
     Ctl *ctl = c.ctl;
     const DevWork &w = c.w;
@@ -1312,7 +1312,10 @@ __device__ bool recorded_dag(const Ctx &c, long long *sh, QOut *qo) {
         }
     }
     __syncthreads();
-    if (s_rec[1]) {   // a region overflowed: forget the compact ids, use the pre-pass
+    // a region overflowed, or the record is large while pruning will run (the lists of every touched node
+    // cost more than the pre-pass's targeted closures and the lazy round 2, r02ai): forget the compact ids,
+    // use the pre-pass
+    if (s_rec[1] || s_rec[0] > max_arcs) {
         for (int64_t j = G.gtid(); j < nt; j += G.gsz) {   // the pre-pass reads both for its (touched) nodes
             const int32_t v = __ldcg(w.pd_touched + j);
             w.pd_cid[v] = -1;
@@ -2357,7 +2360,8 @@ __device__ void topdown(const Ctx &c, BigTile &S, long long *sh, char *dsmem, QO
     const uint32_t kk = (uint32_t)a.k < nc ? (uint32_t)a.k : nc;
     const uint32_t mcap = min((uint32_t)KGS_MAX_K, max(8u * kk, (uint32_t)a.prune_min));
     // predecessor lists: from the arcs the search recorded, else by the in-arc pre-pass (pred_dag)
-    const bool rec = a.dag_record && recorded_dag(c, sh, qo);
+    const bool rec = a.dag_record &&
+                     recorded_dag(c, sh, qo, a.prune && nc > mcap ? (unsigned long long)a.rec_max : ~0ull);
     if (!a.prune || nc <= mcap) {
         if (!rec) {
             seed_pd(c, nullptr, nc);

@@ -213,6 +213,7 @@ struct EngineArgs {
     int mk_min;                 // round 2: per-candidate s* >= 2 test (mk_reach) from this many candidates
     int rm_ok;                  // the search's rm bits decide the s* >= 2 test (hitting arcs = Thm. V.4 arcs)
     int lazy_dag;               // pruning round 2 builds the predecessor DAG only as far as the cut needs
+    int rec_max;                // with pruning, a recorded DAG of more arcs is dropped for the pre-pass
     int dag_record;             // 1: the search records its Thm. V.4 arcs (predecessor lists without the pre-pass)
     int direction;              // KGS_DIR_AUTO / _PUSH / _PULL
     int pull_ratio;             // auto: pull once the frontier's out-arcs exceed m / pull_ratio

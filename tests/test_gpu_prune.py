@@ -238,9 +238,9 @@ def test_key_cutoff_per_candidate_multi_keyword_sources():
         runs = []
         for mk in (0, 1 << 30):
             for lz in (1, 0):
-                for rec in (1, 0):
-                    p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, dag_record=rec, lazy_dag=lz)
-                    runs.append((f"mk={mk} lazy={lz} rec={rec}", kgs.kgs_query(G, kw, k, p), mk))
+                for rec, rmax in ((1, 1 << 22), (1, 0), (0, 1 << 22)):
+                    p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, dag_record=rec, lazy_dag=lz, rec_max=rmax)
+                    runs.append((f"mk={mk} lazy={lz} rec={rec} rec_max={rmax}", kgs.kgs_query(G, kw, k, p), mk))
                 p = kgs.make_params(prune=1, prune_min=40, mk_min=mk, lazy_dag=lz)
                 for j, r in enumerate(kgs.kgs_query_batch(G, [kw, kw[::-1], kw], k, p, 3)):
                     runs.append((f"mk={mk} lazy={lz} batch {j}", r, mk))
@@ -350,9 +350,9 @@ def test_key_cutoff_never_drops_a_two_level_winner(q):
     runs = []
     for mk in (0, 1 << 30):
         for lz in (1, 0):
-            for rec in (1, 0):
-                runs.append((mk, f"{rec} lazy={lz}", kgs.kgs_query(G, kw, 5, kgs.make_params(
-                    prune_min=8, mk_min=mk, dag_record=rec, lazy_dag=lz))))
+            for rec, rmax in ((1, 1 << 22), (1, 0), (0, 1 << 22)):   # rec_max 0: the record is dropped
+                runs.append((mk, f"{rec} rec_max={rmax} lazy={lz}", kgs.kgs_query(G, kw, 5, kgs.make_params(
+                    prune_min=8, mk_min=mk, dag_record=rec, lazy_dag=lz, rec_max=rmax))))
             for r in kgs.kgs_query_batch(G, [kw, kw[::-1]], 5,
                                          kgs.make_params(prune_min=8, mk_min=mk, lazy_dag=lz), 2):
                 runs.append((mk, f"batch lazy={lz}", r))
