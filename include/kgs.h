@@ -149,7 +149,7 @@ typedef struct kgs_result kgs_result; /* opaque: host copy of the answers (+ opt
  *   lazy_dag       0 / 1 [1]: pruning round 2 extends the shared predecessor DAG only as far as the
  *                  candidates' walks need before the exact key cut-off stops them (candidates whose cut is
  *                  valid, decided from the search's rm bits); 0 builds every round-2 closure first
- *   rec_max        >= 0 [2^22]: a recorded DAG (dag_record) of more arcs is dropped for the pre-pass when
+ *   rec_max        >= 0 [2^24]: a recorded DAG (dag_record) of more arcs is dropped for the pre-pass when
  *                  pruning runs (more than max(8k, prune_min) central nodes): its lists cover every touched
  *                  node, the pre-pass only the candidates' closures (with the lazy round 2) */
 typedef struct {

@@ -259,7 +259,7 @@ void kgs_params_default(kgs_params *p) {
     p->mk_min = 4096;
     p->defer_min = 1 << 16;
     p->lazy_dag = 1;
-    p->rec_max = 1 << 22;
+    p->rec_max = 1 << 24;
 }
 
 void kgs_free_graph(kgs_graph *g) {
