@@ -273,15 +273,32 @@ class Answer:
     arcs: np.ndarray   # [n_arcs, 2]
 
 
-@dataclass
 class Result:
-    answers: list
-    stats: dict
-    M: np.ndarray | None = None
-    a: np.ndarray | None = None
-    centrals: np.ndarray | None = None
-    central_depth: np.ndarray | None = None
-    central_key: np.ndarray | None = None
+    """One query's answers (kgs_result_*), plus its statistics.  The statistics dict (with the per-phase
+    times) is built on first access from the raw copies taken before the handle was freed: a batch of
+    thousands of results does not pay for it unless it is read."""
+
+    def __init__(self, answers, raw_stats, tags, tns, nph):
+        self.answers = answers
+        self._raw = (raw_stats, tags, tns, nph)
+        self._stats = None
+        self.M = self.a = self.centrals = self.central_depth = self.central_key = None
+
+    @property
+    def stats(self) -> dict:
+        if self._stats is None:
+            st, tags, tns, m = self._raw
+            stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
+            # per-phase durations (us): time from the previous stamp to this one, summed by phase name
+            ph = {}
+            if m > 1:
+                dur = np.diff(tns[:m].astype(np.int64)) / 1e3
+                sums = np.bincount(tags[1:m], weights=dur)
+                for t in np.flatnonzero(np.bincount(tags[1:m])):
+                    ph[PHASE_NAMES[t] if t < len(PHASE_NAMES) else str(t)] = float(sums[t])
+            stats["phases_us"] = ph
+            self._stats = stats
+        return self._stats
 
 
 def _read_result(h, n, q, want_levels) -> Result:
@@ -301,26 +318,19 @@ def _read_result(h, n, q, want_levels) -> Result:
         _check(L.kgs_result_export(h, cen.ctypes.data, dep.ctypes.data, key.ctypes.data, noff.ctypes.data,
                                    nodes.ctypes.data, aoff.ctypes.data, arcs.ctypes.data))
         arcs2 = arcs.reshape(-1, 2)
-        score = key.astype(np.float32)
-        answers = [Answer(int(cen[i]), int(dep[i]), float(score[i]), float(key[i]), nodes[noff[i]:noff[i + 1]],
-                          arcs2[aoff[i]:aoff[i + 1]]) for i in range(cnt)]
+        # Python scalars in one conversion per array (indexing numpy element by element is the slow part)
+        cl, dl, kl = cen.tolist(), dep.tolist(), key.tolist()
+        sl = key.astype(np.float32).tolist()
+        nl, al = noff.tolist(), aoff.tolist()
+        answers = [Answer(cl[i], dl[i], sl[i], kl[i], nodes[nl[i]:nl[i + 1]], arcs2[al[i]:al[i + 1]])
+                   for i in range(cnt)]
         st = kgs_stats()
         _check(L.kgs_result_stats(h, ctypes.byref(st)))
-        stats = {f: getattr(st, f) for f, _ in kgs_stats._fields_}
         tags = np.zeros(64, np.int32)
         tns = np.zeros(64, np.uint64)
         nph = ctypes.c_int32()
         _check(L.kgs_result_phases(h, tags.ctypes.data, tns.ctypes.data, 64, ctypes.byref(nph)))
-        m = min(nph.value, 64)
-        # per-phase durations (us): time from the previous stamp to this one, summed by phase name
-        ph = {}
-        if m > 1:
-            dur = np.diff(tns[:m].astype(np.int64)) / 1e3
-            sums = np.bincount(tags[1:m], weights=dur)
-            for t in np.flatnonzero(np.bincount(tags[1:m])):
-                ph[PHASE_NAMES[t] if t < len(PHASE_NAMES) else str(t)] = float(sums[t])
-        stats["phases_us"] = ph
-        res = Result(answers, stats)
+        res = Result(answers, st, tags, tns, min(nph.value, 64))
         if want_levels:
             M = np.empty(n * q, np.uint8)
             _check(L.kgs_result_levels(h, M.ctypes.data, M.size))
